@@ -1,0 +1,206 @@
+/*
+ * gd.h — C ABI of the B200-native GNNDrive sample + extract hot path.
+ *
+ * Paper: Jiang, Jia, Wang, "Reducing Memory Contention and I/O Congestion for
+ * Disk-based GNN Training" (ICPP'24, "GNNDrive").  "P:NNN" cites line NNN of the
+ * paper text (reference PAPER.md); "Alg. 1" is its Algorithm 1;
+ * readings R<k> are listed in DESIGN.md §3.
+ *
+ * Conventions for every entry point
+ *   - Returns a gd_status; no exception crosses the ABI.  On a non-OK status
+ *     gd_last_error() gives a thread-local message and no library state changed.
+ *   - "device" pointers are CUDA device (or managed) pointers on the handle's
+ *     device; "host or device" pointers are detected with cudaPointerGetAttributes.
+ *   - Every array argument is caller-owned; the library never frees it.  Library
+ *     state (HBM topology copy, hash workspace, mapping table, reverse map,
+ *     standby ring, slots, internal side stream and events) is owned by the handle
+ *     and released by the matching *_destroy.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).
+ *     Every call is stream-ordered on it and does NOT synchronise the host on the
+ *     hot path (gd_sample / gd_extract / gd_buffer_release).  Calls on one handle
+ *     must be externally serialised and ordered on one stream.
+ *   - Device-side precondition violations (duplicate / out-of-range seed or node
+ *     id, refcount underflow, exhausted standby list) cannot be detected on the
+ *     host without a sync; they set a sticky status word on the handle, reported
+ *     by gd_check_device_status().  Outputs of such a call are unspecified but all
+ *     memory accesses stay in bounds.
+ */
+#ifndef GD_H_
+#define GD_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define GD_MAX_HOPS 8
+#define GD_MAX_FANOUT 256   /* largest sampled fanout; -1 (= whole row) is also allowed */
+
+typedef enum {
+    GD_OK = 0,
+    GD_ERR_INVALID = 1,     /* bad argument (null pointer, size, hop count, fanout, CSR) */
+    GD_ERR_OOM = 2,         /* device or pinned allocation failed */
+    GD_ERR_CUDA = 3,        /* a CUDA runtime call failed */
+    GD_ERR_CAPACITY = 4,    /* buffer capacity / in-flight rule violated */
+    GD_ERR_DEVICE = 5       /* a device-side precondition check tripped (sticky) */
+} gd_status;
+
+/* device status bits (gd_check_device_status sets *bits) */
+#define GD_DEV_BAD_ID       0x1u   /* seed or node id outside [0, N) */
+#define GD_DEV_DUP_SEED     0x2u   /* a seed appears twice in one gd_sample call */
+#define GD_DEV_UNDERFLOW    0x4u   /* gd_buffer_release of a node with refcount 0 */
+#define GD_DEV_STANDBY_DRY  0x8u   /* fewer standby slots than misses (capacity rule broken) */
+
+typedef struct gd_graph gd_graph;
+typedef struct gd_buffer gd_buffer;
+
+/* Thread-local message describing the last non-OK status ("" if none). */
+const char* gd_last_error(void);
+
+/* Library version (major*10000 + minor*100 + patch). */
+int gd_version(void);
+
+/* ----------------------------------------------------------------------------
+ * Topology.  GNNDrive "forms the topological data of a graph as an adjacency
+ * matrix for efficient sampling" in compressed form (indptr / indices,
+ * P:146).  Reading R6: row v lists the nodes v samples from (pass the CSC
+ * of A, i.e. the CSR of A^T, to sample in-neighbours as P:41 does).
+ *
+ *   indptr   host or device int64[num_nodes+1], indptr[0] = 0, non-decreasing,
+ *            indptr[num_nodes] = num_edges.
+ *   indices  host or device int32[num_edges], each in [0, num_nodes).
+ *   validate nonzero: check the CSR on the device once (GD_ERR_INVALID on failure).
+ * The library copies both arrays into HBM on `device` (a replica per GPU)
+ * and keeps no reference to the caller's arrays.  num_nodes <= 2^31-1.
+ * ------------------------------------------------------------------------- */
+gd_status gd_graph_create(const int64_t* indptr, const int32_t* indices, int64_t num_nodes,
+                          int64_t num_edges, int device, int validate, gd_graph** out);
+gd_status gd_graph_destroy(gd_graph* g);
+
+/* Host-only worst-case sizes of one gd_sample call (no device work):
+ *   max_nodes[0] = num_seeds,
+ *   max_edges[h-1] = f_h < 0 ? num_edges : min(num_edges, max_nodes[h-1] * f_h),
+ *   max_nodes[h]   = min(num_nodes, max_nodes[h-1] + max_edges[h-1]),  h = 1..num_hops.
+ * max_nodes has num_hops+1 entries, max_edges num_hops. */
+gd_status gd_sample_bounds(int64_t num_seeds, const int32_t* fanouts, int32_t num_hops,
+                           int64_t num_nodes, int64_t num_edges, int64_t* max_nodes,
+                           int64_t* max_edges);
+
+/* Caller-allocated device outputs of gd_sample, sized from gd_sample_bounds. */
+typedef struct {
+    int32_t* n_id;                    /* [max_nodes[K]] sampled node ids, seeds first       */
+    int64_t* rowptr[GD_MAX_HOPS];     /* hop h: [max_nodes[h-1]+1] row offsets of block h   */
+    int32_t* col[GD_MAX_HOPS];        /* hop h: [max_edges[h-1]] local (relabelled) src ids */
+    int64_t* eid[GD_MAX_HOPS];        /* hop h: [max_edges[h-1]] CSR edge offsets, or NULL  */
+    int64_t* sizes;                   /* [2K+1]: n_0..n_K, e_1..e_K (device-resident)       */
+} gd_sample_out;
+
+/* ----------------------------------------------------------------------------
+ * Multi-hop neighbour sampling + relabel of one mini-batch (the sampler stage,
+ * "each sampler generates a subgraph for a mini-batch from which a list of
+ * sampled node IDs is made"; "3-hop random neighborhood sampling").
+ *
+ *   seeds      host or device int32[num_seeds], distinct, in [0, N) (the
+ *              mini-batch's training nodes).  n_id[0:num_seeds] = seeds.
+ *   fanouts    host int32[num_hops]; f in [0, GD_MAX_FANOUT] or -1 (whole row).
+ *   rng_seed   64-bit key of the counter-based Philox4x32-10 stream (R1).
+ *   batch_id   global mini-batch index; part of the Philox counter, so results
+ *              do not depend on the GPU count or call order (R2).
+ * Semantics (R3-R5): hop h expands every node of n_id[0:n_{h-1}] (cumulative
+ * frontier).  Node v of degree d gets min(f, d) distinct CSR positions (all of
+ * them if f < 0 or d <= f), drawn by Floyd's algorithm with draw t =
+ * floor(u_t * (j+1) / 2^64), u_t = Philox(ctr=(t, v, h-1, batch_id), key=rng_seed)
+ * words (y<<32|x), and listed in ascending position order.  Unseen neighbours
+ * get the next local ids in first-occurrence order and are appended to n_id.
+ * Block h = (rowptr[h], col[h], eid[h]) has dst = n_id[0:n_{h-1}], src =
+ * n_id[0:n_h].  sizes is written on the device; nothing is copied to the host.
+ * ------------------------------------------------------------------------- */
+gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const int32_t* fanouts,
+                    int32_t num_hops, uint64_t rng_seed, uint32_t batch_id, gd_sample_out* out,
+                    void* stream);
+
+/* ----------------------------------------------------------------------------
+ * Feature buffer: `capacity_slots` rows of `row_bytes` in HBM, a
+ * mapping table {slot, reference count, valid bit} per node, a reverse
+ * mapping array and an LRU standby list of slots with refcount 0
+ * (P:109).  The feature table (ascending node id) lives in
+ * pinned host memory, the SSD stand-in:
+ *
+ *   host_feat        host pointer to num_nodes*row_bytes bytes.  If not already
+ *                    page-locked it is registered (cudaHostRegisterMapped |
+ *                    Portable) and unregistered at destroy.  It must stay alive
+ *                    and unmodified until gd_buffer_destroy.
+ *   row_bytes        bytes per row, a multiple of 4 (16 for the vector path).
+ *   capacity_slots   S.  Must be >= min(N, max_inflight * max_nodes_per_batch):
+ *                    the paper's N_e x M_b reservation as a check
+ *                    (GD_ERR_CAPACITY), since a caller-driven API cannot wait
+ *                    for a releaser (R12).
+ *   max_inflight     most extracted-but-unreleased batches at any time (Q).
+ *   preload          nonzero: S >= N, node v resident in slot v from the start.
+ * Initial state: map = {-1, 0, 0}, reverse = -1, standby = [0, 1, .., S-1] (R10).
+ * ------------------------------------------------------------------------- */
+gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_bytes,
+                         int64_t capacity_slots, int32_t max_inflight,
+                         int64_t max_nodes_per_batch, int preload, int device, gd_buffer** out);
+gd_status gd_buffer_destroy(gd_buffer* b);
+
+/* ----------------------------------------------------------------------------
+ * Extraction of one mini-batch (Alg. 1):
+ *   loop 1: hits (valid) take their slot, leaving the standby list if their
+ *           refcount was 0; every node's refcount++;
+ *   loop 2: misses, in list order, take successive LRU standby slots; a slot's
+ *           previous node is invalidated (R9); map / reverse / alias updated;
+ *   the missed rows stream from the pinned host table into their slots and into
+ *   `out` on the library's side stream (asynchronous extraction),
+ *   overlapping the caller's next gd_sample; hit rows are gathered from the slots
+ *   into `out` on `stream` (the trainer's alias indexing, materialised).
+ *
+ *   node_ids  device int32[n], distinct, in [0, N) (normally gd_sample's n_id).
+ *   n_dev     device int64*: n (normally &sizes[K]); n <= n_max.
+ *   n_max     host bound on n (grid sizing); must be <= max_nodes_per_batch.
+ *   out       device [n_max * row_bytes] (16-byte aligned): out[i] = feat[node_ids[i]].
+ *   alias     device int32[n_max] or NULL: slot of node_ids[i] (Alg. 1 ids_r).
+ *   stats     device int64[2] or NULL: {hits, misses} of this batch.
+ *   done      cudaEvent_t (void*) or NULL: recorded when `out` is complete.
+ *             `out` is valid only after `done`; `stream` itself does NOT wait
+ *             for the misses.  node_ids must stay unmodified until `done`.
+ * GD_ERR_CAPACITY if this would exceed max_inflight unreleased batches.
+ * ------------------------------------------------------------------------- */
+gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,
+                     void* out, int32_t* alias, int64_t* stats, void* stream, void* done);
+
+/* ----------------------------------------------------------------------------
+ * Release stage: for node_ids in list order decrement the refcount; a
+ * slot whose count reaches zero is appended at the tail (MRU end) of the standby
+ * list.  The node stays valid until its slot is reused (delayed invalidation).
+ * Arguments as in gd_extract.  Stream-ordered; no host sync.
+ * ------------------------------------------------------------------------- */
+gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev,
+                            int64_t n_max, void* stream);
+
+/* Synchronises the handle's device and returns GD_ERR_DEVICE (and the sticky
+ * GD_DEV_* bits in *bits, if non-NULL) if a device-side check tripped since the
+ * handle was created.  `handle` is a gd_graph* or a gd_buffer*. */
+gd_status gd_check_device_status(void* handle, uint32_t* bits);
+
+/* ----------------------------------------------------------------------------
+ * Debug / test surface (synchronising; not for the hot path).
+ * ------------------------------------------------------------------------- */
+/* Copy the buffer state to host arrays (any may be NULL): map_slot/map_rc/
+ * map_valid [N], reverse [S], standby [S] in LRU order (head first); the number
+ * of standby slots is stored in *standby_len. */
+gd_status gd_buffer_snapshot(gd_buffer* b, int32_t* map_slot, int32_t* map_rc, uint8_t* map_valid,
+                             int32_t* reverse, int32_t* standby, int64_t* standby_len);
+/* Install an explicit state from host arrays (used for the Fig. 6 example,
+ * P:131); slot contents of valid nodes are loaded from the host table. */
+gd_status gd_buffer_set_state(gd_buffer* b, const int32_t* map_slot, const int32_t* map_rc,
+                              const uint8_t* map_valid, const int32_t* reverse,
+                              const int32_t* standby, int64_t standby_len);
+/* The internal side stream (cudaStream_t as void*) misses are copied on. */
+void* gd_buffer_side_stream(gd_buffer* b);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* GD_H_ */

@@ -1,0 +1,226 @@
+"""B200-native sample + extract hot path of GNNDrive (Jiang, Jia, Wang, ICPP'24).
+
+Thin Python binding over libgd.so (include/gd.h): argument marshalling only.  Every step
+of the path runs in the library's sm_100a kernels; torch provides device memory, streams
+and events.  Importing the package loads libgd.so and raises if it is missing.
+
+    g = Graph(indptr, indices, device=0)
+    out = g.sample(seeds, fanouts=(15, 10, 5), rng_seed=3, batch_id=b)     # gd_sample
+    buf = FeatureBuffer(host_feat_u8, capacity=S, max_inflight=4, max_nodes_per_batch=out.max_nodes)
+    feats, alias, done = buf.extract(out.n_id, out.num_nodes_dev, out.max_nodes)    # gd_extract
+    ...                                   # consumer waits `done`, trains on feats
+    buf.release(out.n_id, out.num_nodes_dev, out.max_nodes)                # gd_buffer_release
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import _lib
+from ._lib import GD_MAX_HOPS, GdError, SampleOutC, check, lib
+
+__all__ = ["Graph", "SampleOut", "FeatureBuffer", "GdError", "sample_bounds", "check_device_status", "lib"]
+
+
+def _ptr(t):
+    return ctypes.c_void_p(t.data_ptr()) if t is not None else None
+
+
+def _stream_ptr(stream, device):
+    s = stream if stream is not None else torch.cuda.current_stream(device)
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def sample_bounds(num_seeds: int, fanouts, num_nodes: int, num_edges: int):
+    """gd_sample_bounds: (max_nodes[K+1], max_edges[K]) as Python lists."""
+    K = len(fanouts)
+    f = (ctypes.c_int32 * K)(*fanouts)
+    nm = (ctypes.c_int64 * (K + 1))()
+    em = (ctypes.c_int64 * K)()
+    check(lib.gd_sample_bounds(num_seeds, f, K, num_nodes, num_edges, nm, em))
+    return list(nm), list(em)
+
+
+class SampleOut:
+    """Device outputs of one gd_sample call, allocated at the worst-case bounds."""
+
+    def __init__(self, max_nodes, max_edges, device, with_eid=False):
+        K = len(max_edges)
+        self.K = K
+        self.max_nodes_list = list(max_nodes)
+        self.max_edges_list = list(max_edges)
+        self.max_nodes = int(max_nodes[-1])
+        dev = torch.device("cuda", device)
+        self.n_id = torch.empty(max(1, self.max_nodes), dtype=torch.int32, device=dev)
+        self.rowptr = [torch.empty(max_nodes[h] + 1, dtype=torch.int64, device=dev) for h in range(K)]
+        self.col = [torch.empty(max(1, max_edges[h]), dtype=torch.int32, device=dev) for h in range(K)]
+        self.eid = [torch.empty(max(1, max_edges[h]), dtype=torch.int64, device=dev) for h in range(K)] if with_eid else None
+        self.sizes = torch.zeros(2 * K + 1, dtype=torch.int64, device=dev)
+
+    @property
+    def num_nodes_dev(self) -> torch.Tensor:
+        """Device int64 scalar n_K (a view of sizes[K]) for gd_extract / gd_buffer_release."""
+        return self.sizes[self.K:self.K + 1]
+
+    def cstruct(self) -> SampleOutC:
+        c = SampleOutC()
+        c.n_id = self.n_id.data_ptr()
+        for h in range(self.K):
+            c.rowptr[h] = self.rowptr[h].data_ptr()
+            c.col[h] = self.col[h].data_ptr()
+            c.eid[h] = self.eid[h].data_ptr() if self.eid is not None else None
+        c.sizes = self.sizes.data_ptr()
+        return c
+
+    def to_host(self):
+        """Synchronising copy of the trimmed result (tests / inspection only)."""
+        sizes = self.sizes.cpu()
+        K = self.K
+        nK = int(sizes[K])
+        res = {"sizes": sizes.numpy(), "n_id": self.n_id[:nK].cpu().numpy(), "rowptr": [], "col": [], "eid": []}
+        for h in range(K):
+            n_prev, e_h = int(sizes[h]), int(sizes[K + 1 + h])
+            res["rowptr"].append(self.rowptr[h][:n_prev + 1].cpu().numpy())
+            res["col"].append(self.col[h][:e_h].cpu().numpy())
+            res["eid"].append(self.eid[h][:e_h].cpu().numpy() if self.eid is not None else None)
+        return res
+
+
+class Graph:
+    """gd_graph: an HBM replica of a CSR topology (int64 indptr, int32 indices)."""
+
+    def __init__(self, indptr: torch.Tensor, indices: torch.Tensor, device: int = 0, validate: bool = True):
+        assert indptr.dtype == torch.int64 and indices.dtype == torch.int32
+        indptr = indptr.contiguous()
+        indices = indices.contiguous()
+        self.num_nodes = indptr.numel() - 1
+        self.num_edges = indices.numel()
+        self.device = device
+        h = ctypes.c_void_p()
+        check(lib.gd_graph_create(_ptr(indptr), _ptr(indices), self.num_nodes, self.num_edges, device,
+                                  int(validate), ctypes.byref(h)))
+        self._h = h
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.gd_graph_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    def bounds(self, num_seeds: int, fanouts):
+        return sample_bounds(num_seeds, fanouts, self.num_nodes, self.num_edges)
+
+    def alloc_out(self, num_seeds: int, fanouts, with_eid=False) -> SampleOut:
+        nm, em = self.bounds(num_seeds, fanouts)
+        return SampleOut(nm, em, self.device, with_eid)
+
+    def sample(self, seeds: torch.Tensor, fanouts, rng_seed: int, batch_id: int, out: SampleOut | None = None,
+               stream=None, with_eid: bool = False) -> SampleOut:
+        """gd_sample.  `seeds` int32 on the device or in (pinned) host memory."""
+        assert seeds.dtype == torch.int32 and seeds.is_contiguous()
+        fanouts = list(fanouts)
+        if out is None:
+            out = self.alloc_out(seeds.numel(), fanouts, with_eid)
+        K = len(fanouts)
+        f = (ctypes.c_int32 * K)(*fanouts)
+        cs = out.cstruct()
+        check(lib.gd_sample(self._h, _ptr(seeds), seeds.numel(), f, K, ctypes.c_uint64(rng_seed),
+                            ctypes.c_uint32(batch_id & 0xFFFFFFFF), ctypes.byref(cs), _stream_ptr(stream, self.device)))
+        return out
+
+    def check(self):
+        return check_device_status(self._h)
+
+
+class FeatureBuffer:
+    """gd_buffer: slot-managed HBM feature buffer over a pinned host table (the SSD stand-in)."""
+
+    def __init__(self, host_feat: torch.Tensor, capacity: int, max_inflight: int, max_nodes_per_batch: int,
+                 preload: bool = False, device: int = 0):
+        assert host_feat.device.type == "cpu" and host_feat.dtype == torch.uint8 and host_feat.dim() == 2
+        assert host_feat.is_contiguous()
+        self.host_feat = host_feat          # keep alive until destroy
+        self.num_nodes, self.row_bytes = host_feat.shape
+        self.capacity = int(capacity)
+        self.max_inflight = int(max_inflight)
+        self.max_nodes_per_batch = int(max_nodes_per_batch)
+        self.device = device
+        h = ctypes.c_void_p()
+        check(lib.gd_buffer_init(_ptr(host_feat), self.num_nodes, self.row_bytes, self.capacity, self.max_inflight,
+                                 self.max_nodes_per_batch, int(preload), device, ctypes.byref(h)))
+        self._h = h
+        sp = lib.gd_buffer_side_stream(h)
+        self.side_stream = torch.cuda.ExternalStream(sp, device=torch.device("cuda", device))
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.gd_buffer_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
+
+    def alloc_out(self, n_max: int) -> torch.Tensor:
+        return torch.empty((max(1, n_max), self.row_bytes), dtype=torch.uint8, device=torch.device("cuda", self.device))
+
+    def extract(self, node_ids: torch.Tensor, n_dev: torch.Tensor, n_max: int, out: torch.Tensor | None = None,
+                alias: torch.Tensor | None = None, stats: torch.Tensor | None = None, stream=None,
+                done: torch.cuda.Event | None = None):
+        """gd_extract.  Returns (out, alias, done); `out` is valid after `done`."""
+        if out is None:
+            out = self.alloc_out(n_max)
+        if done is None:
+            done = torch.cuda.Event()
+        check(lib.gd_extract(self._h, _ptr(node_ids), _ptr(n_dev), int(n_max), _ptr(out), _ptr(alias), _ptr(stats),
+                             _stream_ptr(stream, self.device), ctypes.c_void_p(done.cuda_event)))
+        return out, alias, done
+
+    def release(self, node_ids: torch.Tensor, n_dev: torch.Tensor, n_max: int, stream=None):
+        check(lib.gd_buffer_release(self._h, _ptr(node_ids), _ptr(n_dev), int(n_max), _stream_ptr(stream, self.device)))
+
+    def snapshot(self):
+        import numpy as np
+        N, S = self.num_nodes, self.capacity
+        ms = np.zeros(N, dtype=np.int32)
+        mr = np.zeros(N, dtype=np.int32)
+        mv = np.zeros(N, dtype=np.uint8)
+        rv = np.zeros(S, dtype=np.int32)
+        sb = np.zeros(S, dtype=np.int32)
+        k = ctypes.c_int64()
+        p = lambda a: a.ctypes.data_as(ctypes.c_void_p)  # noqa: E731
+        check(lib.gd_buffer_snapshot(self._h, p(ms), p(mr), p(mv), p(rv), p(sb), ctypes.byref(k)))
+        return {"slot": ms, "rc": mr, "valid": mv, "reverse": rv, "standby": sb[:k.value].copy()}
+
+    def set_state(self, slot, rc, valid, reverse, standby):
+        import numpy as np
+        a = [np.ascontiguousarray(x, dtype=t) for x, t in
+             ((slot, np.int32), (rc, np.int32), (valid, np.uint8), (reverse, np.int32), (standby, np.int32))]
+        p = lambda x: x.ctypes.data_as(ctypes.c_void_p)  # noqa: E731
+        check(lib.gd_buffer_set_state(self._h, p(a[0]), p(a[1]), p(a[2]), p(a[3]), p(a[4]), len(a[4])))
+
+    def check(self):
+        return check_device_status(self._h)
+
+
+def check_device_status(handle) -> int:
+    """gd_check_device_status: raises GdError if a device-side check tripped."""
+    bits = ctypes.c_uint32()
+    check(lib.gd_check_device_status(handle, ctypes.byref(bits)))
+    return bits.value

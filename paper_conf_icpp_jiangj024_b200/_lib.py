@@ -1,0 +1,79 @@
+"""ctypes declarations of libgd.so (include/gd.h).  Argument marshalling only.
+
+The library is REQUIRED: importing this module raises if libgd.so is missing or does not
+load.  There is no fallback path of any kind.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libgd.so")
+GD_MAX_HOPS = 8
+GD_MAX_FANOUT = 256
+
+STATUS = {0: "GD_OK", 1: "GD_ERR_INVALID", 2: "GD_ERR_OOM", 3: "GD_ERR_CUDA", 4: "GD_ERR_CAPACITY",
+          5: "GD_ERR_DEVICE"}
+DEV_BITS = {0x1: "GD_DEV_BAD_ID", 0x2: "GD_DEV_DUP_SEED", 0x4: "GD_DEV_UNDERFLOW", 0x8: "GD_DEV_STANDBY_DRY"}
+
+# every entry point include/gd.h declares (checked by tests/test_abi.py)
+EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy", "gd_sample_bounds", "gd_sample",
+           "gd_buffer_init", "gd_buffer_destroy", "gd_extract", "gd_buffer_release", "gd_check_device_status",
+           "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream"]
+
+
+class GdError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+        self.status = status
+
+
+class SampleOutC(ctypes.Structure):
+    _fields_ = [("n_id", ctypes.c_void_p),
+                ("rowptr", ctypes.c_void_p * GD_MAX_HOPS),
+                ("col", ctypes.c_void_p * GD_MAX_HOPS),
+                ("eid", ctypes.c_void_p * GD_MAX_HOPS),
+                ("sizes", ctypes.c_void_p)]
+
+
+_vp = ctypes.c_void_p
+_i64 = ctypes.c_int64
+_i32 = ctypes.c_int32
+_st = ctypes.c_int
+
+
+def _load():
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_jiangj024_b200._build` "
+                          "(or __graft_entry__.build()); there is no non-CUDA fallback")
+    L = ctypes.CDLL(LIB_PATH)
+    L.gd_last_error.restype = ctypes.c_char_p
+    L.gd_last_error.argtypes = []
+    L.gd_version.restype = ctypes.c_int
+    L.gd_graph_create.argtypes = [_vp, _vp, _i64, _i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)]
+    L.gd_graph_destroy.argtypes = [_vp]
+    L.gd_sample_bounds.argtypes = [_i64, _vp, _i32, _i64, _i64, _vp, _vp]
+    L.gd_sample.argtypes = [_vp, _vp, _i64, _vp, _i32, ctypes.c_uint64, ctypes.c_uint32,
+                            ctypes.POINTER(SampleOutC), _vp]
+    L.gd_buffer_init.argtypes = [_vp, _i64, _i64, _i64, _i32, _i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)]
+    L.gd_buffer_destroy.argtypes = [_vp]
+    L.gd_extract.argtypes = [_vp, _vp, _vp, _i64, _vp, _vp, _vp, _vp, _vp]
+    L.gd_buffer_release.argtypes = [_vp, _vp, _vp, _i64, _vp]
+    L.gd_check_device_status.argtypes = [_vp, ctypes.POINTER(ctypes.c_uint32)]
+    L.gd_buffer_snapshot.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, ctypes.POINTER(_i64)]
+    L.gd_buffer_set_state.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i64]
+    L.gd_buffer_side_stream.argtypes = [_vp]
+    L.gd_buffer_side_stream.restype = _vp
+    for name in EXPORTS:
+        if name not in ("gd_last_error", "gd_version", "gd_buffer_side_stream"):
+            getattr(L, name).restype = _st
+    return L
+
+
+lib = _load()
+
+
+def check(status: int):
+    if status != 0:
+        raise GdError(status, lib.gd_last_error().decode())

@@ -1,0 +1,876 @@
+// gd_buffer.cu — the slot-managed feature buffer and extraction (rows a5-a9).
+//
+// gd_extract(b), all stream-ordered, no host sync:
+//   caller stream:  k_lookup (Alg. 1 loop 1 + miss ranks) -> k_pop_assign (loop 2:
+//                   LRU standby slots, eviction, map/reverse/alias) -> [L_b]
+//                   -> wait X_{b-1} -> k_gather_hits (slots -> out) -> [G_b]
+//   side stream:    wait L_b -> k_miss_copy (pinned host -> slot + out) -> [X_b]
+//                   -> wait G_b -> [done]
+// gd_buffer_release(b): k_compact (only when the ring is nearly full; exits at once
+//   otherwise) -> k_release (refcount--, became-zero slots appended at the tail).
+//
+// Standby list: a ring of slot ids in LRU order with lazy deletion.  A slot's
+// live entry is the one at pos_of_slot[slot]; removing a slot (a hit whose refcount was
+// 0, Alg. 1 line 11) just sets pos_of_slot = -1.  Popping takes the first M live entries
+// from head (a ticketed look-back scan that stops at the M-th), pushing appends at tail.
+#include <algorithm>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "gd_common.cuh"
+#include "gd_handles.cuh"
+
+namespace gd {
+
+constexpr int kBThreads = 256;
+constexpr int kBItems = 8;
+constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
+constexpr int kBWarps = kBThreads / 32;
+
+static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// Block-wide ordered scan of per-item 0/1 flags in striped arrangement
+// (item k of thread t = element k*256 + t).  ball[k] = warp ballot of round k.
+// Fills s_cnt[k*8+warp] with the exclusive block offset of (round k, warp) and
+// returns the block aggregate in every thread of warp 0 (others: unspecified).
+__device__ __forceinline__ int block_flag_offsets(const unsigned (&ball)[kBItems], int* s_cnt) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k)
+        if (lane == 0) s_cnt[k * kBWarps + warp] = __popc(ball[k]);
+    __syncthreads();
+    int agg = 0;
+    if (warp == 0) {
+        const int c0 = s_cnt[2 * lane], c1 = s_cnt[2 * lane + 1];
+        const int inc = warp_inclusive_sum(c0 + c1);
+        agg = __shfl_sync(0xffffffffu, inc, 31);
+        __syncwarp();
+        s_cnt[2 * lane] = inc - c0 - c1;
+        s_cnt[2 * lane + 1] = inc - c1;
+    }
+    return agg;
+}
+
+// ------------------------------------------------------------------ a5: lookup
+struct LookupArgs {
+    const int32_t* ids;
+    const int64_t* n_dev;
+    int64_t N;
+    int2* map;
+    int32_t* pos_of_slot;
+    int32_t* alias;
+    uint8_t* missflag;
+    int32_t* misslist;
+    int64_t* mcount;
+    int64_t* stats;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+    unsigned int* status;
+};
+
+__global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const int64_t n = *a.n_dev;
+    const int64_t tile = blockIdx.x;
+    const int64_t i0 = tile * kBTile;
+    if (i0 >= n && tile != 0) return;
+    __shared__ int s_cnt[kBItems * kBWarps];
+    __shared__ long long s_base;
+    const int t = threadIdx.x, lane = t & 31;
+    unsigned ball[kBItems];
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k) {
+        const int64_t i = i0 + (int64_t)k * kBThreads + t;
+        bool miss = false;
+        if (i < n) {
+            const int32_t v = a.ids[i];
+            int32_t al = -1;
+            if (v < 0 || (int64_t)v >= a.N) {
+                atomicOr(a.status, GD_DEV_BAD_ID);
+            } else {
+                const int2 m = a.map[v];
+                const int valid = m.y & 1;
+                const int rc = m.y >> 1;
+                if (valid) {                                   // Alg. 1 lines 8-13
+                    al = m.x;
+                    if (rc == 0) a.pos_of_slot[m.x] = -1;      // line 11: leave the standby list
+                } else if (rc > 0) {                           // lines 14-17 (R8: not reachable
+                    al = m.x;                                  // on the GPU, valid is set at alloc)
+                } else {
+                    miss = true;
+                }
+                a.map[v].y = ((rc + 1) << 1) | valid;           // line 19
+            }
+            a.alias[i] = al;
+            a.missflag[i] = miss ? 1 : 0;
+        }
+        ball[k] = __ballot_sync(0xffffffffu, miss);
+    }
+    const int agg = block_flag_offsets(ball, s_cnt);
+    if ((t >> 5) == 0) {
+        const long long base = lookback_exclusive(a.st, tile, agg, 0);
+        if (lane == 0) {
+            s_base = base;
+            const bool last = (n == 0) ? (tile == 0) : (tile == (n - 1) / kBTile);
+            if (last) {
+                const long long M = base + agg;
+                *a.mcount = M;
+                if (a.stats) {
+                    a.stats[0] = n - M;
+                    a.stats[1] = M;
+                }
+            }
+        }
+    }
+    __syncthreads();
+    const long long base = s_base;
+    const int warp = t >> 5;
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k)
+        if (ball[k] & (1u << lane))
+            a.misslist[base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt)] =
+                (int32_t)(i0 + (int64_t)k * kBThreads + t);
+}
+
+// ------------------------------------------------------- a6: pop + assign (loop 2)
+struct PopArgs {
+    const int32_t* ring;
+    const GdCtl* ctl_in;
+    GdCtl* ctl_out;
+    int32_t* pos_of_slot;
+    int2* map;
+    int32_t* reverse;
+    const int32_t* ids;
+    const int32_t* misslist;
+    const int64_t* mcount;
+    int32_t* alias;
+    int4* trip;
+    int64_t* trip_count;
+    unsigned long long* ticket;     // [2]: next tile, blocks finished
+    unsigned long long* done_word;
+    unsigned long long epoch;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+    unsigned int* status;
+};
+
+__device__ __forceinline__ void ticket_finish(unsigned long long* ticket) {
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        __threadfence();
+        const unsigned long long old = atomicAdd(ticket + 1, 1ull);
+        if (old == gridDim.x - 1) {   // last block out resets the counters for the next launch
+            ticket[0] = 0;
+            ticket[1] = 0;
+            __threadfence();
+        }
+    }
+}
+
+__global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const long long M = *a.mcount;
+    const GdCtl c = *a.ctl_in;
+    __shared__ long long s_tile;
+    __shared__ int s_stop;
+    __shared__ int s_cnt[kBItems * kBWarps];
+    __shared__ long long s_base;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    if (M == 0) {
+        if (blockIdx.x == 0 && t == 0) {
+            *a.ctl_out = c;
+            *a.trip_count = 0;
+        }
+        ticket_finish(a.ticket);
+        return;
+    }
+    while (true) {
+        if (t == 0) {
+            const long long tl = (long long)atomicAdd(a.ticket, 1ull);
+            s_tile = tl;
+            s_stop = (ld_relaxed_u64(a.done_word) == a.epoch) || (c.head + tl * kBTile >= c.tail && tl > 0);
+        }
+        __syncthreads();
+        if (s_stop) break;
+        const long long tl = s_tile;
+        const long long p0 = c.head + tl * kBTile;
+        unsigned ball[kBItems];
+        int32_t slot[kBItems];
+#pragma unroll
+        for (int k = 0; k < kBItems; ++k) {
+            const long long p = p0 + (long long)k * kBThreads + t;
+            bool live = false;
+            slot[k] = -1;
+            if (p < c.tail) {
+                slot[k] = a.ring[p];
+                live = (a.pos_of_slot[slot[k]] == (int32_t)p);
+            }
+            ball[k] = __ballot_sync(0xffffffffu, live);
+        }
+        const int agg = block_flag_offsets(ball, s_cnt);
+        if (warp == 0) {
+            const long long base = lookback_exclusive(a.st, tl, agg, 0);
+            if (lane == 0) {
+                s_base = base;
+                const bool last_tile = (p0 + kBTile >= c.tail);
+                if (last_tile && base + agg < M) {       // standby list ran dry (capacity rule)
+                    atomicOr(a.status, GD_DEV_STANDBY_DRY);
+                    GdCtl o = c;
+                    o.head = c.tail;
+                    *a.ctl_out = o;
+                    *a.trip_count = base + agg;
+                    __threadfence();
+                    st_relaxed_u64(a.done_word, a.epoch);
+                }
+            }
+        }
+        __syncthreads();
+        const long long base = s_base;
+        if (base < M) {
+            const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+            for (int k = 0; k < kBItems; ++k) {
+                if (!(ball[k] & (1u << lane))) continue;
+                const long long rank = base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);
+                if (rank >= M) continue;
+                const int32_t s = slot[k];
+                const int32_t i = a.misslist[rank];
+                const int32_t v = a.ids[i];
+                const int32_t old = a.reverse[s];
+                if (old >= 0) a.map[old] = make_int2(-1, 0);   // invalidate (R9)
+                const int2 m = a.map[v];
+                a.map[v] = make_int2(s, m.y | 1);               // lines 27, 37
+                a.reverse[s] = v;                               // line 28
+                a.alias[i] = s;                                 // line 29
+                a.pos_of_slot[s] = -1;
+                a.trip[rank] = make_int4(v, s, i, 0);
+                if (rank == M - 1) {
+                    const long long p = p0 + (long long)k * kBThreads + t;
+                    GdCtl o = c;
+                    o.head = p + 1;
+                    *a.ctl_out = o;
+                    *a.trip_count = M;
+                    __threadfence();
+                    st_relaxed_u64(a.done_word, a.epoch);
+                }
+            }
+        }
+        __syncthreads();
+    }
+    ticket_finish(a.ticket);
+}
+
+// ------------------------------------------------------------ a7: miss stream
+// One 16-byte chunk per thread-iteration, UNROLL chunks in flight per thread.
+template <int UNROLL>
+__global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ count,
+                                                   const uint8_t* __restrict__ feat, uint8_t* __restrict__ slots,
+                                                   uint8_t* __restrict__ out, int64_t R) {
+    const int64_t M = *count;
+    const int64_t cpr = R >> 4;                     // 16-byte chunks per row
+    const int64_t total = M * cpr;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; base < total; base += stride * UNROLL) {
+        uint4 val[UNROLL];
+        int64_t dsl[UNROLL], dout[UNROLL];
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) {
+            const int64_t idx = base + (int64_t)u * stride;
+            dsl[u] = -1;
+            if (idx < total) {
+                const int64_t r = idx / cpr, c = idx - r * cpr;
+                const int4 tr = __ldg(trip + r);
+                const uint4* src = (const uint4*)(feat + (int64_t)tr.x * R) + c;
+                asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                             : "=r"(val[u].x), "=r"(val[u].y), "=r"(val[u].z), "=r"(val[u].w)
+                             : "l"(src));
+                dsl[u] = (int64_t)tr.y * R + c * 16;
+                dout[u] = (int64_t)tr.z * R + c * 16;
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) {
+            if (dsl[u] >= 0) {
+                *(uint4*)(slots + dsl[u]) = val[u];
+                *(uint4*)(out + dout[u]) = val[u];
+            }
+        }
+    }
+}
+
+// 4-byte fallback for rows that are not a multiple of 16 bytes
+__global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __restrict__ count,
+                               const uint8_t* __restrict__ feat, uint8_t* __restrict__ slots,
+                               uint8_t* __restrict__ out, int64_t R) {
+    const int64_t M = *count;
+    const int64_t cpr = R >> 2;
+    const int64_t total = M * cpr;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = idx / cpr, c = idx - r * cpr;
+        const int4 tr = trip[r];
+        const uint32_t v = ((const uint32_t*)(feat + (int64_t)tr.x * R))[c];
+        ((uint32_t*)(slots + (int64_t)tr.y * R))[c] = v;
+        ((uint32_t*)(out + (int64_t)tr.z * R))[c] = v;
+    }
+}
+
+// ------------------------------------------------------------- a8: hit gather
+template <int UNROLL>
+__global__ void __launch_bounds__(256) k_gather_hits(const int32_t* __restrict__ alias, const uint8_t* __restrict__ missflag,
+                                                     const int64_t* __restrict__ n_dev, const uint8_t* __restrict__ slots,
+                                                     uint8_t* __restrict__ out, int64_t R) {
+    const int64_t n = *n_dev;
+    const int64_t cpr = R >> 4;
+    const int64_t total = n * cpr;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; base < total; base += stride * UNROLL) {
+        uint4 val[UNROLL];
+        int64_t dst[UNROLL];
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u) {
+            const int64_t idx = base + (int64_t)u * stride;
+            dst[u] = -1;
+            if (idx < total) {
+                const int64_t r = idx / cpr, c = idx - r * cpr;
+                const int32_t s = __ldg(alias + r);
+                if (!__ldg(missflag + r) && s >= 0) {
+                    const uint4* src = (const uint4*)(slots + (int64_t)s * R) + c;
+                    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                                 : "=r"(val[u].x), "=r"(val[u].y), "=r"(val[u].z), "=r"(val[u].w)
+                                 : "l"(src));
+                    dst[u] = idx * 16;   // out row r chunk c = flat idx
+                }
+            }
+        }
+#pragma unroll
+        for (int u = 0; u < UNROLL; ++u)
+            if (dst[u] >= 0) *(uint4*)(out + dst[u]) = val[u];
+    }
+}
+
+__global__ void k_gather_hits_w4(const int32_t* __restrict__ alias, const uint8_t* __restrict__ missflag,
+                                 const int64_t* __restrict__ n_dev, const uint8_t* __restrict__ slots,
+                                 uint8_t* __restrict__ out, int64_t R) {
+    const int64_t n = *n_dev;
+    const int64_t cpr = R >> 2;
+    const int64_t total = n * cpr;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = idx / cpr, c = idx - r * cpr;
+        const int32_t s = alias[r];
+        if (missflag[r] || s < 0) continue;
+        ((uint32_t*)out)[idx] = ((const uint32_t*)(slots + (int64_t)s * R))[c];
+    }
+}
+
+// ------------------------------------------------------------ a9: release
+struct ReleaseArgs {
+    const int32_t* ids;
+    const int64_t* n_dev;
+    int64_t N;
+    int2* map;
+    int32_t* ring;
+    int32_t* pos_of_slot;
+    const GdCtl* ctl_in;
+    GdCtl* ctl_out;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+    unsigned int* status;
+};
+
+__global__ void __launch_bounds__(kBThreads) k_release(ReleaseArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const int64_t n = *a.n_dev;
+    const int64_t tile = blockIdx.x;
+    const int64_t i0 = tile * kBTile;
+    const GdCtl c = *a.ctl_in;
+    if (i0 >= n && tile != 0) return;
+    __shared__ int s_cnt[kBItems * kBWarps];
+    __shared__ long long s_base;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    unsigned ball[kBItems];
+    int32_t slot[kBItems];
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k) {
+        const int64_t i = i0 + (int64_t)k * kBThreads + t;
+        bool zero = false;
+        slot[k] = -1;
+        if (i < n) {
+            const int32_t v = a.ids[i];
+            if (v < 0 || (int64_t)v >= a.N) {
+                atomicOr(a.status, GD_DEV_BAD_ID);
+            } else {
+                const int2 m = a.map[v];
+                const int rc = m.y >> 1;
+                if (rc <= 0) {
+                    atomicOr(a.status, GD_DEV_UNDERFLOW);
+                } else {
+                    a.map[v].y = ((rc - 1) << 1) | (m.y & 1);
+                    zero = (rc == 1) && m.x >= 0;
+                    slot[k] = m.x;
+                }
+            }
+        }
+        ball[k] = __ballot_sync(0xffffffffu, zero);
+    }
+    const int agg = block_flag_offsets(ball, s_cnt);
+    if (warp == 0) {
+        const long long base = lookback_exclusive(a.st, tile, agg, 0);
+        if (lane == 0) {
+            s_base = base;
+            const bool last = (n == 0) ? (tile == 0) : (tile == (n - 1) / kBTile);
+            if (last) {
+                GdCtl o = c;
+                o.tail = c.tail + base + agg;
+                *a.ctl_out = o;
+            }
+        }
+    }
+    __syncthreads();
+    const long long base = s_base;
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k) {
+        if (!(ball[k] & (1u << lane))) continue;
+        const long long p = c.tail + base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);
+        a.ring[p] = slot[k];                 // append at the tail of the standby list
+        a.pos_of_slot[slot[k]] = (int32_t)p;
+    }
+}
+
+// ------------------------------------------- ring compaction (rare, before a release)
+struct CompactArgs {
+    int32_t* ring;
+    int32_t* pos_of_slot;
+    const GdCtl* ctl_in;
+    GdCtl* ctl_out;
+    int64_t C;
+    int64_t n_max;
+    unsigned long long* ticket;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+};
+
+__global__ void __launch_bounds__(kBThreads) k_compact(CompactArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const GdCtl c = *a.ctl_in;
+    const bool need = (c.tail + a.n_max > c.base + a.C);
+    if (!need) {
+        if (blockIdx.x == 0 && threadIdx.x == 0) *a.ctl_out = c;
+        return;
+    }
+    const long long nbase = (c.base == 0) ? a.C : 0;
+    __shared__ long long s_tile;
+    __shared__ int s_cnt[kBItems * kBWarps];
+    __shared__ long long s_base;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    const long long ntiles = (c.tail - c.head + kBTile - 1) / kBTile;
+    while (true) {
+        if (t == 0) s_tile = (long long)atomicAdd(a.ticket, 1ull);
+        __syncthreads();
+        const long long tl = s_tile;
+        if (tl >= ntiles && !(tl == 0)) break;
+        const long long p0 = c.head + tl * kBTile;
+        unsigned ball[kBItems];
+        int32_t slot[kBItems];
+#pragma unroll
+        for (int k = 0; k < kBItems; ++k) {
+            const long long p = p0 + (long long)k * kBThreads + t;
+            bool live = false;
+            slot[k] = -1;
+            if (p < c.tail) {
+                slot[k] = a.ring[p];
+                live = (a.pos_of_slot[slot[k]] == (int32_t)p);
+            }
+            ball[k] = __ballot_sync(0xffffffffu, live);
+        }
+        const int agg = block_flag_offsets(ball, s_cnt);
+        if (warp == 0) {
+            const long long base = lookback_exclusive(a.st, tl, agg, 0);
+            if (lane == 0) {
+                s_base = base;
+                if (tl == (ntiles > 0 ? ntiles - 1 : 0)) {
+                    GdCtl o;
+                    o.base = nbase;
+                    o.head = nbase;
+                    o.tail = nbase + base + agg;
+                    *a.ctl_out = o;
+                }
+            }
+        }
+        __syncthreads();
+        const long long base = s_base;
+        const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+        for (int k = 0; k < kBItems; ++k) {
+            if (!(ball[k] & (1u << lane))) continue;
+            const long long q = nbase + base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);
+            a.ring[q] = slot[k];
+            a.pos_of_slot[slot[k]] = (int32_t)q;
+        }
+        __syncthreads();
+        if (tl >= ntiles - 1) break;
+    }
+    ticket_finish(a.ticket);
+}
+
+// ------------------------------------------------------------------- init
+__global__ void k_init_map(int2* map, int64_t N, int preload) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N; v += (int64_t)gridDim.x * blockDim.x)
+        map[v] = preload ? make_int2((int32_t)v, 1) : make_int2(-1, 0);
+}
+__global__ void k_init_slots(int32_t* reverse, int32_t* pos_of_slot, int32_t* ring, int64_t S, int64_t N,
+                             int preload) {
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < S; s += (int64_t)gridDim.x * blockDim.x) {
+        reverse[s] = (preload && s < N) ? (int32_t)s : -1;
+        pos_of_slot[s] = (int32_t)s;
+        ring[s] = (int32_t)s;
+    }
+}
+
+}  // namespace gd
+
+using namespace gd;
+
+static void buffer_free(gd_buffer* b) {
+    if (!b) return;
+    DeviceGuard guard(b->hdr.device);
+    if (b->side) cudaStreamSynchronize(b->side);
+    void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->missflag,
+                    b->alias_ws, b->mcount, b->trip, b->trip_count, b->tickets, b->done_word, b->hdr.dev_status};
+    for (void* p : ptrs)
+        if (p) cudaFree(p);
+    b->scan.release();
+    for (cudaEvent_t e : b->ev_trip)
+        if (e) cudaEventDestroy(e);
+    if (b->ev_L) cudaEventDestroy(b->ev_L);
+    if (b->ev_X) cudaEventDestroy(b->ev_X);
+    if (b->ev_G) cudaEventDestroy(b->ev_G);
+    if (b->side) cudaStreamDestroy(b->side);
+    if (b->registered) cudaHostUnregister((void*)b->host_feat);
+    b->hdr.magic = 0;
+    delete b;
+}
+
+extern "C" {
+
+gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_bytes, int64_t capacity_slots,
+                         int32_t max_inflight, int64_t max_nodes_per_batch, int preload, int device,
+                         gd_buffer** out) {
+    if (!host_feat || !out) return set_error(GD_ERR_INVALID, "gd_buffer_init: null pointer");
+    if (num_nodes < 1 || num_nodes > 0x7FFFFFFFLL || row_bytes < 4 || (row_bytes & 3) ||
+        capacity_slots < 1 || max_inflight < 1 || max_nodes_per_batch < 1)
+        return set_error(GD_ERR_INVALID, "gd_buffer_init: bad size (row_bytes must be a positive multiple of 4)");
+    if (preload && capacity_slots < num_nodes)
+        return set_error(GD_ERR_INVALID, "gd_buffer_init: preload needs capacity_slots >= num_nodes");
+    const int64_t need = std::min<int64_t>(num_nodes, (int64_t)max_inflight * max_nodes_per_batch);
+    if (capacity_slots < need)
+        return set_error(GD_ERR_CAPACITY, "gd_buffer_init: capacity_slots < min(N, max_inflight * max_nodes_per_batch)"
+                                          " (the N_e x M_b reservation, P:122)");
+    const int64_t C = 2 * capacity_slots + max_nodes_per_batch;
+    if (2 * C >= 0x7FFFFFFFLL) return set_error(GD_ERR_INVALID, "gd_buffer_init: capacity too large");
+    DeviceGuard guard(device);
+    GD_CUDA(cudaSetDevice(device));
+    gd_buffer* b = new gd_buffer();
+    b->hdr.magic = kMagicBuffer;
+    b->hdr.device = device;
+    b->N = num_nodes;
+    b->R = row_bytes;
+    b->S = capacity_slots;
+    b->C = C;
+    b->n_max = max_nodes_per_batch;
+    b->Q = max_inflight;
+    b->preload = preload;
+    b->host_feat = host_feat;
+    b->D = max_inflight + 2;
+    auto fail = [&](gd_status s) {
+        buffer_free(b);
+        return s;
+    };
+    // map the pinned host table (the SSD stand-in) into the device address space
+    cudaPointerAttributes pa;
+    bool pinned = (cudaPointerGetAttributes(&pa, host_feat) == cudaSuccess && pa.type == cudaMemoryTypeHost);
+    cudaGetLastError();
+    if (!pinned) {
+        cudaError_t e = cudaHostRegister((void*)host_feat, (size_t)num_nodes * row_bytes,
+                                         cudaHostRegisterMapped | cudaHostRegisterPortable);
+        if (e != cudaSuccess) return fail(cuda_error(e, "cudaHostRegister(host_feat)"));
+        b->registered = true;
+    }
+    void* dptr = nullptr;
+    {
+        cudaError_t e = cudaHostGetDevicePointer(&dptr, (void*)host_feat, 0);
+        if (e != cudaSuccess) return fail(cuda_error(e, "cudaHostGetDevicePointer(host_feat)"));
+    }
+    b->feat_dev = (const uint8_t*)dptr;
+
+    const int64_t nm = max_nodes_per_batch;
+#define GD_ALLOC(ptr, bytes)                                                          \
+    do {                                                                              \
+        cudaError_t e_ = cudaMalloc((void**)&(ptr), (size_t)(bytes));                 \
+        if (e_ != cudaSuccess) return fail(cuda_error(e_, "cudaMalloc " #ptr));       \
+    } while (0)
+    GD_ALLOC(b->hdr.dev_status, sizeof(unsigned int));
+    GD_ALLOC(b->slots, capacity_slots * row_bytes);
+    GD_ALLOC(b->map, num_nodes * sizeof(int2));
+    GD_ALLOC(b->reverse, capacity_slots * sizeof(int32_t));
+    GD_ALLOC(b->pos_of_slot, capacity_slots * sizeof(int32_t));
+    GD_ALLOC(b->ring, 2 * C * sizeof(int32_t));
+    GD_ALLOC(b->ctl, 2 * sizeof(GdCtl));
+    GD_ALLOC(b->misslist, nm * sizeof(int32_t));
+    GD_ALLOC(b->missflag, nm);
+    GD_ALLOC(b->alias_ws, nm * sizeof(int32_t));
+    GD_ALLOC(b->mcount, sizeof(int64_t));
+    GD_ALLOC(b->trip, (int64_t)b->D * nm * sizeof(int4));
+    GD_ALLOC(b->trip_count, b->D * sizeof(int64_t));
+    GD_ALLOC(b->tickets, 4 * sizeof(unsigned long long));
+    GD_ALLOC(b->done_word, sizeof(unsigned long long));
+#undef GD_ALLOC
+    gd_status s = b->scan.ensure(std::max(cdiv(nm, kBTile), cdiv(C, kBTile)) + 1);
+    if (s != GD_OK) return fail(s);
+    GdCtl c0[2];
+    c0[0].head = 0;
+    c0[0].tail = capacity_slots;
+    c0[0].base = 0;
+    c0[1] = c0[0];
+    if (cudaMemcpy(b->ctl, c0, sizeof(c0), cudaMemcpyHostToDevice) != cudaSuccess ||
+        cudaMemset(b->hdr.dev_status, 0, sizeof(unsigned int)) != cudaSuccess ||
+        cudaMemset(b->tickets, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(b->done_word, 0, sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(b->trip_count, 0, b->D * sizeof(int64_t)) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: init copies"));
+    k_init_map<<<148 * 8, 256>>>(b->map, num_nodes, preload);
+    k_init_slots<<<148 * 8, 256>>>(b->reverse, b->pos_of_slot, b->ring, capacity_slots, num_nodes, preload);
+    if (preload) {
+        cudaError_t e = cudaMemcpy(b->slots, host_feat, (size_t)num_nodes * row_bytes, cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: preload copy"));
+    }
+    {
+        cudaError_t e = cudaDeviceSynchronize();
+        if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: init kernels"));
+    }
+    if (cudaStreamCreateWithFlags(&b->side, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaEventCreateWithFlags(&b->ev_L, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&b->ev_X, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventCreateWithFlags(&b->ev_G, cudaEventDisableTiming) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream/event"));
+    b->ev_trip.assign(b->D, nullptr);
+    for (int d = 0; d < b->D; ++d)
+        if (cudaEventCreateWithFlags(&b->ev_trip[d], cudaEventDisableTiming) != cudaSuccess)
+            return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
+    *out = b;
+    return GD_OK;
+}
+
+gd_status gd_buffer_destroy(gd_buffer* b) {
+    if (!b) return GD_OK;
+    if (b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_destroy: bad handle");
+    buffer_free(b);
+    return GD_OK;
+}
+
+void* gd_buffer_side_stream(gd_buffer* b) { return (b && b->hdr.magic == kMagicBuffer) ? (void*)b->side : nullptr; }
+
+gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max, void* out,
+                     int32_t* alias, int64_t* stats, void* stream_v, void* done_v) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_extract: bad buffer handle");
+    if (!node_ids || !n_dev || !out) return set_error(GD_ERR_INVALID, "gd_extract: null pointer");
+    if (n_max < 0 || n_max > b->n_max)
+        return set_error(GD_ERR_INVALID, "gd_extract: n_max exceeds max_nodes_per_batch");
+    if (b->inflight >= b->Q)
+        return set_error(GD_ERR_CAPACITY, "gd_extract: max_inflight unreleased batches already extracted");
+    if (((uintptr_t)out & 15) && (b->R % 16 == 0)) return set_error(GD_ERR_INVALID, "gd_extract: out must be 16-byte aligned");
+    DeviceGuard guard(b->hdr.device);
+    cudaStream_t st = (cudaStream_t)stream_v;
+    int32_t* al = alias ? alias : b->alias_ws;
+    const int d = (int)(b->batch_counter % b->D);
+    int4* trip = b->trip + (int64_t)d * b->n_max;
+    int64_t* tcount = b->trip_count + d;
+    const int64_t lt = std::max<int64_t>(1, cdiv(n_max, kBTile));
+
+    GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));   // side stream done with trip slot d
+
+    LookupArgs la;
+    la.ids = node_ids;
+    la.n_dev = n_dev;
+    la.N = b->N;
+    la.map = b->map;
+    la.pos_of_slot = b->pos_of_slot;
+    la.alias = al;
+    la.missflag = b->missflag;
+    la.misslist = b->misslist;
+    la.mcount = b->mcount;
+    la.stats = stats;
+    la.st = b->scan.use();
+    la.st_clear = b->scan.other();
+    la.st_clear_n = b->scan.cap;
+    la.status = b->hdr.dev_status;
+    k_lookup<<<(unsigned)lt, kBThreads, 0, st>>>(la);
+    b->scan.flip();
+
+    PopArgs pa;
+    pa.ring = b->ring;
+    pa.ctl_in = b->ctl + b->ctl_parity;
+    pa.ctl_out = b->ctl + (b->ctl_parity ^ 1);
+    pa.pos_of_slot = b->pos_of_slot;
+    pa.map = b->map;
+    pa.reverse = b->reverse;
+    pa.ids = node_ids;
+    pa.misslist = b->misslist;
+    pa.mcount = b->mcount;
+    pa.alias = al;
+    pa.trip = trip;
+    pa.trip_count = tcount;
+    pa.ticket = b->tickets;
+    pa.done_word = b->done_word;
+    pa.epoch = ++b->epoch;
+    pa.st = b->scan.use();
+    pa.st_clear = b->scan.other();
+    pa.st_clear_n = b->scan.cap;
+    pa.status = b->hdr.dev_status;
+    k_pop_assign<<<148 * 2, kBThreads, 0, st>>>(pa);
+    b->scan.flip();
+    b->ctl_parity ^= 1;
+    GD_CUDA(cudaEventRecord(b->ev_L, st));
+
+    // hits: their rows were written by earlier miss streams, all ordered before X_{b-1}
+    GD_CUDA(cudaStreamWaitEvent(st, b->ev_X, 0));
+    if (b->R % 16 == 0)
+        k_gather_hits<4><<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
+    else
+        k_gather_hits_w4<<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
+    GD_CUDA(cudaEventRecord(b->ev_G, st));
+
+    // misses: pinned host -> slot + out on the side stream (asynchronous extraction)
+    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
+    if (b->R % 16 == 0)
+        k_miss_copy<4><<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+    else
+        k_miss_copy_w4<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+    GD_CUDA(cudaEventRecord(b->ev_X, b->side));
+    GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side));
+    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
+    if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side));
+    GD_CUDA(cudaGetLastError());
+    b->inflight++;
+    b->batch_counter++;
+    return GD_OK;
+}
+
+gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,
+                            void* stream_v) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_release: bad buffer handle");
+    if (!node_ids || !n_dev) return set_error(GD_ERR_INVALID, "gd_buffer_release: null pointer");
+    if (n_max < 0 || n_max > b->n_max)
+        return set_error(GD_ERR_INVALID, "gd_buffer_release: n_max exceeds max_nodes_per_batch");
+    if (b->inflight <= 0) return set_error(GD_ERR_INVALID, "gd_buffer_release: no extracted batch to release");
+    DeviceGuard guard(b->hdr.device);
+    cudaStream_t st = (cudaStream_t)stream_v;
+
+    CompactArgs ca;
+    ca.ring = b->ring;
+    ca.pos_of_slot = b->pos_of_slot;
+    ca.ctl_in = b->ctl + b->ctl_parity;
+    ca.ctl_out = b->ctl + (b->ctl_parity ^ 1);
+    ca.C = b->C;
+    ca.n_max = b->n_max;
+    ca.ticket = b->tickets + 2;
+    ca.st = b->scan.use();
+    ca.st_clear = b->scan.other();
+    ca.st_clear_n = b->scan.cap;
+    k_compact<<<148 * 2, kBThreads, 0, st>>>(ca);
+    b->scan.flip();
+    b->ctl_parity ^= 1;
+
+    ReleaseArgs ra;
+    ra.ids = node_ids;
+    ra.n_dev = n_dev;
+    ra.N = b->N;
+    ra.map = b->map;
+    ra.ring = b->ring;
+    ra.pos_of_slot = b->pos_of_slot;
+    ra.ctl_in = b->ctl + b->ctl_parity;
+    ra.ctl_out = b->ctl + (b->ctl_parity ^ 1);
+    ra.st = b->scan.use();
+    ra.st_clear = b->scan.other();
+    ra.st_clear_n = b->scan.cap;
+    ra.status = b->hdr.dev_status;
+    k_release<<<(unsigned)std::max<int64_t>(1, cdiv(n_max, kBTile)), kBThreads, 0, st>>>(ra);
+    b->scan.flip();
+    b->ctl_parity ^= 1;
+    GD_CUDA(cudaGetLastError());
+    b->inflight--;
+    return GD_OK;
+}
+
+gd_status gd_buffer_snapshot(gd_buffer* b, int32_t* map_slot, int32_t* map_rc, uint8_t* map_valid, int32_t* reverse,
+                             int32_t* standby, int64_t* standby_len) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_snapshot: bad handle");
+    DeviceGuard guard(b->hdr.device);
+    GD_CUDA(cudaDeviceSynchronize());
+    if (map_slot || map_rc || map_valid) {
+        std::vector<int2> m(b->N);
+        GD_CUDA(cudaMemcpy(m.data(), b->map, b->N * sizeof(int2), cudaMemcpyDeviceToHost));
+        for (int64_t v = 0; v < b->N; ++v) {
+            if (map_slot) map_slot[v] = m[v].x;
+            if (map_rc) map_rc[v] = m[v].y >> 1;
+            if (map_valid) map_valid[v] = (uint8_t)(m[v].y & 1);
+        }
+    }
+    if (reverse) GD_CUDA(cudaMemcpy(reverse, b->reverse, b->S * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    if (standby || standby_len) {
+        GdCtl c;
+        GD_CUDA(cudaMemcpy(&c, b->ctl + b->ctl_parity, sizeof(c), cudaMemcpyDeviceToHost));
+        std::vector<int32_t> pos(b->S), ring(std::max<long long>(1, c.tail - c.head));
+        GD_CUDA(cudaMemcpy(pos.data(), b->pos_of_slot, b->S * sizeof(int32_t), cudaMemcpyDeviceToHost));
+        if (c.tail > c.head)
+            GD_CUDA(cudaMemcpy(ring.data(), b->ring + c.head, (c.tail - c.head) * sizeof(int32_t), cudaMemcpyDeviceToHost));
+        int64_t k = 0;
+        for (long long p = c.head; p < c.tail; ++p) {
+            const int32_t s = ring[p - c.head];
+            if (pos[s] == (int32_t)p) {
+                if (standby) standby[k] = s;
+                ++k;
+            }
+        }
+        if (standby_len) *standby_len = k;
+    }
+    return GD_OK;
+}
+
+gd_status gd_buffer_set_state(gd_buffer* b, const int32_t* map_slot, const int32_t* map_rc, const uint8_t* map_valid,
+                              const int32_t* reverse, const int32_t* standby, int64_t standby_len) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_set_state: bad handle");
+    if (!map_slot || !map_rc || !map_valid || !reverse || (standby_len > 0 && !standby) || standby_len > b->S)
+        return set_error(GD_ERR_INVALID, "gd_buffer_set_state: bad arguments");
+    DeviceGuard guard(b->hdr.device);
+    GD_CUDA(cudaDeviceSynchronize());
+    std::vector<int2> m(b->N);
+    for (int64_t v = 0; v < b->N; ++v) m[v] = make_int2(map_slot[v], (map_rc[v] << 1) | (map_valid[v] & 1));
+    GD_CUDA(cudaMemcpy(b->map, m.data(), b->N * sizeof(int2), cudaMemcpyHostToDevice));
+    GD_CUDA(cudaMemcpy(b->reverse, reverse, b->S * sizeof(int32_t), cudaMemcpyHostToDevice));
+    std::vector<int32_t> pos(b->S, -1);
+    for (int64_t k = 0; k < standby_len; ++k) pos[standby[k]] = (int32_t)k;
+    GD_CUDA(cudaMemcpy(b->pos_of_slot, pos.data(), b->S * sizeof(int32_t), cudaMemcpyHostToDevice));
+    if (standby_len > 0) GD_CUDA(cudaMemcpy(b->ring, standby, standby_len * sizeof(int32_t), cudaMemcpyHostToDevice));
+    GdCtl c[2];
+    c[0].head = 0;
+    c[0].tail = standby_len;
+    c[0].base = 0;
+    c[1] = c[0];
+    GD_CUDA(cudaMemcpy(b->ctl, c, sizeof(c), cudaMemcpyHostToDevice));
+    for (int64_t v = 0; v < b->N; ++v)
+        if ((map_valid[v] & 1) && map_slot[v] >= 0)
+            GD_CUDA(cudaMemcpy(b->slots + (int64_t)map_slot[v] * b->R, (const uint8_t*)b->host_feat + v * b->R, b->R,
+                               cudaMemcpyHostToDevice));
+    return GD_OK;
+}
+
+}  // extern "C"

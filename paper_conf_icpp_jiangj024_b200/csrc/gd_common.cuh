@@ -1,0 +1,182 @@
+// gd_common.cuh — device helpers shared by the sm_100a kernels of libgd.so:
+// error plumbing, handle header, Philox4x32-10, decoupled look-back tile scan,
+// open-addressing hash primitives.  Independent of oracle/ (no shared code).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "../../include/gd.h"
+
+namespace gd {
+
+// ---------------------------------------------------------------- errors (host)
+gd_status set_error(gd_status s, const std::string& msg);
+gd_status cuda_error(cudaError_t e, const char* what);
+#define GD_CUDA(call)                                              \
+    do {                                                           \
+        cudaError_t e_ = (call);                                   \
+        if (e_ != cudaSuccess) return ::gd::cuda_error(e_, #call); \
+    } while (0)
+
+constexpr uint32_t kMagicGraph = 0x47444752u;   // "GDGR"
+constexpr uint32_t kMagicBuffer = 0x47444246u;  // "GDBF"
+
+struct HandleHdr {
+    uint32_t magic;
+    int device;
+    unsigned int* dev_status;   // sticky GD_DEV_* bits (device memory)
+};
+
+struct DeviceGuard {            // switch to the handle's device for one API call
+    int prev = -1;
+    explicit DeviceGuard(int dev) {
+        cudaGetDevice(&prev);
+        if (prev != dev) cudaSetDevice(dev);
+    }
+    ~DeviceGuard() {
+        int cur = -1;
+        cudaGetDevice(&cur);
+        if (prev >= 0 && cur != prev) cudaSetDevice(prev);
+    }
+};
+
+// Pointer kind: true if `p` is device-accessible memory of the current context
+// (device / managed), false for host memory (pageable or pinned).
+bool is_device_pointer(const void* p);
+
+// --------------------------------------------------------- scan tile states (host)
+// Decoupled look-back needs one 64-bit status word per tile, zero before a launch.
+// Two arrays alternate: each scan launch uses one and clears the other for the next
+// launch on the same stream, so no memset node is needed between launches.
+struct ScanState {
+    unsigned long long* buf[2] = {nullptr, nullptr};
+    int64_t cap = 0;     // tiles per array
+    int parity = 0;
+    gd_status ensure(int64_t tiles);
+    void release();
+    unsigned long long* use() const { return buf[parity]; }
+    unsigned long long* other() const { return buf[parity ^ 1]; }
+    void flip() { parity ^= 1; }
+};
+
+// ----------------------------------------------------------------- device side
+constexpr unsigned long long kFlagA = 1ull << 62;   // tile aggregate published
+constexpr unsigned long long kFlagP = 2ull << 62;   // tile inclusive prefix published
+constexpr unsigned long long kValMask = (1ull << 62) - 1;
+constexpr uint32_t kEmpty = 0xFFFFFFFFu;            // empty hash key
+constexpr uint32_t kPending = 0x80000000u;          // hash value tag: first position this hop
+
+__device__ __forceinline__ void st_relaxed_u64(unsigned long long* p, unsigned long long v) {
+    asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+__device__ __forceinline__ uint32_t ld_relaxed_u32(const uint32_t* p) {
+    uint32_t v;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ void clear_tile_state(unsigned long long* p, int64_t n) {
+    if (p == nullptr) return;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+         i += (int64_t)gridDim.x * blockDim.x)
+        p[i] = 0ull;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_sum(T v) {
+    const int lane = threadIdx.x & 31;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        T n = __shfl_up_sync(0xffffffffu, v, o);
+        if (lane >= o) v += n;
+    }
+    return v;
+}
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+    return v;
+}
+
+// Decoupled look-back (Merrill & Garland 2016).  Called by all 32 lanes of ONE warp
+// of the block owning `tile`, after the block computed its aggregate `agg`.  Tiles
+// are processed by blocks that start in tile order (blockIdx order or a ticket), so
+// every predecessor is running or done.  `base` is added to tile 0's prefix.
+// Returns the exclusive prefix of `tile` (same value in every lane).
+__device__ __forceinline__ long long lookback_exclusive(unsigned long long* st, long long tile,
+                                                        long long agg, long long base) {
+    const int lane = threadIdx.x & 31;
+    if (tile == 0) {
+        if (lane == 0) st_relaxed_u64(st, kFlagP | (unsigned long long)(base + agg));
+        return base;
+    }
+    if (lane == 0) st_relaxed_u64(st + tile, kFlagA | (unsigned long long)agg);
+    long long excl = 0;
+    long long t = tile - 1 - lane;
+    while (true) {
+        unsigned long long w;
+        int spins = 0;
+        while (true) {
+            w = (t >= 0) ? ld_relaxed_u64(st + t) : kFlagP;
+            if (__all_sync(0xffffffffu, (w >> 62) != 0)) break;
+            if (++spins > 8) __nanosleep(64);
+        }
+        const unsigned pmask = __ballot_sync(0xffffffffu, (w >> 62) == 2);
+        const int first_p = pmask ? (__ffs(pmask) - 1) : 32;
+        long long v = (lane <= first_p) ? (long long)(w & kValMask) : 0;
+        excl += warp_sum(v);
+        if (pmask) break;
+        t -= 32;
+    }
+    if (lane == 0) st_relaxed_u64(st + tile, kFlagP | (unsigned long long)(excl + agg));
+    return excl;
+}
+
+// Philox4x32-10 (Salmon et al., SC'11), the counter-based generator of reading R1.
+__device__ __forceinline__ void philox4x32_10(uint32_t c[4], uint32_t k0, uint32_t k1) {
+#pragma unroll
+    for (int r = 0; r < 10; ++r) {
+        const uint32_t lo0 = 0xD2511F53u * c[0];
+        const uint32_t hi0 = __umulhi(0xD2511F53u, c[0]);
+        const uint32_t lo1 = 0xCD9E8D57u * c[2];
+        const uint32_t hi1 = __umulhi(0xCD9E8D57u, c[2]);
+        const uint32_t n0 = hi1 ^ c[1] ^ k0;
+        const uint32_t n2 = hi0 ^ c[3] ^ k1;
+        c[0] = n0;
+        c[1] = lo1;
+        c[2] = n2;
+        c[3] = lo0;
+        k0 += 0x9E3779B9u;
+        k1 += 0xBB67AE85u;
+    }
+}
+
+// Draw t for node v at 0-based hop h of batch b, mapped to [0, j] (reading R2):
+// u = y << 32 | x of Philox(ctr=(t, v, h, b), key=(lo, hi of seed)); floor(u (j+1) / 2^64).
+__device__ __forceinline__ uint64_t draw_uniform(uint32_t t, uint32_t v, uint32_t h, uint32_t b,
+                                                 uint64_t seed, uint64_t j) {
+    uint32_t c[4] = {t, v, h, b};
+    philox4x32_10(c, (uint32_t)seed, (uint32_t)(seed >> 32));
+    const uint64_t u = ((uint64_t)c[1] << 32) | (uint64_t)c[0];
+    return __umul64hi(u, j + 1);
+}
+
+__device__ __forceinline__ uint32_t fmix32(uint32_t h) {   // MurmurHash3 finaliser
+    h ^= h >> 16;
+    h *= 0x85EBCA6Bu;
+    h ^= h >> 13;
+    h *= 0xC2B2AE35u;
+    h ^= h >> 16;
+    return h;
+}
+
+}  // namespace gd

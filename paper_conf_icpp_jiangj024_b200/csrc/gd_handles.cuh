@@ -1,0 +1,71 @@
+// gd_handles.cuh — layouts of the two opaque handles of libgd.so.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <vector>
+
+#include "gd_common.cuh"
+
+// Topology replica + per-call sampling workspace.
+struct gd_graph {
+    gd::HandleHdr hdr;
+    int64_t N = 0, E = 0;
+    int64_t* indptr = nullptr;      // HBM int64[N+1]
+    int32_t* indices = nullptr;     // HBM int32[E]
+    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident)
+    int64_t hcap = 0;               // power of two >= 2 * max_nodes[K]
+    int32_t* seeds_ws = nullptr;    // staging for host seed arrays
+    int64_t seeds_cap = 0;
+    gd::ScanState scan;
+};
+
+// Control block of the standby ring.  Kernels that move head/tail read ctl[p] and
+// write ctl[p^1]; the host flips p after each such launch (no in-kernel RAW race).
+// The ring is one array of 2C positions: the live window [head, tail) lies in the
+// half starting at `base` (0 or C); compaction copies the live entries to the other
+// half, so a new position can never equal a stale one.
+struct GdCtl {
+    long long head;       // first ring position that may hold a live entry
+    long long tail;       // next free ring position
+    long long base;       // start of the current half (0 or C)
+};
+
+// Feature buffer + extraction workspace.
+struct gd_buffer {
+    gd::HandleHdr hdr;
+    int64_t N = 0, R = 0, S = 0;     // nodes, row bytes, slots
+    int64_t C = 0;                   // ring capacity per half
+    int64_t n_max = 0;               // max nodes per batch
+    int32_t Q = 0;                   // max in-flight (extracted, unreleased) batches
+    int preload = 0;
+    const void* host_feat = nullptr;
+    const uint8_t* feat_dev = nullptr;   // device alias of the pinned host table
+    bool registered = false;             // we registered host_feat ourselves
+    uint8_t* slots = nullptr;            // HBM [S x R]
+    int2* map = nullptr;                 // HBM [N]: {slot, rc << 1 | valid}
+    int32_t* reverse = nullptr;          // HBM [S]
+    int32_t* pos_of_slot = nullptr;      // HBM [S]: ring position of a slot's live entry, or -1
+    int32_t* ring = nullptr;             // HBM [2C]: slots in LRU order, lazy deletion
+    GdCtl* ctl = nullptr;                // HBM [2]
+    int ctl_parity = 0;
+    // per-batch workspace used on the caller's stream
+    int32_t* misslist = nullptr;         // [n_max] batch positions of misses, list order
+    uint8_t* missflag = nullptr;         // [n_max]
+    int32_t* alias_ws = nullptr;         // [n_max] used when the caller passes alias = NULL
+    int64_t* mcount = nullptr;           // [1] misses of the current batch
+    // miss triples for the side stream, a ring of D batches
+    int D = 0;
+    int4* trip = nullptr;                // [D][n_max] {node, slot, batch position, 0}
+    int64_t* trip_count = nullptr;       // [D]
+    unsigned long long* tickets = nullptr;   // [4] {ticket, finished} x 2 kernels
+    unsigned long long* done_word = nullptr; // [1] epoch-tagged early-exit word of the pop scan
+    gd::ScanState scan;
+    cudaStream_t side = nullptr;
+    cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_G = nullptr;
+    std::vector<cudaEvent_t> ev_trip;    // [D] side stream finished with trip ring slot
+    int64_t batch_counter = 0;
+    int64_t inflight = 0;
+    unsigned long long epoch = 1;
+};

@@ -1,0 +1,549 @@
+// gd_sample.cu — topology replica and the multi-hop sampler (rows a1-a4 of the hot path).
+//
+// One gd_sample call = 3 + 2K launches on the caller's stream, no host sync:
+//   memset(hash) ; k_seed_intake ; K x { k_sample_hop ; k_relabel_hop } ; k_col_resolve
+//
+// k_sample_hop  (S1, a2+a3): tile of 64 frontier nodes per 256-thread block.  Counts
+//   cnt = min(f, deg) are scanned with a decoupled look-back (rowptr), then one warp per
+//   node draws Floyd positions with Philox (lane t = draw t, resolution by ballots, rank
+//   sort by shuffles) and inserts every neighbour into the global open-addressing hash
+//   with atomicMin of its flat position (first occurrence).  col temporarily holds the
+//   neighbour's hash slot.
+// k_relabel_hop (S2, a4): flag = "this edge is the first occurrence of a new node";
+//   warp ballots + popc give in-warp ranks (warp-aggregated compaction), a look-back scan
+//   gives the global rank; new nodes get local ids n_{h-1} + rank, are appended to n_id
+//   and finalised in the hash.
+// k_col_resolve: col[e] = local id of the slot (one launch for all hops).
+#include <algorithm>
+#include <cstring>
+#include <string>
+
+#include "gd_common.cuh"
+#include "gd_handles.cuh"
+
+namespace gd {
+
+constexpr int kThreads = 256;
+constexpr int kWarps = kThreads / 32;
+constexpr int kNodesPerTile = 64;          // frontier nodes per sampler block
+constexpr int kRelabelItems = 8;
+constexpr int kEdgesPerTile = kThreads * kRelabelItems;   // 2048 edges per relabel block
+constexpr int kMaxFanSmem = GD_MAX_FANOUT;
+
+struct SampleHopArgs {
+    const int64_t* indptr;
+    const int32_t* indices;
+    int64_t N;
+    int32_t* n_id;
+    int64_t* sizes;
+    int hop;          // 1-based
+    int K;
+    int fanout;
+    uint32_t batch;
+    uint64_t seed;
+    int64_t* rowptr;
+    int32_t* col;
+    int64_t* eid;
+    uint32_t* hkeys;
+    uint32_t* hvals;
+    uint32_t mask;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+    unsigned int* status;
+};
+
+// Insert neighbour u seen at flat position e of this hop; returns its hash slot.
+__device__ __forceinline__ uint32_t hash_insert(uint32_t* __restrict__ hk, uint32_t* __restrict__ hv,
+                                                uint32_t mask, uint32_t u, uint32_t e) {
+    uint32_t h = fmix32(u) & mask;
+    while (true) {
+        const uint32_t k = ld_relaxed_u32(hk + h);
+        if (k == u) break;
+        if (k == kEmpty) {
+            const uint32_t old = atomicCAS(hk + h, kEmpty, u);
+            if (old == kEmpty || old == u) break;
+        }
+        h = (h + 1) & mask;
+    }
+    const uint32_t tag = kPending | e;
+    if (ld_relaxed_u32(hv + h) > tag) atomicMin(hv + h, tag);
+    return h;
+}
+
+__global__ void __launch_bounds__(kThreads) k_seed_intake(const int32_t* __restrict__ seeds, int64_t B,
+                                                          int64_t N, uint32_t* hk, uint32_t* hv,
+                                                          uint32_t mask, int32_t* n_id, int64_t* sizes,
+                                                          unsigned int* status) {
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i == 0) sizes[0] = B;
+    if (i >= B) return;
+    const int32_t v = seeds[i];
+    n_id[i] = v;
+    if (v < 0 || (int64_t)v >= N) {
+        atomicOr(status, GD_DEV_BAD_ID);
+        return;
+    }
+    uint32_t h = fmix32((uint32_t)v) & mask;
+    while (true) {
+        const uint32_t old = atomicCAS(hk + h, kEmpty, (uint32_t)v);
+        if (old == kEmpty) {
+            hv[h] = (uint32_t)i;   // finalised local id = position
+            return;
+        }
+        if (old == (uint32_t)v) {
+            atomicOr(status, GD_DEV_DUP_SEED);
+            return;
+        }
+        h = (h + 1) & mask;
+    }
+}
+
+// Emit neighbour at CSR position p of node (start) as flat edge e.
+__device__ __forceinline__ void emit_edge(const SampleHopArgs& a, int64_t start, int64_t p, int64_t e) {
+    const uint32_t u = (uint32_t)__ldg(a.indices + start + p);
+    const uint32_t slot = hash_insert(a.hkeys, a.hvals, a.mask, u, (uint32_t)e);
+    a.col[e] = (int32_t)slot;
+    if (a.eid) a.eid[e] = start + p;
+}
+
+__global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const int64_t n_prev = a.sizes[a.hop - 1];
+    const int64_t tile = blockIdx.x;
+    const int64_t i0 = tile * kNodesPerTile;
+    if (i0 >= n_prev && tile != 0) return;
+
+    __shared__ int64_t s_start[kNodesPerTile];
+    __shared__ int64_t s_deg[kNodesPerTile];
+    __shared__ int64_t s_off[kNodesPerTile];
+    __shared__ int32_t s_v[kNodesPerTile];
+    __shared__ long long s_wtot[2];
+    __shared__ long long s_base;
+    __shared__ int64_t s_sel[kWarps][kMaxFanSmem];   // f > 32 path only
+
+    const int t = threadIdx.x;
+    const int lane = t & 31;
+    const int warp = t >> 5;
+    const int f = a.fanout;
+
+    // ---- a2: counts and their exclusive scan (rowptr)
+    long long cnt = 0;
+    if (t < kNodesPerTile) {
+        const int64_t i = i0 + t;
+        int64_t start = 0, d = 0;
+        int32_t v = 0;
+        if (i < n_prev) {
+            v = a.n_id[i];
+            if (v >= 0 && (int64_t)v < a.N) {
+                start = a.indptr[v];
+                d = a.indptr[v + 1] - start;
+            }
+            cnt = (f < 0) ? d : (d < f ? d : f);
+        }
+        s_v[t] = v;
+        s_start[t] = start;
+        s_deg[t] = d;
+    }
+    long long incl = 0;
+    if (t < kNodesPerTile) {
+        incl = warp_inclusive_sum(cnt);
+        if (lane == 31) s_wtot[warp] = incl;
+    }
+    __syncthreads();
+    if (warp == 0) {
+        const long long agg = s_wtot[0] + s_wtot[1];
+        const long long base = lookback_exclusive(a.st, tile, agg, 0);
+        if (lane == 0) s_base = base;
+    }
+    __syncthreads();
+    const long long base = s_base;
+    if (t < kNodesPerTile) {
+        const long long excl = base + incl - cnt + (warp == 1 ? s_wtot[0] : 0);
+        s_off[t] = excl;
+        const int64_t i = i0 + t;
+        if (i < n_prev) a.rowptr[i] = excl;
+        const bool last = (n_prev == 0) ? (tile == 0 && t == 0) : (i == n_prev - 1);
+        if (last) {
+            const long long total = (n_prev == 0) ? 0 : excl + cnt;
+            a.rowptr[n_prev] = total;
+            a.sizes[a.K + a.hop] = total;
+        }
+    }
+    __syncthreads();
+
+    // ---- a3: one warp per frontier node
+    const uint32_t hidx = (uint32_t)(a.hop - 1);
+    for (int ln = warp; ln < kNodesPerTile; ln += kWarps) {
+        const int64_t i = i0 + ln;
+        if (i >= n_prev) break;
+        const int64_t start = s_start[ln];
+        const int64_t d = s_deg[ln];
+        const int64_t off = s_off[ln];
+        const uint32_t v = (uint32_t)s_v[ln];
+        if (f < 0 || d <= f) {
+            // the row verbatim (reading R4): coalesced copy
+            for (int64_t p = lane; p < d; p += 32) emit_edge(a, start, p, off + p);
+        } else if (f <= 32) {
+            // Floyd: lane t holds draw t in [0, d-f+t]
+            int64_t sel = INT64_MAX;
+            if (lane < f) {
+                const uint64_t j = (uint64_t)(d - f + lane);
+                sel = (int64_t)draw_uniform((uint32_t)lane, v, hidx, a.batch, a.seed, j);
+            }
+            for (int s = 1; s < f; ++s) {
+                const int64_t rs = __shfl_sync(0xffffffffu, sel, s);
+                const bool present = __ballot_sync(0xffffffffu, lane < s && sel == rs) != 0;
+                if (lane == s && present) sel = d - f + s;
+            }
+            int rank = 0;
+            for (int s = 0; s < f; ++s) {
+                const int64_t o = __shfl_sync(0xffffffffu, sel, s);
+                rank += (o < sel);
+            }
+            if (lane < f) emit_edge(a, start, sel, off + rank);
+        } else {
+            // f in (32, 256]: resolution in shared memory, O(f^2/32) per node
+            int64_t* ss = s_sel[warp];
+            for (int c = 0; c < f; c += 32) {
+                const int tt = c + lane;
+                int64_t r = 0;
+                if (tt < f) {
+                    const uint64_t j = (uint64_t)(d - f + tt);
+                    r = (int64_t)draw_uniform((uint32_t)tt, v, hidx, a.batch, a.seed, j);
+                }
+                const int cend = min(32, f - c);
+                for (int s = 0; s < cend; ++s) {
+                    const int step = c + s;
+                    const int64_t rs = __shfl_sync(0xffffffffu, r, s);
+                    bool hit = false;
+                    for (int q = lane; q < step; q += 32) hit |= (ss[q] == rs);
+                    const bool present = __ballot_sync(0xffffffffu, hit) != 0;
+                    if (lane == 0) ss[step] = present ? (d - f + step) : rs;
+                    __syncwarp();
+                }
+            }
+            __syncwarp();
+            for (int q = lane; q < f; q += 32) {
+                const int64_t me = ss[q];
+                int rank = 0;
+                for (int x = 0; x < f; ++x) rank += (ss[x] < me);
+                emit_edge(a, start, me, off + rank);
+            }
+            __syncwarp();
+        }
+    }
+}
+
+struct RelabelArgs {
+    int32_t* col;
+    int32_t* n_id;
+    int64_t* sizes;
+    int hop;
+    int K;
+    uint32_t* hkeys;
+    uint32_t* hvals;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+};
+
+__global__ void __launch_bounds__(kThreads) k_relabel_hop(RelabelArgs a) {
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const int64_t e_h = a.sizes[a.K + a.hop];
+    const int64_t n_prev = a.sizes[a.hop - 1];
+    const int64_t tile = blockIdx.x;
+    const int64_t e0 = tile * kEdgesPerTile;
+    if (e0 >= e_h && tile != 0) return;
+
+    __shared__ int s_cnt[kRelabelItems * kWarps];
+    __shared__ long long s_base;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+
+    uint32_t slot[kRelabelItems];
+    unsigned ball[kRelabelItems];
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        const int64_t e = e0 + (int64_t)k * kThreads + t;
+        bool flag = false;
+        slot[k] = 0;
+        if (e < e_h) {
+            slot[k] = (uint32_t)a.col[e];
+            flag = (ld_relaxed_u32(a.hvals + slot[k]) == (kPending | (uint32_t)e));
+        }
+        ball[k] = __ballot_sync(0xffffffffu, flag);
+        if (lane == 0) s_cnt[k * kWarps + warp] = __popc(ball[k]);
+    }
+    __syncthreads();
+    if (warp == 0) {
+        // exclusive scan over the 64 (round, warp) counts in edge order
+        const int c0 = s_cnt[2 * lane], c1 = s_cnt[2 * lane + 1];
+        const int inc = warp_inclusive_sum(c0 + c1);
+        const int ex = inc - c0 - c1;
+        const int agg = __shfl_sync(0xffffffffu, inc, 31);
+        __syncwarp();
+        s_cnt[2 * lane] = ex;
+        s_cnt[2 * lane + 1] = ex + c0;
+        const long long base = lookback_exclusive(a.st, tile, agg, 0);
+        if (lane == 0) {
+            s_base = base;
+            const bool last = (e_h == 0) ? (tile == 0) : (tile == (e_h - 1) / kEdgesPerTile);
+            if (last) a.sizes[a.hop] = n_prev + base + agg;
+        }
+    }
+    __syncthreads();
+    const long long base = s_base;
+    const unsigned lt = (1u << lane) - 1u;
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        if (ball[k] & (1u << lane)) {
+            const long long rank = base + s_cnt[k * kWarps + warp] + __popc(ball[k] & lt);
+            const int64_t local = n_prev + rank;
+            a.n_id[local] = (int32_t)a.hkeys[slot[k]];
+            a.hvals[slot[k]] = (uint32_t)local;
+        }
+    }
+}
+
+struct ColResolveArgs {
+    int32_t* col[GD_MAX_HOPS];
+    const int64_t* sizes;
+    int K;
+    const uint32_t* hvals;
+};
+
+__global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
+    const int hop = blockIdx.y;
+    const int64_t e_h = a.sizes[a.K + 1 + hop];
+    int32_t* col = a.col[hop];
+    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_h;
+         e += (int64_t)gridDim.x * blockDim.x)
+        col[e] = (int32_t)__ldg(a.hvals + col[e]);
+}
+
+__global__ void k_validate_csr(const int64_t* indptr, const int32_t* indices, int64_t N, int64_t E,
+                               unsigned int* bad) {
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    for (int64_t v = t0; v < N; v += stride)
+        if (indptr[v + 1] < indptr[v]) atomicOr(bad, 1u);
+    if (t0 == 0 && (indptr[0] != 0 || indptr[N] != E)) atomicOr(bad, 2u);
+    for (int64_t e = t0; e < E; e += stride) {
+        const int32_t u = indices[e];
+        if (u < 0 || (int64_t)u >= N) atomicOr(bad, 4u);
+    }
+}
+
+static int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+static gd_status copy_in(void* dst, const void* src, size_t bytes) {
+    GD_CUDA(cudaMemcpy(dst, src, bytes, cudaMemcpyDefault));
+    return GD_OK;
+}
+
+}  // namespace gd
+
+using namespace gd;
+
+extern "C" {
+
+gd_status gd_sample_bounds(int64_t num_seeds, const int32_t* fanouts, int32_t num_hops, int64_t num_nodes,
+                           int64_t num_edges, int64_t* max_nodes, int64_t* max_edges) {
+    if (!fanouts || !max_nodes || !max_edges)
+        return set_error(GD_ERR_INVALID, "gd_sample_bounds: null pointer");
+    if (num_hops < 1 || num_hops > GD_MAX_HOPS)
+        return set_error(GD_ERR_INVALID, "gd_sample_bounds: num_hops must be in [1, GD_MAX_HOPS]");
+    if (num_seeds < 0 || num_nodes < 0 || num_edges < 0)
+        return set_error(GD_ERR_INVALID, "gd_sample_bounds: negative size");
+    max_nodes[0] = num_seeds;
+    for (int h = 1; h <= num_hops; ++h) {
+        const int32_t f = fanouts[h - 1];
+        if (f < -1 || f > GD_MAX_FANOUT)
+            return set_error(GD_ERR_INVALID, "gd_sample_bounds: fanout must be -1 or in [0, 256]");
+        int64_t e;
+        if (f < 0) {
+            e = num_edges;
+        } else {
+            const int64_t prev = max_nodes[h - 1];
+            e = (f == 0 || prev <= num_edges / f) ? std::min<int64_t>(num_edges, prev * f) : num_edges;
+        }
+        max_edges[h - 1] = e;
+        max_nodes[h] = std::min<int64_t>(num_nodes, max_nodes[h - 1] + e);
+    }
+    return GD_OK;
+}
+
+gd_status gd_graph_create(const int64_t* indptr, const int32_t* indices, int64_t num_nodes, int64_t num_edges,
+                          int device, int validate, gd_graph** out) {
+    if (!indptr || !out || (num_edges > 0 && !indices))
+        return set_error(GD_ERR_INVALID, "gd_graph_create: null pointer");
+    if (num_nodes < 1 || num_nodes > 0x7FFFFFFFLL || num_edges < 0)
+        return set_error(GD_ERR_INVALID, "gd_graph_create: need 1 <= num_nodes <= 2^31-1, num_edges >= 0");
+    DeviceGuard guard(device);
+    GD_CUDA(cudaSetDevice(device));
+    gd_graph* g = new gd_graph();
+    g->hdr.magic = kMagicGraph;
+    g->hdr.device = device;
+    g->N = num_nodes;
+    g->E = num_edges;
+    auto fail = [&](gd_status s) {
+        gd_graph_destroy(g);
+        return s;
+    };
+    if (cudaMalloc(&g->hdr.dev_status, sizeof(unsigned int)) != cudaSuccess ||
+        cudaMalloc(&g->indptr, (num_nodes + 1) * sizeof(int64_t)) != cudaSuccess ||
+        cudaMalloc(&g->indices, std::max<int64_t>(1, num_edges) * sizeof(int32_t)) != cudaSuccess) {
+        cudaGetLastError();
+        return fail(set_error(GD_ERR_OOM, "gd_graph_create: cudaMalloc failed for the topology replica"));
+    }
+    gd_status s;
+    if ((s = copy_in(g->indptr, indptr, (num_nodes + 1) * sizeof(int64_t))) != GD_OK) return fail(s);
+    if (num_edges > 0 && (s = copy_in(g->indices, indices, num_edges * sizeof(int32_t))) != GD_OK) return fail(s);
+    if (cudaMemset(g->hdr.dev_status, 0, sizeof(unsigned int)) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "cudaMemset"));
+    if (validate) {
+        unsigned int* bad = nullptr;
+        if (cudaMalloc(&bad, sizeof(unsigned int)) != cudaSuccess) return fail(cuda_error(cudaGetLastError(), "cudaMalloc"));
+        cudaMemset(bad, 0, sizeof(unsigned int));
+        k_validate_csr<<<148 * 8, 256>>>(g->indptr, g->indices, num_nodes, num_edges, bad);
+        unsigned int hb = 0;
+        cudaError_t e = cudaMemcpy(&hb, bad, sizeof(hb), cudaMemcpyDeviceToHost);
+        cudaFree(bad);
+        if (e != cudaSuccess) return fail(cuda_error(e, "k_validate_csr"));
+        if (hb)
+            return fail(set_error(GD_ERR_INVALID, std::string("gd_graph_create: invalid CSR (") +
+                                                      ((hb & 1) ? "indptr not monotone " : "") +
+                                                      ((hb & 2) ? "indptr[0]!=0 or indptr[N]!=E " : "") +
+                                                      ((hb & 4) ? "index out of range" : "") + ")"));
+    }
+    *out = g;
+    return GD_OK;
+}
+
+gd_status gd_graph_destroy(gd_graph* g) {
+    if (!g) return GD_OK;
+    DeviceGuard guard(g->hdr.device);
+    if (g->indptr) cudaFree(g->indptr);
+    if (g->indices) cudaFree(g->indices);
+    if (g->hash) cudaFree(g->hash);
+    if (g->seeds_ws) cudaFree(g->seeds_ws);
+    if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
+    g->scan.release();
+    g->hdr.magic = 0;
+    delete g;
+    return GD_OK;
+}
+
+gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const int32_t* fanouts, int32_t num_hops,
+                    uint64_t rng_seed, uint32_t batch_id, gd_sample_out* out, void* stream_v) {
+    if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_sample: bad graph handle");
+    if (!out || !fanouts || (num_seeds > 0 && !seeds) || !out->n_id || !out->sizes)
+        return set_error(GD_ERR_INVALID, "gd_sample: null pointer");
+    int64_t nmax[GD_MAX_HOPS + 1], emax[GD_MAX_HOPS];
+    gd_status s = gd_sample_bounds(num_seeds, fanouts, num_hops, g->N, g->E, nmax, emax);
+    if (s != GD_OK) return s;
+    if (num_seeds > g->N) return set_error(GD_ERR_INVALID, "gd_sample: more seeds than nodes");
+    for (int h = 0; h < num_hops; ++h) {
+        if (!out->rowptr[h] || (!out->col[h] && emax[h] > 0))
+            return set_error(GD_ERR_INVALID, "gd_sample: null rowptr/col for a hop");
+        if (emax[h] >= (int64_t)kPending)
+            return set_error(GD_ERR_INVALID, "gd_sample: a hop may sample >= 2^31 edges");
+    }
+    DeviceGuard guard(g->hdr.device);
+    cudaStream_t st = (cudaStream_t)stream_v;
+
+    // workspace (grows on first use of a larger shape; not on the steady-state path)
+    int64_t want = 1024;
+    while (want < 2 * std::max<int64_t>(nmax[num_hops], 1)) want *= 2;
+    if (want > g->hcap) {
+        if (g->hash) cudaFree(g->hash);
+        g->hash = nullptr;
+        g->hcap = 0;
+        GD_CUDA(cudaMalloc(&g->hash, 2 * want * sizeof(uint32_t)));
+        g->hcap = want;
+    }
+    int64_t tiles = 1;
+    for (int h = 0; h < num_hops; ++h) {
+        tiles = std::max(tiles, ceil_div(nmax[h], kNodesPerTile));
+        tiles = std::max(tiles, ceil_div(emax[h], kEdgesPerTile));
+    }
+    if ((s = g->scan.ensure(tiles)) != GD_OK) return s;
+
+    const int32_t* seeds_d = seeds;
+    if (num_seeds > 0 && !is_device_pointer(seeds)) {
+        if (num_seeds > g->seeds_cap) {
+            if (g->seeds_ws) cudaFree(g->seeds_ws);
+            g->seeds_ws = nullptr;
+            g->seeds_cap = 0;
+            GD_CUDA(cudaMalloc(&g->seeds_ws, num_seeds * sizeof(int32_t)));
+            g->seeds_cap = num_seeds;
+        }
+        GD_CUDA(cudaMemcpyAsync(g->seeds_ws, seeds, num_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, st));
+        seeds_d = g->seeds_ws;
+    }
+
+    uint32_t* hk = g->hash;
+    uint32_t* hv = g->hash + g->hcap;
+    const uint32_t mask = (uint32_t)(g->hcap - 1);
+    GD_CUDA(cudaMemsetAsync(g->hash, 0xFF, 2 * g->hcap * sizeof(uint32_t), st));
+    k_seed_intake<<<(unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads)), kThreads, 0, st>>>(
+        seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status);
+
+    for (int h = 1; h <= num_hops; ++h) {
+        SampleHopArgs a;
+        a.indptr = g->indptr;
+        a.indices = g->indices;
+        a.N = g->N;
+        a.n_id = out->n_id;
+        a.sizes = out->sizes;
+        a.hop = h;
+        a.K = num_hops;
+        a.fanout = fanouts[h - 1];
+        a.batch = batch_id;
+        a.seed = rng_seed;
+        a.rowptr = out->rowptr[h - 1];
+        a.col = out->col[h - 1];
+        a.eid = out->eid[h - 1];
+        a.hkeys = hk;
+        a.hvals = hv;
+        a.mask = mask;
+        a.st = g->scan.use();
+        a.st_clear = g->scan.other();
+        a.st_clear_n = g->scan.cap;
+        a.status = g->hdr.dev_status;
+        const int64_t nt = std::max<int64_t>(1, ceil_div(nmax[h - 1], kNodesPerTile));
+        k_sample_hop<<<(unsigned)nt, kThreads, 0, st>>>(a);
+        g->scan.flip();
+
+        RelabelArgs r;
+        r.col = out->col[h - 1];
+        r.n_id = out->n_id;
+        r.sizes = out->sizes;
+        r.hop = h;
+        r.K = num_hops;
+        r.hkeys = hk;
+        r.hvals = hv;
+        r.st = g->scan.use();
+        r.st_clear = g->scan.other();
+        r.st_clear_n = g->scan.cap;
+        const int64_t et = std::max<int64_t>(1, ceil_div(emax[h - 1], kEdgesPerTile));
+        k_relabel_hop<<<(unsigned)et, kThreads, 0, st>>>(r);
+        g->scan.flip();
+    }
+    ColResolveArgs c;
+    int64_t emax_all = 1;
+    for (int h = 0; h < num_hops; ++h) {
+        c.col[h] = out->col[h];
+        emax_all = std::max(emax_all, emax[h]);
+    }
+    c.sizes = out->sizes;
+    c.K = num_hops;
+    c.hvals = hv;
+    dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
+              (unsigned)num_hops);
+    k_col_resolve<<<grid, kThreads, 0, st>>>(c);
+    GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
+}  // extern "C"

@@ -1,0 +1,270 @@
+"""GPU parity: the sm_100a path (through the C ABI) against the CPU oracle, bit-exact.
+
+Sampling (n_id, rowptr, col, eid, sizes) and extraction (out bytes, alias, hits/misses,
+and the whole buffer state: map, reverse, standby order) must be identical element by
+element.  Sizes span several tiles with ragged tails; edge cases cover empty inputs,
+degree-0 rows, fanout -1 / 0 / > 32, duplicate and out-of-range ids, exhausted capacity.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+import torch
+
+import synth
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+HERE = os.path.dirname(os.path.abspath(__file__))
+
+
+@pytest.fixture(scope="module")
+def gd():
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    import paper_conf_icpp_jiangj024_b200 as gd
+    return gd
+
+
+def make_graph(N, E, seed=1):
+    indptr, indices = synth.chung_lu_csr(N, E, seed=seed)
+    return indptr, indices
+
+
+def compare_sample(res_gpu, res_o, K):
+    h = res_gpu.to_host()
+    assert np.array_equal(h["sizes"], res_o.sizes), (h["sizes"], res_o.sizes)
+    assert np.array_equal(h["n_id"], res_o.n_id)
+    for k in range(K):
+        assert np.array_equal(h["rowptr"][k], res_o.rowptr[k]), f"rowptr hop {k+1}"
+        assert np.array_equal(h["col"][k], res_o.col[k]), f"col hop {k+1}"
+        if h["eid"][k] is not None:
+            assert np.array_equal(h["eid"][k], res_o.eid[k]), f"eid hop {k+1}"
+
+
+@pytest.fixture(scope="module")
+def tiny(gd):
+    cfg = synth.CONFIGS["tiny"]
+    indptr, indices = make_graph(cfg.num_nodes, cfg.num_edges)
+    g = gd.Graph(indptr, indices, device=0)
+    order = synth.epoch_order(synth.train_nodes(cfg.num_nodes, cfg.train_frac))
+    return cfg, g, indptr.numpy(), indices.numpy(), order
+
+
+@pytest.mark.parametrize("fanouts", [(5, 5), (15, 10, 5), (25, 15), (10, 10, 10), (-1, 3), (0, 4), (40, 2),
+                                     (100,), (33, 1), (1, 1, 1, 1, 1, 1, 1, 1)])
+def test_sample_parity_tiny(tiny, gd, fanouts):
+    cfg, g, indptr, indices, order = tiny
+    for b in range(6):
+        seeds = synth.batch_seeds(order, cfg.batch_size, b)
+        res = g.sample(seeds.cuda(), fanouts, synth.RNG_SEED, b, with_eid=True)
+        torch.cuda.synchronize()
+        ref = O.sample(indptr, indices, seeds.numpy(), list(fanouts), synth.RNG_SEED, b)
+        compare_sample(res, ref, len(fanouts))
+    assert g.check() == 0
+
+
+def test_sample_parity_host_seeds_and_no_eid(tiny, gd):
+    cfg, g, indptr, indices, order = tiny
+    seeds = synth.batch_seeds(order, cfg.batch_size, 3).pin_memory()
+    res = g.sample(seeds, (5, 5), 77, 3)          # host seeds, eid not requested
+    torch.cuda.synchronize()
+    compare_sample(res, O.sample(indptr, indices, seeds.numpy(), [5, 5], 77, 3), 2)
+
+
+def test_sample_parity_multi_tile(gd):
+    """~200k nodes, (15,10,5) from 1024 seeds: hundreds of tiles per hop, ragged tails."""
+    N, E = 200_000, 3_000_000
+    indptr, indices = make_graph(N, E, seed=9)
+    g = gd.Graph(indptr, indices)
+    order = synth.epoch_order(synth.train_nodes(N, 0.05))
+    ip, ix = indptr.numpy(), indices.numpy()
+    for b, B in [(0, 1024), (1, 1000), (2, 1), (3, 777)]:
+        seeds = order[b * 1024: b * 1024 + B]
+        res = g.sample(seeds.cuda(), (15, 10, 5), 3, b, with_eid=True)
+        torch.cuda.synchronize()
+        compare_sample(res, O.sample(ip, ix, seeds.numpy(), [15, 10, 5], 3, b), 3)
+
+
+def test_sample_edge_cases(gd):
+    # isolated nodes, self loops, multi-edges; empty seed list
+    rows = [[1, 2], [1, 0, 4], [0, 0, 4], [], [5], [2], [], [3, 3, 3, 3]]
+    indptr = torch.tensor(np.cumsum([0] + [len(r) for r in rows]), dtype=torch.int64)
+    indices = torch.tensor([u for r in rows for u in r], dtype=torch.int32)
+    g = gd.Graph(indptr, indices)
+    for seeds, fan in [([3], [2, 2]), ([6, 3], [5]), ([0, 7, 5], [1, 2, 3]), ([7], [-1, -1, -1]), ([], [2, 2])]:
+        s = torch.tensor(seeds, dtype=torch.int32)
+        res = g.sample(s.cuda() if len(seeds) else s.cuda(), fan, 1, 0, with_eid=True)
+        torch.cuda.synchronize()
+        compare_sample(res, O.sample(indptr.numpy(), indices.numpy(), s.numpy(), fan, 1, 0), len(fan))
+    assert g.check() == 0
+
+
+def test_sample_duplicate_and_bad_seed_flagged(gd):
+    indptr, indices = make_graph(1000, 5000)
+    g = gd.Graph(indptr, indices)
+    g.sample(torch.tensor([1, 2, 1], dtype=torch.int32).cuda(), [3], 1, 0)
+    with pytest.raises(gd.GdError) as e:
+        g.check()
+    assert e.value.status == 5
+    g2 = gd.Graph(indptr, indices)
+    g2.sample(torch.tensor([5, 1000], dtype=torch.int32).cuda(), [3], 1, 0)
+    with pytest.raises(gd.GdError):
+        g2.check()
+
+
+def test_graph_create_rejects_bad_csr(gd):
+    with pytest.raises(gd.GdError):
+        gd.Graph(torch.tensor([0, 2, 1], dtype=torch.int64), torch.tensor([0, 1], dtype=torch.int32))
+    with pytest.raises(gd.GdError):
+        gd.Graph(torch.tensor([0, 1, 2], dtype=torch.int64), torch.tensor([0, 7], dtype=torch.int32))
+
+
+# ----------------------------------------------------------------------- extraction
+
+
+def table_np(N, R, seed=4):
+    return synth.feature_rows(0, N, R, seed).numpy()
+
+
+def compare_state(buf, ob):
+    a, b = buf.snapshot(), ob.state()
+    for k in ("slot", "rc", "valid", "reverse", "standby"):
+        assert np.array_equal(a[k], b[k]), k
+
+
+def run_schedule(gd, g, ip, ix, feat, S, Q, seeds_list, fanouts, preload=False, check_state_every=1):
+    N, R = feat.shape
+    nb, _ = O.sample_bounds(max(len(s) for s in seeds_list), fanouts, N, int(ip[-1]))
+    n_max = nb[-1]
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, Q, n_max, preload=preload)
+    ob = O.Buffer(feat, S, preload=preload)
+    pending = []
+    for b, seeds in enumerate(seeds_list):
+        res = g.sample(torch.as_tensor(seeds).cuda(), fanouts, 3, b)
+        alias = torch.empty(n_max, dtype=torch.int32, device="cuda")
+        stats = torch.zeros(2, dtype=torch.int64, device="cuda")
+        out, _, done = buf.extract(res.n_id, res.num_nodes_dev, res.max_nodes, alias=alias, stats=stats)
+        done.synchronize()
+        n_id = res.to_host()["n_id"]
+        o_out, o_alias, o_stats = ob.extract(n_id)
+        n = len(n_id)
+        assert tuple(stats.cpu().tolist()) == o_stats
+        assert np.array_equal(alias[:n].cpu().numpy(), o_alias)
+        assert np.array_equal(out[:n].cpu().numpy(), o_out)
+        assert np.array_equal(o_out, feat[n_id])                  # closed form
+        pending.append((res, n_id))
+        if len(pending) == Q:
+            r0, n0 = pending.pop(0)
+            buf.release(r0.n_id, r0.num_nodes_dev, r0.max_nodes)
+            ob.release(n0)
+        if check_state_every and b % check_state_every == 0:
+            compare_state(buf, ob)
+    compare_state(buf, ob)
+    assert buf.check() == 0
+    return buf, ob
+
+
+def test_extract_parity_tiny_preload(tiny, gd):
+    cfg, g, ip, ix, order = tiny
+    feat = table_np(cfg.num_nodes, cfg.row_bytes)
+    seeds = [synth.batch_seeds(order, cfg.batch_size, b).numpy() for b in range(12)]
+    run_schedule(gd, g, ip, ix, feat, cfg.num_nodes, 4, seeds, list(cfg.fanouts), preload=True)
+
+
+@pytest.mark.parametrize("Q", [1, 2, 4])
+def test_extract_parity_tiny_evict(tiny, gd, Q):
+    """tiny-evict: S = Q * M_b, the minimum legal capacity: heavy eviction."""
+    cfg, g, ip, ix, order = tiny
+    feat = table_np(cfg.num_nodes, cfg.row_bytes)
+    nb, _ = O.sample_bounds(cfg.batch_size, list(cfg.fanouts), cfg.num_nodes, cfg.num_edges)
+    S = Q * nb[-1]
+    seeds = [synth.batch_seeds(order, cfg.batch_size, b).numpy() for b in range(30)]
+    run_schedule(gd, g, ip, ix, feat, S, Q, seeds, list(cfg.fanouts))
+
+
+@pytest.mark.parametrize("R", [400, 12, 1536])
+def test_extract_parity_row_sizes(gd, R):
+    """Row widths: 16-byte vector path (400 = products, 1536 = mag240m fp16) and the 4-byte path."""
+    N, E = 20_000, 150_000
+    indptr, indices = make_graph(N, E, seed=5)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, R if R % 8 == 0 else 16)[:, :R].copy()
+    order = synth.epoch_order(synth.train_nodes(N, 0.2))
+    seeds = [order[b * 300:(b + 1) * 300].numpy() for b in range(10)]
+    nb, _ = O.sample_bounds(300, [10, 5], N, E)
+    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 2 * nb[-1] + 17, 2, seeds, [10, 5], check_state_every=3)
+
+
+def test_extract_ring_compaction(gd):
+    """Many batches with a small capacity and lag: the standby ring compacts repeatedly."""
+    N, E = 3000, 30000
+    indptr, indices = make_graph(N, E, seed=6)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, 32)
+    order = synth.epoch_order(synth.train_nodes(N, 0.5))
+    seeds = [order[(b * 40) % 1400:(b * 40) % 1400 + 40].numpy() for b in range(80)]
+    nb, _ = O.sample_bounds(40, [4, 4], N, E)
+    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 3 * nb[-1], 3, seeds, [4, 4], check_state_every=7)
+
+
+def test_figure6_on_gpu(gd):
+    gdict = json.load(open(os.path.join(HERE, "golden", "fig6.json")))
+    N, S = gdict["num_nodes"], gdict["num_slots"]
+    feat = table_np(N, 16)
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, 2, 8)
+    buf.set_state(gdict["map_slot"], gdict["map_rc"], gdict["map_valid"], gdict["reverse"], gdict["standby"])
+    ids = torch.tensor(gdict["batch"], dtype=torch.int32, device="cuda")
+    n = torch.tensor([len(gdict["batch"])], dtype=torch.int64, device="cuda")
+    alias = torch.empty(8, dtype=torch.int32, device="cuda")
+    stats = torch.zeros(2, dtype=torch.int64, device="cuda")
+    out, _, done = buf.extract(ids, n, 8, alias=alias, stats=stats)
+    done.synchronize()
+    assert alias[:5].cpu().tolist() == gdict["expect_alias"]
+    assert stats.cpu().tolist() == [gdict["expect_hits"], gdict["expect_misses"]]
+    st = buf.snapshot()
+    assert st["reverse"].tolist() == gdict["expect_reverse"]
+    assert st["standby"].tolist() == gdict["expect_standby_after_extract"]
+    for v in gdict["expect_invalidated"]:
+        assert st["valid"][v] == 0 and st["slot"][v] == -1
+    assert np.array_equal(out[:5].cpu().numpy(), feat[gdict["batch"]])
+    rel = torch.tensor(gdict["release"], dtype=torch.int32, device="cuda")
+    buf.release(rel, torch.tensor([1], dtype=torch.int64, device="cuda"), 8)
+    assert buf.snapshot()["standby"].tolist() == gdict["expect_standby_after_release"]
+
+
+def test_extract_capacity_and_errors(gd):
+    feat = table_np(100, 16)
+    with pytest.raises(gd.GdError) as e:
+        gd.FeatureBuffer(torch.from_numpy(feat), 10, 2, 8)          # 10 < min(100, 2*8)
+    assert e.value.status == 4
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), 16, 2, 8)
+    ids = torch.arange(8, dtype=torch.int32, device="cuda")
+    n = torch.tensor([8], dtype=torch.int64, device="cuda")
+    buf.extract(ids, n, 8)
+    buf.extract(ids + 8, n, 8)
+    with pytest.raises(gd.GdError) as e:
+        buf.extract(ids + 16, n, 8)                                   # third unreleased batch
+    assert e.value.status == 4
+    with pytest.raises(gd.GdError):
+        buf.extract(ids, n, 9)                                        # n_max > max_nodes_per_batch
+    buf.release(ids, n, 8)
+    buf.release(ids, n, 8)                                            # refcount underflow
+    with pytest.raises(gd.GdError) as e:
+        buf.check()
+    assert e.value.status == 5
+
+
+def test_extract_empty_batch(gd):
+    feat = table_np(50, 16)
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), 20, 2, 8)
+    ids = torch.empty(8, dtype=torch.int32, device="cuda")
+    n = torch.zeros(1, dtype=torch.int64, device="cuda")
+    stats = torch.full((2,), -1, dtype=torch.int64, device="cuda")
+    _, _, done = buf.extract(ids, n, 8, stats=stats)
+    done.synchronize()
+    assert stats.cpu().tolist() == [0, 0]
+    buf.release(ids, n, 8)
+    assert buf.check() == 0
+    assert buf.snapshot()["standby"].tolist() == list(range(20))

@@ -15,7 +15,7 @@ import pytest
 import torch
 
 from oracle import oracle as O
-from paper_conf_icpp_jiangj024_b200 import synth
+import synth
 
 
 @pytest.mark.parametrize("d,f", [(5, 3), (6, 2), (7, 4), (8, 8), (9, 1), (10, 5), (4, 0)])
