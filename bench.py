@@ -1,0 +1,526 @@
+#!/usr/bin/env python
+"""Benchmark of the GNNDrive sample + extract hot path on B200 (BASELINE.json metric:
+sampled+extracted mini-batches/s; gather GB/s vs HBM, misses vs the host link).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config papers100m]
+    python -m torch.distributed.run --nnodes=1 --nproc-per-node N --master-addr 127.0.0.1 \\
+        --master-port P bench.py --gpus N ...
+    python bench.py --impl reference ...      # the CPU oracle as the reference arm
+
+One step = one mini-batch through every §8(a) row: gd_sample (seed intake, counts,
+Floyd/Philox sampling, relabel) -> gd_extract (lookup, LRU alloc/evict, hit gather, miss
+stream from the pinned host table) -> gd_buffer_release of the batch Q=4 steps earlier
+(P:177 training-queue depth).  Inputs are synthetic (synth/), shaped like the paper's
+workloads; the default workload is the Papers100M-shaped config (BASELINE.json configs[2]).
+Rank 0 prints ONE JSON line.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+
+Q = 4   # release lag = training-queue capacity
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=64)
+    p.add_argument("--warmup", type=int, default=16)
+    p.add_argument("--config", default="papers100m", choices=sorted(synth.CONFIGS))
+    p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the oracle cpu_baseline sample")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
+    p.add_argument("--out", default=None, help="also write the JSON line to this file")
+    return p.parse_args()
+
+
+# ----------------------------------------------------------------------------- helpers
+
+def log(*a):
+    if int(os.environ.get("RANK", "0")) == 0:
+        print("[bench]", *a, file=sys.stderr, flush=True)
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu = gpu_index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
+                                     timeout=5).stdout.strip()
+                if out:
+                    self.rows.append([x.strip() for x in out.split(",")])
+            except Exception:  # noqa: BLE001
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self._t:
+            self._t.join(timeout=10)
+
+    def summary(self):
+        sm = [float(r[1]) for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for k, nm in enumerate(names):
+                if len(r) > 5 + k and r[5 + k].lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+def h2d_peak_gbps(device) -> float:
+    """Host-link roofline measured in-run: pinned 1 GiB cudaMemcpyAsync H2D, best of 10."""
+    n = 1 << 30
+    h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
+    h.fill_(1)
+    d = torch.empty(n, dtype=torch.uint8, device=device)
+    s = torch.cuda.Stream(device)
+    best = 0.0
+    with torch.cuda.stream(s):
+        for _ in range(10):
+            a = torch.cuda.Event(enable_timing=True)
+            b = torch.cuda.Event(enable_timing=True)
+            a.record(s)
+            d.copy_(h, non_blocking=True)
+            b.record(s)
+            b.synchronize()
+            best = max(best, n / (a.elapsed_time(b) * 1e6))
+    del h, d
+    return best
+
+
+def measured_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:  # noqa: BLE001
+        return {}
+
+
+def capacity_for(cfg, n_max: int) -> int:
+    if cfg.preload:
+        return cfg.num_nodes
+    if cfg.buffer_frac < 0:                           # "miss heavy": the minimum legal size
+        return min(cfg.num_nodes, Q * n_max)
+    return max(int(cfg.buffer_frac * cfg.num_nodes), min(cfg.num_nodes, Q * n_max))
+
+
+def train_batches(cfg, device):
+    train = synth.train_nodes(cfg.num_nodes, cfg.train_frac, device=device)
+    nb = max(1, len(train) // cfg.batch_size)
+    return train, nb
+
+
+class Workload:
+    """Graph, host table, seeds of one config on this rank (setup, not timed)."""
+
+    def __init__(self, cfg, rank, world, device, need_host_csr):
+        from paper_conf_icpp_jiangj024_b200.multigpu import HostTable, barrier
+        self.cfg = cfg
+        t0 = time.time()
+        indptr, indices = synth.chung_lu_csr(cfg.num_nodes, cfg.num_edges, device=device)
+        torch.cuda.synchronize(device)
+        self.t_graph = time.time() - t0
+        deg = (indptr[1:] - indptr[:-1])
+        self.deg_stats = {"max": int(deg.max()), "mean": float(cfg.num_edges / cfg.num_nodes),
+                          "p99": int(torch.quantile(deg[:: max(1, cfg.num_nodes // 1_000_000)].double(), 0.99))}
+        del deg
+        self.host_indptr = indptr.cpu().numpy() if need_host_csr else None
+        self.host_indices = indices.cpu().numpy() if need_host_csr else None
+        self.indptr, self.indices = indptr, indices
+        t0 = time.time()
+        self.table = HostTable(cfg.num_nodes, cfg.row_bytes, cfg.name, rank, world)
+        # page-lock + map once here, so FeatureBuffer re-inits (parity / preload) skip it
+        rc = torch.cuda.cudart().cudaHostRegister(self.table.tensor.data_ptr(), cfg.num_nodes * cfg.row_bytes, 3)
+        if int(rc) != 0:
+            raise RuntimeError(f"cudaHostRegister(host table) failed: {rc}")
+        self.t_table_alloc = time.time() - t0
+        self.rank, self.world, self.device = rank, world, device
+        train, nb = train_batches(cfg, device)
+        self.train, self.num_batches = train, nb
+        self._orders = {}
+        self._barrier = barrier
+
+    def fill_table(self):
+        """Rank 0 writes the feature rows (generated on the GPU) into the host table."""
+        t0 = time.time()
+        if self.table.owner:
+            cfg = self.cfg
+            chunk = max(1, (256 << 20) // cfg.row_bytes)
+            for s in range(0, cfg.num_nodes, chunk):
+                e = min(cfg.num_nodes, s + chunk)
+                self.table.tensor[s:e].copy_(synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
+        torch.cuda.synchronize(self.device)
+        self._barrier()
+        self.t_fill = time.time() - t0
+
+    def close(self):
+        torch.cuda.cudart().cudaHostUnregister(self.table.tensor.data_ptr())
+        self.table.close()
+
+    def seeds(self, b, epoch):
+        if epoch not in self._orders:
+            self._orders[epoch] = synth.epoch_order(self.train, epoch)
+        o = self._orders[epoch]
+        B = self.cfg.batch_size
+        return o[b * B:(b + 1) * B]
+
+
+# ----------------------------------------------------------------------------- our arm
+
+def run_ours(args, rank, world, local_rank):
+    import paper_conf_icpp_jiangj024_b200 as gd
+    from paper_conf_icpp_jiangj024_b200.multigpu import barrier, batch_schedule, max_over_ranks, sum_over_ranks
+
+    cfg = synth.CONFIGS[args.config]
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    want_cpu = (not args.no_cpu_baseline) and rank == 0 and world == 1
+    need_host_csr = want_cpu or (rank == 0 and args.parity_batches > 0)
+    W, K = args.warmup, args.steps
+    t_setup = time.time()
+    wl = Workload(cfg, rank, world, dev, need_host_csr)
+    g = gd.Graph(wl.indptr, wl.indices, device=local_rank, validate=False)
+    del wl.indptr, wl.indices
+    torch.cuda.empty_cache()
+    fan = list(cfg.fanouts)
+    nm, em = g.bounds(cfg.batch_size, fan)
+    n_max = nm[-1]
+    S = capacity_for(cfg, n_max)
+    t0 = time.time()
+    buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=False, device=local_rank)
+    t_register = time.time() - t0
+    wl.fill_table()
+    if cfg.preload:   # "all features resident": rebuild with the filled table preloaded
+        buf.close()
+        buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=True, device=local_rank)
+    log(f"setup: graph {wl.t_graph:.1f}s table alloc {wl.t_table_alloc:.1f}s register {t_register:.1f}s "
+        f"fill {wl.t_fill:.1f}s; N={cfg.num_nodes} E={cfg.num_edges} S={S} n_max={n_max} deg={wl.deg_stats}")
+
+    total = W + K + (0 if args.no_e2e else K)
+    sched = batch_schedule(wl.num_batches, rank, world, total)
+    seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
+    seeds_host = seeds_dev.cpu().pin_memory()
+    batch_ids = [ep * wl.num_batches + b for b, ep in sched]
+
+    outs = [g.alloc_out(cfg.batch_size, fan) for _ in range(Q + 1)]
+    feats = [buf.alloc_out(n_max) for _ in range(Q)]
+    aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(Q)]
+    dones = [torch.cuda.Event() for _ in range(Q)]
+    stats = torch.zeros((total, 2), dtype=torch.int64, device=dev)
+    sizes_log = torch.zeros((total, 2 * len(fan) + 1), dtype=torch.int64, device=dev)
+    main = torch.cuda.current_stream(dev)
+    pending = []
+
+    def step(j, host_inputs=False, host_out=None):
+        o = outs[j % (Q + 1)]
+        sd = seeds_host[j] if host_inputs else seeds_dev[j]
+        g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
+        s = j % Q
+        buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, out=feats[s], alias=aliases[s], stats=stats[j],
+                    stream=main, done=dones[s])
+        pending.append(o)
+        if len(pending) == Q:
+            r = pending.pop(0)
+            buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
+        sizes_log[j].copy_(o.sizes, non_blocking=True)
+        if host_out is not None:               # e2e: read this step's result on the host
+            host_out[0].copy_(o.sizes, non_blocking=True)
+            host_out[1].copy_(stats[j], non_blocking=True)
+            main.synchronize()
+
+    # ---- full-size sampled parity vs the oracle (untimed; first batches of this rank)
+    parity = None
+    if rank == 0 and args.parity_batches > 0:
+        parity = check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev)
+        buf.close()
+        buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
+    barrier()
+
+    # ---- warm-up
+    for j in range(W):
+        step(j)
+    torch.cuda.synchronize(dev)
+    barrier()
+    torch.cuda.synchronize(dev)
+
+    # ---- timed region (device events on the launching stream)
+    g.timing(True)
+    buf.timing(True)
+    ev0 = torch.cuda.Event(enable_timing=True)
+    ev1 = torch.cuda.Event(enable_timing=True)
+    with ClockSampler(local_rank) as clk:
+        ev0.record(main)
+        for j in range(W, W + K):
+            step(j)
+        main.wait_event(dones[(W + K - 1) % Q])     # the last batch's misses are in `out`
+        ev1.record(main)
+        ev1.synchronize()
+    torch.cuda.synchronize(dev)
+    g.timing(False)
+    buf.timing(False)
+    ms = ev0.elapsed_time(ev1)
+    ms_max = max_over_ranks(ms, dev)
+    tg = g.timing_read()
+    tb = buf.timing_read()
+    st = stats[W:W + K].sum(0).cpu().tolist()
+    sz = sizes_log[W:W + K].double().mean(0).cpu().tolist()
+    hits, misses = int(st[0]), int(st[1])
+    barrier()
+
+    # ---- e2e through the public API with host inputs / host-read results
+    e2e = None
+    if not args.no_e2e:
+        h_sizes = torch.zeros(2 * len(fan) + 1, dtype=torch.int64).pin_memory()
+        h_stats = torch.zeros(2, dtype=torch.int64).pin_memory()
+        torch.cuda.synchronize(dev)
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(main)
+        for j in range(W + K, W + 2 * K):
+            step(j, host_inputs=True, host_out=(h_sizes, h_stats))
+        main.wait_event(dones[(W + 2 * K - 1) % Q])
+        e1.record(main)
+        e1.synchronize()
+        e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)
+        e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s",
+               "h2d_bytes_per_step": cfg.batch_size * 4,
+               "d2h_bytes_per_step": (2 * len(fan) + 1) * 8 + 16}
+    status_g = g.check()
+    status_b = buf.check()
+
+    # ---- reference measurements for the roofline
+    hbm_peak = measured_peaks().get("hbm_gbs")
+    link_peak = h2d_peak_gbps(dev)
+    R = cfg.row_bytes
+    gather_bytes = 2 * R * hits + 5 * (hits + misses)       # read slot + write out, alias+flag reads
+    miss_link_bytes = R * misses                            # pinned host -> GPU over the host link
+    gather_gbs = gather_bytes / (tb["gather_ms"] * 1e6) if tb["gather_ms"] > 0 else None
+    miss_gbs = miss_link_bytes / (tb["miss_ms"] * 1e6) if tb["miss_ms"] > 0 else None
+    kern = {"sample_ms_per_batch": tg["sample_ms"] / max(1, tg["calls"]),
+            "bookkeeping_ms_per_batch": tb["bookkeeping_ms"] / max(1, tb["batches"]),
+            "gather_ms_per_batch": tb["gather_ms"] / max(1, tb["batches"]),
+            "miss_ms_per_batch": tb["miss_ms"] / max(1, tb["batches"])}
+    roof_gather = {"bound": "hbm", "achieved": round(gather_gbs, 1) if gather_gbs else None, "peak": hbm_peak,
+                   "unit": "GB/s", "frac": round(gather_gbs / hbm_peak, 4) if gather_gbs and hbm_peak else None,
+                   "traffic": None, "kernel": "k_gather_hits", "peak_source": "MEASURED_PEAKS.json hbm_gbs"}
+    roof_miss = {"bound": "host_link", "achieved": round(miss_gbs, 2) if miss_gbs else None,
+                 "peak": round(link_peak, 2), "unit": "GB/s",
+                 "frac": round(miss_gbs / link_peak, 4) if miss_gbs else None, "traffic": None,
+                 "kernel": "k_miss_copy", "peak_source": "in-run pinned 1 GiB H2D cudaMemcpyAsync, best of 10"}
+    dominant = roof_miss if kern["miss_ms_per_batch"] >= kern["gather_ms_per_batch"] and misses > 0 else roof_gather
+    traffic = load_traffic(cfg.name)
+    if traffic:
+        for r in (roof_gather, roof_miss):
+            if r["kernel"] in traffic:
+                r["traffic"] = traffic[r["kernel"]]
+
+    cpu = None
+    if want_cpu:
+        cpu = cpu_baseline(cfg, wl, sched, batch_ids, fan, S, args.cpu_seconds)
+    total_batches = sum_over_ranks(K, dev)
+    value = total_batches / (ms_max / 1e3)
+    line = {
+        "metric": "sampled+extracted mini-batches/s",
+        "value": round(value, 2), "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
+        "ms_per_step": round(ms_max / K, 4), "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
+        "config": {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
+                   "feat_dim": cfg.feat_dim, "feat_bytes": R, "batch_size": cfg.batch_size, "fanouts": fan,
+                   "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
+                   "parallelism": f"dp{world} (batch segments, no collective)",
+                   "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
+                       (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.num_nodes * R * 1e-9)},
+        "e2e": e2e,
+        "gpu_launches": K * (2 * len(fan) + 8),
+        "roofline": dominant,
+        "roofline_gather": roof_gather,
+        "roofline_miss": roof_miss,
+        "cpu_baseline": cpu,
+        "clocks": clk.summary(),
+        "per_batch": {"n_nodes": round(sz[len(fan)], 1), "edges": [round(x, 1) for x in sz[len(fan) + 1:]],
+                      "hits": hits / K, "misses": misses / K,
+                      "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
+        "parity": parity,
+        "device_status": {"graph": status_g, "buffer": status_b},
+        "setup_s": round(time.time() - t_setup, 1),
+    }
+    if rank == 0:
+        s = json.dumps(line)
+        print(s, flush=True)
+        if args.out:
+            with open(args.out, "w") as f:
+                f.write(s + "\n")
+    buf.close()
+    g.close()
+    wl.close()
+
+
+def load_traffic(config_name):
+    """dram bytes per launch from the committed ncu --set full summary, if any."""
+    p = os.path.join(ROOT, "profiles", "traffic.json")
+    try:
+        return json.load(open(p)).get(config_name)
+    except Exception:  # noqa: BLE001
+        return None
+
+
+def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
+    """Full-size sampled parity: the first batches in the bench's launch configuration,
+    checked bit-exactly against the oracle (sampling outputs, alias, hit/miss, out rows)."""
+    from oracle import oracle as O
+    t0 = time.time()
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    res_ok = True
+    checked = 0
+    for j in range(min(args.parity_batches, len(sched))):
+        b, ep = sched[j]
+        seeds = wl.seeds(b, ep)
+        o = g.sample(seeds.to(dev), fan, synth.RNG_SEED, batch_ids[j], with_eid=True)
+        alias = torch.empty(n_max, dtype=torch.int32, device=dev)
+        st = torch.zeros(2, dtype=torch.int64, device=dev)
+        out, _, done = buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, alias=alias, stats=st)
+        done.synchronize()
+        h = o.to_host()
+        ref = O.sample(wl.host_indptr, wl.host_indices, seeds.cpu().numpy(), fan, synth.RNG_SEED, batch_ids[j])
+        ok = np.array_equal(h["sizes"], ref.sizes) and np.array_equal(h["n_id"], ref.n_id)
+        for k in range(len(fan)):
+            ok &= np.array_equal(h["rowptr"][k], ref.rowptr[k]) and np.array_equal(h["col"][k], ref.col[k])
+            ok &= np.array_equal(h["eid"][k], ref.eid[k])
+        o_out, o_alias, o_st = ob.extract(ref.n_id)
+        n = len(ref.n_id)
+        ok &= tuple(st.cpu().tolist()) == o_st
+        ok &= np.array_equal(alias[:n].cpu().numpy(), o_alias)
+        ok &= np.array_equal(out[:n].cpu().numpy(), o_out)
+        res_ok &= bool(ok)
+        checked += 1
+    return {"batches": checked, "bit_exact": res_ok, "seconds": round(time.time() - t0, 1)}
+
+
+def cpu_baseline(cfg, wl, sched, batch_ids, fan, S, budget_s):
+    """The oracle as it stands, single-threaded on this host, on a bounded sample of the same
+    workload: full steps (sample + Alg. 1 extract + release with lag Q) until budget_s."""
+    from oracle import oracle as O
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    pend = []
+    n = 0
+    t0 = time.perf_counter()
+    while True:
+        b, ep = sched[n % len(sched)]
+        ref = O.sample(wl.host_indptr, wl.host_indices, wl.seeds(b, ep).cpu().numpy(), fan, synth.RNG_SEED,
+                       batch_ids[n % len(sched)])
+        ob.extract(ref.n_id)
+        pend.append(ref.n_id)
+        if len(pend) == Q:
+            ob.release(pend.pop(0))
+        n += 1
+        el = time.perf_counter() - t0
+        if el >= budget_s or n >= 10_000:
+            break
+    return {"value": round(n / el, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
+            "sample": f"{n} consecutive full mini-batches of {cfg.name} (sample+extract+release, Q={Q}), "
+                      f"{el:.1f} s on 1 host thread"}
+
+
+# ----------------------------------------------------------------------- reference arm
+
+def run_reference(args, rank, world, local_rank):
+    """The oracle (oracle/) as the reference arm: W + K full steps on the host CPU."""
+    if rank != 0:
+        return
+    from oracle import oracle as O
+    cfg = synth.CONFIGS[args.config]
+    dev = torch.device("cuda", local_rank) if torch.cuda.is_available() else torch.device("cpu")
+    wl = Workload(cfg, 0, 1, dev, True)
+    del wl.indptr, wl.indices
+    wl.fill_table()
+    fan = list(cfg.fanouts)
+    nm = O.sample_bounds(cfg.batch_size, fan, cfg.num_nodes, cfg.num_edges)[0]
+    S = capacity_for(cfg, nm[-1])
+    from paper_conf_icpp_jiangj024_b200.multigpu import batch_schedule
+    sched = batch_schedule(wl.num_batches, 0, 1, args.warmup + args.steps)
+    bids = [ep * wl.num_batches + b for b, ep in sched]
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    pend = []
+    t0 = None
+    for j, (b, ep) in enumerate(sched):
+        if j == args.warmup:
+            t0 = time.perf_counter()
+        ref = O.sample(wl.host_indptr, wl.host_indices, wl.seeds(b, ep).cpu().numpy(), fan, synth.RNG_SEED, bids[j])
+        ob.extract(ref.n_id)
+        pend.append(ref.n_id)
+        if len(pend) == Q:
+            ob.release(pend.pop(0))
+    el = time.perf_counter() - t0
+    v = args.steps / el
+    line = {"impl": "reference", "metric": "sampled+extracted mini-batches/s", "value": round(v, 3),
+            "unit": "batches/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
+            "ms_per_step": round(el * 1e3 / args.steps, 2), "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
+            "config": {"workload": cfg.name, "batch_size": cfg.batch_size, "fanouts": fan, "buffer_slots": S},
+            "cpu_baseline": {"value": round(v, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{args.steps} timed full mini-batches after {args.warmup} warm-up, 1 thread"},
+            "e2e": {"value": round(v, 3), "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    wl.close()
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        if args.impl == "reference":
+            run_reference(args, rank, world, local_rank)
+        else:
+            run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

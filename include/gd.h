@@ -200,6 +200,17 @@ gd_status gd_buffer_set_state(gd_buffer* b, const int32_t* map_slot, const int32
 /* The internal side stream (cudaStream_t as void*) misses are copied on. */
 void* gd_buffer_side_stream(gd_buffer* b);
 
+/* Per-kernel timing with CUDA events recorded on the streams the kernels run on
+ * (the caller's stream for bookkeeping / gather / sampling, the side stream for
+ * misses).  enable != 0 starts collecting (and clears what was collected);
+ * enable == 0 stops.  *_timing_read synchronises and sums the collected
+ * durations in milliseconds.  Used by bench.py for the roofline fractions. */
+gd_status gd_buffer_timing(gd_buffer* b, int enable);
+gd_status gd_buffer_timing_read(gd_buffer* b, double* bookkeeping_ms, double* gather_ms, double* miss_ms,
+                                int64_t* batches);
+gd_status gd_graph_timing(gd_graph* g, int enable);
+gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls);
+
 #ifdef __cplusplus
 }
 #endif

@@ -141,6 +141,15 @@ class Graph:
     def check(self):
         return check_device_status(self._h)
 
+    def timing(self, enable: bool):
+        check(lib.gd_graph_timing(self._h, int(enable)))
+
+    def timing_read(self):
+        ms = ctypes.c_double()
+        n = ctypes.c_int64()
+        check(lib.gd_graph_timing_read(self._h, ctypes.byref(ms), ctypes.byref(n)))
+        return {"sample_ms": ms.value, "calls": n.value}
+
 
 class FeatureBuffer:
     """gd_buffer: slot-managed HBM feature buffer over a pinned host table (the SSD stand-in)."""
@@ -217,6 +226,15 @@ class FeatureBuffer:
 
     def check(self):
         return check_device_status(self._h)
+
+    def timing(self, enable: bool):
+        check(lib.gd_buffer_timing(self._h, int(enable)))
+
+    def timing_read(self):
+        a, g, m = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+        n = ctypes.c_int64()
+        check(lib.gd_buffer_timing_read(self._h, ctypes.byref(a), ctypes.byref(g), ctypes.byref(m), ctypes.byref(n)))
+        return {"bookkeeping_ms": a.value, "gather_ms": g.value, "miss_ms": m.value, "batches": n.value}
 
 
 def check_device_status(handle) -> int:

@@ -20,7 +20,8 @@ DEV_BITS = {0x1: "GD_DEV_BAD_ID", 0x2: "GD_DEV_DUP_SEED", 0x4: "GD_DEV_UNDERFLOW
 # every entry point include/gd.h declares (checked by tests/test_abi.py)
 EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy", "gd_sample_bounds", "gd_sample",
            "gd_buffer_init", "gd_buffer_destroy", "gd_extract", "gd_buffer_release", "gd_check_device_status",
-           "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream"]
+           "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream", "gd_buffer_timing",
+           "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read"]
 
 
 class GdError(RuntimeError):
@@ -45,7 +46,7 @@ _st = ctypes.c_int
 
 def _load():
     if not os.path.exists(LIB_PATH):
-        raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_jiangj024_b200._build` "
+        raise ImportError(f"{LIB_PATH} is missing: build it with `python tools/build_native.py` "
                           "(or __graft_entry__.build()); there is no non-CUDA fallback")
     L = ctypes.CDLL(LIB_PATH)
     L.gd_last_error.restype = ctypes.c_char_p
@@ -65,6 +66,11 @@ def _load():
     L.gd_buffer_set_state.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _i64]
     L.gd_buffer_side_stream.argtypes = [_vp]
     L.gd_buffer_side_stream.restype = _vp
+    _dp = ctypes.POINTER(ctypes.c_double)
+    L.gd_buffer_timing.argtypes = [_vp, ctypes.c_int]
+    L.gd_buffer_timing_read.argtypes = [_vp, _dp, _dp, _dp, ctypes.POINTER(_i64)]
+    L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
+    L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:
         if name not in ("gd_last_error", "gd_version", "gd_buffer_side_stream"):
             getattr(L, name).restype = _st

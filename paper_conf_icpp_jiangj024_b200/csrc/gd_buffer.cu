@@ -548,6 +548,7 @@ static void buffer_free(gd_buffer* b) {
     for (void* p : ptrs)
         if (p) cudaFree(p);
     b->scan.release();
+    b->timer.destroy();
     for (cudaEvent_t e : b->ev_trip)
         if (e) cudaEventDestroy(e);
     if (b->ev_L) cudaEventDestroy(b->ev_L);
@@ -676,6 +677,26 @@ gd_status gd_buffer_destroy(gd_buffer* b) {
     return GD_OK;
 }
 
+gd_status gd_buffer_timing(gd_buffer* b, int enable) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing: bad handle");
+    DeviceGuard guard(b->hdr.device);
+    if (enable) b->timer.reset();
+    b->timer.on = enable != 0;
+    return GD_OK;
+}
+
+gd_status gd_buffer_timing_read(gd_buffer* b, double* bookkeeping_ms, double* gather_ms, double* miss_ms,
+                                int64_t* batches) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing_read: bad handle");
+    DeviceGuard guard(b->hdr.device);
+    if (bookkeeping_ms) *bookkeeping_ms = b->timer.total_ms(3, 0);
+    if (gather_ms) *gather_ms = b->timer.total_ms(3, 1);
+    if (miss_ms) *miss_ms = b->timer.total_ms(3, 2);
+    if (batches) *batches = (int64_t)b->timer.pairs.size() / 3;
+    GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
 void* gd_buffer_side_stream(gd_buffer* b) { return (b && b->hdr.magic == kMagicBuffer) ? (void*)b->side : nullptr; }
 
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max, void* out,
@@ -696,6 +717,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     const int64_t lt = std::max<int64_t>(1, cdiv(n_max, kBTile));
 
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));   // side stream done with trip slot d
+    const bool timed = b->timer.on;
+    const int t_book = timed ? b->timer.begin(st) : -1;
 
     LookupArgs la;
     la.ids = node_ids;
@@ -738,22 +761,27 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     k_pop_assign<<<148 * 2, kBThreads, 0, st>>>(pa);
     b->scan.flip();
     b->ctl_parity ^= 1;
+    if (timed) b->timer.end(t_book, st);
     GD_CUDA(cudaEventRecord(b->ev_L, st));
 
     // hits: their rows were written by earlier miss streams, all ordered before X_{b-1}
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_X, 0));
+    const int t_gat = timed ? b->timer.begin(st) : -1;
     if (b->R % 16 == 0)
         k_gather_hits<4><<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
     else
         k_gather_hits_w4<<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
+    if (timed) b->timer.end(t_gat, st);
     GD_CUDA(cudaEventRecord(b->ev_G, st));
 
     // misses: pinned host -> slot + out on the side stream (asynchronous extraction)
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
+    const int t_miss = timed ? b->timer.begin(b->side) : -1;
     if (b->R % 16 == 0)
         k_miss_copy<4><<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     else
         k_miss_copy_w4<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+    if (timed) b->timer.end(t_miss, b->side);
     GD_CUDA(cudaEventRecord(b->ev_X, b->side));
     GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side));
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));

@@ -7,6 +7,8 @@
 #include <stdint.h>
 
 #include <string>
+#include <utility>
+#include <vector>
 
 #include "../../include/gd.h"
 
@@ -46,6 +48,51 @@ struct DeviceGuard {            // switch to the handle's device for one API cal
 // Pointer kind: true if `p` is device-accessible memory of the current context
 // (device / managed), false for host memory (pageable or pinned).
 bool is_device_pointer(const void* p);
+
+// ------------------------------------------------------------ event timing (host)
+// Pairs of events recorded around kernel groups; summed on read (which syncs).
+struct EventTimer {
+    bool on = false;
+    std::vector<cudaEvent_t> pool;
+    std::vector<std::pair<int, int>> pairs;   // indices into pool
+    int used = 0;
+    cudaEvent_t next() {
+        if (used == (int)pool.size()) {
+            cudaEvent_t e;
+            cudaEventCreate(&e);
+            pool.push_back(e);
+        }
+        return pool[used++];
+    }
+    void reset() { used = 0; pairs.clear(); }
+    // record the start of a group on `s`; returns the pair slot
+    int begin(cudaStream_t s) {
+        const int a = used;
+        cudaEventRecord(next(), s);
+        pairs.push_back({a, -1});
+        return (int)pairs.size() - 1;
+    }
+    void end(int slot, cudaStream_t s) {
+        pairs[slot].second = used;
+        cudaEventRecord(next(), s);
+    }
+    double total_ms(int stride, int which) {   // sum the pairs with index % stride == which
+        double t = 0;
+        for (size_t i = which; i < pairs.size(); i += stride) {
+            if (pairs[i].second < 0) continue;
+            float ms = 0;
+            cudaEventSynchronize(pool[pairs[i].second]);
+            cudaEventElapsedTime(&ms, pool[pairs[i].first], pool[pairs[i].second]);
+            t += ms;
+        }
+        return t;
+    }
+    void destroy() {
+        for (auto e : pool) cudaEventDestroy(e);
+        pool.clear();
+        reset();
+    }
+};
 
 // --------------------------------------------------------- scan tile states (host)
 // Decoupled look-back needs one 64-bit status word per tile, zero before a launch.

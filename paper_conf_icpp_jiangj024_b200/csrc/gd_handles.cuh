@@ -19,6 +19,7 @@ struct gd_graph {
     int32_t* seeds_ws = nullptr;    // staging for host seed arrays
     int64_t seeds_cap = 0;
     gd::ScanState scan;
+    gd::EventTimer timer;            // one pair per gd_sample call
 };
 
 // Control block of the standby ring.  Kernels that move head/tail read ctl[p] and
@@ -65,6 +66,7 @@ struct gd_buffer {
     cudaStream_t side = nullptr;
     cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_G = nullptr;
     std::vector<cudaEvent_t> ev_trip;    // [D] side stream finished with trip ring slot
+    gd::EventTimer timer;                // 3 pairs per gd_extract: bookkeeping, gather, miss
     int64_t batch_counter = 0;
     int64_t inflight = 0;
     unsigned long long epoch = 1;

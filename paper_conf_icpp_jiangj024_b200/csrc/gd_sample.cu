@@ -429,6 +429,7 @@ gd_status gd_graph_destroy(gd_graph* g) {
     if (g->seeds_ws) cudaFree(g->seeds_ws);
     if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
     g->scan.release();
+    g->timer.destroy();
     g->hdr.magic = 0;
     delete g;
     return GD_OK;
@@ -485,6 +486,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     uint32_t* hk = g->hash;
     uint32_t* hv = g->hash + g->hcap;
     const uint32_t mask = (uint32_t)(g->hcap - 1);
+    const int tslot = g->timer.on ? g->timer.begin(st) : -1;
     GD_CUDA(cudaMemsetAsync(g->hash, 0xFF, 2 * g->hcap * sizeof(uint32_t), st));
     k_seed_intake<<<(unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads)), kThreads, 0, st>>>(
         seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status);
@@ -542,6 +544,24 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
               (unsigned)num_hops);
     k_col_resolve<<<grid, kThreads, 0, st>>>(c);
+    if (tslot >= 0) g->timer.end(tslot, st);
+    GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
+gd_status gd_graph_timing(gd_graph* g, int enable) {
+    if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_graph_timing: bad handle");
+    DeviceGuard guard(g->hdr.device);
+    if (enable) g->timer.reset();
+    g->timer.on = enable != 0;
+    return GD_OK;
+}
+
+gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls) {
+    if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_graph_timing_read: bad handle");
+    DeviceGuard guard(g->hdr.device);
+    if (sample_ms) *sample_ms = g->timer.total_ms(1, 0);
+    if (calls) *calls = (int64_t)g->timer.pairs.size();
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }

@@ -18,8 +18,8 @@ def declared_functions():
 
 @pytest.fixture(scope="module")
 def gd():
-    from paper_conf_icpp_jiangj024_b200 import _build
-    _build.build()
+    from tools import build_native
+    build_native.build()
     from paper_conf_icpp_jiangj024_b200 import _lib
     return _lib
 

@@ -213,13 +213,13 @@ def test_figure6_on_gpu(gd):
     gdict = json.load(open(os.path.join(HERE, "golden", "fig6.json")))
     N, S = gdict["num_nodes"], gdict["num_slots"]
     feat = table_np(N, 16)
-    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, 2, 8)
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, 1, 5)     # S=6 >= min(N, 1 x 5)
     buf.set_state(gdict["map_slot"], gdict["map_rc"], gdict["map_valid"], gdict["reverse"], gdict["standby"])
     ids = torch.tensor(gdict["batch"], dtype=torch.int32, device="cuda")
     n = torch.tensor([len(gdict["batch"])], dtype=torch.int64, device="cuda")
-    alias = torch.empty(8, dtype=torch.int32, device="cuda")
+    alias = torch.empty(5, dtype=torch.int32, device="cuda")
     stats = torch.zeros(2, dtype=torch.int64, device="cuda")
-    out, _, done = buf.extract(ids, n, 8, alias=alias, stats=stats)
+    out, _, done = buf.extract(ids, n, 5, alias=alias, stats=stats)
     done.synchronize()
     assert alias[:5].cpu().tolist() == gdict["expect_alias"]
     assert stats.cpu().tolist() == [gdict["expect_hits"], gdict["expect_misses"]]
@@ -230,7 +230,7 @@ def test_figure6_on_gpu(gd):
         assert st["valid"][v] == 0 and st["slot"][v] == -1
     assert np.array_equal(out[:5].cpu().numpy(), feat[gdict["batch"]])
     rel = torch.tensor(gdict["release"], dtype=torch.int32, device="cuda")
-    buf.release(rel, torch.tensor([1], dtype=torch.int64, device="cuda"), 8)
+    buf.release(rel, torch.tensor([1], dtype=torch.int64, device="cuda"), 5)
     assert buf.snapshot()["standby"].tolist() == gdict["expect_standby_after_release"]
 
 

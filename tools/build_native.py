@@ -1,6 +1,8 @@
-"""Build libgd.so (the sm_100a kernels + C ABI) in-tree with nvcc.
+"""Build paper_conf_icpp_jiangj024_b200/libgd.so (the sm_100a kernels + C ABI) in-tree with nvcc.
 
-    python -m paper_conf_icpp_jiangj024_b200._build [--force] [--verbose]
+    python tools/build_native.py [--force] [--verbose]
+
+Lives outside the package so that building never imports (and loads) a stale libgd.so.
 """
 from __future__ import annotations
 
@@ -9,8 +11,8 @@ import os
 import subprocess
 import sys
 
-PKG = os.path.dirname(os.path.abspath(__file__))
-ROOT = os.path.dirname(PKG)
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+PKG = os.path.join(ROOT, "paper_conf_icpp_jiangj024_b200")
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libgd.so")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
