@@ -243,22 +243,34 @@ def run_ours(args, rank, world, local_rank):
     feats = [buf.alloc_out(n_max) for _ in range(Q)]
     aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(Q)]
     dones = [torch.cuda.Event() for _ in range(Q)]
+    for e in dones:
+        e.record(torch.cuda.current_stream(dev))     # create the events (torch creates lazily)
     stats = torch.zeros((total, 2), dtype=torch.int64, device=dev)
     sizes_log = torch.zeros((total, 2 * len(fan) + 1), dtype=torch.int64, device=dev)
     main = torch.cuda.current_stream(dev)
     pending = []
 
+    dbg = os.environ.get("GD_DEBUG_SYNC") == "1"
+
+    def dsync(what, j):
+        if dbg:
+            torch.cuda.synchronize(dev)
+            log(f"  step {j}: {what} ok")
+
     def step(j, host_inputs=False, host_out=None):
         o = outs[j % (Q + 1)]
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
         g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
+        dsync("sample", j)
         s = j % Q
         buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, out=feats[s], alias=aliases[s], stats=stats[j],
                     stream=main, done=dones[s])
+        dsync("extract", j)
         pending.append(o)
         if len(pending) == Q:
             r = pending.pop(0)
             buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
+            dsync("release", j)
         sizes_log[j].copy_(o.sizes, non_blocking=True)
         if host_out is not None:               # e2e: read this step's result on the host
             host_out[0].copy_(o.sizes, non_blocking=True)
@@ -268,12 +280,14 @@ def run_ours(args, rank, world, local_rank):
     # ---- full-size sampled parity vs the oracle (untimed; first batches of this rank)
     parity = None
     if rank == 0 and args.parity_batches > 0:
+        log("parity check ...")
         parity = check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev)
         buf.close()
         buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
     barrier()
 
     # ---- warm-up
+    log(f"parity {parity}; warm-up ...")
     for j in range(W):
         step(j)
     torch.cuda.synchronize(dev)
@@ -281,6 +295,7 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize(dev)
 
     # ---- timed region (device events on the launching stream)
+    log("timed region ...")
     g.timing(True)
     buf.timing(True)
     ev0 = torch.cuda.Event(enable_timing=True)
@@ -305,6 +320,7 @@ def run_ours(args, rank, world, local_rank):
     barrier()
 
     # ---- e2e through the public API with host inputs / host-read results
+    log(f"timed: {ms:.2f} ms for {K} steps; e2e ...")
     e2e = None
     if not args.no_e2e:
         h_sizes = torch.zeros(2 * len(fan) + 1, dtype=torch.int64).pin_memory()
@@ -353,6 +369,7 @@ def run_ours(args, rank, world, local_rank):
                 r["traffic"] = traffic[r["kernel"]]
 
     cpu = None
+    log("cpu baseline ...")
     if want_cpu:
         cpu = cpu_baseline(cfg, wl, sched, batch_ids, fan, S, args.cpu_seconds)
     total_batches = sum_over_ranks(K, dev)
@@ -408,6 +425,7 @@ def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
     from oracle import oracle as O
     t0 = time.time()
     ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    log(f"  oracle buffer ready {time.time() - t0:.1f}s")
     res_ok = True
     checked = 0
     for j in range(min(args.parity_batches, len(sched))):
@@ -424,6 +442,7 @@ def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
         for k in range(len(fan)):
             ok &= np.array_equal(h["rowptr"][k], ref.rowptr[k]) and np.array_equal(h["col"][k], ref.col[k])
             ok &= np.array_equal(h["eid"][k], ref.eid[k])
+        log(f"  batch {j}: gpu+oracle sample done {time.time() - t0:.1f}s, ok={ok}")
         o_out, o_alias, o_st = ob.extract(ref.n_id)
         n = len(ref.n_id)
         ok &= tuple(st.cpu().tolist()) == o_st
@@ -503,6 +522,8 @@ def run_reference(args, rank, world, local_rank):
 
 
 def main():
+    import faulthandler
+    faulthandler.dump_traceback_later(float(os.environ.get("GD_BENCH_WATCHDOG", "240")), repeat=True)
     args = parse()
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))

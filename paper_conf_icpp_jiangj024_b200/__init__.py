@@ -197,6 +197,8 @@ class FeatureBuffer:
             out = self.alloc_out(n_max)
         if done is None:
             done = torch.cuda.Event()
+        if done.cuda_event == 0:        # torch creates events lazily on first record
+            done.record(torch.cuda.current_stream(self.device))
         check(lib.gd_extract(self._h, _ptr(node_ids), _ptr(n_dev), int(n_max), _ptr(out), _ptr(alias), _ptr(stats),
                              _stream_ptr(stream, self.device), ctypes.c_void_p(done.cuda_event)))
         return out, alias, done

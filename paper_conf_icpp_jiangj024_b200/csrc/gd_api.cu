@@ -1,6 +1,7 @@
 // gd_api.cu — host plumbing shared by the C ABI: thread-local errors, pointer
 // classification, scan-state allocation, sticky device status.
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -20,6 +21,20 @@ gd_status cuda_error(cudaError_t e, const char* what) {
     std::string m = std::string(what) + ": " + cudaGetErrorString(e);
     cudaGetLastError();   // clear non-sticky errors
     return set_error(e == cudaErrorMemoryAllocation ? GD_ERR_OOM : GD_ERR_CUDA, m);
+}
+
+bool debug_kernels() {
+    static const bool on = [] {
+        const char* e = std::getenv("GD_DEBUG_KERNELS");
+        return e && e[0] == '1';
+    }();
+    return on;
+}
+
+void debug_after(const char* what, cudaStream_t s) {
+    cudaError_t e = cudaStreamSynchronize(s);
+    std::fprintf(stderr, "[gd] %s -> %s\n", what, cudaGetErrorString(e));
+    std::fflush(stderr);
 }
 
 bool is_device_pointer(const void* p) {

@@ -190,9 +190,15 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
     }
     while (true) {
         if (t == 0) {
-            const long long tl = (long long)atomicAdd(a.ticket, 1ull);
-            s_tile = tl;
-            s_stop = (ld_relaxed_u64(a.done_word) == a.epoch) || (c.head + tl * kBTile >= c.tail && tl > 0);
+            // Check `done` BEFORE taking a ticket: every ticket taken must be processed and
+            // published, or the block holding the next ticket would spin on it forever.
+            if (ld_relaxed_u64(a.done_word) == a.epoch) {
+                s_stop = 1;
+            } else {
+                const long long tl = (long long)atomicAdd(a.ticket, 1ull);
+                s_tile = tl;
+                s_stop = (c.head + tl * kBTile >= c.tail && tl > 0);   // monotone in tl
+            }
         }
         __syncthreads();
         if (s_stop) break;
@@ -736,6 +742,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     la.st_clear_n = b->scan.cap;
     la.status = b->hdr.dev_status;
     k_lookup<<<(unsigned)lt, kBThreads, 0, st>>>(la);
+    GD_DEBUG_AFTER("k_lookup", st);
     b->scan.flip();
 
     PopArgs pa;
@@ -759,6 +766,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.st_clear_n = b->scan.cap;
     pa.status = b->hdr.dev_status;
     k_pop_assign<<<148 * 2, kBThreads, 0, st>>>(pa);
+    GD_DEBUG_AFTER("k_pop_assign", st);
     b->scan.flip();
     b->ctl_parity ^= 1;
     if (timed) b->timer.end(t_book, st);
@@ -771,6 +779,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         k_gather_hits<4><<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
     else
         k_gather_hits_w4<<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
+    GD_DEBUG_AFTER("k_gather_hits", st);
     if (timed) b->timer.end(t_gat, st);
     GD_CUDA(cudaEventRecord(b->ev_G, st));
 
@@ -781,6 +790,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         k_miss_copy<4><<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     else
         k_miss_copy_w4<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+    GD_DEBUG_AFTER("k_miss_copy", b->side);
     if (timed) b->timer.end(t_miss, b->side);
     GD_CUDA(cudaEventRecord(b->ev_X, b->side));
     GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side));
@@ -814,6 +824,7 @@ gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t
     ca.st_clear = b->scan.other();
     ca.st_clear_n = b->scan.cap;
     k_compact<<<148 * 2, kBThreads, 0, st>>>(ca);
+    GD_DEBUG_AFTER("k_compact", st);
     b->scan.flip();
     b->ctl_parity ^= 1;
 
@@ -831,6 +842,7 @@ gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t
     ra.st_clear_n = b->scan.cap;
     ra.status = b->hdr.dev_status;
     k_release<<<(unsigned)std::max<int64_t>(1, cdiv(n_max, kBTile)), kBThreads, 0, st>>>(ra);
+    GD_DEBUG_AFTER("k_release", st);
     b->scan.flip();
     b->ctl_parity ^= 1;
     GD_CUDA(cudaGetLastError());

@@ -45,6 +45,14 @@ struct DeviceGuard {            // switch to the handle's device for one API cal
     }
 };
 
+// Debug trace (env GD_DEBUG_KERNELS=1): synchronise after each launch and log it.
+bool debug_kernels();
+void debug_after(const char* what, cudaStream_t s);
+#define GD_DEBUG_AFTER(what, s)                       \
+    do {                                              \
+        if (::gd::debug_kernels()) ::gd::debug_after(what, s); \
+    } while (0)
+
 // Pointer kind: true if `p` is device-accessible memory of the current context
 // (device / managed), false for host memory (pageable or pinned).
 bool is_device_pointer(const void* p);

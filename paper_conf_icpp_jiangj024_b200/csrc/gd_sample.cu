@@ -515,6 +515,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
         a.status = g->hdr.dev_status;
         const int64_t nt = std::max<int64_t>(1, ceil_div(nmax[h - 1], kNodesPerTile));
         k_sample_hop<<<(unsigned)nt, kThreads, 0, st>>>(a);
+        GD_DEBUG_AFTER("k_sample_hop", st);
         g->scan.flip();
 
         RelabelArgs r;
@@ -530,6 +531,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
         r.st_clear_n = g->scan.cap;
         const int64_t et = std::max<int64_t>(1, ceil_div(emax[h - 1], kEdgesPerTile));
         k_relabel_hop<<<(unsigned)et, kThreads, 0, st>>>(r);
+        GD_DEBUG_AFTER("k_relabel_hop", st);
         g->scan.flip();
     }
     ColResolveArgs c;
@@ -544,6 +546,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
               (unsigned)num_hops);
     k_col_resolve<<<grid, kThreads, 0, st>>>(c);
+        GD_DEBUG_AFTER("k_col_resolve", st);
     if (tslot >= 0) g->timer.end(tslot, st);
     GD_CUDA(cudaGetLastError());
     return GD_OK;
