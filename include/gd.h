@@ -161,7 +161,8 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  *   n_max     host bound on n (grid sizing); must be <= max_nodes_per_batch.
  *   out       device [n_max * row_bytes] (16-byte aligned): out[i] = feat[node_ids[i]].
  *   alias     device int32[n_max] or NULL: slot of node_ids[i] (Alg. 1 ids_r).
- *   stats     device int64[2] or NULL: {hits, misses} of this batch.
+ *   stats     device int64[4] or NULL: {hits, misses, misses copied zero-copy,
+ *             misses copied through the staged path} of this batch.
  *   done      cudaEvent_t (void*) or NULL: recorded when `out` is complete.
  *             `out` is valid only after `done`; `stream` itself does NOT wait
  *             for the misses.  node_ids must stay unmodified until `done`.
@@ -169,6 +170,21 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  * ------------------------------------------------------------------------- */
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,
                      void* out, int32_t* alias, int64_t* stats, void* stream, void* done);
+
+/* ----------------------------------------------------------------------------
+ * Miss-stream configuration.  The misses of a batch are split in list order: ranks
+ * [0, K0) are copied zero-copy from the pinned table by SM loads; ranks [K0, M) take
+ * the paper's two-phase path: phase 1, `host_threads` library-owned
+ * CPU threads gather the rows into a pinned staging slot (run from a CUDA host
+ * function, so still stream-ordered, no caller sync); phase 2, a kernel pulls the
+ * slot contiguously over the host link.  K0 = floor(M * zero_copy_share).
+ *   host_threads     0 disables the staged path (all misses zero-copy).
+ *   zero_copy_share  in [0, 1]; < 0 = adaptive (balance the two paths' measured rates).
+ * Default at init: host_threads = min(8, cores/2) (0 with preload), adaptive share;
+ * env GD_HOST_THREADS / GD_ZERO_COPY_SHARE override.  Synchronises the buffer's
+ * internal streams; call between batches.
+ * ------------------------------------------------------------------------- */
+gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share);
 
 /* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a
@@ -206,8 +222,9 @@ void* gd_buffer_side_stream(gd_buffer* b);
  * enable == 0 stops.  *_timing_read synchronises and sums the collected
  * durations in milliseconds.  Used by bench.py for the roofline fractions. */
 gd_status gd_buffer_timing(gd_buffer* b, int enable);
-gd_status gd_buffer_timing_read(gd_buffer* b, double* bookkeeping_ms, double* gather_ms, double* miss_ms,
-                                int64_t* batches);
+/* ms[6] = {bookkeeping (lookup + pop/assign), hit gather, zero-copy miss copy,
+ *          staged miss pull, host gather (phase 1, summed), current zero-copy share}. */
+gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches);
 gd_status gd_graph_timing(gd_graph* g, int enable);
 gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls);
 

@@ -233,10 +233,15 @@ class FeatureBuffer:
         check(lib.gd_buffer_timing(self._h, int(enable)))
 
     def timing_read(self):
-        a, g, m = ctypes.c_double(), ctypes.c_double(), ctypes.c_double()
+        ms = (ctypes.c_double * 6)()
         n = ctypes.c_int64()
-        check(lib.gd_buffer_timing_read(self._h, ctypes.byref(a), ctypes.byref(g), ctypes.byref(m), ctypes.byref(n)))
-        return {"bookkeeping_ms": a.value, "gather_ms": g.value, "miss_ms": m.value, "batches": n.value}
+        check(lib.gd_buffer_timing_read(self._h, ms, ctypes.byref(n)))
+        return {"bookkeeping_ms": ms[0], "gather_ms": ms[1], "miss_zero_copy_ms": ms[2], "miss_staged_ms": ms[3],
+                "host_gather_ms": ms[4], "zero_copy_share": ms[5], "batches": n.value}
+
+    def config(self, host_threads: int, zero_copy_share: float = -1.0):
+        """gd_buffer_config: staged miss path width and zero-copy share (< 0: adaptive)."""
+        check(lib.gd_buffer_config(self._h, int(host_threads), float(zero_copy_share)))
 
 
 def check_device_status(handle) -> int:

@@ -4,8 +4,10 @@
 //   caller stream:  k_lookup (Alg. 1 loop 1 + miss ranks) -> k_pop_assign (loop 2:
 //                   LRU standby slots, eviction, map/reverse/alias) -> [L_b]
 //                   -> wait X_{b-1} -> k_gather_hits (slots -> out) -> [G_b]
-//   side stream:    wait L_b -> k_miss_copy (pinned host -> slot + out) -> [X_b]
-//                   -> wait G_b -> [done]
+//   stream Z:       wait L_b -> k_miss_copy<zero-copy> misses [0, K0) -> [X_b]
+//   stream H:       wait L_b -> host gather (thread pool) of misses [K0, M) -> [E_b]
+//   stream P:       wait E_b -> k_miss_copy<staged> pull of the staging slot -> [Xs_b]
+//   stream J:       wait X_b, Xs_b, G_b -> [done]
 // gd_buffer_release(b): k_compact (only when the ring is nearly full; exits at once
 //   otherwise) -> k_release (refcount--, became-zero slots appended at the tail).
 //
@@ -17,6 +19,8 @@
 #include <cstring>
 #include <string>
 #include <vector>
+#include <cstdlib>
+#include <thread>
 
 #include "gd_common.cuh"
 #include "gd_handles.cuh"
@@ -149,6 +153,11 @@ struct PopArgs {
     int32_t* alias;
     int4* trip;
     int64_t* trip_count;
+    int64_t* trip_split;            // K0 = floor(M * alpha_q16 / 2^16): first staged rank
+    uint32_t alpha_q16;
+    int32_t* h_nodes;               // mapped host: node ids of ranks [K0, M) (staged share)
+    int64_t* h_meta;                // mapped host: {M, K0, M - K0}
+    int64_t* stats;                 // caller's stats or null: [2] = K0, [3] = M - K0
     unsigned long long* ticket;     // [2]: next tile, blocks finished
     unsigned long long* done_word;
     unsigned long long epoch;
@@ -180,10 +189,21 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
     __shared__ int s_cnt[kBItems * kBWarps];
     __shared__ long long s_base;
     const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+    const long long K0 = (long long)(((unsigned long long)M * a.alpha_q16) >> 16);
     if (M == 0) {
         if (blockIdx.x == 0 && t == 0) {
             *a.ctl_out = c;
             *a.trip_count = 0;
+            *a.trip_split = 0;
+            if (a.h_meta) {
+                a.h_meta[0] = 0;
+                a.h_meta[1] = 0;
+                a.h_meta[2] = 0;
+            }
+            if (a.stats) {
+                a.stats[2] = 0;
+                a.stats[3] = 0;
+            }
         }
         ticket_finish(a.ticket);
         return;
@@ -228,7 +248,18 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                     GdCtl o = c;
                     o.head = c.tail;
                     *a.ctl_out = o;
-                    *a.trip_count = base + agg;
+                    const long long Mx = base + agg, K0x = K0 < Mx ? K0 : Mx;
+                    *a.trip_count = Mx;
+                    *a.trip_split = K0x;
+                    if (a.h_meta) {
+                        a.h_meta[0] = Mx;
+                        a.h_meta[1] = K0x;
+                        a.h_meta[2] = Mx - K0x;
+                    }
+                    if (a.stats) {
+                        a.stats[2] = K0x;
+                        a.stats[3] = Mx - K0x;
+                    }
                     __threadfence();
                     st_relaxed_u64(a.done_word, a.epoch);
                 }
@@ -254,12 +285,23 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                 a.alias[i] = s;                                 // line 29
                 a.pos_of_slot[s] = -1;
                 a.trip[rank] = make_int4(v, s, i, 0);
+                if (rank >= K0 && a.h_nodes) a.h_nodes[rank - K0] = v;
                 if (rank == M - 1) {
                     const long long p = p0 + (long long)k * kBThreads + t;
                     GdCtl o = c;
                     o.head = p + 1;
                     *a.ctl_out = o;
                     *a.trip_count = M;
+                    *a.trip_split = K0;
+                    if (a.h_meta) {
+                        a.h_meta[0] = M;
+                        a.h_meta[1] = K0;
+                        a.h_meta[2] = M - K0;
+                    }
+                    if (a.stats) {
+                        a.stats[2] = K0;
+                        a.stats[3] = M - K0;
+                    }
                     __threadfence();
                     st_relaxed_u64(a.done_word, a.epoch);
                 }
@@ -271,12 +313,17 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
 }
 
 // ------------------------------------------------------------ a7: miss stream
+// Copies miss ranks k in [*begin, *end) (begin == nullptr: 0) into their slot and
+// their `out` row.  STAGED = false: source row = pinned host table row trip[k].x
+// (zero-copy over the host link).  STAGED = true: source row = staging row k - begin
+// (the contiguous phase-2 pull of rows the host gathered in phase 1).
 // One 16-byte chunk per thread-iteration, UNROLL chunks in flight per thread.
-template <int UNROLL>
-__global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ count,
-                                                   const uint8_t* __restrict__ feat, uint8_t* __restrict__ slots,
-                                                   uint8_t* __restrict__ out, int64_t R) {
-    const int64_t M = *count;
+template <int UNROLL, bool STAGED>
+__global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
+                                                   const int64_t* __restrict__ end, const uint8_t* __restrict__ src,
+                                                   uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+    const int64_t k0 = begin ? *begin : 0;
+    const int64_t M = *end - k0;
     const int64_t cpr = R >> 4;                     // 16-byte chunks per row
     const int64_t total = M * cpr;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -289,11 +336,11 @@ __global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip
             dsl[u] = -1;
             if (idx < total) {
                 const int64_t r = idx / cpr, c = idx - r * cpr;
-                const int4 tr = __ldg(trip + r);
-                const uint4* src = (const uint4*)(feat + (int64_t)tr.x * R) + c;
+                const int4 tr = __ldg(trip + k0 + r);
+                const uint4* sp = STAGED ? (const uint4*)(src + r * R) + c : (const uint4*)(src + (int64_t)tr.x * R) + c;
                 asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                              : "=r"(val[u].x), "=r"(val[u].y), "=r"(val[u].z), "=r"(val[u].w)
-                             : "l"(src));
+                             : "l"(sp));
                 dsl[u] = (int64_t)tr.y * R + c * 16;
                 dout[u] = (int64_t)tr.z * R + c * 16;
             }
@@ -309,17 +356,19 @@ __global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip
 }
 
 // 4-byte fallback for rows that are not a multiple of 16 bytes
-__global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __restrict__ count,
-                               const uint8_t* __restrict__ feat, uint8_t* __restrict__ slots,
-                               uint8_t* __restrict__ out, int64_t R) {
-    const int64_t M = *count;
+template <bool STAGED>
+__global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
+                               const int64_t* __restrict__ end, const uint8_t* __restrict__ src,
+                               uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+    const int64_t k0 = begin ? *begin : 0;
+    const int64_t M = *end - k0;
     const int64_t cpr = R >> 2;
     const int64_t total = M * cpr;
     for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = idx / cpr, c = idx - r * cpr;
-        const int4 tr = trip[r];
-        const uint32_t v = ((const uint32_t*)(feat + (int64_t)tr.x * R))[c];
+        const int4 tr = trip[k0 + r];
+        const uint32_t v = STAGED ? ((const uint32_t*)(src + r * R))[c] : ((const uint32_t*)(src + (int64_t)tr.x * R))[c];
         ((uint32_t*)(slots + (int64_t)tr.y * R))[c] = v;
         ((uint32_t*)(out + (int64_t)tr.z * R))[c] = v;
     }
@@ -549,18 +598,25 @@ static void buffer_free(gd_buffer* b) {
     if (!b) return;
     DeviceGuard guard(b->hdr.device);
     if (b->side) cudaStreamSynchronize(b->side);
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+        if (s) cudaStreamSynchronize(s);
     void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->missflag,
-                    b->alias_ws, b->mcount, b->trip, b->trip_count, b->tickets, b->done_word, b->hdr.dev_status};
+                    b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
+                    b->hdr.dev_status};
     for (void* p : ptrs)
         if (p) cudaFree(p);
+    for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem})
+        if (p) cudaFreeHost(p);
+    delete b->pool;
     b->scan.release();
     b->timer.destroy();
-    for (cudaEvent_t e : b->ev_trip)
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1})
+        for (cudaEvent_t e : *v)
+            if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G})
         if (e) cudaEventDestroy(e);
-    if (b->ev_L) cudaEventDestroy(b->ev_L);
-    if (b->ev_X) cudaEventDestroy(b->ev_X);
-    if (b->ev_G) cudaEventDestroy(b->ev_G);
-    if (b->side) cudaStreamDestroy(b->side);
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+        if (s) cudaStreamDestroy(s);
     if (b->registered) cudaHostUnregister((void*)b->host_feat);
     b->hdr.magic = 0;
     delete b;
@@ -637,6 +693,7 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     GD_ALLOC(b->mcount, sizeof(int64_t));
     GD_ALLOC(b->trip, (int64_t)b->D * nm * sizeof(int4));
     GD_ALLOC(b->trip_count, b->D * sizeof(int64_t));
+    GD_ALLOC(b->trip_split, b->D * sizeof(int64_t));
     GD_ALLOC(b->tickets, 4 * sizeof(unsigned long long));
     GD_ALLOC(b->done_word, sizeof(unsigned long long));
 #undef GD_ALLOC
@@ -651,7 +708,8 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
         cudaMemset(b->hdr.dev_status, 0, sizeof(unsigned int)) != cudaSuccess ||
         cudaMemset(b->tickets, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
         cudaMemset(b->done_word, 0, sizeof(unsigned long long)) != cudaSuccess ||
-        cudaMemset(b->trip_count, 0, b->D * sizeof(int64_t)) != cudaSuccess)
+        cudaMemset(b->trip_count, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
+        cudaMemset(b->trip_split, 0, b->D * sizeof(int64_t)) != cudaSuccess)
         return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: init copies"));
     k_init_map<<<148 * 8, 256>>>(b->map, num_nodes, preload);
     k_init_slots<<<148 * 8, 256>>>(b->reverse, b->pos_of_slot, b->ring, capacity_slots, num_nodes, preload);
@@ -663,15 +721,27 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: init kernels"));
     }
-    if (cudaStreamCreateWithFlags(&b->side, cudaStreamNonBlocking) != cudaSuccess ||
-        cudaEventCreateWithFlags(&b->ev_L, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&b->ev_X, cudaEventDisableTiming) != cudaSuccess ||
-        cudaEventCreateWithFlags(&b->ev_G, cudaEventDisableTiming) != cudaSuccess)
-        return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream/event"));
-    b->ev_trip.assign(b->D, nullptr);
-    for (int d = 0; d < b->D; ++d)
-        if (cudaEventCreateWithFlags(&b->ev_trip[d], cudaEventDisableTiming) != cudaSuccess)
+    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j})
+        if (cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking) != cudaSuccess)
+            return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
+    for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G})
+        if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1}) {
+        const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1);
+        v->assign(b->D, nullptr);
+        for (int d = 0; d < b->D; ++d)
+            if (cudaEventCreateWithFlags(&(*v)[d], timing ? cudaEventDefault : cudaEventDisableTiming) != cudaSuccess)
+                return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
+    }
+    // staged miss path (phase 1 host gather + phase 2 contiguous pull): on by default
+    // unless every row is resident from the start; GD_HOST_THREADS overrides the width.
+    int threads = preload ? 0 : (int)std::min(8u, std::max(1u, std::thread::hardware_concurrency() / 2));
+    if (const char* e = std::getenv("GD_HOST_THREADS")) threads = std::max(0, std::atoi(e));
+    double share = -1.0;
+    if (const char* e = std::getenv("GD_ZERO_COPY_SHARE")) share = std::atof(e);
+    s = gd_buffer_config(b, threads, share);
+    if (s != GD_OK) return fail(s);
     *out = b;
     return GD_OK;
 }
@@ -683,27 +753,99 @@ gd_status gd_buffer_destroy(gd_buffer* b) {
     return GD_OK;
 }
 
+gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_config: bad handle");
+    if (host_threads < 0 || host_threads > 256 || zero_copy_share > 1.0)
+        return set_error(GD_ERR_INVALID, "gd_buffer_config: host_threads in [0, 256], zero_copy_share <= 1");
+    DeviceGuard guard(b->hdr.device);
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+        if (s) GD_CUDA(cudaStreamSynchronize(s));
+    if (host_threads > 0 && !b->stage_mem) {
+        const int D = b->D;
+        const int64_t nm = b->n_max;
+        GD_CUDA(cudaHostAlloc((void**)&b->stage_mem, (size_t)D * nm * b->R, cudaHostAllocMapped | cudaHostAllocPortable));
+        GD_CUDA(cudaHostAlloc((void**)&b->hnodes_mem, (size_t)D * nm * sizeof(int32_t), cudaHostAllocMapped | cudaHostAllocPortable));
+        GD_CUDA(cudaHostAlloc((void**)&b->hmeta_mem, (size_t)D * 4 * sizeof(int64_t), cudaHostAllocMapped | cudaHostAllocPortable));
+        std::memset(b->hmeta_mem, 0, (size_t)D * 4 * sizeof(int64_t));
+        b->stg.assign(D, StagedSlot());
+        for (int d = 0; d < D; ++d) {
+            b->stg[d].owner = b;
+            b->stg[d].d = d;
+            b->stg[d].staging = b->stage_mem + (size_t)d * nm * b->R;
+            b->stg[d].h_nodes = b->hnodes_mem + (size_t)d * nm;
+            b->stg[d].h_meta = b->hmeta_mem + 4 * d;
+        }
+    }
+    if (b->pool && (host_threads == 0 || b->pool->threads() != host_threads)) {
+        delete b->pool;
+        b->pool = nullptr;
+    }
+    if (host_threads > 0 && !b->pool) b->pool = new HostGatherPool(host_threads);
+    b->host_threads = host_threads;
+    b->alpha_fixed = zero_copy_share >= 0;
+    b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.5);
+    return GD_OK;
+}
+
 gd_status gd_buffer_timing(gd_buffer* b, int enable) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing: bad handle");
     DeviceGuard guard(b->hdr.device);
-    if (enable) b->timer.reset();
+    if (enable) {
+        for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j}) GD_CUDA(cudaStreamSynchronize(s));
+        b->timer.reset();
+        b->timer_host_ms = 0;
+    }
     b->timer.on = enable != 0;
     return GD_OK;
 }
 
-gd_status gd_buffer_timing_read(gd_buffer* b, double* bookkeeping_ms, double* gather_ms, double* miss_ms,
-                                int64_t* batches) {
+gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing_read: bad handle");
     DeviceGuard guard(b->hdr.device);
-    if (bookkeeping_ms) *bookkeeping_ms = b->timer.total_ms(3, 0);
-    if (gather_ms) *gather_ms = b->timer.total_ms(3, 1);
-    if (miss_ms) *miss_ms = b->timer.total_ms(3, 2);
-    if (batches) *batches = (int64_t)b->timer.pairs.size() / 3;
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j}) GD_CUDA(cudaStreamSynchronize(s));
+    if (ms) {
+        for (int k = 0; k < 4; ++k) ms[k] = b->timer.total_ms(4, k);
+        ms[4] = b->timer_host_ms;
+        ms[5] = b->alpha;
+    }
+    if (batches) *batches = (int64_t)b->timer.pairs.size() / 4;
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
 
 void* gd_buffer_side_stream(gd_buffer* b) { return (b && b->hdr.magic == kMagicBuffer) ? (void*)b->side : nullptr; }
+
+// Phase 1 of the staged share, run by the CUDA callback thread of stream H once the
+// pop kernel has written the node list and counts to mapped host memory.
+static void CUDART_CB host_gather_cb(void* arg) {
+    StagedSlot* ss = (StagedSlot*)arg;
+    gd_buffer* b = ss->owner;
+    const int64_t n = ((volatile int64_t*)ss->h_meta)[2];
+    ss->cpu_ms = b->pool->gather((const uint8_t*)b->host_feat, ss->h_nodes, n, b->R, ss->staging);
+    if (b->timer.on) b->timer_host_ms += ss->cpu_ms;   // serialised on stream H
+}
+
+// Zero-copy share alpha from the measured rates of a finished batch: the zero-copy
+// path is bounded by the host's random-translation rate, the staged path by
+// max(host gather, contiguous pull); split the misses so both finish together.
+static void adapt_alpha(gd_buffer* b, int d) {
+    StagedSlot& ss = b->stg[d];
+    if (b->alpha_fixed || ss.batch < 0) return;
+    if (cudaEventQuery(b->ev_z1[d]) != cudaSuccess || cudaEventQuery(b->ev_p1[d]) != cudaSuccess) {
+        cudaGetLastError();
+        return;
+    }
+    const double M = (double)ss.h_meta[0], K0 = (double)ss.h_meta[1];
+    float tz = 0, tp = 0;
+    cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]);
+    cudaEventElapsedTime(&tp, b->ev_p0[d], b->ev_p1[d]);
+    cudaGetLastError();
+    if (M < 4096 || K0 < 256 || M - K0 < 256 || tz <= 0) return;
+    const double rz = K0 / tz;
+    const double rs = (M - K0) / std::max<double>(std::max<double>(tp, ss.cpu_ms), 1e-3);
+    const double target = rz / (rz + rs);
+    b->alpha = std::min(0.95, std::max(0.05, 0.7 * b->alpha + 0.3 * target));
+}
 
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max, void* out,
                      int32_t* alias, int64_t* stats, void* stream_v, void* done_v) {
@@ -720,9 +862,18 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     const int d = (int)(b->batch_counter % b->D);
     int4* trip = b->trip + (int64_t)d * b->n_max;
     int64_t* tcount = b->trip_count + d;
+    int64_t* tsplit = b->trip_split + d;
     const int64_t lt = std::max<int64_t>(1, cdiv(n_max, kBTile));
+    const bool staged = b->host_threads > 0;
+    StagedSlot* ss = staged ? &b->stg[d] : nullptr;
 
-    GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));   // side stream done with trip slot d
+    // every stream is done with trip / host-list slot d (batch - D)
+    GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));
+    if (staged) {
+        adapt_alpha(b, (int)((b->batch_counter + b->D - 2) % b->D));
+        ss->batch = b->batch_counter;
+    }
+    const uint32_t alpha_q16 = staged ? (uint32_t)std::lround(b->alpha * 65536.0) : 65536u;
     const bool timed = b->timer.on;
     const int t_book = timed ? b->timer.begin(st) : -1;
 
@@ -758,6 +909,15 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.alias = al;
     pa.trip = trip;
     pa.trip_count = tcount;
+    pa.trip_split = tsplit;
+    pa.alpha_q16 = alpha_q16;
+    pa.h_nodes = nullptr;
+    pa.h_meta = nullptr;
+    if (staged) {
+        GD_CUDA(cudaHostGetDevicePointer((void**)&pa.h_nodes, ss->h_nodes, 0));
+        GD_CUDA(cudaHostGetDevicePointer((void**)&pa.h_meta, ss->h_meta, 0));
+    }
+    pa.stats = stats;
     pa.ticket = b->tickets;
     pa.done_word = b->done_word;
     pa.epoch = ++b->epoch;
@@ -772,8 +932,10 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (timed) b->timer.end(t_book, st);
     GD_CUDA(cudaEventRecord(b->ev_L, st));
 
-    // hits: their rows were written by earlier miss streams, all ordered before X_{b-1}
+    // a8: hits.  Their rows were written by earlier miss copies, all ordered before the
+    // previous batch's X events (each miss stream is in order).
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_X, 0));
+    GD_CUDA(cudaStreamWaitEvent(st, b->ev_Xs, 0));
     const int t_gat = timed ? b->timer.begin(st) : -1;
     if (b->R % 16 == 0)
         k_gather_hits<4><<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
@@ -783,19 +945,50 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (timed) b->timer.end(t_gat, st);
     GD_CUDA(cudaEventRecord(b->ev_G, st));
 
-    // misses: pinned host -> slot + out on the side stream (asynchronous extraction)
+    // a7, zero-copy share: misses [0, K0) straight from the pinned host table (stream Z)
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
-    const int t_miss = timed ? b->timer.begin(b->side) : -1;
+    const int t_zc = timed ? b->timer.begin(b->side) : -1;
+    GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
     if (b->R % 16 == 0)
-        k_miss_copy<4><<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy<4, false><<<148 * 2, 256, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     else
-        k_miss_copy_w4<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy_w4<false><<<148 * 2, 256, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     GD_DEBUG_AFTER("k_miss_copy", b->side);
-    if (timed) b->timer.end(t_miss, b->side);
+    GD_CUDA(cudaEventRecord(b->ev_z1[d], b->side));
+    if (timed) b->timer.end(t_zc, b->side);
     GD_CUDA(cudaEventRecord(b->ev_X, b->side));
-    GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side));
-    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
-    if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side));
+
+    // a7, staged share: misses [K0, M).  Phase 1 on stream H (host gather into pinned
+    // staging slot d), phase 2 on stream P (contiguous pull into slots + out).
+    if (staged) {
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
+        GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
+        GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));
+        GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_E[d], 0));
+        const uint8_t* stage_dev = nullptr;
+        GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
+        const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
+        GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
+        if (b->R % 16 == 0)
+            k_miss_copy<4, true><<<148 * 2, 256, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+        else
+            k_miss_copy_w4<true><<<148 * 2, 256, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+        GD_DEBUG_AFTER("k_stage_copy", b->side_p);
+        GD_CUDA(cudaEventRecord(b->ev_p1[d], b->side_p));
+        if (timed) b->timer.end(t_pl, b->side_p);
+        GD_CUDA(cudaEventRecord(b->ev_P[d], b->side_p));
+        GD_CUDA(cudaEventRecord(b->ev_Xs, b->side_p));
+    } else if (timed) {
+        b->timer.end(b->timer.begin(b->side), b->side);   // keep 4 timing pairs per batch
+    }
+
+    // join: out complete, trip slot d free
+    GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_X, 0));
+    if (staged) GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_Xs, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_G, 0));
+    GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side_j));
+    if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side_j));
     GD_CUDA(cudaGetLastError());
     b->inflight++;
     b->batch_counter++;

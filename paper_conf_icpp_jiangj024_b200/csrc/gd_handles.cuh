@@ -7,6 +7,7 @@
 #include <vector>
 
 #include "gd_common.cuh"
+#include "gd_hostpool.h"
 
 // Topology replica + per-call sampling workspace.
 struct gd_graph {
@@ -31,6 +32,19 @@ struct GdCtl {
     long long head;       // first ring position that may hold a live entry
     long long tail;       // next free ring position
     long long base;       // start of the current half (0 or C)
+};
+
+struct gd_buffer;
+
+// One slot of the staged miss path (phase 1 host gather -> phase 2 contiguous pull).
+struct StagedSlot {
+    gd_buffer* owner = nullptr;
+    int d = 0;
+    int32_t* h_nodes = nullptr;   // pinned, mapped [n_max]: node ids of the staged share
+    int64_t* h_meta = nullptr;    // pinned, mapped [4]: M, K0, staged rows, 0
+    uint8_t* staging = nullptr;   // pinned, mapped [n_max x R]
+    double cpu_ms = 0;            // duration of the last host gather into this slot
+    int64_t batch = -1;           // batch that last used this slot
 };
 
 // Feature buffer + extraction workspace.
@@ -63,10 +77,25 @@ struct gd_buffer {
     unsigned long long* tickets = nullptr;   // [4] {ticket, finished} x 2 kernels
     unsigned long long* done_word = nullptr; // [1] epoch-tagged early-exit word of the pop scan
     gd::ScanState scan;
-    cudaStream_t side = nullptr;
-    cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_G = nullptr;
-    std::vector<cudaEvent_t> ev_trip;    // [D] side stream finished with trip ring slot
-    gd::EventTimer timer;                // 3 pairs per gd_extract: bookkeeping, gather, miss
+    cudaStream_t side = nullptr;         // Z: zero-copy share of the misses
+    cudaStream_t side_h = nullptr;       // H: host gather (phase 1) of the staged share
+    cudaStream_t side_p = nullptr;       // P: contiguous pull (phase 2) of the staged share
+    cudaStream_t side_j = nullptr;       // J: joins Z, P and the hit gather into `done`
+    cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_Xs = nullptr, ev_G = nullptr;
+    std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
+    std::vector<cudaEvent_t> ev_E, ev_P; // [D] host gather / staged pull of slot d done
+    std::vector<cudaEvent_t> ev_z0, ev_z1, ev_p0, ev_p1;   // [D] timing of the two miss paths
+    int64_t* trip_split = nullptr;       // [D] K0: misses [0, K0) zero-copy, [K0, M) staged
+    int host_threads = 0;                // 0: staged path off (all misses zero-copy)
+    double alpha = 1.0;                  // zero-copy share of the misses (adapted)
+    bool alpha_fixed = false;
+    gd::HostGatherPool* pool = nullptr;
+    std::vector<StagedSlot> stg;
+    uint8_t* stage_mem = nullptr;        // pinned allocations behind stg
+    int32_t* hnodes_mem = nullptr;
+    int64_t* hmeta_mem = nullptr;
+    gd::EventTimer timer;                // 4 pairs per gd_extract: bookkeeping, gather, zero-copy, pull
+    double timer_host_ms = 0;            // host gather time while timing is on
     int64_t batch_counter = 0;
     int64_t inflight = 0;
     unsigned long long epoch = 1;

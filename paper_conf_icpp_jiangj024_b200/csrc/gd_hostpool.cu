@@ -1,0 +1,105 @@
+// gd_hostpool.cu — host worker pool for phase 1 of the staged miss path (host code only).
+//
+// GNNDrive's extractor loads missed rows from storage into a host staging buffer before
+// the GPU transfer ("two-phase extraction").  Here the storage stand-in is
+// the pinned host table, and phase 1 is a multi-threaded CPU gather of the missed rows
+// into a contiguous pinned staging slot, run from a CUDA host function on the library's
+// host-gather stream; phase 2 (k_stage_copy) pulls the slot over the host link with
+// contiguous, translation-friendly reads.
+#include <atomic>
+#include <chrono>
+#include <condition_variable>
+#include <cstring>
+#include <functional>
+#include <mutex>
+#include <thread>
+#include <vector>
+
+#include "gd_hostpool.h"
+
+namespace gd {
+
+struct HostGatherPool::Impl {
+    std::vector<std::thread> workers;
+    std::mutex mu;
+    std::condition_variable cv_work, cv_done;
+    uint64_t generation = 0;
+    int active = 0;
+    bool stop = false;
+    // current job
+    const uint8_t* src = nullptr;
+    const int32_t* rows = nullptr;
+    uint8_t* dst = nullptr;
+    int64_t n = 0, R = 0;
+    std::atomic<int64_t> next{0};
+    static constexpr int64_t kChunk = 512;
+
+    void work() {
+        while (true) {
+            const int64_t lo = next.fetch_add(kChunk, std::memory_order_relaxed);
+            if (lo >= n) break;
+            const int64_t hi = lo + kChunk < n ? lo + kChunk : n;
+            for (int64_t j = lo; j < hi; ++j)
+                std::memcpy(dst + j * R, src + (int64_t)rows[j] * R, (size_t)R);
+        }
+    }
+
+    void loop() {
+        uint64_t seen = 0;
+        while (true) {
+            {
+                std::unique_lock<std::mutex> lk(mu);
+                cv_work.wait(lk, [&] { return stop || generation != seen; });
+                if (stop) return;
+                seen = generation;
+            }
+            work();
+            {
+                std::lock_guard<std::mutex> lk(mu);
+                if (--active == 0) cv_done.notify_one();
+            }
+        }
+    }
+};
+
+HostGatherPool::HostGatherPool(int threads) : impl_(new Impl) {
+    // the calling (CUDA callback) thread works too, so spawn threads-1 helpers
+    for (int t = 1; t < threads; ++t) impl_->workers.emplace_back([this] { impl_->loop(); });
+}
+
+HostGatherPool::~HostGatherPool() {
+    {
+        std::lock_guard<std::mutex> lk(impl_->mu);
+        impl_->stop = true;
+    }
+    impl_->cv_work.notify_all();
+    for (auto& w : impl_->workers) w.join();
+    delete impl_;
+}
+
+int HostGatherPool::threads() const { return (int)impl_->workers.size() + 1; }
+
+double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst) {
+    const auto t0 = std::chrono::steady_clock::now();
+    if (n > 0) {
+        Impl& I = *impl_;
+        {
+            std::lock_guard<std::mutex> lk(I.mu);
+            I.src = src;
+            I.rows = rows;
+            I.dst = dst;
+            I.n = n;
+            I.R = R;
+            I.next.store(0, std::memory_order_relaxed);
+            I.active = (int)I.workers.size();
+            ++I.generation;
+        }
+        I.cv_work.notify_all();
+        I.work();
+        std::unique_lock<std::mutex> lk(I.mu);
+        I.cv_done.wait(lk, [&] { return I.active == 0; });
+    }
+    return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+}
+
+}  // namespace gd

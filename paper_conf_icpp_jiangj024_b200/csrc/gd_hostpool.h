@@ -1,0 +1,21 @@
+// gd_hostpool.h — host worker pool for the staged miss path (see gd_hostpool.cu).
+#pragma once
+
+#include <stdint.h>
+
+namespace gd {
+
+class HostGatherPool {
+   public:
+    explicit HostGatherPool(int threads);
+    ~HostGatherPool();
+    int threads() const;
+    // dst[j*R : (j+1)*R] = src[rows[j]*R : ...] for j < n, on all threads; returns elapsed ms.
+    double gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst);
+
+   private:
+    struct Impl;
+    Impl* impl_;
+};
+
+}  // namespace gd
