@@ -239,10 +239,11 @@ def run_ours(args, rank, world, local_rank):
     seeds_host = seeds_dev.cpu().pin_memory()
     batch_ids = [ep * wl.num_batches + b for b, ep in sched]
 
-    outs = [g.alloc_out(cfg.batch_size, fan) for _ in range(Q + 1)]
-    feats = [buf.alloc_out(n_max) for _ in range(Q)]
-    aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(Q)]
-    dones = [torch.cuda.Event() for _ in range(Q)]
+    RING = Q + 1   # per-batch buffers in flight: Q unreleased batches + the one being sampled
+    outs = [g.alloc_out(cfg.batch_size, fan) for _ in range(RING)]
+    feats = [buf.alloc_out(n_max) for _ in range(RING)]
+    aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(RING)]
+    dones = [torch.cuda.Event() for _ in range(RING)]
     for e in dones:
         e.record(torch.cuda.current_stream(dev))     # create the events (torch creates lazily)
     stats = torch.zeros((total, 4), dtype=torch.int64, device=dev)
@@ -258,11 +259,12 @@ def run_ours(args, rank, world, local_rank):
             log(f"  step {j}: {what} ok")
 
     def step(j, host_inputs=False, host_out=None):
-        o = outs[j % (Q + 1)]
+        s = j % RING
+        o = outs[s]
+        main.wait_event(dones[s])          # batch j - RING is complete: its buffers are free
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
         g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
         dsync("sample", j)
-        s = j % Q
         buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, out=feats[s], alias=aliases[s], stats=stats[j],
                     stream=main, done=dones[s])
         dsync("extract", j)
@@ -304,7 +306,7 @@ def run_ours(args, rank, world, local_rank):
         ev0.record(main)
         for j in range(W, W + K):
             step(j)
-        main.wait_event(dones[(W + K - 1) % Q])     # the last batch's misses are in `out`
+        main.wait_event(dones[(W + K - 1) % RING])  # the last batch's rows are all in `out`
         ev1.record(main)
         ev1.synchronize()
     torch.cuda.synchronize(dev)
@@ -332,7 +334,7 @@ def run_ours(args, rank, world, local_rank):
         e0.record(main)
         for j in range(W + K, W + 2 * K):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats))
-        main.wait_event(dones[(W + 2 * K - 1) % Q])
+        main.wait_event(dones[(W + 2 * K - 1) % RING])
         e1.record(main)
         e1.synchronize()
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)

@@ -165,7 +165,8 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  *             misses copied through the staged path} of this batch.
  *   done      cudaEvent_t (void*) or NULL: recorded when `out` is complete.
  *             `out` is valid only after `done`; `stream` itself does NOT wait
- *             for the misses.  node_ids must stay unmodified until `done`.
+ *             for the misses or the hit gather.  node_ids, *n_dev and alias
+ *             must stay unmodified until `done`.
  * GD_ERR_CAPACITY if this would exceed max_inflight unreleased batches.
  * ------------------------------------------------------------------------- */
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,

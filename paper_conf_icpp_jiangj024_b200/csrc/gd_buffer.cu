@@ -3,7 +3,7 @@
 // gd_extract(b), all stream-ordered, no host sync:
 //   caller stream:  k_lookup (Alg. 1 loop 1 + miss ranks) -> k_pop_assign (loop 2:
 //                   LRU standby slots, eviction, map/reverse/alias) -> [L_b]
-//                   -> wait X_{b-1} -> k_gather_hits (slots -> out) -> [G_b]
+//   stream G:       wait L_b, X_{b-1}, Xs_{b-1} -> k_gather_hits (slots -> out) -> [G_b]
 //   stream Z:       wait L_b -> k_miss_copy<zero-copy> misses [0, K0) -> [X_b]
 //   stream H:       wait L_b -> host gather (thread pool) of misses [K0, M) -> [E_b]
 //   stream P:       wait E_b -> k_miss_copy<staged> pull of the staging slot -> [Xs_b]
@@ -598,7 +598,7 @@ static void buffer_free(gd_buffer* b) {
     if (!b) return;
     DeviceGuard guard(b->hdr.device);
     if (b->side) cudaStreamSynchronize(b->side);
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) cudaStreamSynchronize(s);
     void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->missflag,
                     b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
@@ -615,7 +615,7 @@ static void buffer_free(gd_buffer* b) {
             if (e) cudaEventDestroy(e);
     for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G})
         if (e) cudaEventDestroy(e);
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) cudaStreamDestroy(s);
     if (b->registered) cudaHostUnregister((void*)b->host_feat);
     b->hdr.magic = 0;
@@ -688,8 +688,8 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     GD_ALLOC(b->ring, 2 * C * sizeof(int32_t));
     GD_ALLOC(b->ctl, 2 * sizeof(GdCtl));
     GD_ALLOC(b->misslist, nm * sizeof(int32_t));
-    GD_ALLOC(b->missflag, nm);
-    GD_ALLOC(b->alias_ws, nm * sizeof(int32_t));
+    GD_ALLOC(b->missflag, (int64_t)b->D * nm);
+    GD_ALLOC(b->alias_ws, (int64_t)b->D * nm * sizeof(int32_t));
     GD_ALLOC(b->mcount, sizeof(int64_t));
     GD_ALLOC(b->trip, (int64_t)b->D * nm * sizeof(int4));
     GD_ALLOC(b->trip_count, b->D * sizeof(int64_t));
@@ -721,7 +721,7 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: init kernels"));
     }
-    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j})
+    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_g})
         if (cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
     for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G})
@@ -758,7 +758,7 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     if (host_threads < 0 || host_threads > 256 || zero_copy_share > 1.0)
         return set_error(GD_ERR_INVALID, "gd_buffer_config: host_threads in [0, 256], zero_copy_share <= 1");
     DeviceGuard guard(b->hdr.device);
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) GD_CUDA(cudaStreamSynchronize(s));
     if (host_threads > 0 && !b->stage_mem) {
         const int D = b->D;
@@ -791,7 +791,7 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing: bad handle");
     DeviceGuard guard(b->hdr.device);
     if (enable) {
-        for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j}) GD_CUDA(cudaStreamSynchronize(s));
+        for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g}) GD_CUDA(cudaStreamSynchronize(s));
         b->timer.reset();
         b->timer_host_ms = 0;
     }
@@ -802,7 +802,7 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable) {
 gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing_read: bad handle");
     DeviceGuard guard(b->hdr.device);
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j}) GD_CUDA(cudaStreamSynchronize(s));
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g}) GD_CUDA(cudaStreamSynchronize(s));
     if (ms) {
         for (int k = 0; k < 4; ++k) ms[k] = b->timer.total_ms(4, k);
         ms[4] = b->timer_host_ms;
@@ -858,8 +858,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (((uintptr_t)out & 15) && (b->R % 16 == 0)) return set_error(GD_ERR_INVALID, "gd_extract: out must be 16-byte aligned");
     DeviceGuard guard(b->hdr.device);
     cudaStream_t st = (cudaStream_t)stream_v;
-    int32_t* al = alias ? alias : b->alias_ws;
     const int d = (int)(b->batch_counter % b->D);
+    int32_t* al = alias ? alias : b->alias_ws + (int64_t)d * b->n_max;
+    uint8_t* mflag = b->missflag + (int64_t)d * b->n_max;
     int4* trip = b->trip + (int64_t)d * b->n_max;
     int64_t* tcount = b->trip_count + d;
     int64_t* tsplit = b->trip_split + d;
@@ -884,7 +885,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     la.map = b->map;
     la.pos_of_slot = b->pos_of_slot;
     la.alias = al;
-    la.missflag = b->missflag;
+    la.missflag = mflag;
     la.misslist = b->misslist;
     la.mcount = b->mcount;
     la.stats = stats;
@@ -932,21 +933,32 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (timed) b->timer.end(t_book, st);
     GD_CUDA(cudaEventRecord(b->ev_L, st));
 
-    // a8: hits.  Their rows were written by earlier miss copies, all ordered before the
-    // previous batch's X events (each miss stream is in order).
-    GD_CUDA(cudaStreamWaitEvent(st, b->ev_X, 0));
-    GD_CUDA(cudaStreamWaitEvent(st, b->ev_Xs, 0));
-    const int t_gat = timed ? b->timer.begin(st) : -1;
+    // Stream order (the host enqueue order below matters: each wait captures the event's
+    // latest record):  G(b) waits X/Xs of b-1 (hits may sit in slots the previous
+    // batch's misses are still filling); Z(b)/P(b) wait G(b-1) (their slots were freed
+    // by releases of batches whose gathers are <= b-1, so no live gather reads them).
+    GD_CUDA(cudaStreamWaitEvent(b->side_g, b->ev_L, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side_g, b->ev_X, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side_g, b->ev_Xs, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
+    if (staged) {
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
+        GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_G, 0));
+    }
+
+    // a8: hits, slots -> out (stream G)
+    const int t_gat = timed ? b->timer.begin(b->side_g) : -1;
     if (b->R % 16 == 0)
-        k_gather_hits<4><<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
+        k_gather_hits<4><<<148 * 8, 256, 0, b->side_g>>>(al, mflag, n_dev, b->slots, (uint8_t*)out, b->R);
     else
-        k_gather_hits_w4<<<148 * 8, 256, 0, st>>>(al, b->missflag, n_dev, b->slots, (uint8_t*)out, b->R);
-    GD_DEBUG_AFTER("k_gather_hits", st);
-    if (timed) b->timer.end(t_gat, st);
-    GD_CUDA(cudaEventRecord(b->ev_G, st));
+        k_gather_hits_w4<<<148 * 8, 256, 0, b->side_g>>>(al, mflag, n_dev, b->slots, (uint8_t*)out, b->R);
+    GD_DEBUG_AFTER("k_gather_hits", b->side_g);
+    if (timed) b->timer.end(t_gat, b->side_g);
+    GD_CUDA(cudaEventRecord(b->ev_G, b->side_g));
 
     // a7, zero-copy share: misses [0, K0) straight from the pinned host table (stream Z)
-    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
     const int t_zc = timed ? b->timer.begin(b->side) : -1;
     GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
     if (b->R % 16 == 0)
@@ -961,8 +973,6 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // a7, staged share: misses [K0, M).  Phase 1 on stream H (host gather into pinned
     // staging slot d), phase 2 on stream P (contiguous pull into slots + out).
     if (staged) {
-        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
-        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
         GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
         GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));
         GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_E[d], 0));

@@ -67,8 +67,8 @@ struct gd_buffer {
     int ctl_parity = 0;
     // per-batch workspace used on the caller's stream
     int32_t* misslist = nullptr;         // [n_max] batch positions of misses, list order
-    uint8_t* missflag = nullptr;         // [n_max]
-    int32_t* alias_ws = nullptr;         // [n_max] used when the caller passes alias = NULL
+    uint8_t* missflag = nullptr;         // [D][n_max] (read by the gather on stream G)
+    int32_t* alias_ws = nullptr;         // [D][n_max] used when the caller passes alias = NULL
     int64_t* mcount = nullptr;           // [1] misses of the current batch
     // miss triples for the side stream, a ring of D batches
     int D = 0;
@@ -81,6 +81,7 @@ struct gd_buffer {
     cudaStream_t side_h = nullptr;       // H: host gather (phase 1) of the staged share
     cudaStream_t side_p = nullptr;       // P: contiguous pull (phase 2) of the staged share
     cudaStream_t side_j = nullptr;       // J: joins Z, P and the hit gather into `done`
+    cudaStream_t side_g = nullptr;       // G: hit gather (slots -> out)
     cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_Xs = nullptr, ev_G = nullptr;
     std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
     std::vector<cudaEvent_t> ev_E, ev_P; // [D] host gather / staged pull of slot d done
