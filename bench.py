@@ -48,6 +48,8 @@ def parse():
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
+    p.add_argument("--miss-sweep", default="", help="tuning: 'threads:share:zc_blocks:pull_blocks,...' timed "
+                   "one after another in this process (results under 'sweep')")
     return p.parse_args()
 
 
@@ -233,7 +235,8 @@ def run_ours(args, rank, world, local_rank):
     log(f"setup: graph {wl.t_graph:.1f}s table alloc {wl.t_table_alloc:.1f}s register {t_register:.1f}s "
         f"fill {wl.t_fill:.1f}s; N={cfg.num_nodes} E={cfg.num_edges} S={S} n_max={n_max} deg={wl.deg_stats}")
 
-    total = W + K + (0 if args.no_e2e else K)
+    sweep_cfgs = [tuple(float(x) for x in c.split(":")) for c in args.miss_sweep.split(",") if c]
+    total = W + K + (0 if args.no_e2e else K) + len(sweep_cfgs) * (W + K)
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -341,6 +344,36 @@ def run_ours(args, rank, world, local_rank):
         e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s",
                "h2d_bytes_per_step": cfg.batch_size * 4,
                "d2h_bytes_per_step": (2 * len(fan) + 1) * 8 + 32}
+    # ---- optional in-process sweep of the miss-stream configuration (tuning only)
+    sweep = []
+    j0 = W + K + (0 if args.no_e2e else K)
+    for (thr, share, zcb, plb) in sweep_cfgs:
+        torch.cuda.synchronize(dev)
+        buf.config(int(thr), share, int(zcb), int(plb))
+        for j in range(j0, j0 + W):
+            step(j)
+        torch.cuda.synchronize(dev)
+        buf.timing(True)
+        a = torch.cuda.Event(enable_timing=True)
+        z = torch.cuda.Event(enable_timing=True)
+        a.record(main)
+        for j in range(j0 + W, j0 + W + K):
+            step(j)
+        main.wait_event(dones[(j0 + W + K - 1) % RING])
+        z.record(main)
+        z.synchronize()
+        buf.timing(False)
+        t = buf.timing_read()
+        sst = stats[j0 + W:j0 + W + K].sum(0).cpu().tolist()
+        el = a.elapsed_time(z)
+        rec = {"host_threads": int(thr), "share": share, "zc_blocks": int(zcb), "pull_blocks": int(plb),
+               "batches_per_s": round(K / (el / 1e3), 1),
+               "link_GBps": round(cfg.row_bytes * sst[1] / (el / 1e3) / 1e9, 2),
+               "ms": {k: round(v / max(1, t["batches"]), 3) for k, v in t.items() if k.endswith("_ms")},
+               "zero_copy_share_final": round(t["zero_copy_share"], 3)}
+        log("sweep", rec)
+        sweep.append(rec)
+        j0 += W + K
     status_g = g.check()
     status_b = buf.check()
 
@@ -413,6 +446,7 @@ def run_ours(args, rank, world, local_rank):
                       "hits": hits / K, "misses": misses / K,
                       "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
         "parity": parity,
+        "sweep": sweep or None,
         "device_status": {"graph": status_g, "buffer": status_b},
         "setup_s": round(time.time() - t_setup, 1),
     }

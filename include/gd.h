@@ -181,11 +181,17 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  * slot contiguously over the host link.  K0 = floor(M * zero_copy_share).
  *   host_threads     0 disables the staged path (all misses zero-copy).
  *   zero_copy_share  in [0, 1]; < 0 = adaptive (balance the two paths' measured rates).
- * Default at init: host_threads = min(8, cores/2) (0 with preload), adaptive share;
- * env GD_HOST_THREADS / GD_ZERO_COPY_SHARE override.  Synchronises the buffer's
+ *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
+ *                    copy kernels; <= 0 keeps the current value (defaults 24 and 8).
+ *                    Few whole-SM blocks keep long-latency host loads off the SMs
+ *                    that run sampling / bookkeeping / the hit gather.
+ * Default at init: host_threads = min(12, 3/4 of the cores) (0 with preload),
+ * adaptive share; env GD_HOST_THREADS / GD_ZERO_COPY_SHARE / GD_ZC_BLOCKS /
+ * GD_PULL_BLOCKS override.  Synchronises the buffer's
  * internal streams; call between batches.
  * ------------------------------------------------------------------------- */
-gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share);
+gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share, int zc_blocks,
+                           int pull_blocks);
 
 /* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a

@@ -239,9 +239,10 @@ class FeatureBuffer:
         return {"bookkeeping_ms": ms[0], "gather_ms": ms[1], "miss_zero_copy_ms": ms[2], "miss_staged_ms": ms[3],
                 "host_gather_ms": ms[4], "zero_copy_share": ms[5], "batches": n.value}
 
-    def config(self, host_threads: int, zero_copy_share: float = -1.0):
-        """gd_buffer_config: staged miss path width and zero-copy share (< 0: adaptive)."""
-        check(lib.gd_buffer_config(self._h, int(host_threads), float(zero_copy_share)))
+    def config(self, host_threads: int, zero_copy_share: float = -1.0, zc_blocks: int = 0, pull_blocks: int = 0):
+        """gd_buffer_config: staged miss path width, zero-copy share (< 0: adaptive), copy grids."""
+        check(lib.gd_buffer_config(self._h, int(host_threads), float(zero_copy_share), int(zc_blocks),
+                                   int(pull_blocks)))
 
 
 def check_device_status(handle) -> int:

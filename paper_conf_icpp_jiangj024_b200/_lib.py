@@ -69,7 +69,7 @@ def _load():
     _dp = ctypes.POINTER(ctypes.c_double)
     L.gd_buffer_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_buffer_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
-    L.gd_buffer_config.argtypes = [_vp, ctypes.c_int, ctypes.c_double]
+    L.gd_buffer_config.argtypes = [_vp, ctypes.c_int, ctypes.c_double, ctypes.c_int, ctypes.c_int]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:

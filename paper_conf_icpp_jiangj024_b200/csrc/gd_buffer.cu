@@ -319,7 +319,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
 // (the contiguous phase-2 pull of rows the host gathered in phase 1).
 // One 16-byte chunk per thread-iteration, UNROLL chunks in flight per thread.
 template <int UNROLL, bool STAGED>
-__global__ void __launch_bounds__(256) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
+__global__ void __launch_bounds__(1024, 1) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
                                                    const int64_t* __restrict__ end, const uint8_t* __restrict__ src,
                                                    uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
     const int64_t k0 = begin ? *begin : 0;
@@ -736,11 +736,14 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     }
     // staged miss path (phase 1 host gather + phase 2 contiguous pull): on by default
     // unless every row is resident from the start; GD_HOST_THREADS overrides the width.
-    int threads = preload ? 0 : (int)std::min(8u, std::max(1u, std::thread::hardware_concurrency() / 2));
+    int threads = preload ? 0 : (int)std::min(12u, std::max(1u, std::thread::hardware_concurrency() * 3 / 4));
     if (const char* e = std::getenv("GD_HOST_THREADS")) threads = std::max(0, std::atoi(e));
     double share = -1.0;
     if (const char* e = std::getenv("GD_ZERO_COPY_SHARE")) share = std::atof(e);
-    s = gd_buffer_config(b, threads, share);
+    int zcb = 0, plb = 0;
+    if (const char* e = std::getenv("GD_ZC_BLOCKS")) zcb = std::atoi(e);
+    if (const char* e = std::getenv("GD_PULL_BLOCKS")) plb = std::atoi(e);
+    s = gd_buffer_config(b, threads, share, zcb, plb);
     if (s != GD_OK) return fail(s);
     *out = b;
     return GD_OK;
@@ -753,10 +756,12 @@ gd_status gd_buffer_destroy(gd_buffer* b) {
     return GD_OK;
 }
 
-gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share) {
+gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share, int zc_blocks, int pull_blocks) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_config: bad handle");
-    if (host_threads < 0 || host_threads > 256 || zero_copy_share > 1.0)
-        return set_error(GD_ERR_INVALID, "gd_buffer_config: host_threads in [0, 256], zero_copy_share <= 1");
+    if (host_threads < 0 || host_threads > 256 || zero_copy_share > 1.0 || zc_blocks > 4096 || pull_blocks > 4096)
+        return set_error(GD_ERR_INVALID, "gd_buffer_config: host_threads in [0, 256], zero_copy_share <= 1, blocks <= 4096");
+    if (zc_blocks > 0) b->zc_blocks = zc_blocks;
+    if (pull_blocks > 0) b->pull_blocks = pull_blocks;
     DeviceGuard guard(b->hdr.device);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) GD_CUDA(cudaStreamSynchronize(s));
@@ -962,9 +967,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     const int t_zc = timed ? b->timer.begin(b->side) : -1;
     GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
     if (b->R % 16 == 0)
-        k_miss_copy<4, false><<<148 * 2, 256, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     else
-        k_miss_copy_w4<false><<<148 * 2, 256, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     GD_DEBUG_AFTER("k_miss_copy", b->side);
     GD_CUDA(cudaEventRecord(b->ev_z1[d], b->side));
     if (timed) b->timer.end(t_zc, b->side);
@@ -981,9 +986,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
         GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
         if (b->R % 16 == 0)
-            k_miss_copy<4, true><<<148 * 2, 256, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+            k_miss_copy<4, true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
         else
-            k_miss_copy_w4<true><<<148 * 2, 256, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+            k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
         GD_DEBUG_AFTER("k_stage_copy", b->side_p);
         GD_CUDA(cudaEventRecord(b->ev_p1[d], b->side_p));
         if (timed) b->timer.end(t_pl, b->side_p);

@@ -252,6 +252,17 @@ int main(int argc, char** argv) {
         int32_t* d_seq;
         CK(cudaMalloc(&d_seq, n * 4));
         CK(cudaMemcpy(d_seq, seq.data(), n * 4, cudaMemcpyHostToDevice));
+        if (getenv("ZC_SMS")) {   // few whole-SM blocks (1024 threads)
+            for (int G : {2, 4, 8, 12, 16, 24, 32, 48}) {
+                float a1 = timeit([&] { k_flat<0, 4><<<G, 1024>>>(d_rows, n, src, d_dst, R); });
+                float a2 = timeit([&] { k_flat<0, 8><<<G, 1024>>>(d_rows, n, src, d_dst, R); });
+                float c1 = timeit([&] { k_flat<0, 4><<<G, 1024>>>(d_seq, n, src, d_dst, R); });
+                float c2 = timeit([&] { k_flat<0, 8><<<G, 1024>>>(d_seq, n, src, d_dst, R); });
+                printf("SMs=%2d x1024thr: random u4 %.1f u8 %.1f | contiguous u4 %.1f u8 %.1f GB/s\n", G, mb / a1 / 1e6,
+                       mb / a2 / 1e6, mb / c1 / 1e6, mb / c2 / 1e6);
+            }
+            return 0;
+        }
         float a = timeit([&] { k_flat<0, 4><<<296, 256>>>(d_rows, n, src, d_dst, R); });
         float b = timeit([&] { k_flat<0, 4><<<296, 256>>>(d_srt, n, src, d_dst, R); });
         float c = timeit([&] { k_flat<0, 4><<<296, 256>>>(d_seq, n, src, d_dst, R); });
