@@ -47,6 +47,8 @@ def parse():
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
+    p.add_argument("--prewarm-max", type=int, default=400,
+                   help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
     p.add_argument("--miss-sweep", default="", help="tuning: 'threads:share:zc_blocks:pull_blocks,...' timed "
                    "one after another in this process (results under 'sweep')")
@@ -228,6 +230,9 @@ def run_ours(args, rank, world, local_rank):
     t0 = time.time()
     buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=False, device=local_rank)
     t_register = time.time() - t0
+    host_threads = max(1, min(14, len(os.sched_getaffinity(0)) // world - 2))
+    if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
+        buf.config(host_threads)
     wl.fill_table()
     if cfg.preload:   # "all features resident": rebuild with the filled table preloaded
         buf.close()
@@ -236,7 +241,8 @@ def run_ours(args, rank, world, local_rank):
         f"fill {wl.t_fill:.1f}s; N={cfg.num_nodes} E={cfg.num_edges} S={S} n_max={n_max} deg={wl.deg_stats}")
 
     sweep_cfgs = [tuple(float(x) for x in c.split(":")) for c in args.miss_sweep.split(",") if c]
-    total = W + K + (0 if args.no_e2e else K) + len(sweep_cfgs) * (W + K)
+    PRE = 0 if cfg.preload else args.prewarm_max
+    total = PRE + W + K + (0 if args.no_e2e else K) + len(sweep_cfgs) * (W + K)
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -289,11 +295,26 @@ def run_ours(args, rank, world, local_rank):
         parity = check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev)
         buf.close()
         buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
+        if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
+            buf.config(host_threads)
     barrier()
 
-    # ---- warm-up
-    log(f"parity {parity}; warm-up ...")
-    for j in range(W):
+    # ---- buffer pre-warm (untimed): the feature buffer reaches steady state once the
+    # cumulative misses exceed its capacity; stats are read every 8 batches
+    log(f"parity {parity}; pre-warm ...")
+    jp = 0
+    while jp < PRE:
+        for _ in range(8):
+            if jp < PRE:
+                step(jp)
+                jp += 1
+        if int(stats[:jp, 1].sum().item()) >= S:
+            break
+    prewarm_batches = jp
+    torch.cuda.synchronize(dev)
+    off = jp              # schedule offset: everything below uses batches after the pre-warm
+    log(f"pre-warm: {prewarm_batches} batches; warm-up ...")
+    for j in range(off, off + W):
         step(j)
     torch.cuda.synchronize(dev)
     barrier()
@@ -307,9 +328,9 @@ def run_ours(args, rank, world, local_rank):
     ev1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local_rank) as clk:
         ev0.record(main)
-        for j in range(W, W + K):
+        for j in range(off + W, off + W + K):
             step(j)
-        main.wait_event(dones[(W + K - 1) % RING])  # the last batch's rows are all in `out`
+        main.wait_event(dones[(off + W + K - 1) % RING])  # the last batch's rows are all in `out`
         ev1.record(main)
         ev1.synchronize()
     torch.cuda.synchronize(dev)
@@ -319,8 +340,8 @@ def run_ours(args, rank, world, local_rank):
     ms_max = max_over_ranks(ms, dev)
     tg = g.timing_read()
     tb = buf.timing_read()
-    st = stats[W:W + K].sum(0).cpu().tolist()
-    sz = sizes_log[W:W + K].double().mean(0).cpu().tolist()
+    st = stats[off + W:off + W + K].sum(0).cpu().tolist()
+    sz = sizes_log[off + W:off + W + K].double().mean(0).cpu().tolist()
     hits, misses, miss_zc, miss_staged = (int(x) for x in st)
     barrier()
 
@@ -335,9 +356,9 @@ def run_ours(args, rank, world, local_rank):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(main)
-        for j in range(W + K, W + 2 * K):
+        for j in range(off + W + K, off + W + 2 * K):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats))
-        main.wait_event(dones[(W + 2 * K - 1) % RING])
+        main.wait_event(dones[(off + W + 2 * K - 1) % RING])
         e1.record(main)
         e1.synchronize()
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)
@@ -346,7 +367,7 @@ def run_ours(args, rank, world, local_rank):
                "d2h_bytes_per_step": (2 * len(fan) + 1) * 8 + 32}
     # ---- optional in-process sweep of the miss-stream configuration (tuning only)
     sweep = []
-    j0 = W + K + (0 if args.no_e2e else K)
+    j0 = off + W + K + (0 if args.no_e2e else K)
     for (thr, share, zcb, plb) in sweep_cfgs:
         torch.cuda.synchronize(dev)
         buf.config(int(thr), share, int(zcb), int(plb))
@@ -432,6 +453,7 @@ def run_ours(args, rank, world, local_rank):
         "config": {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
                    "feat_dim": cfg.feat_dim, "feat_bytes": R, "batch_size": cfg.batch_size, "fanouts": fan,
                    "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
+                   "buffer_prewarm_batches": prewarm_batches,
                    "parallelism": f"dp{world} (batch segments, no collective)",
                    "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
                        (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.num_nodes * R * 1e-9)},

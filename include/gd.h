@@ -180,12 +180,14 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  * function, so still stream-ordered, no caller sync); phase 2, a kernel pulls the
  * slot contiguously over the host link.  K0 = floor(M * zero_copy_share).
  *   host_threads     0 disables the staged path (all misses zero-copy).
- *   zero_copy_share  in [0, 1]; < 0 = adaptive (balance the two paths' measured rates).
+ *   zero_copy_share  in [0, 1]; < 0 = adaptive: 1 - r_host / r_link, with r_host the
+ *                    measured host gather rate and r_link the contiguous pull rate of
+ *                    the host link, calibrated when this call enables adaptation.
  *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
- *                    copy kernels; <= 0 keeps the current value (defaults 24 and 8).
+ *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs
  *                    that run sampling / bookkeeping / the hit gather.
- * Default at init: host_threads = min(12, 3/4 of the cores) (0 with preload),
+ * Default at init: host_threads = min(14, cores - 2) (0 with preload),
  * adaptive share; env GD_HOST_THREADS / GD_ZERO_COPY_SHARE / GD_ZC_BLOCKS /
  * GD_PULL_BLOCKS override.  Synchronises the buffer's
  * internal streams; call between batches.

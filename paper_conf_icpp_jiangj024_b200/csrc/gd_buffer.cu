@@ -594,6 +594,10 @@ __global__ void k_init_slots(int32_t* reverse, int32_t* pos_of_slot, int32_t* ri
 
 using namespace gd;
 
+extern "C" {
+static gd_status calibrate_link(gd_buffer* b);
+}
+
 static void buffer_free(gd_buffer* b) {
     if (!b) return;
     DeviceGuard guard(b->hdr.device);
@@ -736,7 +740,8 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     }
     // staged miss path (phase 1 host gather + phase 2 contiguous pull): on by default
     // unless every row is resident from the start; GD_HOST_THREADS overrides the width.
-    int threads = preload ? 0 : (int)std::min(12u, std::max(1u, std::thread::hardware_concurrency() * 3 / 4));
+    const int hw = (int)std::thread::hardware_concurrency();
+    int threads = preload ? 0 : std::min(14, std::max(1, hw - 2));
     if (const char* e = std::getenv("GD_HOST_THREADS")) threads = std::max(0, std::atoi(e));
     double share = -1.0;
     if (const char* e = std::getenv("GD_ZERO_COPY_SHARE")) share = std::atof(e);
@@ -788,7 +793,12 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     if (host_threads > 0 && !b->pool) b->pool = new HostGatherPool(host_threads);
     b->host_threads = host_threads;
     b->alpha_fixed = zero_copy_share >= 0;
-    b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.5);
+    b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.2);
+    b->r_host = 0;
+    if (host_threads > 0 && !b->alpha_fixed) {
+        gd_status st = calibrate_link(b);
+        if (st != GD_OK) return st;
+    }
     return GD_OK;
 }
 
@@ -830,26 +840,61 @@ static void CUDART_CB host_gather_cb(void* arg) {
     if (b->timer.on) b->timer_host_ms += ss->cpu_ms;   // serialised on stream H
 }
 
-// Zero-copy share alpha from the measured rates of a finished batch: the zero-copy
-// path is bounded by the host's random-translation rate, the staged path by
-// max(host gather, contiguous pull); split the misses so both finish together.
+// Zero-copy share alpha.  The staged path moves rows with contiguous (cheap to
+// translate) host-link reads but is capped by the host gather rate r_host; the
+// zero-copy path is capped by the host's random-translation rate and competes for the
+// same link.  The fastest split lets the staged path run at r_host and tops the link
+// up with zero-copy: alpha = 1 - r_host / r_link (r_link calibrated at config time).
 static void adapt_alpha(gd_buffer* b, int d) {
     StagedSlot& ss = b->stg[d];
-    if (b->alpha_fixed || ss.batch < 0) return;
-    if (cudaEventQuery(b->ev_z1[d]) != cudaSuccess || cudaEventQuery(b->ev_p1[d]) != cudaSuccess) {
+    if (b->alpha_fixed || ss.batch < 0 || b->r_link <= 0) return;
+    if (cudaEventQuery(b->ev_E[d]) != cudaSuccess) {   // that batch's host gather still running
         cudaGetLastError();
         return;
     }
-    const double M = (double)ss.h_meta[0], K0 = (double)ss.h_meta[1];
-    float tz = 0, tp = 0;
-    cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]);
-    cudaEventElapsedTime(&tp, b->ev_p0[d], b->ev_p1[d]);
-    cudaGetLastError();
-    if (M < 4096 || K0 < 256 || M - K0 < 256 || tz <= 0) return;
-    const double rz = K0 / tz;
-    const double rs = (M - K0) / std::max<double>(std::max<double>(tp, ss.cpu_ms), 1e-3);
-    const double target = rz / (rz + rs);
-    b->alpha = std::min(0.95, std::max(0.05, 0.7 * b->alpha + 0.3 * target));
+    const double staged_rows = (double)ss.h_meta[2];
+    if (staged_rows < 2048 || ss.cpu_ms <= 0) return;
+    const double r = staged_rows * (double)b->R / ss.cpu_ms;
+    b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
+    b->alpha = std::min(0.9, std::max(0.0, 1.0 - b->r_host / b->r_link));
+}
+
+// Contiguous host-link pull rate (bytes/ms), measured once on the staging memory.
+__global__ void __launch_bounds__(1024, 1) k_link_calib(const uint4* __restrict__ src, uint4* __restrict__ dst, int64_t n16) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n16; i += (int64_t)gridDim.x * blockDim.x) {
+        uint4 v;
+        asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                     : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(src + i));
+        dst[i] = v;
+    }
+}
+
+static gd_status calibrate_link(gd_buffer* b) {
+    const int64_t bytes = std::min<int64_t>(64ll << 20, (int64_t)b->n_max * b->R) & ~(int64_t)15;
+    if (bytes < (1 << 20)) return GD_OK;
+    const uint8_t* src = nullptr;
+    GD_CUDA(cudaHostGetDevicePointer((void**)&src, b->stage_mem, 0));
+    uint8_t* dst = nullptr;
+    GD_CUDA(cudaMalloc(&dst, bytes));
+    cudaEvent_t e0, e1;
+    cudaEventCreate(&e0);
+    cudaEventCreate(&e1);
+    float best = 1e30f;
+    for (int rep = 0; rep < 4; ++rep) {
+        cudaEventRecord(e0, b->side_p);
+        k_link_calib<<<b->pull_blocks, 1024, 0, b->side_p>>>((const uint4*)src, (uint4*)dst, bytes / 16);
+        cudaEventRecord(e1, b->side_p);
+        cudaEventSynchronize(e1);
+        float ms = 0;
+        cudaEventElapsedTime(&ms, e0, e1);
+        if (rep > 0 && ms > 0 && ms < best) best = ms;
+    }
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    cudaFree(dst);
+    GD_CUDA(cudaGetLastError());
+    b->r_link = (double)bytes / best;
+    return GD_OK;
 }
 
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max, void* out,

@@ -88,9 +88,11 @@ struct gd_buffer {
     std::vector<cudaEvent_t> ev_z0, ev_z1, ev_p0, ev_p1;   // [D] timing of the two miss paths
     int64_t* trip_split = nullptr;       // [D] K0: misses [0, K0) zero-copy, [K0, M) staged
     int host_threads = 0;                // 0: staged path off (all misses zero-copy)
-    int zc_blocks = 24;                  // 1024-thread blocks (~whole SMs) of the zero-copy copy
+    int zc_blocks = 16;                  // 1024-thread blocks (~whole SMs) of the zero-copy copy
     int pull_blocks = 8;                 // 1024-thread blocks of the staged pull
     double alpha = 1.0;                  // zero-copy share of the misses (adapted)
+    double r_host = 0;                   // EMA of the host gather rate (bytes/ms)
+    double r_link = 0;                   // contiguous pull rate of the host link (bytes/ms), calibrated
     bool alpha_fixed = false;
     gd::HostGatherPool* pool = nullptr;
     std::vector<StagedSlot> stg;
