@@ -1,0 +1,103 @@
+"""Multi-GPU host logic on CPU: world-size-2 gloo process groups (no GPU needed).
+
+Covers the data-parallel sharding of §8(e) ("segments", P:142 shared host data):
+contiguous, disjoint, complete batch segments; per-rank schedules with epoch wrap; the
+/dev/shm host table created by rank 0 and mapped by every rank; max/sum over ranks.
+"""
+import os
+import socket
+import tempfile
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, shm_dir, q):
+    import sys
+    sys.path.insert(0, ROOT)
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_icpp_jiangj024_b200 import multigpu as M
+        out = {}
+        out["seg"] = list(M.segment(1209, rank, world))
+        out["sched"] = M.batch_schedule(10, rank, world, 12)
+        t = M.HostTable(1000, 64, "test", rank, world, shm_dir=shm_dir)
+        if rank == 0:
+            t.array[:] = (np.arange(1000 * 64) % 251).astype(np.uint8).reshape(1000, 64)
+        M.barrier()
+        out["table_sum"] = int(t.array.astype(np.int64).sum())
+        out["table_row7"] = t.array[7].tolist()
+        out["max"] = M.max_over_ranks(float(rank * 10 + 1))
+        out["sum"] = M.sum_over_ranks(float(rank + 1))
+        M.barrier()
+        t.close(unlink=True)
+        q.put((rank, out))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.fixture(scope="module")
+def results():
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    with tempfile.TemporaryDirectory() as d:
+        port = _free_port()
+        procs = [ctx.Process(target=_worker, args=(r, world, port, d, q)) for r in range(world)]
+        for p in procs:
+            p.start()
+        res = dict(q.get(timeout=120) for _ in range(world))
+        for p in procs:
+            p.join(timeout=60)
+            assert p.exitcode == 0
+        assert not os.listdir(d)        # rank 0 unlinked the shared table
+    return res
+
+
+def test_segments_disjoint_and_complete(results):
+    a, b = results[0]["seg"], results[1]["seg"]
+    assert a == list(range(0, 604)) and b == list(range(604, 1209))
+    assert sorted(a + b) == list(range(1209))
+
+
+def test_schedule_wraps_with_epochs(results):
+    s0, s1 = results[0]["sched"], results[1]["sched"]
+    assert s0[:5] == [(b, 0) for b in range(5)] and s0[5:10] == [(b, 1) for b in range(5)]
+    assert s1[:5] == [(b, 0) for b in range(5, 10)]
+    # the Philox batch key epoch * num_batches + b is distinct across ranks and epochs
+    keys = [ep * 10 + b for b, ep in s0 + s1]
+    assert len(set(keys)) == len(keys)
+
+
+def test_shared_host_table_visible_to_all_ranks(results):
+    expect = (np.arange(1000 * 64) % 251).astype(np.int64)
+    assert results[0]["table_sum"] == results[1]["table_sum"] == int(expect.sum())
+    assert results[1]["table_row7"] == expect.reshape(1000, 64)[7].tolist()
+
+
+def test_max_and_sum_over_ranks(results):
+    assert results[0]["max"] == results[1]["max"] == 11.0
+    assert results[0]["sum"] == results[1]["sum"] == 3.0
+
+
+def test_single_process_fallbacks():
+    from paper_conf_icpp_jiangj024_b200 import multigpu as M
+    assert M.max_over_ranks(3.5) == 3.5 and M.sum_over_ranks(2.0) == 2.0
+    assert list(M.segment(7, 0, 1)) == list(range(7))
+    assert M.batch_schedule(3, 0, 1, 7) == [(0, 0), (1, 0), (2, 0), (0, 1), (1, 1), (2, 1), (0, 2)]
+    assert M.batch_schedule(1, 1, 4, 3) == []       # more ranks than batches: an empty segment
