@@ -6,6 +6,8 @@
 // into a contiguous pinned staging slot, run from a CUDA host function on the library's
 // host-gather stream; phase 2 (k_stage_copy) pulls the slot over the host link with
 // contiguous, translation-friendly reads.
+#include <emmintrin.h>   // SSE2 streaming stores (baseline x86-64)
+
 #include <atomic>
 #include <chrono>
 #include <condition_variable>
@@ -34,14 +36,37 @@ struct HostGatherPool::Impl {
     std::atomic<int64_t> next{0};
     static constexpr int64_t kChunk = 512;
 
+    // Row copy with non-temporal stores: the staging slot is read next by the GPU over
+    // PCIe, so keeping it out of the CPU caches avoids snoop hits on dirty lines, and
+    // streaming stores skip the read-for-ownership of every destination line.
+    static void copy_row(uint8_t* d, const uint8_t* s, int64_t R) {
+        if ((R & 15) == 0 && (((uintptr_t)d) & 15) == 0) {
+            const __m128i* sp = (const __m128i*)s;
+            __m128i* dp = (__m128i*)d;
+            const int64_t n16 = R >> 4;
+            int64_t c = 0;
+            for (; c + 4 <= n16; c += 4) {
+                const __m128i a = _mm_loadu_si128(sp + c), b = _mm_loadu_si128(sp + c + 1);
+                const __m128i e = _mm_loadu_si128(sp + c + 2), f = _mm_loadu_si128(sp + c + 3);
+                _mm_stream_si128(dp + c, a);
+                _mm_stream_si128(dp + c + 1, b);
+                _mm_stream_si128(dp + c + 2, e);
+                _mm_stream_si128(dp + c + 3, f);
+            }
+            for (; c < n16; ++c) _mm_stream_si128(dp + c, _mm_loadu_si128(sp + c));
+        } else {
+            std::memcpy(d, s, (size_t)R);
+        }
+    }
+
     void work() {
         while (true) {
             const int64_t lo = next.fetch_add(kChunk, std::memory_order_relaxed);
             if (lo >= n) break;
             const int64_t hi = lo + kChunk < n ? lo + kChunk : n;
-            for (int64_t j = lo; j < hi; ++j)
-                std::memcpy(dst + j * R, src + (int64_t)rows[j] * R, (size_t)R);
+            for (int64_t j = lo; j < hi; ++j) copy_row(dst + j * R, src + (int64_t)rows[j] * R, R);
         }
+        _mm_sfence();   // streaming stores globally visible before the GPU pull is released
     }
 
     void loop() {

@@ -2,6 +2,7 @@
 //   g++ -O3 -march=native -pthread -o cg tools/cpu_gather_bench.cpp
 //   ./cg <table_GB> <row_bytes> <rows> <thp 0/1>
 #include <sys/mman.h>
+#include <emmintrin.h>
 
 #include <algorithm>
 #include <atomic>
@@ -32,9 +33,9 @@ int main(int argc, char** argv) {
     std::vector<int32_t> rows(n);
     std::mt19937_64 rng(1);
     for (auto& r : rows) r = (int32_t)(rng() % N);
-    std::vector<uint8_t> stage(n * R);
+    uint8_t* stage = (uint8_t*)aligned_alloc(64, n * R);
     for (int T : {1, 2, 4, 8, 12, 16}) {
-        for (int pf : {0, 8}) {
+        for (int pf : {0, 1}) {   // 1 = non-temporal stores
             double best = 0;
             for (int rep = 0; rep < 3; ++rep) {
                 auto t0 = std::chrono::steady_clock::now();
@@ -43,18 +44,21 @@ int main(int argc, char** argv) {
                     th.emplace_back([&, k] {
                         const size_t lo = n * k / T, hi = n * (k + 1) / T;
                         for (size_t i = lo; i < hi; ++i) {
-                            if (pf && i + pf < hi) {
-                                const uint8_t* p = t + (size_t)rows[i + pf] * R;
-                                for (size_t c = 0; c < R; c += 64) __builtin_prefetch(p + c);
+                            if (pf) {
+                                const __m128i* sp = (const __m128i*)(t + (size_t)rows[i] * R);
+                                __m128i* dp = (__m128i*)&stage[i * R];
+                                for (size_t c = 0; c < R / 16; ++c) _mm_stream_si128(dp + c, _mm_loadu_si128(sp + c));
+                            } else {
+                                memcpy(&stage[i * R], t + (size_t)rows[i] * R, R);
                             }
-                            memcpy(&stage[i * R], t + (size_t)rows[i] * R, R);
                         }
+                        _mm_sfence();
                     });
                 for (auto& x : th) x.join();
                 const double s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
                 best = std::max(best, n * R / s / 1e9);
             }
-            printf("table %.0f GB R=%zu thp=%d threads=%2d prefetch=%d: %.1f GB/s\n", GB, R, thp, T, pf, best);
+            printf("table %.0f GB R=%zu thp=%d threads=%2d nt_store=%d: %.1f GB/s\n", GB, R, thp, T, pf, best);
         }
     }
     return 0;
