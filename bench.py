@@ -63,10 +63,8 @@ def log(*a):
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled every 200 ms during the timed region."""
-    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clocks and throttle reasons sampled every 200 ms during the timed region, in-process
+    through NVML (spawning nvidia-smi would steal a host core from the miss-path gather)."""
 
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
@@ -75,13 +73,21 @@ class ClockSampler:
         self._t = None
 
     def _run(self):
+        try:
+            import pynvml as N
+            N.nvmlInit()
+            h = N.nvmlDeviceGetHandleByIndex(self.gpu)
+        except Exception:  # noqa: BLE001
+            return
+        bits = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
+                "sw_power_cap": 0x4}
         while not self._stop.is_set():
             try:
-                out = subprocess.run(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
-                                      "--format=csv,noheader,nounits"], capture_output=True, text=True,
-                                     timeout=5).stdout.strip()
-                if out:
-                    self.rows.append([x.strip() for x in out.split(",")])
+                sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+                mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+                r = N.nvmlDeviceGetCurrentClocksEventReasons(h) if hasattr(N, "nvmlDeviceGetCurrentClocksEventReasons") \
+                    else N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+                self.rows.append((sm, mx, [k for k, b in bits.items() if r & b]))
             except Exception:  # noqa: BLE001
                 pass
             self._stop.wait(0.2)
@@ -97,16 +103,11 @@ class ClockSampler:
             self._t.join(timeout=10)
 
     def summary(self):
-        sm = [float(r[1]) for r in self.rows if len(r) > 8 and r[1].replace(".", "").isdigit()]
-        mx = [float(r[2]) for r in self.rows if len(r) > 8 and r[2].replace(".", "").isdigit()]
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = set()
-        for r in self.rows:
-            for k, nm in enumerate(names):
-                if len(r) > 5 + k and r[5 + k].lower().startswith("active"):
-                    reasons.add(nm)
+        sm = [r[0] for r in self.rows]
+        mx = [r[1] for r in self.rows]
+        reasons = sorted({x for r in self.rows for x in r[2]})
         return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(self.rows)}
+                "reasons": reasons, "samples": len(self.rows), "source": "NVML, 200 ms"}
 
 
 def h2d_peak_gbps(device) -> float:
@@ -230,7 +231,7 @@ def run_ours(args, rank, world, local_rank):
     t0 = time.time()
     buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=False, device=local_rank)
     t_register = time.time() - t0
-    host_threads = max(1, min(14, len(os.sched_getaffinity(0)) // world - 2))
+    host_threads = max(1, min(13, len(os.sched_getaffinity(0)) // world - 3))
     if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
         buf.config(host_threads)
     wl.fill_table()

@@ -187,7 +187,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs
  *                    that run sampling / bookkeeping / the hit gather.
- * Default at init: host_threads = min(14, cores - 2) (0 with preload),
+ * Default at init: host_threads = min(13, cores - 3) (0 with preload),
  * adaptive share; env GD_HOST_THREADS / GD_ZERO_COPY_SHARE / GD_ZC_BLOCKS /
  * GD_PULL_BLOCKS override.  Synchronises the buffer's
  * internal streams; call between batches.

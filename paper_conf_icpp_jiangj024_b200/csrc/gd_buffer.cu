@@ -741,7 +741,7 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     // staged miss path (phase 1 host gather + phase 2 contiguous pull): on by default
     // unless every row is resident from the start; GD_HOST_THREADS overrides the width.
     const int hw = (int)std::thread::hardware_concurrency();
-    int threads = preload ? 0 : std::min(14, std::max(1, hw - 2));
+    int threads = preload ? 0 : std::min(13, std::max(1, hw - 3));
     if (const char* e = std::getenv("GD_HOST_THREADS")) threads = std::max(0, std::atoi(e));
     double share = -1.0;
     if (const char* e = std::getenv("GD_ZERO_COPY_SHARE")) share = std::atof(e);
