@@ -3,9 +3,10 @@
 // One gd_sample call = 3 + 2K launches on the caller's stream, no host sync:
 //   memset(hash) ; k_seed_intake ; K x { k_sample_hop ; k_relabel_hop } ; k_col_resolve
 //
-// k_sample_hop  (S1, a2+a3): tile of 64 frontier nodes per 256-thread block.  Counts
-//   cnt = min(f, deg) are scanned with a decoupled look-back (rowptr), then one warp per
-//   node draws Floyd positions with Philox (lane t = draw t, resolution by ballots, rank
+// k_sample_hop  (S1, a2+a3): tile of 64-256 frontier nodes per 256-thread block.  Counts
+//   cnt = min(f, deg) are scanned with a decoupled look-back (rowptr), then a group of
+//   G = pow2 >= f lanes per node (32/G nodes per warp at once; a whole warp for f > 16)
+//   draws Floyd positions with Philox (lane t = draw t, resolution by ballots, rank
 //   sort by shuffles) and inserts every neighbour into the global open-addressing hash
 //   with atomicMin of its flat position (first occurrence).  col temporarily holds the
 //   neighbour's hash slot.
@@ -25,7 +26,6 @@ namespace gd {
 
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
-constexpr int kNodesPerTile = 64;          // frontier nodes per sampler block
 constexpr int kRelabelItems = 8;
 constexpr int kEdgesPerTile = kThreads * kRelabelItems;   // 2048 edges per relabel block
 constexpr int kMaxFanSmem = GD_MAX_FANOUT;
@@ -107,29 +107,33 @@ __device__ __forceinline__ void emit_edge(const SampleHopArgs& a, int64_t start,
     if (a.eid) a.eid[e] = start + p;
 }
 
+// G = lanes per frontier node (a power of two >= fanout, or 32 for the generic paths);
+// NPB = frontier nodes per 256-thread block (8 node-iterations per warp).
+template <int G, int NPB>
 __global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
+    static_assert(NPB <= kThreads && (32 % G) == 0, "tile shape");
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t n_prev = a.sizes[a.hop - 1];
     const int64_t tile = blockIdx.x;
-    const int64_t i0 = tile * kNodesPerTile;
+    const int64_t i0 = tile * NPB;
     if (i0 >= n_prev && tile != 0) return;
 
-    __shared__ int64_t s_start[kNodesPerTile];
-    __shared__ int64_t s_deg[kNodesPerTile];
-    __shared__ int64_t s_off[kNodesPerTile];
-    __shared__ int32_t s_v[kNodesPerTile];
-    __shared__ long long s_wtot[2];
+    __shared__ int64_t s_start[NPB];
+    __shared__ int64_t s_deg[NPB];
+    __shared__ int64_t s_off[NPB];
+    __shared__ int32_t s_v[NPB];
+    __shared__ long long s_wtot[kWarps];
     __shared__ long long s_base;
-    __shared__ int64_t s_sel[kWarps][kMaxFanSmem];   // f > 32 path only
+    __shared__ int64_t s_sel[G == 32 ? kWarps : 1][G == 32 ? kMaxFanSmem : 1];   // f > 32 path only
 
     const int t = threadIdx.x;
     const int lane = t & 31;
     const int warp = t >> 5;
     const int f = a.fanout;
 
-    // ---- a2: counts and their exclusive scan (rowptr)
+    // ---- a2: counts (one frontier node per thread) and their exclusive scan (rowptr)
     long long cnt = 0;
-    if (t < kNodesPerTile) {
+    if (t < NPB) {
         const int64_t i = i0 + t;
         int64_t start = 0, d = 0;
         int32_t v = 0;
@@ -145,21 +149,21 @@ __global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
         s_start[t] = start;
         s_deg[t] = d;
     }
-    long long incl = 0;
-    if (t < kNodesPerTile) {
-        incl = warp_inclusive_sum(cnt);
-        if (lane == 31) s_wtot[warp] = incl;
-    }
+    const long long incl = warp_inclusive_sum(cnt);
+    if (lane == 31) s_wtot[warp] = incl;
     __syncthreads();
     if (warp == 0) {
-        const long long agg = s_wtot[0] + s_wtot[1];
+        const long long wt = lane < kWarps ? s_wtot[lane] : 0;
+        const long long winc = warp_inclusive_sum(wt);
+        const long long agg = __shfl_sync(0xffffffffu, winc, kWarps - 1);
+        __syncwarp();
+        if (lane < kWarps) s_wtot[lane] = winc - wt;          // exclusive warp offsets
         const long long base = lookback_exclusive(a.st, tile, agg, 0);
         if (lane == 0) s_base = base;
     }
     __syncthreads();
-    const long long base = s_base;
-    if (t < kNodesPerTile) {
-        const long long excl = base + incl - cnt + (warp == 1 ? s_wtot[0] : 0);
+    if (t < NPB) {
+        const long long excl = s_base + s_wtot[warp] + incl - cnt;
         s_off[t] = excl;
         const int64_t i = i0 + t;
         if (i < n_prev) a.rowptr[i] = excl;
@@ -172,66 +176,132 @@ __global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
     }
     __syncthreads();
 
-    // ---- a3: one warp per frontier node
+    // ---- a3: Floyd sampling, G lanes per frontier node
     const uint32_t hidx = (uint32_t)(a.hop - 1);
-    for (int ln = warp; ln < kNodesPerTile; ln += kWarps) {
-        const int64_t i = i0 + ln;
-        if (i >= n_prev) break;
-        const int64_t start = s_start[ln];
-        const int64_t d = s_deg[ln];
-        const int64_t off = s_off[ln];
-        const uint32_t v = (uint32_t)s_v[ln];
-        if (f < 0 || d <= f) {
-            // the row verbatim (reading R4): coalesced copy
-            for (int64_t p = lane; p < d; p += 32) emit_edge(a, start, p, off + p);
-        } else if (f <= 32) {
-            // Floyd: lane t holds draw t in [0, d-f+t]
+    if constexpr (G < 32) {
+        // 0 <= f <= G: lane gl of the group holds draw gl; groups are independent nodes
+        constexpr int P = 32 / G;
+        const int gl = lane & (G - 1);
+        const int gbase = lane & ~(G - 1);
+        const unsigned gmask = ((G == 32) ? 0xffffffffu : ((1u << G) - 1u)) << gbase;
+        for (int ln0 = warp * P; ln0 < NPB; ln0 += kWarps * P) {
+            const int ln = ln0 + lane / G;
+            const int64_t i = i0 + ln;
+            const bool active = (ln < NPB) && (i < n_prev);
+            int64_t d = 0, start = 0, off = 0;
+            uint32_t v = 0;
+            if (active) {
+                d = s_deg[ln];
+                start = s_start[ln];
+                off = s_off[ln];
+                v = (uint32_t)s_v[ln];
+            }
+            const bool fl = active && d > f;           // Floyd; otherwise the row verbatim
             int64_t sel = INT64_MAX;
-            if (lane < f) {
-                const uint64_t j = (uint64_t)(d - f + lane);
-                sel = (int64_t)draw_uniform((uint32_t)lane, v, hidx, a.batch, a.seed, j);
+            if (fl) {
+                if (gl < f) sel = (int64_t)draw_uniform((uint32_t)gl, v, hidx, a.batch, a.seed, (uint64_t)(d - f + gl));
+            } else if (active && gl < d) {
+                sel = gl;
             }
             for (int s = 1; s < f; ++s) {
-                const int64_t rs = __shfl_sync(0xffffffffu, sel, s);
-                const bool present = __ballot_sync(0xffffffffu, lane < s && sel == rs) != 0;
-                if (lane == s && present) sel = d - f + s;
+                const int64_t rs = __shfl_sync(0xffffffffu, sel, gbase + s);
+                const unsigned bl = __ballot_sync(0xffffffffu, fl && gl < s && sel == rs);
+                if (fl && gl == s && (bl & gmask)) sel = d - f + s;
             }
-            int rank = 0;
-            for (int s = 0; s < f; ++s) {
-                const int64_t o = __shfl_sync(0xffffffffu, sel, s);
-                rank += (o < sel);
-            }
-            if (lane < f) emit_edge(a, start, sel, off + rank);
-        } else {
-            // f in (32, 256]: resolution in shared memory, O(f^2/32) per node
-            int64_t* ss = s_sel[warp];
-            for (int c = 0; c < f; c += 32) {
-                const int tt = c + lane;
-                int64_t r = 0;
-                if (tt < f) {
-                    const uint64_t j = (uint64_t)(d - f + tt);
-                    r = (int64_t)draw_uniform((uint32_t)tt, v, hidx, a.batch, a.seed, j);
+            int rank = gl;
+            if (f > 1) {
+                int r = 0;
+                for (int s = 0; s < f; ++s) {
+                    const int64_t o = __shfl_sync(0xffffffffu, sel, gbase + s);
+                    r += (o < sel);
                 }
-                const int cend = min(32, f - c);
-                for (int s = 0; s < cend; ++s) {
-                    const int step = c + s;
-                    const int64_t rs = __shfl_sync(0xffffffffu, r, s);
-                    bool hit = false;
-                    for (int q = lane; q < step; q += 32) hit |= (ss[q] == rs);
-                    const bool present = __ballot_sync(0xffffffffu, hit) != 0;
-                    if (lane == 0) ss[step] = present ? (d - f + step) : rs;
-                    __syncwarp();
-                }
+                if (fl) rank = r;
             }
-            __syncwarp();
-            for (int q = lane; q < f; q += 32) {
-                const int64_t me = ss[q];
-                int rank = 0;
-                for (int x = 0; x < f; ++x) rank += (ss[x] < me);
-                emit_edge(a, start, me, off + rank);
-            }
-            __syncwarp();
+            if (sel != INT64_MAX) emit_edge(a, start, sel, off + rank);
         }
+    } else {
+        for (int ln = warp; ln < NPB; ln += kWarps) {
+            const int64_t i = i0 + ln;
+            if (i >= n_prev) break;
+            const int64_t start = s_start[ln];
+            const int64_t d = s_deg[ln];
+            const int64_t off = s_off[ln];
+            const uint32_t v = (uint32_t)s_v[ln];
+            if (f < 0 || d <= f) {
+                // the row verbatim (reading R5): coalesced copy
+                for (int64_t p = lane; p < d; p += 32) emit_edge(a, start, p, off + p);
+            } else if (f <= 32) {
+                // Floyd: lane t holds draw t in [0, d-f+t]
+                int64_t sel = INT64_MAX;
+                if (lane < f) {
+                    const uint64_t j = (uint64_t)(d - f + lane);
+                    sel = (int64_t)draw_uniform((uint32_t)lane, v, hidx, a.batch, a.seed, j);
+                }
+                for (int s = 1; s < f; ++s) {
+                    const int64_t rs = __shfl_sync(0xffffffffu, sel, s);
+                    const bool present = __ballot_sync(0xffffffffu, lane < s && sel == rs) != 0;
+                    if (lane == s && present) sel = d - f + s;
+                }
+                int rank = 0;
+                for (int s = 0; s < f; ++s) {
+                    const int64_t o = __shfl_sync(0xffffffffu, sel, s);
+                    rank += (o < sel);
+                }
+                if (lane < f) emit_edge(a, start, sel, off + rank);
+            } else {
+                // f in (32, 256]: resolution in shared memory, O(f^2/32) per node
+                int64_t* ss = s_sel[warp];
+                for (int c = 0; c < f; c += 32) {
+                    const int tt = c + lane;
+                    int64_t r = 0;
+                    if (tt < f) {
+                        const uint64_t j = (uint64_t)(d - f + tt);
+                        r = (int64_t)draw_uniform((uint32_t)tt, v, hidx, a.batch, a.seed, j);
+                    }
+                    const int cend = min(32, f - c);
+                    for (int s = 0; s < cend; ++s) {
+                        const int step = c + s;
+                        const int64_t rs = __shfl_sync(0xffffffffu, r, s);
+                        bool hit = false;
+                        for (int q = lane; q < step; q += 32) hit |= (ss[q] == rs);
+                        const bool present = __ballot_sync(0xffffffffu, hit) != 0;
+                        if (lane == 0) ss[step] = present ? (d - f + step) : rs;
+                        __syncwarp();
+                    }
+                }
+                __syncwarp();
+                for (int q = lane; q < f; q += 32) {
+                    const int64_t me = ss[q];
+                    int rank = 0;
+                    for (int x = 0; x < f; ++x) rank += (ss[x] < me);
+                    emit_edge(a, start, me, off + rank);
+                }
+                __syncwarp();
+            }
+        }
+    }
+}
+
+// Tile shape for a fanout: lanes per node G and nodes per block NPB.
+static int sampler_group(int f) {
+    if (f < 0 || f > 16) return 32;
+    int g = 1;
+    while (g < f) g *= 2;
+    return g;
+}
+static int sampler_npb(int g) { return g >= 32 ? 64 : (g == 16 ? 128 : 256); }
+
+static void launch_sample_hop(const SampleHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
+    const int g = sampler_group(a.fanout);
+    const int npb = sampler_npb(g);
+    const unsigned nt = (unsigned)std::max<int64_t>(1, (n_frontier_max + npb - 1) / npb);
+    switch (g) {
+        case 1: k_sample_hop<1, 256><<<nt, kThreads, 0, st>>>(a); break;
+        case 2: k_sample_hop<2, 256><<<nt, kThreads, 0, st>>>(a); break;
+        case 4: k_sample_hop<4, 256><<<nt, kThreads, 0, st>>>(a); break;
+        case 8: k_sample_hop<8, 256><<<nt, kThreads, 0, st>>>(a); break;
+        case 16: k_sample_hop<16, 128><<<nt, kThreads, 0, st>>>(a); break;
+        default: k_sample_hop<32, 64><<<nt, kThreads, 0, st>>>(a); break;
     }
 }
 
@@ -465,7 +535,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     }
     int64_t tiles = 1;
     for (int h = 0; h < num_hops; ++h) {
-        tiles = std::max(tiles, ceil_div(nmax[h], kNodesPerTile));
+        tiles = std::max(tiles, ceil_div(nmax[h], 64));
         tiles = std::max(tiles, ceil_div(emax[h], kEdgesPerTile));
     }
     if ((s = g->scan.ensure(tiles)) != GD_OK) return s;
@@ -513,8 +583,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
         a.st_clear = g->scan.other();
         a.st_clear_n = g->scan.cap;
         a.status = g->hdr.dev_status;
-        const int64_t nt = std::max<int64_t>(1, ceil_div(nmax[h - 1], kNodesPerTile));
-        k_sample_hop<<<(unsigned)nt, kThreads, 0, st>>>(a);
+        launch_sample_hop(a, nmax[h - 1], st);
         GD_DEBUG_AFTER("k_sample_hop", st);
         g->scan.flip();
 
