@@ -1008,10 +1008,12 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (timed) b->timer.end(t_gat, b->side_g);
     GD_CUDA(cudaEventRecord(b->ev_G, b->side_g));
 
-    // a7, zero-copy share: misses [0, K0) straight from the pinned host table (stream Z)
+    // a7, zero-copy share: misses [0, K0) straight from the pinned host table (stream Z).
+    // With preload every node is valid from the start and never evicted: no misses, no copy.
     const int t_zc = timed ? b->timer.begin(b->side) : -1;
     GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
-    if (b->R % 16 == 0)
+    if (b->preload) {
+    } else if (b->R % 16 == 0)
         k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
     else
         k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
