@@ -64,7 +64,8 @@ struct LookupArgs {
     int2* map;
     int32_t* pos_of_slot;
     int32_t* alias;
-    uint8_t* missflag;
+    int2* hitlist;                   // [n - M]: {batch position, slot} of the non-misses, list order
+    int64_t* hcount;                 // n - M
     int32_t* misslist;
     int64_t* mcount;
     int64_t* stats;
@@ -84,13 +85,14 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
     __shared__ long long s_base;
     const int t = threadIdx.x, lane = t & 31;
     unsigned ball[kBItems];
+    int32_t alv[kBItems];
 #pragma unroll
     for (int k = 0; k < kBItems; ++k) {
         const int64_t i = i0 + (int64_t)k * kBThreads + t;
         bool miss = false;
+        int32_t al = -1;
         if (i < n) {
             const int32_t v = a.ids[i];
-            int32_t al = -1;
             if (v < 0 || (int64_t)v >= a.N) {
                 atomicOr(a.status, GD_DEV_BAD_ID);
             } else {
@@ -108,8 +110,8 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
                 a.map[v].y = ((rc + 1) << 1) | valid;           // line 19
             }
             a.alias[i] = al;
-            a.missflag[i] = miss ? 1 : 0;
         }
+        alv[k] = al;
         ball[k] = __ballot_sync(0xffffffffu, miss);
     }
     const int agg = block_flag_offsets(ball, s_cnt);
@@ -121,6 +123,7 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
             if (last) {
                 const long long M = base + agg;
                 *a.mcount = M;
+                *a.hcount = n - M;
                 if (a.stats) {
                     a.stats[0] = n - M;
                     a.stats[1] = M;
@@ -133,10 +136,14 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
     const int warp = t >> 5;
     const unsigned lt = (1u << lane) - 1u;
 #pragma unroll
-    for (int k = 0; k < kBItems; ++k)
+    for (int k = 0; k < kBItems; ++k) {
+        const int64_t i = i0 + (int64_t)k * kBThreads + t;
+        const long long mrank = base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);   // misses before i
         if (ball[k] & (1u << lane))
-            a.misslist[base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt)] =
-                (int32_t)(i0 + (int64_t)k * kBThreads + t);
+            a.misslist[mrank] = (int32_t)i;
+        else if (i < n)
+            a.hitlist[i - mrank] = make_int2((int32_t)i, alv[k]);
+    }
 }
 
 // ------------------------------------------------------- a6: pop + assign (loop 2)
@@ -375,13 +382,13 @@ __global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __r
 }
 
 // ------------------------------------------------------------- a8: hit gather
+// out[i] = slots[s] for every (i, s) of the compacted hit list (only hits are visited).
 template <int UNROLL>
-__global__ void __launch_bounds__(256) k_gather_hits(const int32_t* __restrict__ alias, const uint8_t* __restrict__ missflag,
-                                                     const int64_t* __restrict__ n_dev, const uint8_t* __restrict__ slots,
-                                                     uint8_t* __restrict__ out, int64_t R) {
-    const int64_t n = *n_dev;
+__global__ void __launch_bounds__(256) k_gather_hits(const int2* __restrict__ hitlist, const int64_t* __restrict__ hcount,
+                                                     const uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+    const int64_t H = *hcount;
     const int64_t cpr = R >> 4;
-    const int64_t total = n * cpr;
+    const int64_t total = H * cpr;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; base < total; base += stride * UNROLL) {
         uint4 val[UNROLL];
@@ -392,13 +399,13 @@ __global__ void __launch_bounds__(256) k_gather_hits(const int32_t* __restrict__
             dst[u] = -1;
             if (idx < total) {
                 const int64_t r = idx / cpr, c = idx - r * cpr;
-                const int32_t s = __ldg(alias + r);
-                if (!__ldg(missflag + r) && s >= 0) {
-                    const uint4* src = (const uint4*)(slots + (int64_t)s * R) + c;
+                const int2 h = __ldg(hitlist + r);
+                if (h.y >= 0) {
+                    const uint4* src = (const uint4*)(slots + (int64_t)h.y * R) + c;
                     asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                                  : "=r"(val[u].x), "=r"(val[u].y), "=r"(val[u].z), "=r"(val[u].w)
                                  : "l"(src));
-                    dst[u] = idx * 16;   // out row r chunk c = flat idx
+                    dst[u] = (int64_t)h.x * R + c * 16;
                 }
             }
         }
@@ -408,18 +415,17 @@ __global__ void __launch_bounds__(256) k_gather_hits(const int32_t* __restrict__
     }
 }
 
-__global__ void k_gather_hits_w4(const int32_t* __restrict__ alias, const uint8_t* __restrict__ missflag,
-                                 const int64_t* __restrict__ n_dev, const uint8_t* __restrict__ slots,
-                                 uint8_t* __restrict__ out, int64_t R) {
-    const int64_t n = *n_dev;
+__global__ void k_gather_hits_w4(const int2* __restrict__ hitlist, const int64_t* __restrict__ hcount,
+                                 const uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+    const int64_t H = *hcount;
     const int64_t cpr = R >> 2;
-    const int64_t total = n * cpr;
+    const int64_t total = H * cpr;
     for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = idx / cpr, c = idx - r * cpr;
-        const int32_t s = alias[r];
-        if (missflag[r] || s < 0) continue;
-        ((uint32_t*)out)[idx] = ((const uint32_t*)(slots + (int64_t)s * R))[c];
+        const int2 h = hitlist[r];
+        if (h.y < 0) continue;
+        ((uint32_t*)(out + (int64_t)h.x * R))[c] = ((const uint32_t*)(slots + (int64_t)h.y * R))[c];
     }
 }
 
@@ -604,7 +610,7 @@ static void buffer_free(gd_buffer* b) {
     if (b->side) cudaStreamSynchronize(b->side);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) cudaStreamSynchronize(s);
-    void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->missflag,
+    void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->hitlist, b->hcount,
                     b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
                     b->hdr.dev_status};
     for (void* p : ptrs)
@@ -692,7 +698,8 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     GD_ALLOC(b->ring, 2 * C * sizeof(int32_t));
     GD_ALLOC(b->ctl, 2 * sizeof(GdCtl));
     GD_ALLOC(b->misslist, nm * sizeof(int32_t));
-    GD_ALLOC(b->missflag, (int64_t)b->D * nm);
+    GD_ALLOC(b->hitlist, (int64_t)b->D * nm * sizeof(int2));
+    GD_ALLOC(b->hcount, (int64_t)b->D * sizeof(int64_t));
     GD_ALLOC(b->alias_ws, (int64_t)b->D * nm * sizeof(int32_t));
     GD_ALLOC(b->mcount, sizeof(int64_t));
     GD_ALLOC(b->trip, (int64_t)b->D * nm * sizeof(int4));
@@ -910,7 +917,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     cudaStream_t st = (cudaStream_t)stream_v;
     const int d = (int)(b->batch_counter % b->D);
     int32_t* al = alias ? alias : b->alias_ws + (int64_t)d * b->n_max;
-    uint8_t* mflag = b->missflag + (int64_t)d * b->n_max;
+    int2* hlist = b->hitlist + (int64_t)d * b->n_max;
+    int64_t* hcnt = b->hcount + d;
     int4* trip = b->trip + (int64_t)d * b->n_max;
     int64_t* tcount = b->trip_count + d;
     int64_t* tsplit = b->trip_split + d;
@@ -935,7 +943,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     la.map = b->map;
     la.pos_of_slot = b->pos_of_slot;
     la.alias = al;
-    la.missflag = mflag;
+    la.hitlist = hlist;
+    la.hcount = hcnt;
     la.misslist = b->misslist;
     la.mcount = b->mcount;
     la.stats = stats;
@@ -1001,9 +1010,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // a8: hits, slots -> out (stream G)
     const int t_gat = timed ? b->timer.begin(b->side_g) : -1;
     if (b->R % 16 == 0)
-        k_gather_hits<4><<<148 * 8, 256, 0, b->side_g>>>(al, mflag, n_dev, b->slots, (uint8_t*)out, b->R);
+        k_gather_hits<4><<<148 * 8, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
     else
-        k_gather_hits_w4<<<148 * 8, 256, 0, b->side_g>>>(al, mflag, n_dev, b->slots, (uint8_t*)out, b->R);
+        k_gather_hits_w4<<<148 * 8, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
     GD_DEBUG_AFTER("k_gather_hits", b->side_g);
     if (timed) b->timer.end(t_gat, b->side_g);
     GD_CUDA(cudaEventRecord(b->ev_G, b->side_g));

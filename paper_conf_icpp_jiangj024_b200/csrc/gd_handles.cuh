@@ -67,7 +67,8 @@ struct gd_buffer {
     int ctl_parity = 0;
     // per-batch workspace used on the caller's stream
     int32_t* misslist = nullptr;         // [n_max] batch positions of misses, list order
-    uint8_t* missflag = nullptr;         // [D][n_max] (read by the gather on stream G)
+    int2* hitlist = nullptr;             // [D][n_max] {position, slot} of the hits (read on stream G)
+    int64_t* hcount = nullptr;           // [D] number of hits
     int32_t* alias_ws = nullptr;         // [D][n_max] used when the caller passes alias = NULL
     int64_t* mcount = nullptr;           // [1] misses of the current batch
     // miss triples for the side stream, a ring of D batches
