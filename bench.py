@@ -39,7 +39,7 @@ Q = 4   # release lag = training-queue capacity
 def parse():
     p = argparse.ArgumentParser()
     p.add_argument("--gpus", type=int, default=1)
-    p.add_argument("--steps", type=int, default=64)
+    p.add_argument("--steps", type=int, default=200)
     p.add_argument("--warmup", type=int, default=16)
     p.add_argument("--config", default="papers100m", choices=sorted(synth.CONFIGS))
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])

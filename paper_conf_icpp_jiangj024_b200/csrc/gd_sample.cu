@@ -282,26 +282,45 @@ __global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
     }
 }
 
-// Tile shape for a fanout: lanes per node G and nodes per block NPB.
+// Tile shape: G lanes per node (pow2 >= fanout; 32 for f > 16 or f < 0), ITERS node
+// iterations per warp, NPB = 8 warps x ITERS x (32 / G) nodes per block (<= 256, one per
+// thread in the count phase).  ITERS is chosen from the frontier bound so that small
+// frontiers get many short warps (latency) and large ones still fill every SM.
 static int sampler_group(int f) {
     if (f < 0 || f > 16) return 32;
     int g = 1;
     while (g < f) g *= 2;
     return g;
 }
-static int sampler_npb(int g) { return g >= 32 ? 64 : (g == 16 ? 128 : 256); }
+
+template <int G, int ITERS>
+static void launch_hop_t(const SampleHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
+    constexpr int NPB = kWarps * ITERS * (32 / G);
+    const unsigned nt = (unsigned)std::max<int64_t>(1, (n_frontier_max + NPB - 1) / NPB);
+    k_sample_hop<G, NPB><<<nt, kThreads, 0, st>>>(a);
+}
+
+template <int G>
+static void launch_hop_g(const SampleHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
+    constexpr int P = 32 / G;
+    constexpr int CAP = (256 / (kWarps * P)) < 8 ? (256 / (kWarps * P)) : 8;   // max ITERS
+    const int64_t warp_iters = (n_frontier_max + P - 1) / P;
+    int iters = 1;
+    while (iters < CAP && warp_iters / (iters * 2) >= 8192) iters *= 2;      // keep >= 8k warps
+    if constexpr (CAP >= 8) { if (iters == 8) return launch_hop_t<G, 8>(a, n_frontier_max, st); }
+    if constexpr (CAP >= 4) { if (iters == 4) return launch_hop_t<G, 4>(a, n_frontier_max, st); }
+    if constexpr (CAP >= 2) { if (iters == 2) return launch_hop_t<G, 2>(a, n_frontier_max, st); }
+    launch_hop_t<G, 1>(a, n_frontier_max, st);
+}
 
 static void launch_sample_hop(const SampleHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
-    const int g = sampler_group(a.fanout);
-    const int npb = sampler_npb(g);
-    const unsigned nt = (unsigned)std::max<int64_t>(1, (n_frontier_max + npb - 1) / npb);
-    switch (g) {
-        case 1: k_sample_hop<1, 256><<<nt, kThreads, 0, st>>>(a); break;
-        case 2: k_sample_hop<2, 256><<<nt, kThreads, 0, st>>>(a); break;
-        case 4: k_sample_hop<4, 256><<<nt, kThreads, 0, st>>>(a); break;
-        case 8: k_sample_hop<8, 256><<<nt, kThreads, 0, st>>>(a); break;
-        case 16: k_sample_hop<16, 128><<<nt, kThreads, 0, st>>>(a); break;
-        default: k_sample_hop<32, 64><<<nt, kThreads, 0, st>>>(a); break;
+    switch (sampler_group(a.fanout)) {
+        case 1: launch_hop_g<1>(a, n_frontier_max, st); break;
+        case 2: launch_hop_g<2>(a, n_frontier_max, st); break;
+        case 4: launch_hop_g<4>(a, n_frontier_max, st); break;
+        case 8: launch_hop_g<8>(a, n_frontier_max, st); break;
+        case 16: launch_hop_g<16>(a, n_frontier_max, st); break;
+        default: launch_hop_g<32>(a, n_frontier_max, st); break;
     }
 }
 
@@ -537,7 +556,7 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     }
     int64_t tiles = 1;
     for (int h = 0; h < num_hops; ++h) {
-        tiles = std::max(tiles, ceil_div(nmax[h], 64));
+        tiles = std::max(tiles, ceil_div(nmax[h], 8));   // smallest sampler tile: 8 nodes
         tiles = std::max(tiles, ceil_div(emax[h], kEdgesPerTile));
     }
     if ((s = g->scan.ensure(tiles)) != GD_OK) return s;
