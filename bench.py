@@ -50,6 +50,8 @@ def parse():
     p.add_argument("--prewarm-max", type=int, default=400,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
+    p.add_argument("--pipeline-sweep", default="", help="f1: 'samplers:reorder,...' SET pipeline runs "
+                   "(concurrent sampler streams, out-of-order extraction), results under 'pipeline'")
     p.add_argument("--miss-sweep", default="", help="tuning: 'threads:share:zc_blocks:pull_blocks,...' timed "
                    "one after another in this process (results under 'sweep')")
     return p.parse_args()
@@ -243,7 +245,8 @@ def run_ours(args, rank, world, local_rank):
 
     sweep_cfgs = [tuple(float(x) for x in c.split(":")) for c in args.miss_sweep.split(",") if c]
     PRE = 0 if cfg.preload else args.prewarm_max
-    total = PRE + W + K + (0 if args.no_e2e else K) + len(sweep_cfgs) * (W + K)
+    n_pipe = len([x for x in args.pipeline_sweep.split(",") if x])
+    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe) * (W + K)
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -396,6 +399,35 @@ def run_ours(args, rank, world, local_rank):
         log("sweep", rec)
         sweep.append(rec)
         j0 += W + K
+    # ---- f1: the SET pipeline with S concurrent samplers (optionally out-of-order extraction)
+    pipe_res = []
+    if args.pipeline_sweep:
+        from paper_conf_icpp_jiangj024_b200.pipeline import SETPipeline
+        torch.cuda.synchronize(dev)
+        while pending:                              # hand the buffer over with nothing in flight
+            r = pending.pop(0)
+            buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
+        torch.cuda.synchronize(dev)
+        for spec in args.pipeline_sweep.split(","):
+            S_, ro = spec.split(":")
+            pipe = SETPipeline(g, buf, fan, cfg.batch_size, synth.RNG_SEED, samplers=int(S_), release_lag=Q,
+                               reorder=bool(int(ro)), device=local_rank)
+            nrun = W + K
+            base_j = j0
+            sd = [seeds_dev[(base_j + j) % len(seeds_dev)] for j in range(nrun)]
+            bi = [batch_ids[(base_j + j) % len(batch_ids)] for j in range(nrun)]
+            pipe.run(sd[:W], bi[:W])
+            torch.cuda.synchronize(dev)
+            t0 = time.perf_counter()
+            order, pst = pipe.run(sd[W:], bi[W:])
+            torch.cuda.synchronize(dev)
+            el = time.perf_counter() - t0
+            inversions = sum(1 for a_, b_ in zip(order, order[1:]) if b_ < a_)
+            rec = {"samplers": int(S_), "reorder": bool(int(ro)), "batches_per_s": round(K / el, 1),
+                   "out_of_order_extractions": inversions}
+            log("pipeline", rec)
+            pipe_res.append(rec)
+            j0 += nrun
     status_g = g.check()
     status_b = buf.check()
 
@@ -470,6 +502,7 @@ def run_ours(args, rank, world, local_rank):
                       "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
         "parity": parity,
         "sweep": sweep or None,
+        "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
         "setup_s": round(time.time() - t_setup, 1),
     }

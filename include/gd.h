@@ -120,6 +120,19 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
                     int32_t num_hops, uint64_t rng_seed, uint32_t batch_id, gd_sample_out* out,
                     void* stream);
 
+/* Sampling workspaces.  gd_sample uses the graph's default workspace, so calls on
+ * one graph are stream-ordered on one stream.  Several samplers ("a pool of
+ * threads as samplers") may run concurrently on different streams, each with its own
+ * workspace (relabel hash, scan tile states, seed staging), via gd_sample_ws.  A
+ * workspace must not be used by two calls that may overlap in time. */
+typedef struct gd_workspace gd_workspace;
+gd_status gd_workspace_create(gd_graph* g, gd_workspace** out);
+gd_status gd_workspace_destroy(gd_workspace* w);
+/* gd_sample with an explicit workspace (w = NULL: the graph's default). */
+gd_status gd_sample_ws(gd_graph* g, gd_workspace* w, const int32_t* seeds, int64_t num_seeds,
+                       const int32_t* fanouts, int32_t num_hops, uint64_t rng_seed, uint32_t batch_id,
+                       gd_sample_out* out, void* stream);
+
 /* ----------------------------------------------------------------------------
  * Feature buffer: `capacity_slots` rows of `row_bytes` in HBM, a
  * mapping table {slot, reference count, valid bit} per node, a reverse

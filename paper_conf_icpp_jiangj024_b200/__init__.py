@@ -20,7 +20,7 @@ import torch
 from . import _lib
 from ._lib import GD_MAX_HOPS, GdError, SampleOutC, check, lib
 
-__all__ = ["Graph", "SampleOut", "FeatureBuffer", "GdError", "sample_bounds", "check_device_status", "lib"]
+__all__ = ["Graph", "SampleOut", "Workspace", "FeatureBuffer", "GdError", "sample_bounds", "check_device_status", "lib"]
 
 
 def _ptr(t):
@@ -125,8 +125,8 @@ class Graph:
         return SampleOut(nm, em, self.device, with_eid)
 
     def sample(self, seeds: torch.Tensor, fanouts, rng_seed: int, batch_id: int, out: SampleOut | None = None,
-               stream=None, with_eid: bool = False) -> SampleOut:
-        """gd_sample.  `seeds` int32 on the device or in (pinned) host memory."""
+               stream=None, with_eid: bool = False, workspace: "Workspace | None" = None) -> SampleOut:
+        """gd_sample (gd_sample_ws with a workspace).  `seeds` int32 on the device or in (pinned) host memory."""
         assert seeds.dtype == torch.int32 and seeds.is_contiguous()
         fanouts = list(fanouts)
         if out is None:
@@ -134,9 +134,18 @@ class Graph:
         K = len(fanouts)
         f = (ctypes.c_int32 * K)(*fanouts)
         cs = out.cstruct()
-        check(lib.gd_sample(self._h, _ptr(seeds), seeds.numel(), f, K, ctypes.c_uint64(rng_seed),
-                            ctypes.c_uint32(batch_id & 0xFFFFFFFF), ctypes.byref(cs), _stream_ptr(stream, self.device)))
+        if workspace is None:
+            check(lib.gd_sample(self._h, _ptr(seeds), seeds.numel(), f, K, ctypes.c_uint64(rng_seed),
+                                ctypes.c_uint32(batch_id & 0xFFFFFFFF), ctypes.byref(cs),
+                                _stream_ptr(stream, self.device)))
+        else:
+            check(lib.gd_sample_ws(self._h, workspace.handle, _ptr(seeds), seeds.numel(), f, K,
+                                   ctypes.c_uint64(rng_seed), ctypes.c_uint32(batch_id & 0xFFFFFFFF),
+                                   ctypes.byref(cs), _stream_ptr(stream, self.device)))
         return out
+
+    def workspace(self) -> "Workspace":
+        return Workspace(self)
 
     def check(self):
         return check_device_status(self._h)
@@ -149,6 +158,31 @@ class Graph:
         n = ctypes.c_int64()
         check(lib.gd_graph_timing_read(self._h, ctypes.byref(ms), ctypes.byref(n)))
         return {"sample_ms": ms.value, "calls": n.value}
+
+
+class Workspace:
+    """gd_workspace: sampling scratch for one concurrently sampling stream."""
+
+    def __init__(self, graph: Graph):
+        h = ctypes.c_void_p()
+        check(lib.gd_workspace_create(graph.handle, ctypes.byref(h)))
+        self._h = h
+        self.graph = graph      # keep the graph alive
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            lib.gd_workspace_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:  # noqa: BLE001
+            pass
 
 
 class FeatureBuffer:

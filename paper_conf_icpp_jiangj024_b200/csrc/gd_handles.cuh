@@ -9,18 +9,25 @@
 #include "gd_common.cuh"
 #include "gd_hostpool.h"
 
-// Topology replica + per-call sampling workspace.
+// Per-call sampling workspace; one per concurrently sampling stream.
+struct gd_workspace {
+    uint32_t magic = 0x47445753u;   // "GDWS"
+    int device = 0;
+    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident)
+    int64_t hcap = 0;               // power of two >= 1.25 x max_nodes[K]
+    int32_t* seeds_ws = nullptr;    // staging for host seed arrays
+    int64_t seeds_cap = 0;
+    gd::ScanState scan;
+};
+
+// Topology replica + its default workspace.
 struct gd_graph {
     gd::HandleHdr hdr;
     int64_t N = 0, E = 0;
     int64_t* indptr = nullptr;      // HBM int64[N+1]
     int32_t* indices = nullptr;     // HBM int32[E]
-    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident)
-    int64_t hcap = 0;               // power of two >= 2 * max_nodes[K]
-    int32_t* seeds_ws = nullptr;    // staging for host seed arrays
-    int64_t seeds_cap = 0;
-    gd::ScanState scan;
-    gd::EventTimer timer;            // one pair per gd_sample call
+    gd_workspace ws;                // used by gd_sample
+    gd::EventTimer timer;           // one pair per gd_sample call
 };
 
 // Control block of the standby ring.  Kernels that move head/tail read ctl[p] and

@@ -514,19 +514,48 @@ gd_status gd_graph_destroy(gd_graph* g) {
     DeviceGuard guard(g->hdr.device);
     if (g->indptr) cudaFree(g->indptr);
     if (g->indices) cudaFree(g->indices);
-    if (g->hash) cudaFree(g->hash);
-    if (g->seeds_ws) cudaFree(g->seeds_ws);
+    if (g->ws.hash) cudaFree(g->ws.hash);
+    if (g->ws.seeds_ws) cudaFree(g->ws.seeds_ws);
     if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
-    g->scan.release();
+    g->ws.scan.release();
     g->timer.destroy();
     g->hdr.magic = 0;
     delete g;
     return GD_OK;
 }
 
+gd_status gd_workspace_create(gd_graph* g, gd_workspace** out) {
+    if (!g || g->hdr.magic != kMagicGraph || !out) return set_error(GD_ERR_INVALID, "gd_workspace_create: bad argument");
+    gd_workspace* w = new gd_workspace();
+    w->device = g->hdr.device;
+    *out = w;
+    return GD_OK;
+}
+
+gd_status gd_workspace_destroy(gd_workspace* w) {
+    if (!w) return GD_OK;
+    if (w->magic != 0x47445753u) return set_error(GD_ERR_INVALID, "gd_workspace_destroy: bad handle");
+    DeviceGuard guard(w->device);
+    if (w->hash) cudaFree(w->hash);
+    if (w->seeds_ws) cudaFree(w->seeds_ws);
+    w->scan.release();
+    w->magic = 0;
+    delete w;
+    return GD_OK;
+}
+
 gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const int32_t* fanouts, int32_t num_hops,
                     uint64_t rng_seed, uint32_t batch_id, gd_sample_out* out, void* stream_v) {
+    return gd_sample_ws(g, nullptr, seeds, num_seeds, fanouts, num_hops, rng_seed, batch_id, out, stream_v);
+}
+
+gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int64_t num_seeds,
+                       const int32_t* fanouts, int32_t num_hops, uint64_t rng_seed, uint32_t batch_id,
+                       gd_sample_out* out, void* stream_v) {
     if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_sample: bad graph handle");
+    if (wsp && (wsp->magic != 0x47445753u || wsp->device != g->hdr.device))
+        return set_error(GD_ERR_INVALID, "gd_sample_ws: bad workspace handle");
+    gd_workspace& w = wsp ? *wsp : g->ws;
     if (!out || !fanouts || (num_seeds > 0 && !seeds) || !out->n_id || !out->sizes)
         return set_error(GD_ERR_INVALID, "gd_sample: null pointer");
     int64_t nmax[GD_MAX_HOPS + 1], emax[GD_MAX_HOPS];
@@ -547,38 +576,38 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
     // real batches reach 30-70% of the bound), so the per-batch clear stays small
     int64_t want = 1024;
     while (want < std::max<int64_t>(nmax[num_hops], 1) * 5 / 4 + 1) want *= 2;
-    if (want > g->hcap) {
-        if (g->hash) cudaFree(g->hash);
-        g->hash = nullptr;
-        g->hcap = 0;
-        GD_CUDA(cudaMalloc(&g->hash, 2 * want * sizeof(uint32_t)));
-        g->hcap = want;
+    if (want > w.hcap) {
+        if (w.hash) cudaFree(w.hash);
+        w.hash = nullptr;
+        w.hcap = 0;
+        GD_CUDA(cudaMalloc(&w.hash, 2 * want * sizeof(uint32_t)));
+        w.hcap = want;
     }
     int64_t tiles = 1;
     for (int h = 0; h < num_hops; ++h) {
         tiles = std::max(tiles, ceil_div(nmax[h], 8));   // smallest sampler tile: 8 nodes
         tiles = std::max(tiles, ceil_div(emax[h], kEdgesPerTile));
     }
-    if ((s = g->scan.ensure(tiles)) != GD_OK) return s;
+    if ((s = w.scan.ensure(tiles)) != GD_OK) return s;
 
     const int32_t* seeds_d = seeds;
     if (num_seeds > 0 && !is_device_pointer(seeds)) {
-        if (num_seeds > g->seeds_cap) {
-            if (g->seeds_ws) cudaFree(g->seeds_ws);
-            g->seeds_ws = nullptr;
-            g->seeds_cap = 0;
-            GD_CUDA(cudaMalloc(&g->seeds_ws, num_seeds * sizeof(int32_t)));
-            g->seeds_cap = num_seeds;
+        if (num_seeds > w.seeds_cap) {
+            if (w.seeds_ws) cudaFree(w.seeds_ws);
+            w.seeds_ws = nullptr;
+            w.seeds_cap = 0;
+            GD_CUDA(cudaMalloc(&w.seeds_ws, num_seeds * sizeof(int32_t)));
+            w.seeds_cap = num_seeds;
         }
-        GD_CUDA(cudaMemcpyAsync(g->seeds_ws, seeds, num_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, st));
-        seeds_d = g->seeds_ws;
+        GD_CUDA(cudaMemcpyAsync(w.seeds_ws, seeds, num_seeds * sizeof(int32_t), cudaMemcpyHostToDevice, st));
+        seeds_d = w.seeds_ws;
     }
 
-    uint32_t* hk = g->hash;
-    uint32_t* hv = g->hash + g->hcap;
-    const uint32_t mask = (uint32_t)(g->hcap - 1);
+    uint32_t* hk = w.hash;
+    uint32_t* hv = w.hash + w.hcap;
+    const uint32_t mask = (uint32_t)(w.hcap - 1);
     const int tslot = g->timer.on ? g->timer.begin(st) : -1;
-    GD_CUDA(cudaMemsetAsync(g->hash, 0xFF, 2 * g->hcap * sizeof(uint32_t), st));
+    GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 2 * w.hcap * sizeof(uint32_t), st));
     k_seed_intake<<<(unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads)), kThreads, 0, st>>>(
         seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status);
 
@@ -600,13 +629,13 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
         a.hkeys = hk;
         a.hvals = hv;
         a.mask = mask;
-        a.st = g->scan.use();
-        a.st_clear = g->scan.other();
-        a.st_clear_n = g->scan.cap;
+        a.st = w.scan.use();
+        a.st_clear = w.scan.other();
+        a.st_clear_n = w.scan.cap;
         a.status = g->hdr.dev_status;
         launch_sample_hop(a, nmax[h - 1], st);
         GD_DEBUG_AFTER("k_sample_hop", st);
-        g->scan.flip();
+        w.scan.flip();
 
         RelabelArgs r;
         r.col = out->col[h - 1];
@@ -616,13 +645,13 @@ gd_status gd_sample(gd_graph* g, const int32_t* seeds, int64_t num_seeds, const 
         r.K = num_hops;
         r.hkeys = hk;
         r.hvals = hv;
-        r.st = g->scan.use();
-        r.st_clear = g->scan.other();
-        r.st_clear_n = g->scan.cap;
+        r.st = w.scan.use();
+        r.st_clear = w.scan.other();
+        r.st_clear_n = w.scan.cap;
         const int64_t et = std::max<int64_t>(1, ceil_div(emax[h - 1], kEdgesPerTile));
         k_relabel_hop<<<(unsigned)et, kThreads, 0, st>>>(r);
         GD_DEBUG_AFTER("k_relabel_hop", st);
-        g->scan.flip();
+        w.scan.flip();
     }
     ColResolveArgs c;
     int64_t emax_all = 1;

@@ -285,3 +285,51 @@ def test_extract_empty_batch(gd):
     buf.release(ids, n, 8)
     assert buf.check() == 0
     assert buf.snapshot()["standby"].tolist() == list(range(20))
+
+
+# ----------------------------------------------------------------------- f1 pipeline
+
+
+@pytest.mark.parametrize("samplers,reorder", [(1, False), (3, False), (3, True), (4, True)])
+def test_pipeline_parity_in_extraction_order(gd, samplers, reorder):
+    """SET pipeline with S concurrent sampler streams (own workspaces) and out-of-order
+    extraction: the oracle replayed in the recorded extraction order gives the same
+    alias, hit/miss counts and rows, and the same final buffer state."""
+    from paper_conf_icpp_jiangj024_b200.pipeline import SETPipeline
+    N, E, B, fan, Q = 40_000, 400_000, 300, [10, 5], 3
+    indptr, indices = make_graph(N, E, seed=12)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, 64)
+    nb, _ = O.sample_bounds(B, fan, N, E)
+    S = Q * nb[-1]
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, Q, nb[-1])
+    order = synth.epoch_order(synth.train_nodes(N, 0.3))
+    seeds = [order[b * B:(b + 1) * B].cuda() for b in range(24)]
+    bids = list(range(100, 124))
+    rows = {}
+
+    def consumer(k, out, alias, done):
+        done.synchronize()
+        rows[k] = (out.cpu().numpy().copy(), alias.cpu().numpy().copy())
+
+    pipe = SETPipeline(g, buf, fan, B, 7, samplers=samplers, release_lag=Q, reorder=reorder)
+    ext_order, stats = pipe.run(seeds, bids, consumer=consumer)
+    torch.cuda.synchronize()
+    assert sorted(ext_order) == list(range(24))
+    ob = O.Buffer(feat, S)
+    pend = []
+    ip, ix = indptr.numpy(), indices.numpy()
+    for k in ext_order:
+        ref = O.sample(ip, ix, seeds[k].cpu().numpy(), fan, 7, bids[k])
+        o_out, o_alias, o_st = ob.extract(ref.n_id)
+        n = len(ref.n_id)
+        out, alias = rows[k]
+        assert tuple(stats[k].cpu().tolist()[:2]) == o_st
+        assert np.array_equal(alias[:n], o_alias) and np.array_equal(out[:n], o_out)
+        pend.append(ref.n_id)
+        if len(pend) == Q:
+            ob.release(pend.pop(0))
+    while pend:
+        ob.release(pend.pop(0))
+    compare_state(buf, ob)
+    assert buf.check() == 0 and g.check() == 0
