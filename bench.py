@@ -453,7 +453,7 @@ def run_ours(args, rank, world, local_rank):
     rnd = lambda x, k=2: round(x, k) if x is not None else None  # noqa: E731
     roof_gather = {"bound": "hbm", "achieved": rnd(gather_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
                    "frac": rnd(gather_gbs / hbm_peak, 4) if gather_gbs and hbm_peak else None, "traffic": None,
-                   "kernel": "k_gather_hits", "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+                   "kernel": "k_gather_rows", "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
     roof_miss = {"bound": "host_link", "achieved": rnd(link_gbs), "peak": round(link_peak, 2), "unit": "GB/s",
                  "frac": rnd(link_gbs / link_peak, 4) if link_gbs else None, "traffic": None,
                  "kernel": "k_miss_copy (zero-copy share) + k_miss_copy<staged> (pull of the host-gathered share)",
