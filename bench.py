@@ -491,7 +491,10 @@ def run_ours(args, rank, world, local_rank):
                    "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
                        (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.num_nodes * R * 1e-9)},
         "e2e": e2e,
-        "gpu_launches": K * (2 * len(fan) + 8),
+        # per step: seed intake + K x (sample, relabel) + col resolve | lookup, pop/assign, hit gather
+        # [+ zero-copy miss copy unless preload] [+ staged pull when the host path is on] | compact, release
+        "gpu_launches": K * ((2 * len(fan) + 2) + 3 + (0 if cfg.preload else 1)
+                             + (1 if (miss_staged > 0 or tb["miss_staged_ms"] > 1e-3) and not cfg.preload else 0) + 2),
         "roofline": dominant,
         "roofline_gather": roof_gather,
         "roofline_miss": roof_miss,
