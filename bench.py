@@ -43,6 +43,9 @@ def parse():
     p.add_argument("--warmup", type=int, default=16)
     p.add_argument("--config", default="papers100m", choices=sorted(synth.CONFIGS))
     p.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    p.add_argument("--batch-size", type=int, default=None, help="f3 sweep override (Fig. 10)")
+    p.add_argument("--feat-dim", type=int, default=None, help="f3 sweep override (Fig. 8)")
+    p.add_argument("--buffer-frac", type=float, default=None, help="f3 sweep override (Fig. 12)")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the oracle cpu_baseline sample")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
@@ -211,11 +214,25 @@ class Workload:
 
 # ----------------------------------------------------------------------------- our arm
 
+def config_from_args(args):
+    import dataclasses
+    cfg = synth.CONFIGS[args.config]
+    over = {}
+    if args.batch_size:
+        over["batch_size"] = args.batch_size
+    if args.feat_dim:
+        over["feat_dim"] = args.feat_dim
+    if args.buffer_frac is not None:
+        over["buffer_frac"] = args.buffer_frac
+        over["preload"] = False
+    return dataclasses.replace(cfg, **over) if over else cfg
+
+
 def run_ours(args, rank, world, local_rank):
     import paper_conf_icpp_jiangj024_b200 as gd
     from paper_conf_icpp_jiangj024_b200.multigpu import barrier, batch_schedule, max_over_ranks, sum_over_ranks
 
-    cfg = synth.CONFIGS[args.config]
+    cfg = config_from_args(args)
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
     want_cpu = (not args.no_cpu_baseline) and rank == 0 and world == 1
@@ -595,7 +612,7 @@ def run_reference(args, rank, world, local_rank):
     if rank != 0:
         return
     from oracle import oracle as O
-    cfg = synth.CONFIGS[args.config]
+    cfg = config_from_args(args)
     dev = torch.device("cuda", local_rank) if torch.cuda.is_available() else torch.device("cpu")
     wl = Workload(cfg, 0, 1, dev, True)
     del wl.indptr, wl.indices
