@@ -193,9 +193,11 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  * function, so still stream-ordered, no caller sync); phase 2, a kernel pulls the
  * slot contiguously over the host link.  K0 = floor(M * zero_copy_share).
  *   host_threads     0 disables the staged path (all misses zero-copy).
- *   zero_copy_share  in [0, 1]; < 0 = adaptive: 1 - r_host / r_link, with r_host the
- *                    measured host gather rate and r_link the contiguous pull rate of
- *                    the host link, calibrated when this call enables adaptation.
+ *   zero_copy_share  in [0, 1]; < 0 = adaptive, from the measured zero-copy rate r_zc
+ *                    and host gather rate r_host and the contiguous pull rate r_link of
+ *                    the host link (calibrated when this call enables adaptation):
+ *                    r_zc / (r_zc + r_host) if r_zc + r_host <= r_link, else
+ *                    1 - r_host / r_link; clamped to [0.05, 0.9].
  *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
  *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs

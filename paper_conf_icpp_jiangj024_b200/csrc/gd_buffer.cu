@@ -834,6 +834,7 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     b->alpha_fixed = zero_copy_share >= 0;
     b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.2);
     b->r_host = 0;
+    b->r_zc = 0;
     if (host_threads > 0 && !b->alpha_fixed) {
         gd_status st = calibrate_link(b);
         if (st != GD_OK) return st;
@@ -879,23 +880,39 @@ static void CUDART_CB host_gather_cb(void* arg) {
     if (b->timer.on) b->timer_host_ms += ss->cpu_ms;   // serialised on stream H
 }
 
-// Zero-copy share alpha.  The staged path moves rows with contiguous (cheap to
-// translate) host-link reads but is capped by the host gather rate r_host; the
-// zero-copy path is capped by the host's random-translation rate and competes for the
-// same link.  The fastest split lets the staged path run at r_host and tops the link
-// up with zero-copy: alpha = 1 - r_host / r_link (r_link calibrated at config time).
+// Zero-copy share alpha.  Both miss paths have their own cap: the zero-copy copy the
+// host's random-translation rate (r_zc; a row rate, so small rows move few bytes), the
+// staged path the host gather rate r_host; both share the host link r_link.  Minimising
+// max(alpha B / r_zc, (1 - alpha) B / r_host, B / r_link):
+//   r_zc + r_host <= r_link: balance the paths, alpha = r_zc / (r_zc + r_host);
+//   otherwise the link binds and the smallest zero-copy share that keeps the staged path
+//   within it is best (zero-copy loads also slow the SMs they run on):
+//   alpha = 1 - r_host / r_link.
 static void adapt_alpha(gd_buffer* b, int d) {
     StagedSlot& ss = b->stg[d];
     if (b->alpha_fixed || ss.batch < 0 || b->r_link <= 0) return;
-    if (cudaEventQuery(b->ev_E[d]) != cudaSuccess) {   // that batch's host gather still running
-        cudaGetLastError();
+    if (cudaEventQuery(b->ev_E[d]) != cudaSuccess || cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
+        cudaGetLastError();                     // that batch is still in flight
         return;
     }
-    const double staged_rows = (double)ss.h_meta[2];
-    if (staged_rows < 2048 || ss.cpu_ms <= 0) return;
-    const double r = staged_rows * (double)b->R / ss.cpu_ms;
-    b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
-    b->alpha = std::min(0.9, std::max(0.0, 1.0 - b->r_host / b->r_link));
+    const double staged_rows = (double)ss.h_meta[2], zc_rows = (double)ss.h_meta[1];
+    if (staged_rows >= 2048 && ss.cpu_ms > 0) {
+        const double r = staged_rows * (double)b->R / ss.cpu_ms;
+        b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
+    }
+    float tz = 0;
+    if (zc_rows >= 2048 && cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]) == cudaSuccess && tz > 0) {
+        const double r = zc_rows * (double)b->R / tz;
+        b->r_zc = b->r_zc > 0 ? 0.7 * b->r_zc + 0.3 * r : r;
+    }
+    cudaGetLastError();
+    if (b->r_host <= 0) return;
+    double a;
+    if (b->r_zc > 0 && b->r_zc + b->r_host <= b->r_link)
+        a = b->r_zc / (b->r_zc + b->r_host);
+    else
+        a = 1.0 - b->r_host / b->r_link;
+    b->alpha = std::min(0.9, std::max(0.05, a));
 }
 
 // Contiguous host-link pull rate (bytes/ms), measured once on the staging memory.

@@ -100,6 +100,7 @@ struct gd_buffer {
     int pull_blocks = 8;                 // 1024-thread blocks of the staged pull
     double alpha = 1.0;                  // zero-copy share of the misses (adapted)
     double r_host = 0;                   // EMA of the host gather rate (bytes/ms)
+    double r_zc = 0;                     // EMA of the zero-copy copy rate (bytes/ms)
     double r_link = 0;                   // contiguous pull rate of the host link (bytes/ms), calibrated
     bool alpha_fixed = false;
     gd::HostGatherPool* pool = nullptr;
