@@ -657,8 +657,14 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch.distributed as dist
-        torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        if os.environ.get("GD_BENCH_SAME_DEVICE") == "1":
+            # test mode for 1-GPU boxes: every rank on cuda:0, gloo (NCCL refuses shared GPUs)
+            local_rank = 0
+            torch.cuda.set_device(0)
+            dist.init_process_group("gloo")
+        else:
+            torch.cuda.set_device(local_rank)
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
     try:
         if args.impl == "reference":
             run_reference(args, rank, world, local_rank)

@@ -44,6 +44,8 @@ def max_over_ranks(x: float, device=None) -> float:
     """Max of a per-rank scalar (timings are reported as the slowest rank)."""
     if not (dist.is_available() and dist.is_initialized()):
         return float(x)
+    if dist.get_backend() == "gloo":
+        device = None
     t = torch.tensor([float(x)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.MAX)
     return float(t.item())
@@ -52,6 +54,8 @@ def max_over_ranks(x: float, device=None) -> float:
 def sum_over_ranks(x: float, device=None) -> float:
     if not (dist.is_available() and dist.is_initialized()):
         return float(x)
+    if dist.get_backend() == "gloo":
+        device = None
     t = torch.tensor([float(x)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
