@@ -176,19 +176,29 @@ class Workload:
         self.indptr, self.indices = indptr, indices
         t0 = time.time()
         self.table = HostTable(cfg.num_nodes, cfg.row_bytes, cfg.name, rank, world)
-        # page-lock + map once here, so FeatureBuffer re-inits (parity / preload) skip it
-        rc = torch.cuda.cudart().cudaHostRegister(self.table.tensor.data_ptr(), cfg.num_nodes * cfg.row_bytes, 3)
-        if int(rc) != 0:
-            raise RuntimeError(f"cudaHostRegister(host table) failed: {rc}")
-        self.t_table_alloc = time.time() - t0
+        # page-lock + map once here, so FeatureBuffer re-inits (parity / preload) skip it.
+        # Multi-rank: rank 0 registers (faulting the shared pages in) and fills first; the
+        # others register afterwards, one at a time (concurrent first-touch pinning of the
+        # same tmpfs pages by several processes fails).
         self.rank, self.world, self.device = rank, world, device
+        self._barrier = barrier
+        if rank == 0:
+            self._register()
+        self.t_table_alloc = time.time() - t0
         train, nb = train_batches(cfg, device)
         self.train, self.num_batches = train, nb
         self._orders = {}
         self._barrier = barrier
 
+    def _register(self):
+        n = self.cfg.num_nodes * self.cfg.row_bytes
+        rc = torch.cuda.cudart().cudaHostRegister(self.table.tensor.data_ptr(), n, 3)
+        if int(rc) != 0:
+            raise RuntimeError(f"cudaHostRegister(host table, {n} bytes) failed: code {int(rc)}")
+
     def fill_table(self):
-        """Rank 0 writes the feature rows (generated on the GPU) into the host table."""
+        """Rank 0 writes the feature rows (generated on the GPU) into the host table; then
+        the other ranks register the (now resident) shared pages one after another."""
         t0 = time.time()
         if self.table.owner:
             cfg = self.cfg
@@ -198,6 +208,10 @@ class Workload:
                 self.table.tensor[s:e].copy_(synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
         torch.cuda.synchronize(self.device)
         self._barrier()
+        for r in range(1, self.world):
+            if self.rank == r:
+                self._register()
+            self._barrier()
         self.t_fill = time.time() - t0
 
     def close(self):
@@ -247,16 +261,13 @@ def run_ours(args, rank, world, local_rank):
     nm, em = g.bounds(cfg.batch_size, fan)
     n_max = nm[-1]
     S = capacity_for(cfg, n_max)
+    wl.fill_table()
     t0 = time.time()
-    buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=False, device=local_rank)
+    buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
     t_register = time.time() - t0
     host_threads = max(1, min(13, len(os.sched_getaffinity(0)) // world - 3))
     if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
         buf.config(host_threads)
-    wl.fill_table()
-    if cfg.preload:   # "all features resident": rebuild with the filled table preloaded
-        buf.close()
-        buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=True, device=local_rank)
     log(f"setup: graph {wl.t_graph:.1f}s table alloc {wl.t_table_alloc:.1f}s register {t_register:.1f}s "
         f"fill {wl.t_fill:.1f}s; N={cfg.num_nodes} E={cfg.num_edges} S={S} n_max={n_max} deg={wl.deg_stats}")
 
