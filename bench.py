@@ -175,7 +175,7 @@ class Workload:
         self.host_indices = indices.cpu().numpy() if need_host_csr else None
         self.indptr, self.indices = indptr, indices
         t0 = time.time()
-        self.table = HostTable(cfg.num_nodes, cfg.row_bytes, cfg.name, rank, world)
+        self.table = HostTable(cfg.host_rows, cfg.row_bytes, cfg.name, rank, world)
         # page-lock + map once here, so FeatureBuffer re-inits (parity / preload) skip it.
         # Multi-rank: rank 0 registers (faulting the shared pages in) and fills first; the
         # others register afterwards, one at a time (concurrent first-touch pinning of the
@@ -191,7 +191,7 @@ class Workload:
         self._barrier = barrier
 
     def _register(self):
-        n = self.cfg.num_nodes * self.cfg.row_bytes
+        n = self.cfg.host_rows * self.cfg.row_bytes
         rc = torch.cuda.cudart().cudaHostRegister(self.table.tensor.data_ptr(), n, 3)
         if int(rc) != 0:
             raise RuntimeError(f"cudaHostRegister(host table, {n} bytes) failed: code {int(rc)}")
@@ -203,8 +203,8 @@ class Workload:
         if self.table.owner:
             cfg = self.cfg
             chunk = max(1, (256 << 20) // cfg.row_bytes)
-            for s in range(0, cfg.num_nodes, chunk):
-                e = min(cfg.num_nodes, s + chunk)
+            for s in range(0, cfg.host_rows, chunk):
+                e = min(cfg.host_rows, s + chunk)
                 self.table.tensor[s:e].copy_(synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
         torch.cuda.synchronize(self.device)
         self._barrier()
@@ -263,7 +263,8 @@ def run_ours(args, rank, world, local_rank):
     S = capacity_for(cfg, n_max)
     wl.fill_table()
     t0 = time.time()
-    buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
+    buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank,
+                           num_nodes=cfg.num_nodes)
     t_register = time.time() - t0
     host_threads = max(1, min(13, len(os.sched_getaffinity(0)) // world - 3))
     if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
@@ -326,7 +327,8 @@ def run_ours(args, rank, world, local_rank):
         log("parity check ...")
         parity = check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev)
         buf.close()
-        buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank)
+        buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank,
+                               num_nodes=cfg.num_nodes)
         if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
             buf.config(host_threads)
     barrier()
@@ -517,7 +519,8 @@ def run_ours(args, rank, world, local_rank):
                    "buffer_prewarm_batches": prewarm_batches,
                    "parallelism": f"dp{world} (batch segments, no collective)",
                    "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
-                       (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.num_nodes * R * 1e-9)},
+                       (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.host_rows * R * 1e-9),
+                   "host_table_rows": cfg.host_rows},
         "e2e": e2e,
         # per step: seed intake + K x (sample, relabel) + col resolve | lookup, pop/assign, hit gather
         # [+ zero-copy miss copy unless preload] [+ staged pull when the host path is on] | compact, release
@@ -562,7 +565,7 @@ def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
     checked bit-exactly against the oracle (sampling outputs, alias, hit/miss, out rows)."""
     from oracle import oracle as O
     t0 = time.time()
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
     log(f"  oracle buffer ready {time.time() - t0:.1f}s")
     res_ok = True
     checked = 0
@@ -595,7 +598,7 @@ def cpu_baseline(cfg, wl, sched, batch_ids, fan, S, budget_s):
     """The oracle as it stands, single-threaded on this host, on a bounded sample of the same
     workload: full steps (sample + Alg. 1 extract + release with lag Q) until budget_s."""
     from oracle import oracle as O
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
     pend = []
     n = 0
     t0 = time.perf_counter()
@@ -634,7 +637,7 @@ def run_reference(args, rank, world, local_rank):
     from paper_conf_icpp_jiangj024_b200.multigpu import batch_schedule
     sched = batch_schedule(wl.num_batches, 0, 1, args.warmup + args.steps)
     bids = [ep * wl.num_batches + b for b, ep in sched]
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload)
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
     pend = []
     t0 = None
     for j, (b, ep) in enumerate(sched):

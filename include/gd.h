@@ -156,6 +156,13 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* w, const int32_t* seeds, int64
 gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_bytes,
                          int64_t capacity_slots, int32_t max_inflight,
                          int64_t max_nodes_per_batch, int preload, int device, gd_buffer** out);
+/* As gd_buffer_init, but the host table holds only `table_rows` rows (1 <= table_rows <=
+ * num_nodes) and node v's feature row is table row (v mod table_rows): a bounded physical
+ * table for workloads whose full table exceeds host memory (the mag240m config: 375 GB
+ * logical).  The same bytes cross the host link per miss. */
+gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t num_nodes, int64_t row_bytes,
+                             int64_t capacity_slots, int32_t max_inflight, int64_t max_nodes_per_batch,
+                             int preload, int device, gd_buffer** out);
 gd_status gd_buffer_destroy(gd_buffer* b);
 
 /* ----------------------------------------------------------------------------

@@ -197,8 +197,8 @@ int oracle_sample(const int64_t* indptr, const int32_t* indices, int64_t num_nod
 struct MapEntry { int32_t slot; int32_t rc; uint8_t valid; };
 
 struct OracleBuffer {
-    const uint8_t* feat;      /* host table [N x R], ascending node id */
-    int64_t N, R, S;
+    const uint8_t* feat;      /* host table [P x R]; node v's row is row v mod P (P = N normally) */
+    int64_t N, R, S, P;
     std::vector<MapEntry> map;             /* mapping table */
     std::vector<int32_t> reverse;          /* reverse mapping array */
     std::list<int32_t> standby;            /* LRU order: head = least recently used */
@@ -222,11 +222,16 @@ static void standby_remove(OracleBuffer* B, int32_t s) {   /* Alg. 1 line 11 */
 /* Initial state (C6, C14): every map entry {-1, 0, 0}, reverse = -1, standby =
  * [0, 1, ..., S-1] (ascending; "slot 2 is the first available free slot").
  * preload (requires S >= N): node v resident in slot v, valid, rc 0. */
+/* Feature row of node v: the table holds P rows, node v's features are row (v mod P)
+ * (P = N is the paper's layout; P < N is the bounded table of the mag240m config). */
+static const uint8_t* feat_row(const OracleBuffer* B, int64_t v) { return B->feat + (size_t)(v % B->P) * B->R; }
+
 void* oracle_buffer_create(const uint8_t* host_feat, int64_t num_nodes, int64_t row_bytes,
-                           int64_t capacity_slots, int preload) {
+                           int64_t capacity_slots, int preload, int64_t table_rows) {
     if (preload && capacity_slots < num_nodes) return nullptr;
+    if (table_rows < 1 || table_rows > num_nodes) return nullptr;
     OracleBuffer* B = new OracleBuffer();
-    B->feat = host_feat; B->N = num_nodes; B->R = row_bytes; B->S = capacity_slots;
+    B->feat = host_feat; B->N = num_nodes; B->R = row_bytes; B->S = capacity_slots; B->P = table_rows;
     B->map.assign(num_nodes, MapEntry{-1, 0, 0});
     B->reverse.assign(capacity_slots, -1);
     B->where.resize(capacity_slots);
@@ -238,7 +243,7 @@ void* oracle_buffer_create(const uint8_t* host_feat, int64_t num_nodes, int64_t 
         for (int64_t v = 0; v < num_nodes; ++v) {
             B->map[v] = MapEntry{(int32_t)v, 0, 1};
             B->reverse[v] = (int32_t)v;
-            std::memcpy(&B->slots[(size_t)v * row_bytes], host_feat + (size_t)v * row_bytes, row_bytes);
+            std::memcpy(&B->slots[(size_t)v * row_bytes], feat_row(B, v), row_bytes);
         }
     }
     return B;
@@ -284,7 +289,7 @@ int oracle_extract(void* h, const int32_t* ids, int64_t n, uint8_t* out, int32_t
         B->reverse[index] = id;                               /* line 28 */
         ids_r[i] = index;                                     /* line 29 */
         /* lines 30-36: load from the table (the SSD stand-in) into the slot */
-        std::memcpy(&B->slots[(size_t)index * B->R], B->feat + (size_t)id * B->R, B->R);
+        std::memcpy(&B->slots[(size_t)index * B->R], feat_row(B, id), B->R);
         B->map[id].valid = 1;                                 /* line 37 */
         ++misses;
     }
@@ -340,7 +345,7 @@ int oracle_buffer_set_state(void* h, const int32_t* map_slot, const int32_t* map
     for (int64_t k = 0; k < standby_len; ++k) standby_push_back(B, standby[k]);
     for (int64_t v = 0; v < B->N; ++v)
         if (B->map[v].valid && B->map[v].slot >= 0)
-            std::memcpy(&B->slots[(size_t)B->map[v].slot * B->R], B->feat + (size_t)v * B->R, B->R);
+            std::memcpy(&B->slots[(size_t)B->map[v].slot * B->R], feat_row(B, v), B->R);
     return 0;
 }
 

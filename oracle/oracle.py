@@ -56,7 +56,8 @@ def lib():
                                     ctypes.POINTER(_i64p), ctypes.POINTER(_i32p),
                                     ctypes.POINTER(_i64p), _i64p]
         L.oracle_sample.restype = ctypes.c_int
-        L.oracle_buffer_create.argtypes = [_u8p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int]
+        L.oracle_buffer_create.argtypes = [_u8p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                                           ctypes.c_int64]
         L.oracle_buffer_create.restype = ctypes.c_void_p
         L.oracle_buffer_destroy.argtypes = [ctypes.c_void_p]
         L.oracle_buffer_destroy.restype = None
@@ -161,14 +162,16 @@ def sample(indptr: np.ndarray, indices: np.ndarray, seeds: np.ndarray, fanouts, 
 class Buffer:
     """Algorithm 1 feature buffer over a host table feat[N, R] (uint8 view)."""
 
-    def __init__(self, feat_u8: np.ndarray, capacity_slots: int, preload: bool = False):
+    def __init__(self, feat_u8: np.ndarray, capacity_slots: int, preload: bool = False, num_nodes: int | None = None):
+        """feat_u8 [P, R]: node v's row is feat_u8[v mod P]; num_nodes defaults to P."""
         assert feat_u8.dtype == np.uint8 and feat_u8.ndim == 2 and feat_u8.flags.c_contiguous
         self.feat = feat_u8
-        self.N, self.R = feat_u8.shape
+        self.P, self.R = feat_u8.shape
+        self.N = int(num_nodes) if num_nodes is not None else self.P
         self.S = int(capacity_slots)
-        self.h = lib().oracle_buffer_create(_p(feat_u8, _u8p), self.N, self.R, self.S, int(preload))
+        self.h = lib().oracle_buffer_create(_p(feat_u8, _u8p), self.N, self.R, self.S, int(preload), self.P)
         if not self.h:
-            raise ValueError("oracle_buffer_create: preload requires capacity >= N")
+            raise ValueError("oracle_buffer_create: preload requires capacity >= N, and 1 <= P <= N")
 
     def __del__(self):
         if getattr(self, "h", None):

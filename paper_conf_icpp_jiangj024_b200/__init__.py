@@ -189,18 +189,22 @@ class FeatureBuffer:
     """gd_buffer: slot-managed HBM feature buffer over a pinned host table (the SSD stand-in)."""
 
     def __init__(self, host_feat: torch.Tensor, capacity: int, max_inflight: int, max_nodes_per_batch: int,
-                 preload: bool = False, device: int = 0):
+                 preload: bool = False, device: int = 0, num_nodes: int | None = None):
+        """`host_feat` [P, R] uint8; node v's row is host_feat[v mod P] when num_nodes > P
+        (gd_buffer_init_mod), else P = num_nodes (gd_buffer_init)."""
         assert host_feat.device.type == "cpu" and host_feat.dtype == torch.uint8 and host_feat.dim() == 2
         assert host_feat.is_contiguous()
         self.host_feat = host_feat          # keep alive until destroy
-        self.num_nodes, self.row_bytes = host_feat.shape
+        self.table_rows, self.row_bytes = host_feat.shape
+        self.num_nodes = int(num_nodes) if num_nodes is not None else self.table_rows
         self.capacity = int(capacity)
         self.max_inflight = int(max_inflight)
         self.max_nodes_per_batch = int(max_nodes_per_batch)
         self.device = device
         h = ctypes.c_void_p()
-        check(lib.gd_buffer_init(_ptr(host_feat), self.num_nodes, self.row_bytes, self.capacity, self.max_inflight,
-                                 self.max_nodes_per_batch, int(preload), device, ctypes.byref(h)))
+        check(lib.gd_buffer_init_mod(_ptr(host_feat), self.table_rows, self.num_nodes, self.row_bytes, self.capacity,
+                                     self.max_inflight, self.max_nodes_per_batch, int(preload), device,
+                                     ctypes.byref(h)))
         self._h = h
         sp = lib.gd_buffer_side_stream(h)
         self.side_stream = torch.cuda.ExternalStream(sp, device=torch.device("cuda", device))

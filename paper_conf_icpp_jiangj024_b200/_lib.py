@@ -22,7 +22,7 @@ EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy",
            "gd_buffer_init", "gd_buffer_destroy", "gd_extract", "gd_buffer_release", "gd_check_device_status",
            "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream", "gd_buffer_timing",
            "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config",
-           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws"]
+           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod"]
 
 
 class GdError(RuntimeError):
@@ -63,6 +63,8 @@ def _load():
     L.gd_sample_ws.argtypes = [_vp, _vp, _vp, _i64, _vp, _i32, ctypes.c_uint64, ctypes.c_uint32,
                                ctypes.POINTER(SampleOutC), _vp]
     L.gd_buffer_init.argtypes = [_vp, _i64, _i64, _i64, _i32, _i64, ctypes.c_int, ctypes.c_int, ctypes.POINTER(_vp)]
+    L.gd_buffer_init_mod.argtypes = [_vp, _i64, _i64, _i64, _i64, _i32, _i64, ctypes.c_int, ctypes.c_int,
+                                     ctypes.POINTER(_vp)]
     L.gd_buffer_destroy.argtypes = [_vp]
     L.gd_extract.argtypes = [_vp, _vp, _vp, _i64, _vp, _vp, _vp, _vp, _vp]
     L.gd_buffer_release.argtypes = [_vp, _vp, _vp, _i64, _vp]

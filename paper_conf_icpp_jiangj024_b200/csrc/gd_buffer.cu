@@ -328,7 +328,8 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
 template <int UNROLL, bool STAGED>
 __global__ void __launch_bounds__(1024, 1) k_miss_copy(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
                                                    const int64_t* __restrict__ end, const uint8_t* __restrict__ src,
-                                                   uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+                                                   uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R,
+                                                   int64_t P) {
     const int64_t k0 = begin ? *begin : 0;
     const int64_t M = *end - k0;
     const int64_t cpr = R >> 4;                     // 16-byte chunks per row
@@ -344,7 +345,8 @@ __global__ void __launch_bounds__(1024, 1) k_miss_copy(const int4* __restrict__ 
             if (idx < total) {
                 const int64_t r = idx / cpr, c = idx - r * cpr;
                 const int4 tr = __ldg(trip + k0 + r);
-                const uint4* sp = STAGED ? (const uint4*)(src + r * R) + c : (const uint4*)(src + (int64_t)tr.x * R) + c;
+                const int64_t row = (int64_t)tr.x < P ? (int64_t)tr.x : (int64_t)tr.x % P;   // table row of node
+                const uint4* sp = STAGED ? (const uint4*)(src + r * R) + c : (const uint4*)(src + row * R) + c;
                 asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
                              : "=r"(val[u].x), "=r"(val[u].y), "=r"(val[u].z), "=r"(val[u].w)
                              : "l"(sp));
@@ -366,7 +368,7 @@ __global__ void __launch_bounds__(1024, 1) k_miss_copy(const int4* __restrict__ 
 template <bool STAGED>
 __global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __restrict__ begin,
                                const int64_t* __restrict__ end, const uint8_t* __restrict__ src,
-                               uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+                               uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R, int64_t P) {
     const int64_t k0 = begin ? *begin : 0;
     const int64_t M = *end - k0;
     const int64_t cpr = R >> 2;
@@ -375,7 +377,8 @@ __global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __r
          idx += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = idx / cpr, c = idx - r * cpr;
         const int4 tr = trip[k0 + r];
-        const uint32_t v = STAGED ? ((const uint32_t*)(src + r * R))[c] : ((const uint32_t*)(src + (int64_t)tr.x * R))[c];
+        const int64_t row = (int64_t)tr.x % P;
+        const uint32_t v = STAGED ? ((const uint32_t*)(src + r * R))[c] : ((const uint32_t*)(src + row * R))[c];
         ((uint32_t*)(slots + (int64_t)tr.y * R))[c] = v;
         ((uint32_t*)(out + (int64_t)tr.z * R))[c] = v;
     }
@@ -669,7 +672,16 @@ extern "C" {
 gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_bytes, int64_t capacity_slots,
                          int32_t max_inflight, int64_t max_nodes_per_batch, int preload, int device,
                          gd_buffer** out) {
+    return gd_buffer_init_mod(host_feat, num_nodes, num_nodes, row_bytes, capacity_slots, max_inflight,
+                              max_nodes_per_batch, preload, device, out);
+}
+
+gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t num_nodes, int64_t row_bytes,
+                             int64_t capacity_slots, int32_t max_inflight, int64_t max_nodes_per_batch, int preload,
+                             int device, gd_buffer** out) {
     if (!host_feat || !out) return set_error(GD_ERR_INVALID, "gd_buffer_init: null pointer");
+    if (table_rows < 1 || table_rows > num_nodes)
+        return set_error(GD_ERR_INVALID, "gd_buffer_init_mod: need 1 <= table_rows <= num_nodes");
     if (num_nodes < 1 || num_nodes > 0x7FFFFFFFLL || row_bytes < 4 || (row_bytes & 3) ||
         capacity_slots < 1 || max_inflight < 1 || max_nodes_per_batch < 1)
         return set_error(GD_ERR_INVALID, "gd_buffer_init: bad size (row_bytes must be a positive multiple of 4)");
@@ -694,6 +706,7 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     b->Q = max_inflight;
     b->preload = preload;
     b->host_feat = host_feat;
+    b->P = table_rows;
     b->D = max_inflight + 2;
     auto fail = [&](gd_status s) {
         buffer_free(b);
@@ -704,7 +717,7 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     bool pinned = (cudaPointerGetAttributes(&pa, host_feat) == cudaSuccess && pa.type == cudaMemoryTypeHost);
     cudaGetLastError();
     if (!pinned) {
-        cudaError_t e = cudaHostRegister((void*)host_feat, (size_t)num_nodes * row_bytes,
+        cudaError_t e = cudaHostRegister((void*)host_feat, (size_t)table_rows * row_bytes,
                                          cudaHostRegisterMapped | cudaHostRegisterPortable);
         if (e != cudaSuccess) return fail(cuda_error(e, "cudaHostRegister(host_feat)"));
         b->registered = true;
@@ -757,8 +770,12 @@ gd_status gd_buffer_init(const void* host_feat, int64_t num_nodes, int64_t row_b
     k_init_map<<<148 * 8, 256>>>(b->map, num_nodes, preload);
     k_init_slots<<<148 * 8, 256>>>(b->reverse, b->pos_of_slot, b->ring, capacity_slots, num_nodes, preload);
     if (preload) {
-        cudaError_t e = cudaMemcpy(b->slots, host_feat, (size_t)num_nodes * row_bytes, cudaMemcpyHostToDevice);
-        if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: preload copy"));
+        for (int64_t v0 = 0; v0 < num_nodes; v0 += table_rows) {   // slot v holds row v mod P
+            const int64_t nr = std::min(table_rows, num_nodes - v0);
+            cudaError_t e = cudaMemcpy(b->slots + v0 * row_bytes, host_feat, (size_t)nr * row_bytes,
+                                       cudaMemcpyHostToDevice);
+            if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: preload copy"));
+        }
     }
     {
         cudaError_t e = cudaDeviceSynchronize();
@@ -876,7 +893,7 @@ static void CUDART_CB host_gather_cb(void* arg) {
     StagedSlot* ss = (StagedSlot*)arg;
     gd_buffer* b = ss->owner;
     const int64_t n = ((volatile int64_t*)ss->h_meta)[2];
-    ss->cpu_ms = b->pool->gather((const uint8_t*)b->host_feat, ss->h_nodes, n, b->R, ss->staging);
+    ss->cpu_ms = b->pool->gather((const uint8_t*)b->host_feat, ss->h_nodes, n, b->R, ss->staging, b->P);
     if (b->timer.on) b->timer_host_ms += ss->cpu_ms;   // serialised on stream H
 }
 
@@ -1078,9 +1095,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
     if (b->preload) {
     } else if (b->R % 16 == 0)
-        k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
     else
-        k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R);
+        k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
     GD_DEBUG_AFTER("k_miss_copy", b->side);
     GD_CUDA(cudaEventRecord(b->ev_z1[d], b->side));
     if (timed) b->timer.end(t_zc, b->side);
@@ -1097,9 +1114,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
         GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
         if (b->R % 16 == 0)
-            k_miss_copy<4, true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+            k_miss_copy<4, true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         else
-            k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R);
+            k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         GD_DEBUG_AFTER("k_stage_copy", b->side_p);
         GD_CUDA(cudaEventRecord(b->ev_p1[d], b->side_p));
         if (timed) b->timer.end(t_pl, b->side_p);
@@ -1227,7 +1244,7 @@ gd_status gd_buffer_set_state(gd_buffer* b, const int32_t* map_slot, const int32
     GD_CUDA(cudaMemcpy(b->ctl, c, sizeof(c), cudaMemcpyHostToDevice));
     for (int64_t v = 0; v < b->N; ++v)
         if ((map_valid[v] & 1) && map_slot[v] >= 0)
-            GD_CUDA(cudaMemcpy(b->slots + (int64_t)map_slot[v] * b->R, (const uint8_t*)b->host_feat + v * b->R, b->R,
+            GD_CUDA(cudaMemcpy(b->slots + (int64_t)map_slot[v] * b->R, (const uint8_t*)b->host_feat + (v % b->P) * b->R, b->R,
                                cudaMemcpyHostToDevice));
     return GD_OK;
 }

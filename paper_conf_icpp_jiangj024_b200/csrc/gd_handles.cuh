@@ -58,6 +58,7 @@ struct StagedSlot {
 struct gd_buffer {
     gd::HandleHdr hdr;
     int64_t N = 0, R = 0, S = 0;     // nodes, row bytes, slots
+    int64_t P = 0;                   // host table rows: node v's row is v mod P (P = N normally)
     int64_t C = 0;                   // ring capacity per half
     int64_t n_max = 0;               // max nodes per batch
     int32_t Q = 0;                   // max in-flight (extracted, unreleased) batches

@@ -32,7 +32,7 @@ struct HostGatherPool::Impl {
     const uint8_t* src = nullptr;
     const int32_t* rows = nullptr;
     uint8_t* dst = nullptr;
-    int64_t n = 0, R = 0;
+    int64_t n = 0, R = 0, P = 1;
     std::atomic<int64_t> next{0};
     static constexpr int64_t kChunk = 512;
 
@@ -64,7 +64,10 @@ struct HostGatherPool::Impl {
             const int64_t lo = next.fetch_add(kChunk, std::memory_order_relaxed);
             if (lo >= n) break;
             const int64_t hi = lo + kChunk < n ? lo + kChunk : n;
-            for (int64_t j = lo; j < hi; ++j) copy_row(dst + j * R, src + (int64_t)rows[j] * R, R);
+            for (int64_t j = lo; j < hi; ++j) {
+                const int64_t v = rows[j];
+                copy_row(dst + j * R, src + (v < P ? v : v % P) * R, R);
+            }
         }
         _mm_sfence();   // streaming stores globally visible before the GPU pull is released
     }
@@ -104,7 +107,8 @@ HostGatherPool::~HostGatherPool() {
 
 int HostGatherPool::threads() const { return (int)impl_->workers.size() + 1; }
 
-double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst) {
+double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst,
+                              int64_t P) {
     const auto t0 = std::chrono::steady_clock::now();
     if (n > 0) {
         Impl& I = *impl_;
@@ -115,6 +119,7 @@ double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n
             I.dst = dst;
             I.n = n;
             I.R = R;
+            I.P = P;
             I.next.store(0, std::memory_order_relaxed);
             I.active = (int)I.workers.size();
             ++I.generation;

@@ -10,8 +10,8 @@ class HostGatherPool {
     explicit HostGatherPool(int threads);
     ~HostGatherPool();
     int threads() const;
-    // dst[j*R : (j+1)*R] = src[rows[j]*R : ...] for j < n, on all threads; returns elapsed ms.
-    double gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst);
+    // dst[j*R : (j+1)*R] = src[(rows[j] mod P)*R : ...] for j < n, on all threads; returns elapsed ms.
+    double gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst, int64_t P);
 
    private:
     struct Impl;

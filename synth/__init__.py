@@ -61,10 +61,15 @@ class Config:
     buffer_frac: float          # capacity S as a fraction of N (1.0 + preload = all resident)
     preload: bool
     train_frac: float
+    table_rows: int | None = None   # physical host-table rows P (node v -> row v mod P); None = N
 
     @property
     def row_bytes(self) -> int:
         return self.feat_dim * self.elem_bytes
+
+    @property
+    def host_rows(self) -> int:
+        return self.table_rows or self.num_nodes
 
 
 # BASELINE.json configs; shapes from SURVEY.md §8.0
@@ -73,7 +78,10 @@ CONFIGS = {
     "products": Config("products", 2_400_000, 62_000_000, 100, 4, 1024, (15, 10, 5), 1.0, True, 0.08),
     "papers100m": Config("papers100m", 111_000_000, 1_600_000_000, 128, 4, 1000, (15, 10, 5), 0.10, False, 0.0109),
     "friendster": Config("friendster", 65_000_000, 1_800_000_000, 256, 4, 1000, (10, 10, 10), -1.0, False, 0.01),
-    "mag240m": Config("mag240m", 244_000_000, 1_700_000_000, 768, 2, 1000, (25, 15), 0.10, False, 0.0046),
+    # 375 GB logical table > the 196 GB of host RAM of this pool's boxes: a bounded physical
+    # table of 64M rows (98 GB), node v -> row v mod 64M (R15)
+    "mag240m": Config("mag240m", 244_000_000, 1_700_000_000, 768, 2, 1000, (25, 15), 0.10, False, 0.0046,
+                      table_rows=64_000_000),
 }
 
 GRAPH_SEED, TRAIN_SEED, RNG_SEED, FEATURE_SEED = 1, 2, 3, 4

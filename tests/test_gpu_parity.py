@@ -134,14 +134,16 @@ def compare_state(buf, ob):
         assert np.array_equal(a[k], b[k]), k
 
 
-def run_schedule(gd, g, ip, ix, feat, S, Q, seeds_list, fanouts, preload=False, check_state_every=1, config=None):
-    N, R = feat.shape
+def run_schedule(gd, g, ip, ix, feat, S, Q, seeds_list, fanouts, preload=False, check_state_every=1, config=None,
+                 num_nodes=None):
+    P, R = feat.shape
+    N = num_nodes or P
     nb, _ = O.sample_bounds(max(len(s) for s in seeds_list), fanouts, N, int(ip[-1]))
     n_max = nb[-1]
-    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, Q, n_max, preload=preload)
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), S, Q, n_max, preload=preload, num_nodes=N)
     if config is not None:
         buf.config(*config)
-    ob = O.Buffer(feat, S, preload=preload)
+    ob = O.Buffer(feat, S, preload=preload, num_nodes=N)
     pending = []
     for b, seeds in enumerate(seeds_list):
         res = g.sample(torch.as_tensor(seeds).cuda(), fanouts, 3, b)
@@ -155,7 +157,7 @@ def run_schedule(gd, g, ip, ix, feat, S, Q, seeds_list, fanouts, preload=False, 
         assert tuple(stats.cpu().tolist()[:2]) == o_stats
         assert np.array_equal(alias[:n].cpu().numpy(), o_alias)
         assert np.array_equal(out[:n].cpu().numpy(), o_out)
-        assert np.array_equal(o_out, feat[n_id])                  # closed form
+        assert np.array_equal(o_out, feat[n_id % P])              # closed form
         pending.append((res, n_id))
         if len(pending) == Q:
             r0, n0 = pending.pop(0)
@@ -199,6 +201,21 @@ def test_extract_parity_miss_paths(gd, config):
     nb, _ = O.sample_bounds(500, [10, 5], N, E)
     run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 3 * nb[-1], 3, seeds, [10, 5],
                  check_state_every=4, config=config)
+
+
+@pytest.mark.parametrize("preload", [False, True])
+def test_extract_parity_bounded_table(gd, preload):
+    """mag240m-style bounded host table (node v -> row v mod P), zero-copy + staged paths."""
+    N, E, P = 30_000, 240_000, 7_001
+    indptr, indices = make_graph(N, E, seed=13)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(P, 1536)
+    order = synth.epoch_order(synth.train_nodes(N, 0.3))
+    seeds = [order[b * 200:(b + 1) * 200].numpy() for b in range(10)]
+    nb, _ = O.sample_bounds(200, [25, 15], N, E)
+    S = N if preload else 2 * nb[-1]
+    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, S, 2, seeds, [25, 15], preload=preload,
+                 check_state_every=3, num_nodes=N)
 
 
 @pytest.mark.parametrize("R", [400, 12, 1536])

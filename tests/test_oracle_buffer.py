@@ -168,3 +168,21 @@ def test_capacity_violation_and_underflow():
     B2 = O.Buffer(table(10), 4)
     with pytest.raises(RuntimeError):
         B2.release(np.array([3], dtype=np.int32))
+
+
+def test_bounded_table_rows_mod_p():
+    """mag240m's bounded host table: node v's row is table[v mod P] (R15)."""
+    rng = np.random.default_rng(9)
+    N, P = 500, 37
+    feat = table(P, R=32, seed=9)
+    B = O.Buffer(feat, 64, num_nodes=N)
+    pend = []
+    for _ in range(40):
+        ids = rng.choice(N, size=20, replace=False).astype(np.int32)
+        out, alias, _ = B.extract(ids)
+        assert np.array_equal(out, feat[ids % P])
+        pend.append(ids)
+        if len(pend) == 3:
+            B.release(pend.pop(0))
+    with pytest.raises(ValueError):
+        O.Buffer(feat, 600, preload=True, num_nodes=N + 1000)   # preload needs capacity >= N
