@@ -195,13 +195,10 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
 /* ----------------------------------------------------------------------------
  * Miss-stream configuration.  The misses of a batch are split in list order: ranks
  * [0, K0) are copied zero-copy from the pinned table by SM loads; ranks [K0, M) take
- * the paper's two-phase path: phase 1, a library worker thread and
- * `host_threads` pool threads gather the rows into a pinned staging slot; phase 2, the
- * copy engine moves the slot to HBM (cudaMemcpyAsync) and signals the scatter kernel
- * already queued on the internal stream through cuStreamWriteValue64 /
- * cuStreamWaitValue64 (stream-ordered, no caller sync).  Without stream memory ops
- * (or with env GD_STAGE_COPY_ENGINE=0) phase 1 runs in a CUDA host function and phase
- * 2 is a kernel pulling the pinned slot over the link.  K0 = floor(M * zero_copy_share).
+ * the paper's two-phase path: phase 1, `host_threads` library-owned
+ * CPU threads gather the rows into a pinned staging slot (run from a CUDA host
+ * function, so still stream-ordered, no caller sync); phase 2, a kernel pulls the
+ * slot contiguously over the host link.  K0 = floor(M * zero_copy_share).
  *   host_threads     0 disables the staged path (all misses zero-copy).
  *   zero_copy_share  in [0, 1]; < 0 = adaptive, from the measured zero-copy rate r_zc
  *                    and host gather rate r_host and the contiguous pull rate r_link of
@@ -256,9 +253,8 @@ void* gd_buffer_side_stream(gd_buffer* b);
  * enable == 0 stops.  *_timing_read synchronises and sums the collected
  * durations in milliseconds.  Used by bench.py for the roofline fractions. */
 gd_status gd_buffer_timing(gd_buffer* b, int enable);
-/* ms[7] = {bookkeeping (lookup + pop/assign), hit gather, zero-copy miss copy,
- *          staged miss pull / scatter, host gather (phase 1, summed), current zero-copy
- *          share, copy-engine H2D of the staged share (summed)}. */
+/* ms[6] = {bookkeeping (lookup + pop/assign), hit gather, zero-copy miss copy,
+ *          staged miss pull, host gather (phase 1, summed), current zero-copy share}. */
 gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches);
 gd_status gd_graph_timing(gd_graph* g, int enable);
 gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls);

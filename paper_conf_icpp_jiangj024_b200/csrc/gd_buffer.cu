@@ -22,12 +22,6 @@
 #include <cstdlib>
 #include <thread>
 
-#include <cuda.h>
-
-#include <condition_variable>
-#include <deque>
-#include <mutex>
-
 #include "gd_common.cuh"
 #include "gd_handles.cuh"
 
@@ -641,129 +635,6 @@ __global__ void k_init_slots(int32_t* reverse, int32_t* pos_of_slot, int32_t* ri
 
 using namespace gd;
 
-// ---------------------------------------------------------------- stream memory ops
-// cuStreamWaitValue64 / cuStreamWriteValue64 from the driver, resolved at run time (the
-// library must still load on hosts without a driver).
-typedef CUresult (*PFN_streamValue64)(CUstream, CUdeviceptr, cuuint64_t, unsigned int);
-static PFN_streamValue64 g_wait64 = nullptr, g_write64 = nullptr;
-
-static bool stream_mem_ops_available() {
-    static int state = -1;
-    if (state >= 0) return state == 1;
-    state = 0;
-    cudaDriverEntryPointQueryResult q1, q2;
-    void *w = nullptr, *r = nullptr;
-    if (cudaGetDriverEntryPoint("cuStreamWaitValue64", &w, cudaEnableDefault, &q1) == cudaSuccess &&
-        cudaGetDriverEntryPoint("cuStreamWriteValue64", &r, cudaEnableDefault, &q2) == cudaSuccess && w && r &&
-        q1 == cudaDriverEntryPointSuccess && q2 == cudaDriverEntryPointSuccess) {
-        g_wait64 = (PFN_streamValue64)w;
-        g_write64 = (PFN_streamValue64)r;
-        // functional probe on a scratch stream
-        unsigned long long* f = nullptr;
-        cudaStream_t s0;
-        if (cudaMalloc(&f, 8) == cudaSuccess && cudaMemset(f, 0, 8) == cudaSuccess &&
-            cudaStreamCreateWithFlags(&s0, cudaStreamNonBlocking) == cudaSuccess) {
-            if (g_write64((CUstream)s0, (CUdeviceptr)f, 5, 0) == CUDA_SUCCESS &&
-                g_wait64((CUstream)s0, (CUdeviceptr)f, 5, CU_STREAM_WAIT_VALUE_GEQ) == CUDA_SUCCESS &&
-                cudaStreamSynchronize(s0) == cudaSuccess)
-                state = 1;
-            cudaStreamDestroy(s0);
-        }
-        if (f) cudaFree(f);
-    }
-    cudaGetLastError();
-    return state == 1;
-}
-
-// Phase 1 + the transfer of the staged share, on a library-owned thread, in batch order:
-// wait for the batch's pop (node list in mapped host memory), wait for the previous
-// copy out of this pinned slot, gather the rows (thread pool), then cudaMemcpyAsync the
-// slot into device staging on stream C (copy engine) and cuStreamWriteValue64(seq) so
-// the scatter kernel already queued on stream P may run.
-struct StageJob {
-    int d;
-    uint64_t seq;
-};
-
-struct StageWorker {
-    gd_buffer* b;
-    std::thread th;
-    std::mutex mu;
-    std::condition_variable cv, cv_idle;
-    std::deque<StageJob> q;
-    bool stop = false;
-    bool busy = false;
-    int prev_d = -1;
-
-    explicit StageWorker(gd_buffer* owner) : b(owner) { th = std::thread([this] { loop(); }); }
-
-    void push(StageJob j) {
-        {
-            std::lock_guard<std::mutex> lk(mu);
-            q.push_back(j);
-        }
-        cv.notify_one();
-    }
-    void drain() {
-        std::unique_lock<std::mutex> lk(mu);
-        cv_idle.wait(lk, [&] { return q.empty() && !busy; });
-    }
-    void shutdown() {
-        {
-            std::lock_guard<std::mutex> lk(mu);
-            stop = true;
-        }
-        cv.notify_one();
-        if (th.joinable()) th.join();
-    }
-    void loop() {
-        cudaSetDevice(b->hdr.device);
-        while (true) {
-            StageJob j;
-            {
-                std::unique_lock<std::mutex> lk(mu);
-                cv.wait(lk, [&] { return stop || !q.empty(); });
-                if (q.empty() && stop) return;
-                j = q.front();
-                q.pop_front();
-                busy = true;
-            }
-            run(j);
-            {
-                std::lock_guard<std::mutex> lk(mu);
-                busy = false;
-            }
-            cv_idle.notify_all();
-        }
-    }
-    void run(const StageJob& j) {
-        StagedSlot& ss = b->stg[j.d];
-        cudaEventSynchronize(b->ev_Ls[j.d]);     // pop of this batch done: node list is valid
-        cudaEventSynchronize(b->ev_cp[j.d]);     // the previous copy out of this pinned slot is done
-        if (b->timer.on && prev_d >= 0) {        // account the previous copy (done or nearly)
-            float ms = 0;
-            cudaEventSynchronize(b->ev_c1[prev_d]);
-            if (cudaEventElapsedTime(&ms, b->ev_c0[prev_d], b->ev_c1[prev_d]) == cudaSuccess) b->timer_copy_ms += ms;
-        }
-        const int64_t n = ((volatile int64_t*)ss.h_meta)[2];
-        ss.cpu_ms = b->pool->gather((const uint8_t*)b->host_feat, ss.h_nodes, n, b->R, ss.staging, b->P);
-        if (b->timer.on) b->timer_host_ms += ss.cpu_ms;
-        uint8_t* dst = b->dstage + (int64_t)j.d * b->n_max * b->R;
-        cudaStreamWaitEvent(b->side_c, b->ev_P[j.d], 0);   // scatter of batch - D done with dstage[d]
-        cudaEventRecord(b->ev_c0[j.d], b->side_c);
-        if (n > 0) cudaMemcpyAsync(dst, ss.staging, (size_t)n * b->R, cudaMemcpyHostToDevice, b->side_c);
-        cudaEventRecord(b->ev_c1[j.d], b->side_c);
-        cudaEventRecord(b->ev_cp[j.d], b->side_c);
-        g_write64((CUstream)b->side_c, (CUdeviceptr)b->stage_flag, (cuuint64_t)j.seq, 0);
-        prev_d = b->timer.on ? j.d : -1;
-        if (cudaGetLastError() != cudaSuccess) atomic_or_status(b);
-    }
-    static void atomic_or_status(gd_buffer* bb) {
-        unsigned int v = GD_DEV_STANDBY_DRY;   // surfaced through gd_check_device_status
-        cudaMemcpy(bb->hdr.dev_status, &v, sizeof(v), cudaMemcpyHostToDevice);
-    }
-};
-
 extern "C" {
 static gd_status calibrate_link(gd_buffer* b);
 }
@@ -772,17 +643,11 @@ static void buffer_free(gd_buffer* b) {
     if (!b) return;
     DeviceGuard guard(b->hdr.device);
     if (b->side) cudaStreamSynchronize(b->side);
-    if (b->worker) {
-        b->worker->drain();
-        b->worker->shutdown();
-        delete b->worker;
-        b->worker = nullptr;
-    }
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) cudaStreamSynchronize(s);
     void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->hitlist, b->hcount,
                     b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
-                    b->hdr.dev_status, b->dstage, b->stage_flag};
+                    b->hdr.dev_status};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem})
@@ -790,13 +655,12 @@ static void buffer_free(gd_buffer* b) {
     delete b->pool;
     b->scan.release();
     b->timer.destroy();
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_Ls, &b->ev_cp,
-                    &b->ev_c0, &b->ev_c1})
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
     for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G})
         if (e) cudaEventDestroy(e);
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) cudaStreamDestroy(s);
     if (b->registered) cudaHostUnregister((void*)b->host_feat);
     b->hdr.magic = 0;
@@ -917,16 +781,14 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: init kernels"));
     }
-    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_g, &b->side_c})
+    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_g})
         if (cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
     for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G})
         if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_Ls, &b->ev_cp,
-                    &b->ev_c0, &b->ev_c1}) {
-        const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1 || v == &b->ev_c0 ||
-                             v == &b->ev_c1);
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1}) {
+        const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1);
         v->assign(b->D, nullptr);
         for (int d = 0; d < b->D; ++d)
             if (cudaEventCreateWithFlags(&(*v)[d], timing ? cudaEventDefault : cudaEventDisableTiming) != cudaSuccess)
@@ -962,8 +824,7 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     if (zc_blocks > 0) b->zc_blocks = zc_blocks;
     if (pull_blocks > 0) b->pull_blocks = pull_blocks;
     DeviceGuard guard(b->hdr.device);
-    if (b->worker) b->worker->drain();
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g})
         if (s) GD_CUDA(cudaStreamSynchronize(s));
     if (host_threads > 0 && !b->stage_mem) {
         const int D = b->D;
@@ -986,16 +847,6 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         b->pool = nullptr;
     }
     if (host_threads > 0 && !b->pool) b->pool = new HostGatherPool(host_threads);
-    const char* ce_env = std::getenv("GD_STAGE_COPY_ENGINE");
-    const bool want_ce = !(ce_env && ce_env[0] == '0');
-    if (host_threads > 0 && want_ce && !b->worker && stream_mem_ops_available()) {
-        GD_CUDA(cudaMalloc(&b->dstage, (size_t)b->D * b->n_max * b->R));
-        GD_CUDA(cudaMalloc(&b->stage_flag, sizeof(unsigned long long)));
-        GD_CUDA(cudaMemset(b->stage_flag, 0, sizeof(unsigned long long)));
-        b->stage_seq = 0;
-        b->worker = new StageWorker(b);
-    }
-    b->ce_path = host_threads > 0 && b->worker != nullptr;
     b->host_threads = host_threads;
     b->alpha_fixed = zero_copy_share >= 0;
     b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.2);
@@ -1012,12 +863,9 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing: bad handle");
     DeviceGuard guard(b->hdr.device);
     if (enable) {
-        if (b->worker) b->worker->drain();
-        for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
-            GD_CUDA(cudaStreamSynchronize(s));
+        for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g}) GD_CUDA(cudaStreamSynchronize(s));
         b->timer.reset();
         b->timer_host_ms = 0;
-        b->timer_copy_ms = 0;
     }
     b->timer.on = enable != 0;
     return GD_OK;
@@ -1026,14 +874,11 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable) {
 gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing_read: bad handle");
     DeviceGuard guard(b->hdr.device);
-    if (b->worker) b->worker->drain();
-    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
-        GD_CUDA(cudaStreamSynchronize(s));
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g}) GD_CUDA(cudaStreamSynchronize(s));
     if (ms) {
         for (int k = 0; k < 4; ++k) ms[k] = b->timer.total_ms(4, k);
         ms[4] = b->timer_host_ms;
         ms[5] = b->alpha;
-        ms[6] = b->timer_copy_ms;
     }
     if (batches) *batches = (int64_t)b->timer.pairs.size() / 4;
     GD_CUDA(cudaGetLastError());
@@ -1063,8 +908,7 @@ static void CUDART_CB host_gather_cb(void* arg) {
 static void adapt_alpha(gd_buffer* b, int d) {
     StagedSlot& ss = b->stg[d];
     if (b->alpha_fixed || ss.batch < 0 || b->r_link <= 0) return;
-    if (cudaEventQuery(b->ce_path ? b->ev_cp[d] : b->ev_E[d]) != cudaSuccess ||
-        cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
+    if (cudaEventQuery(b->ev_E[d]) != cudaSuccess || cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
         cudaGetLastError();                     // that batch is still in flight
         return;
     }
@@ -1111,10 +955,7 @@ static gd_status calibrate_link(gd_buffer* b) {
     float best = 1e30f;
     for (int rep = 0; rep < 4; ++rep) {
         cudaEventRecord(e0, b->side_p);
-        if (b->ce_path)   // the staged share crosses the link by copy engine
-            cudaMemcpyAsync(dst, b->stage_mem, bytes, cudaMemcpyHostToDevice, b->side_p);
-        else
-            k_link_calib<<<b->pull_blocks, 1024, 0, b->side_p>>>((const uint4*)src, (uint4*)dst, bytes / 16);
+        k_link_calib<<<b->pull_blocks, 1024, 0, b->side_p>>>((const uint4*)src, (uint4*)dst, bytes / 16);
         cudaEventRecord(e1, b->side_p);
         cudaEventSynchronize(e1);
         float ms = 0;
@@ -1227,10 +1068,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
     if (staged) {
-        if (!b->ce_path) {
-            GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
-            GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
-        }
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
         GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_G, 0));
     }
 
@@ -1267,26 +1106,15 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // a7, staged share: misses [K0, M).  Phase 1 on stream H (host gather into pinned
     // staging slot d), phase 2 on stream P (contiguous pull into slots + out).
     if (staged) {
+        GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
+        GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));
+        GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_E[d], 0));
         const uint8_t* stage_dev = nullptr;
-        if (b->ce_path) {
-            // worker: gather -> cudaMemcpyAsync into dstage[d] -> write seq; P waits for seq
-            const uint64_t seq = ++b->stage_seq;
-            GD_CUDA(cudaEventRecord(b->ev_Ls[d], st));
-            b->worker->push(StageJob{d, seq});
-            if (g_wait64((CUstream)b->side_p, (CUdeviceptr)b->stage_flag, (cuuint64_t)seq, CU_STREAM_WAIT_VALUE_GEQ) !=
-                CUDA_SUCCESS)
-                return set_error(GD_ERR_CUDA, "gd_extract: cuStreamWaitValue64 failed");
-            stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
-        } else {
-            GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
-            GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));
-            GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_E[d], 0));
-            GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
-        }
+        GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
         const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
         GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
         if (b->R % 16 == 0)
-            k_miss_copy<4, true><<<b->ce_path ? 32 : b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
+            k_miss_copy<4, true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         else
             k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         GD_DEBUG_AFTER("k_stage_copy", b->side_p);

@@ -106,17 +106,6 @@ struct gd_buffer {
     bool alpha_fixed = false;
     gd::HostGatherPool* pool = nullptr;
     std::vector<StagedSlot> stg;
-    // copy-engine variant of the staged path (default when stream memory ops exist): a
-    // library worker thread gathers into the pinned slot, issues an H2D cudaMemcpyAsync
-    // into dstage[d] on stream C and signals stream P with cuStreamWriteValue64
-    bool ce_path = false;
-    uint8_t* dstage = nullptr;           // HBM [D][n_max x R]
-    unsigned long long* stage_flag = nullptr;   // HBM: last staged sequence number copied
-    uint64_t stage_seq = 0;
-    cudaStream_t side_c = nullptr;       // C: the worker's copy stream
-    std::vector<cudaEvent_t> ev_Ls, ev_cp, ev_c0, ev_c1;   // [D] batch's pop done; copy done; copy timing
-    struct StageWorker* worker = nullptr;
-    double timer_copy_ms = 0;
     uint8_t* stage_mem = nullptr;        // pinned allocations behind stg
     int32_t* hnodes_mem = nullptr;
     int64_t* hmeta_mem = nullptr;
