@@ -463,6 +463,9 @@ def run_ours(args, rank, world, local_rank):
 
     # ---- reference measurements for the roofline
     hbm_peak = measured_peaks().get("hbm_gbs")
+    hbm_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)"
+    if not hbm_peak:   # B200_PROFILING.md: fallback only when the driver-written file is absent
+        hbm_peak, hbm_src = 6650.0, "of fallback: B200_PROFILING.md 6.65 TB/s (MEASURED_PEAKS.json absent)"
     link_peak = h2d_peak_gbps(dev)
     R = cfg.row_bytes
     region_s = ms / 1e3
@@ -483,7 +486,7 @@ def run_ours(args, rank, world, local_rank):
     rnd = lambda x, k=2: round(x, k) if x is not None else None  # noqa: E731
     roof_gather = {"bound": "hbm", "achieved": rnd(gather_gbs, 1), "peak": hbm_peak, "unit": "GB/s",
                    "frac": rnd(gather_gbs / hbm_peak, 4) if gather_gbs and hbm_peak else None, "traffic": None,
-                   "kernel": "k_gather_rows", "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"}
+                   "kernel": "k_gather_rows", "peak_source": hbm_src}
     roof_miss = {"bound": "host_link", "achieved": rnd(link_gbs), "peak": round(link_peak, 2), "unit": "GB/s",
                  "frac": rnd(link_gbs / link_peak, 4) if link_gbs else None, "traffic": None,
                  "kernel": "k_miss_copy (zero-copy share) + k_miss_copy<staged> (pull of the host-gathered share)",

@@ -7,6 +7,10 @@
 // host-gather stream; phase 2 (k_stage_copy) pulls the slot over the host link with
 // contiguous, translation-friendly reads.
 #include <emmintrin.h>   // SSE2 streaming stores (baseline x86-64)
+#include <xmmintrin.h>   // _mm_prefetch
+
+#include <algorithm>
+#include <cstdlib>
 
 #include <atomic>
 #include <chrono>
@@ -59,14 +63,25 @@ struct HostGatherPool::Impl {
         }
     }
 
+    int64_t pf = 8;   // prefetch distance in rows (env GD_GATHER_PF; 0 = off)
+
+    const uint8_t* row_ptr(int64_t v) const { return src + (v < P ? v : v % P) * R; }
+    void prefetch_row(const uint8_t* p) const {
+        for (int64_t c = 0; c < R; c += 64) _mm_prefetch((const char*)p + c, _MM_HINT_T0);
+    }
+
     void work() {
         while (true) {
             const int64_t lo = next.fetch_add(kChunk, std::memory_order_relaxed);
             if (lo >= n) break;
             const int64_t hi = lo + kChunk < n ? lo + kChunk : n;
+            // software prefetch `pf` rows ahead: random rows over a table far larger than
+            // the caches and the TLB reach are latency-bound per thread; prefetching every
+            // line of row j + pf keeps ~pf rows of misses (and their page walks) in flight
+            for (int64_t j = lo; j < hi && j < lo + pf; ++j) prefetch_row(row_ptr(rows[j]));
             for (int64_t j = lo; j < hi; ++j) {
-                const int64_t v = rows[j];
-                copy_row(dst + j * R, src + (v < P ? v : v % P) * R, R);
+                if (j + pf < hi) prefetch_row(row_ptr(rows[j + pf]));
+                copy_row(dst + j * R, row_ptr(rows[j]), R);
             }
         }
         _mm_sfence();   // streaming stores globally visible before the GPU pull is released
@@ -92,6 +107,7 @@ struct HostGatherPool::Impl {
 
 HostGatherPool::HostGatherPool(int threads) : impl_(new Impl) {
     // the calling (CUDA callback) thread works too, so spawn threads-1 helpers
+    if (const char* e = std::getenv("GD_GATHER_PF")) impl_->pf = std::max(0, std::atoi(e));
     for (int t = 1; t < threads; ++t) impl_->workers.emplace_back([this] { impl_->loop(); });
 }
 

@@ -363,7 +363,7 @@ def test_run_twice_bitwise_identical_and_gpu_count_independent(gd):
     seeds = [order[b * 400:(b + 1) * 400].cuda() for b in range(8)]
 
     def run():
-        buf = gd.FeatureBuffer(torch.from_numpy(feat), 20_000, 3, g.bounds(400, [15, 10, 5])[0][-1])
+        buf = gd.FeatureBuffer(torch.from_numpy(feat), N, 3, g.bounds(400, [15, 10, 5])[0][-1])   # S >= min(N, Q M_b)
         outs, pend = [], []
         for b, sd in enumerate(seeds):
             o = g.sample(sd, [15, 10, 5], 3, b)
