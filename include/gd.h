@@ -218,6 +218,21 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
                            int pull_blocks);
 
 /* ----------------------------------------------------------------------------
+ * Phase 2 of the staged share ("CUDA async copy" of the staging buffer).
+ *   copy_engine = 1 (default; env GD_STAGE_COPY_ENGINE=0 at init selects 0): the
+ *     staged share is the FIRST `cap` misses of the batch, cap = (1 - share) x the
+ *     misses of a recently completed batch (the copy size must be known when it is
+ *     enqueued, and nothing may synchronise the host); after the host gather, stream
+ *     H copies cap rows pinned -> HBM staging with cudaMemcpyAsync (DMA, no SM
+ *     loads over the link) and a kernel scatters them into slots + out.  The other
+ *     misses go zero-copy.  HBM cost: D x max_nodes_per_batch x row_bytes.
+ *   copy_engine = 0: ranks [K0, M) are staged and a kernel pulls the pinned slot.
+ * Either way the results (out, alias, buffer state) are identical.  Synchronises the
+ * internal streams (re-runs gd_buffer_config); call between batches.
+ * ------------------------------------------------------------------------- */
+gd_status gd_buffer_stage_mode(gd_buffer* b, int copy_engine);
+
+/* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a
  * slot whose count reaches zero is appended at the tail (MRU end) of the standby
  * list.  The node stays valid until its slot is reused (delayed invalidation).
@@ -253,8 +268,10 @@ void* gd_buffer_side_stream(gd_buffer* b);
  * enable == 0 stops.  *_timing_read synchronises and sums the collected
  * durations in milliseconds.  Used by bench.py for the roofline fractions. */
 gd_status gd_buffer_timing(gd_buffer* b, int enable);
-/* ms[6] = {bookkeeping (lookup + pop/assign), hit gather, zero-copy miss copy,
- *          staged miss pull, host gather (phase 1, summed), current zero-copy share}. */
+/* ms[7] = {bookkeeping (lookup + pop/assign), hit gather, zero-copy miss copy,
+ *          staged miss pull (SM pull mode) or scatter (copy-engine mode), host gather
+ *          (phase 1, summed), current zero-copy share, copy-engine H2D of the staged
+ *          share (copy-engine mode; 0 otherwise)}. */
 gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches);
 gd_status gd_graph_timing(gd_graph* g, int enable);
 gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls);

@@ -271,11 +271,15 @@ class FeatureBuffer:
         check(lib.gd_buffer_timing(self._h, int(enable)))
 
     def timing_read(self):
-        ms = (ctypes.c_double * 6)()
+        ms = (ctypes.c_double * 7)()
         n = ctypes.c_int64()
         check(lib.gd_buffer_timing_read(self._h, ms, ctypes.byref(n)))
         return {"bookkeeping_ms": ms[0], "gather_ms": ms[1], "miss_zero_copy_ms": ms[2], "miss_staged_ms": ms[3],
-                "host_gather_ms": ms[4], "zero_copy_share": ms[5], "batches": n.value}
+                "host_gather_ms": ms[4], "zero_copy_share": ms[5], "staged_copy_ms": ms[6], "batches": n.value}
+
+    def stage_mode(self, copy_engine: bool):
+        """gd_buffer_stage_mode: phase 2 of the staged share by copy engine (True) or SM pull."""
+        check(lib.gd_buffer_stage_mode(self._h, int(bool(copy_engine))))
 
     def config(self, host_threads: int, zero_copy_share: float = -1.0, zc_blocks: int = 0, pull_blocks: int = 0):
         """gd_buffer_config: staged miss path width, zero-copy share (< 0: adaptive), copy grids."""

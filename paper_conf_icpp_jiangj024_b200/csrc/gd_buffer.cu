@@ -31,6 +31,7 @@ constexpr int kBThreads = 256;
 constexpr int kBItems = 8;
 constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
+constexpr int kTimedPairs = 5;   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -162,6 +163,7 @@ struct PopArgs {
     int64_t* trip_count;
     int64_t* trip_split;            // K0 = floor(M * alpha_q16 / 2^16): first staged rank
     uint32_t alpha_q16;
+    long long staged_cap;           // >= 0 (copy-engine staging): K0 = max(0, M - staged_cap)
     int32_t* h_nodes;               // mapped host: node ids of ranks [K0, M) (staged share)
     int64_t* h_meta;                // mapped host: {M, K0, M - K0}
     int64_t* stats;                 // caller's stats or null: [2] = K0, [3] = M - K0
@@ -196,7 +198,8 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
     __shared__ int s_cnt[kBItems * kBWarps];
     __shared__ long long s_base;
     const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
-    const long long K0 = (long long)(((unsigned long long)M * a.alpha_q16) >> 16);
+    const long long K0 = a.staged_cap >= 0 ? (M > a.staged_cap ? M - a.staged_cap : 0)
+                                           : (long long)(((unsigned long long)M * a.alpha_q16) >> 16);
     if (M == 0) {
         if (blockIdx.x == 0 && t == 0) {
             *a.ctl_out = c;
@@ -647,7 +650,7 @@ static void buffer_free(gd_buffer* b) {
         if (s) cudaStreamSynchronize(s);
     void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->hitlist, b->hcount,
                     b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
-                    b->hdr.dev_status};
+                    b->hdr.dev_status, b->dstage};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem})
@@ -804,6 +807,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     int zcb = 0, plb = 0;
     if (const char* e = std::getenv("GD_ZC_BLOCKS")) zcb = std::atoi(e);
     if (const char* e = std::getenv("GD_PULL_BLOCKS")) plb = std::atoi(e);
+    if (const char* e = std::getenv("GD_STAGE_COPY_ENGINE")) b->ce_mode = e[0] != '0';
     s = gd_buffer_config(b, threads, share, zcb, plb);
     if (s != GD_OK) return fail(s);
     *out = b;
@@ -847,7 +851,14 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         b->pool = nullptr;
     }
     if (host_threads > 0 && !b->pool) b->pool = new HostGatherPool(host_threads);
+    if (host_threads > 0 && b->ce_mode && !b->dstage)
+        GD_CUDA(cudaMalloc(&b->dstage, (size_t)b->D * b->n_max * b->R));
+    if ((host_threads == 0 || !b->ce_mode) && b->dstage) {
+        GD_CUDA(cudaFree(b->dstage));
+        b->dstage = nullptr;
+    }
     b->host_threads = host_threads;
+    b->m_est = 0;
     b->alpha_fixed = zero_copy_share >= 0;
     b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.2);
     b->r_host = 0;
@@ -857,6 +868,14 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         if (st != GD_OK) return st;
     }
     return GD_OK;
+}
+
+gd_status gd_buffer_stage_mode(gd_buffer* b, int copy_engine) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_stage_mode: bad handle");
+    if (copy_engine != 0 && copy_engine != 1) return set_error(GD_ERR_INVALID, "gd_buffer_stage_mode: 0 or 1");
+    if ((copy_engine == 1) == b->ce_mode) return GD_OK;
+    b->ce_mode = copy_engine == 1;
+    return gd_buffer_config(b, b->host_threads, b->alpha_fixed ? b->alpha : -1.0, 0, 0);
 }
 
 gd_status gd_buffer_timing(gd_buffer* b, int enable) {
@@ -876,11 +895,12 @@ gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches) {
     DeviceGuard guard(b->hdr.device);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g}) GD_CUDA(cudaStreamSynchronize(s));
     if (ms) {
-        for (int k = 0; k < 4; ++k) ms[k] = b->timer.total_ms(4, k);
+        for (int k = 0; k < 4; ++k) ms[k] = b->timer.total_ms(kTimedPairs, k);
         ms[4] = b->timer_host_ms;
+        ms[6] = b->timer.total_ms(kTimedPairs, 4);
         ms[5] = b->alpha;
     }
-    if (batches) *batches = (int64_t)b->timer.pairs.size() / 4;
+    if (batches) *batches = (int64_t)b->timer.pairs.size() / kTimedPairs;
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
@@ -907,11 +927,14 @@ static void CUDART_CB host_gather_cb(void* arg) {
 //   alpha = 1 - r_host / r_link.
 static void adapt_alpha(gd_buffer* b, int d) {
     StagedSlot& ss = b->stg[d];
-    if (b->alpha_fixed || ss.batch < 0 || b->r_link <= 0) return;
+    if (ss.batch < 0) return;
     if (cudaEventQuery(b->ev_E[d]) != cudaSuccess || cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
         cudaGetLastError();                     // that batch is still in flight
         return;
     }
+    // misses per batch, for the copy-engine staging size (its pop finished long ago)
+    b->m_est = (double)((volatile int64_t*)ss.h_meta)[0];
+    if (b->alpha_fixed || b->r_link <= 0) return;
     const double staged_rows = (double)ss.h_meta[2], zc_rows = (double)ss.h_meta[1];
     if (staged_rows >= 2048 && ss.cpu_ms > 0) {
         const double r = staged_rows * (double)b->R / ss.cpu_ms;
@@ -955,7 +978,10 @@ static gd_status calibrate_link(gd_buffer* b) {
     float best = 1e30f;
     for (int rep = 0; rep < 4; ++rep) {
         cudaEventRecord(e0, b->side_p);
-        k_link_calib<<<b->pull_blocks, 1024, 0, b->side_p>>>((const uint4*)src, (uint4*)dst, bytes / 16);
+        if (b->ce_mode)   // the staged share crosses the link by copy engine
+            cudaMemcpyAsync(dst, b->stage_mem, bytes, cudaMemcpyHostToDevice, b->side_p);
+        else
+            k_link_calib<<<b->pull_blocks, 1024, 0, b->side_p>>>((const uint4*)src, (uint4*)dst, bytes / 16);
         cudaEventRecord(e1, b->side_p);
         cudaEventSynchronize(e1);
         float ms = 0;
@@ -999,6 +1025,12 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         ss->batch = b->batch_counter;
     }
     const uint32_t alpha_q16 = staged ? (uint32_t)std::lround(b->alpha * 65536.0) : 65536u;
+    // Copy-engine staging: the H2D copy is enqueued now, so its size must be known now;
+    // the staged share is the first `cap` misses (cap from the recent misses per batch),
+    // the zero-copy share takes the rest.  A batch with fewer misses copies some unused
+    // staging rows (bounded by the estimate's error).
+    const bool ce = staged && b->ce_mode && b->dstage;
+    const long long cap = ce ? std::min<long long>(b->n_max, (long long)((1.0 - b->alpha) * b->m_est * 0.97)) : -1;
     const bool timed = b->timer.on;
     const int t_book = timed ? b->timer.begin(st) : -1;
 
@@ -1037,6 +1069,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.trip_count = tcount;
     pa.trip_split = tsplit;
     pa.alpha_q16 = alpha_q16;
+    pa.staged_cap = cap;
     pa.h_nodes = nullptr;
     pa.h_meta = nullptr;
     if (staged) {
@@ -1107,14 +1140,25 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // staging slot d), phase 2 on stream P (contiguous pull into slots + out).
     if (staged) {
         GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
+        const uint8_t* stage_dev = nullptr;
+        if (ce) {
+            // phase 2 by the copy engine: pinned slot d -> dstage[d] (stream H still owns
+            // dstage[d]: it waited for the scatter of batch - D above)
+            stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
+            const int t_ce = timed ? b->timer.begin(b->side_h) : -1;
+            if (cap > 0)
+                GD_CUDA(cudaMemcpyAsync((void*)stage_dev, ss->staging, (size_t)cap * b->R, cudaMemcpyHostToDevice, b->side_h));
+            if (timed) b->timer.end(t_ce, b->side_h);
+        } else {
+            GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
+            if (timed) b->timer.end(b->timer.begin(b->side_h), b->side_h);
+        }
         GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));
         GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_E[d], 0));
-        const uint8_t* stage_dev = nullptr;
-        GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
         const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
         GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
         if (b->R % 16 == 0)
-            k_miss_copy<4, true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
+            k_miss_copy<4, true><<<ce ? 64 : b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         else
             k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         GD_DEBUG_AFTER("k_stage_copy", b->side_p);
@@ -1123,7 +1167,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         GD_CUDA(cudaEventRecord(b->ev_P[d], b->side_p));
         GD_CUDA(cudaEventRecord(b->ev_Xs, b->side_p));
     } else if (timed) {
-        b->timer.end(b->timer.begin(b->side), b->side);   // keep 4 timing pairs per batch
+        b->timer.end(b->timer.begin(b->side), b->side);   // keep kTimedPairs timing pairs per batch
+        b->timer.end(b->timer.begin(b->side), b->side);
     }
 
     // join: out complete, trip slot d free

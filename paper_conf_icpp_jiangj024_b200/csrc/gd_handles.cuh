@@ -105,6 +105,11 @@ struct gd_buffer {
     double r_link = 0;                   // contiguous pull rate of the host link (bytes/ms), calibrated
     bool alpha_fixed = false;
     gd::HostGatherPool* pool = nullptr;
+    // phase 2 of the staged share: copy engine (cudaMemcpyAsync pinned slot -> dstage[d]
+    // on stream H, then a scatter kernel on P) or an SM pull kernel reading the pinned slot
+    bool ce_mode = true;
+    uint8_t* dstage = nullptr;           // HBM [D][n_max x R] (copy-engine mode)
+    double m_est = 0;                    // misses of a recently completed batch
     std::vector<StagedSlot> stg;
     uint8_t* stage_mem = nullptr;        // pinned allocations behind stg
     int32_t* hnodes_mem = nullptr;

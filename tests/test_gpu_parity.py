@@ -135,12 +135,14 @@ def compare_state(buf, ob):
 
 
 def run_schedule(gd, g, ip, ix, feat, S, Q, seeds_list, fanouts, preload=False, check_state_every=1, config=None,
-                 num_nodes=None):
+                 num_nodes=None, stage_mode=None):
     P, R = feat.shape
     N = num_nodes or P
     nb, _ = O.sample_bounds(max(len(s) for s in seeds_list), fanouts, N, int(ip[-1]))
     n_max = nb[-1]
     buf = gd.FeatureBuffer(torch.from_numpy(feat), S, Q, n_max, preload=preload, num_nodes=N)
+    if stage_mode is not None:
+        buf.stage_mode(stage_mode)
     if config is not None:
         buf.config(*config)
     ob = O.Buffer(feat, S, preload=preload, num_nodes=N)
@@ -188,10 +190,11 @@ def test_extract_parity_tiny_evict(tiny, gd, Q):
     run_schedule(gd, g, ip, ix, feat, S, Q, seeds, list(cfg.fanouts))
 
 
+@pytest.mark.parametrize("copy_engine", [True, False])
 @pytest.mark.parametrize("config", [(0, -1.0), (4, 0.0), (4, 1.0), (3, 0.3), (8, -1.0), (1, 0.9)])
-def test_extract_parity_miss_paths(gd, config):
-    """The miss stream split between zero-copy and the staged (host gather + pull) path:
-    every split gives the same bytes, alias and state."""
+def test_extract_parity_miss_paths(gd, config, copy_engine):
+    """The miss stream split between zero-copy and the staged (host gather + copy engine
+    or SM pull) path: every split gives the same bytes, alias and state."""
     N, E = 60_000, 600_000
     indptr, indices = make_graph(N, E, seed=8)
     g = gd.Graph(indptr, indices)
@@ -200,7 +203,7 @@ def test_extract_parity_miss_paths(gd, config):
     seeds = [order[b * 500:(b + 1) * 500].numpy() for b in range(16)]
     nb, _ = O.sample_bounds(500, [10, 5], N, E)
     run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 3 * nb[-1], 3, seeds, [10, 5],
-                 check_state_every=4, config=config)
+                 check_state_every=4, config=config, stage_mode=copy_engine)
 
 
 @pytest.mark.parametrize("preload", [False, True])
@@ -218,8 +221,9 @@ def test_extract_parity_bounded_table(gd, preload):
                  check_state_every=3, num_nodes=N)
 
 
+@pytest.mark.parametrize("copy_engine", [True, False])
 @pytest.mark.parametrize("R", [400, 12, 1536])
-def test_extract_parity_row_sizes(gd, R):
+def test_extract_parity_row_sizes(gd, R, copy_engine):
     """Row widths: 16-byte vector path (400 = products, 1536 = mag240m fp16) and the 4-byte path."""
     N, E = 20_000, 150_000
     indptr, indices = make_graph(N, E, seed=5)
@@ -228,7 +232,8 @@ def test_extract_parity_row_sizes(gd, R):
     order = synth.epoch_order(synth.train_nodes(N, 0.2))
     seeds = [order[b * 300:(b + 1) * 300].numpy() for b in range(10)]
     nb, _ = O.sample_bounds(300, [10, 5], N, E)
-    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 2 * nb[-1] + 17, 2, seeds, [10, 5], check_state_every=3)
+    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 2 * nb[-1] + 17, 2, seeds, [10, 5], check_state_every=3,
+                 config=(4, 0.3), stage_mode=copy_engine)
 
 
 def test_extract_ring_compaction(gd):
