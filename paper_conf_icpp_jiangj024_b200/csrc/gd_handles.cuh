@@ -93,7 +93,9 @@ struct gd_buffer {
     cudaStream_t side_g = nullptr;       // G: hit gather (slots -> out)
     cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_Xs = nullptr, ev_G = nullptr;
     std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
-    std::vector<cudaEvent_t> ev_E, ev_P; // [D] host gather / staged pull of slot d done
+    std::vector<cudaEvent_t> ev_E, ev_P; // [D] staging slot d ready in HBM or pinned / staged pull done
+    std::vector<cudaEvent_t> ev_H;       // [D] host gather of slot d done (copy-engine mode)
+    cudaStream_t side_c = nullptr;       // C: copy-engine H2D of the staged share
     std::vector<cudaEvent_t> ev_z0, ev_z1, ev_p0, ev_p1;   // [D] timing of the two miss paths
     int64_t* trip_split = nullptr;       // [D] K0: misses [0, K0) zero-copy, [K0, M) staged
     int host_threads = 0;                // 0: staged path off (all misses zero-copy)
