@@ -31,6 +31,7 @@ constexpr int kBThreads = 256;
 constexpr int kBItems = 8;
 constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
+constexpr int kStageRing = 4;    // pinned chunk buffers of the copy-engine staging ring
 constexpr int kTimedPairs = 5;   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -653,15 +654,15 @@ static void buffer_free(gd_buffer* b) {
                     b->hdr.dev_status, b->dstage};
     for (void* p : ptrs)
         if (p) cudaFree(p);
-    for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem})
+    for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem, (void*)b->ring_mem})
         if (p) cudaFreeHost(p);
     delete b->pool;
     b->scan.release();
     b->timer.destroy();
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H})
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_ring})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
-    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G})
+    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk})
         if (e) cudaEventDestroy(e);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
         if (s) cudaStreamDestroy(s);
@@ -857,6 +858,26 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         GD_CUDA(cudaFree(b->dstage));
         b->dstage = nullptr;
     }
+    // chunked staging ring (copy-engine mode): env GD_STAGE_CHUNK_KB, default 8 MB chunks;
+    // 0 = one chunk per batch into the batch's full pinned staging slot
+    int64_t chunk_kb = 8192;
+    if (const char* e = std::getenv("GD_STAGE_CHUNK_KB")) chunk_kb = std::max<int64_t>(0, std::atoll(e));
+    const int64_t rows = (host_threads > 0 && b->ce_mode && chunk_kb > 0)
+                             ? std::min<int64_t>(b->n_max, std::max<int64_t>(1, (chunk_kb << 10) / b->R)) : 0;
+    if (rows != b->stage_chunk_rows) {
+        if (b->ring_mem) GD_CUDA(cudaFreeHost(b->ring_mem));
+        b->ring_mem = nullptr;
+        b->stage_chunk_rows = rows;
+        if (rows > 0) {
+            GD_CUDA(cudaHostAlloc((void**)&b->ring_mem, (size_t)kStageRing * rows * b->R, cudaHostAllocPortable));
+            if (b->ev_ring.empty()) {
+                b->ev_ring.assign(kStageRing, nullptr);
+                for (auto& e : b->ev_ring) GD_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+                GD_CUDA(cudaEventCreateWithFlags(&b->ev_chunk, cudaEventDisableTiming));
+            }
+            b->jobs.assign((size_t)b->D * cdiv(b->n_max, rows), ChunkJob());
+        }
+    }
     b->host_threads = host_threads;
     b->m_est = 0;
     b->alpha_fixed = zero_copy_share >= 0;
@@ -918,6 +939,22 @@ static void CUDART_CB host_gather_cb(void* arg) {
     const int64_t n = ((volatile int64_t*)ss->h_meta)[2];
     ss->cpu_ms = b->pool->gather((const uint8_t*)b->host_feat, ss->h_nodes, n, b->R, ss->staging, b->P);
     if (b->timer.on) b->timer_host_ms += ss->cpu_ms;   // serialised on stream H
+}
+
+// One chunk of the staged share (copy-engine mode): ranks [lo, min(hi, n)) into a ring
+// buffer with ordinary stores (it is read by DMA right after, while still cached).
+static void CUDART_CB chunk_gather_cb(void* arg) {
+    ChunkJob* j = (ChunkJob*)arg;
+    StagedSlot* ss = j->ss;
+    gd_buffer* b = ss->owner;
+    const int64_t staged = ((volatile int64_t*)ss->h_meta)[2];
+    const int64_t n = std::min<int64_t>(staged, j->hi);
+    if (j->first) ss->cpu_ms = 0;
+    const double ms = n > j->lo ? b->pool->gather((const uint8_t*)b->host_feat, ss->h_nodes + j->lo, n - j->lo, b->R,
+                                                  j->buf, b->P, false)
+                                : 0.0;
+    ss->cpu_ms += ms;
+    if (b->timer.on) b->timer_host_ms += ms;   // serialised on stream H
 }
 
 // Zero-copy share alpha.  Both miss paths have their own cap: the zero-copy copy the
@@ -1142,9 +1179,37 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // a7, staged share: misses [K0, M).  Phase 1 on stream H (host gather into pinned
     // staging slot d), phase 2 on stream P (contiguous pull into slots + out).
     if (staged) {
-        GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
         const uint8_t* stage_dev = nullptr;
-        if (ce) {
+        if (ce && b->stage_chunk_rows > 0) {
+            // chunk c: H waits until the copy out of ring buffer r (chunk k - kStageRing)
+            // is done, gathers into it; C copies it to dstage[d] at rank offset lo
+            stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
+            const int64_t ch = b->stage_chunk_rows, nch = cap > 0 ? cdiv(cap, ch) : 0;
+            const int64_t maxch = cdiv(b->n_max, ch);
+            const int t_ce = timed ? b->timer.begin(b->side_c) : -1;
+            if (nch == 0) ss->cpu_ms = 0;
+            for (int64_t c = 0; c < nch; ++c) {
+                const int r = (int)(b->chunk_counter++ % kStageRing);
+                ChunkJob* j = &b->jobs[(size_t)d * maxch + c];
+                j->ss = ss;
+                j->lo = c * ch;
+                j->hi = std::min<int64_t>(cap, (c + 1) * ch);
+                j->buf = b->ring_mem + (int64_t)r * ch * b->R;
+                j->first = c == 0;
+                GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_ring[r], 0));
+                GD_CUDA(cudaLaunchHostFunc(b->side_h, chunk_gather_cb, j));
+                GD_CUDA(cudaEventRecord(b->ev_chunk, b->side_h));
+                GD_CUDA(cudaStreamWaitEvent(b->side_c, b->ev_chunk, 0));
+                GD_CUDA(cudaMemcpyAsync((void*)(stage_dev + j->lo * b->R), j->buf, (size_t)(j->hi - j->lo) * b->R,
+                                        cudaMemcpyHostToDevice, b->side_c));
+                GD_CUDA(cudaEventRecord(b->ev_ring[r], b->side_c));
+            }
+            if (timed) b->timer.end(t_ce, b->side_c);
+            GD_CUDA(cudaEventRecord(b->ev_H[d], b->side_h));     // every chunk gathered
+            GD_CUDA(cudaStreamWaitEvent(b->side_c, b->ev_H[d], 0));
+            GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_c));
+        } else if (ce) {
+            GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
             // phase 2 by the copy engine on stream C, so that the host gather of the next
             // batch (stream H) overlaps this copy: pinned slot d -> dstage[d].  dstage[d]
             // is free: H waited for the scatter of batch - D before this gather.
@@ -1157,6 +1222,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
             if (timed) b->timer.end(t_ce, b->side_c);
             GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_c));
         } else {
+            GD_CUDA(cudaLaunchHostFunc(b->side_h, host_gather_cb, ss));
             GD_CUDA(cudaHostGetDevicePointer((void**)&stage_dev, ss->staging, 0));
             if (timed) b->timer.end(b->timer.begin(b->side_h), b->side_h);
             GD_CUDA(cudaEventRecord(b->ev_E[d], b->side_h));

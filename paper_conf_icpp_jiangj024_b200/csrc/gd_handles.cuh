@@ -44,6 +44,13 @@ struct GdCtl {
 struct gd_buffer;
 
 // One slot of the staged miss path (phase 1 host gather -> phase 2 contiguous pull).
+struct ChunkJob {
+    struct StagedSlot* ss = nullptr;
+    int64_t lo = 0, hi = 0;   // staged ranks [lo, hi) of this chunk
+    uint8_t* buf = nullptr;   // pinned ring buffer the chunk is gathered into
+    bool first = false;       // first chunk of the batch (resets the batch's cpu_ms)
+};
+
 struct StagedSlot {
     gd_buffer* owner = nullptr;
     int d = 0;
@@ -112,6 +119,15 @@ struct gd_buffer {
     bool ce_mode = true;
     uint8_t* dstage = nullptr;           // HBM [D][n_max x R] (copy-engine mode)
     double m_est = 0;                    // misses of a recently completed batch
+    // chunked copy-engine staging (stage_chunk_rows > 0): the host gathers chunk c of the
+    // staged share into ring buffer (k mod kStageRing) of a small pinned ring that stays
+    // in the CPU caches, and the copy engine moves each chunk as soon as it is gathered
+    int64_t stage_chunk_rows = 0;
+    uint8_t* ring_mem = nullptr;         // pinned [kStageRing x stage_chunk_rows x R]
+    uint64_t chunk_counter = 0;
+    std::vector<cudaEvent_t> ev_ring;    // [kStageRing] copy out of ring buffer r done
+    cudaEvent_t ev_chunk = nullptr;      // chunk gathered (re-recorded per chunk)
+    std::vector<struct ChunkJob> jobs;   // [D x max chunks] host-function arguments
     std::vector<StagedSlot> stg;
     uint8_t* stage_mem = nullptr;        // pinned allocations behind stg
     int32_t* hnodes_mem = nullptr;

@@ -37,14 +37,17 @@ struct HostGatherPool::Impl {
     const int32_t* rows = nullptr;
     uint8_t* dst = nullptr;
     int64_t n = 0, R = 0, P = 1;
+    bool nt = true;
     std::atomic<int64_t> next{0};
-    static constexpr int64_t kChunk = 512;
+    static constexpr int64_t kChunk = 256;
 
     // Row copy with non-temporal stores: the staging slot is read next by the GPU over
     // PCIe, so keeping it out of the CPU caches avoids snoop hits on dirty lines, and
     // streaming stores skip the read-for-ownership of every destination line.
-    static void copy_row(uint8_t* d, const uint8_t* s, int64_t R) {
-        if ((R & 15) == 0 && (((uintptr_t)d) & 15) == 0) {
+    static void copy_row(uint8_t* d, const uint8_t* s, int64_t R, bool nt) {
+        if (!nt) {
+            std::memcpy(d, s, (size_t)R);
+        } else if ((R & 15) == 0 && (((uintptr_t)d) & 15) == 0) {
             const __m128i* sp = (const __m128i*)s;
             __m128i* dp = (__m128i*)d;
             const int64_t n16 = R >> 4;
@@ -81,7 +84,7 @@ struct HostGatherPool::Impl {
             for (int64_t j = lo; j < hi && j < lo + pf; ++j) prefetch_row(row_ptr(rows[j]));
             for (int64_t j = lo; j < hi; ++j) {
                 if (j + pf < hi) prefetch_row(row_ptr(rows[j + pf]));
-                copy_row(dst + j * R, row_ptr(rows[j]), R);
+                copy_row(dst + j * R, row_ptr(rows[j]), R, nt);
             }
         }
         _mm_sfence();   // streaming stores globally visible before the GPU pull is released
@@ -124,7 +127,7 @@ HostGatherPool::~HostGatherPool() {
 int HostGatherPool::threads() const { return (int)impl_->workers.size() + 1; }
 
 double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst,
-                              int64_t P) {
+                              int64_t P, bool nt) {
     const auto t0 = std::chrono::steady_clock::now();
     if (n > 0) {
         Impl& I = *impl_;
@@ -136,6 +139,7 @@ double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n
             I.n = n;
             I.R = R;
             I.P = P;
+            I.nt = nt;
             I.next.store(0, std::memory_order_relaxed);
             I.active = (int)I.workers.size();
             ++I.generation;

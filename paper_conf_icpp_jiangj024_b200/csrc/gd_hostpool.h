@@ -11,7 +11,10 @@ class HostGatherPool {
     ~HostGatherPool();
     int threads() const;
     // dst[j*R : (j+1)*R] = src[(rows[j] mod P)*R : ...] for j < n, on all threads; returns elapsed ms.
-    double gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst, int64_t P);
+    // nt = true: non-temporal stores (the destination is read later, from DRAM); false:
+    // ordinary stores (the destination is a small cache-resident ring read at once by DMA).
+    double gather(const uint8_t* src, const int32_t* rows, int64_t n, int64_t R, uint8_t* dst, int64_t P,
+                  bool nt = true);
 
    private:
     struct Impl;

@@ -190,9 +190,15 @@ def test_extract_parity_tiny_evict(tiny, gd, Q):
     run_schedule(gd, g, ip, ix, feat, S, Q, seeds, list(cfg.fanouts))
 
 
-@pytest.mark.parametrize("copy_engine", [True, False])
+# phase 2 of the staged share: SM pull of the pinned slot, or copy engine with the
+# default 8 MB chunk ring, with 64 KB chunks (many chunks per batch, ring reuse), or
+# with one chunk per batch (GD_STAGE_CHUNK_KB=0)
+STAGE_MODES = {"pull": (False, None), "ce": (True, None), "ce-64k": (True, "64"), "ce-whole": (True, "0")}
+
+
+@pytest.mark.parametrize("mode", list(STAGE_MODES))
 @pytest.mark.parametrize("config", [(0, -1.0), (4, 0.0), (4, 1.0), (3, 0.3), (8, -1.0), (1, 0.9)])
-def test_extract_parity_miss_paths(gd, config, copy_engine):
+def test_extract_parity_miss_paths(gd, config, mode, monkeypatch):
     """The miss stream split between zero-copy and the staged (host gather + copy engine
     or SM pull) path: every split gives the same bytes, alias and state."""
     N, E = 60_000, 600_000
@@ -202,6 +208,9 @@ def test_extract_parity_miss_paths(gd, config, copy_engine):
     order = synth.epoch_order(synth.train_nodes(N, 0.3))
     seeds = [order[b * 500:(b + 1) * 500].numpy() for b in range(16)]
     nb, _ = O.sample_bounds(500, [10, 5], N, E)
+    copy_engine, chunk_kb = STAGE_MODES[mode]
+    if chunk_kb is not None:
+        monkeypatch.setenv("GD_STAGE_CHUNK_KB", chunk_kb)
     run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 3 * nb[-1], 3, seeds, [10, 5],
                  check_state_every=4, config=config, stage_mode=copy_engine)
 
@@ -221,9 +230,9 @@ def test_extract_parity_bounded_table(gd, preload):
                  check_state_every=3, num_nodes=N)
 
 
-@pytest.mark.parametrize("copy_engine", [True, False])
+@pytest.mark.parametrize("mode", list(STAGE_MODES))
 @pytest.mark.parametrize("R", [400, 12, 1536])
-def test_extract_parity_row_sizes(gd, R, copy_engine):
+def test_extract_parity_row_sizes(gd, R, mode, monkeypatch):
     """Row widths: 16-byte vector path (400 = products, 1536 = mag240m fp16) and the 4-byte path."""
     N, E = 20_000, 150_000
     indptr, indices = make_graph(N, E, seed=5)
@@ -232,6 +241,9 @@ def test_extract_parity_row_sizes(gd, R, copy_engine):
     order = synth.epoch_order(synth.train_nodes(N, 0.2))
     seeds = [order[b * 300:(b + 1) * 300].numpy() for b in range(10)]
     nb, _ = O.sample_bounds(300, [10, 5], N, E)
+    copy_engine, chunk_kb = STAGE_MODES[mode]
+    if chunk_kb is not None:
+        monkeypatch.setenv("GD_STAGE_CHUNK_KB", chunk_kb)
     run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 2 * nb[-1] + 17, 2, seeds, [10, 5], check_state_every=3,
                  config=(4, 0.3), stage_mode=copy_engine)
 
