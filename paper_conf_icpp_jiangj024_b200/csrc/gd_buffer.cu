@@ -659,7 +659,8 @@ static void buffer_free(gd_buffer* b) {
     delete b->pool;
     b->scan.release();
     b->timer.destroy();
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_ring})
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_ring,
+                    &b->ev_s0})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
     for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk})
@@ -791,8 +792,9 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G})
         if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H}) {
-        const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1);
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_s0}) {
+        const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1 || v == &b->ev_E ||
+                             v == &b->ev_s0);
         v->assign(b->D, nullptr);
         for (int d = 0; d < b->D; ++d)
             if (cudaEventCreateWithFlags(&(*v)[d], timing ? cudaEventDefault : cudaEventDisableTiming) != cudaSuccess)
@@ -974,7 +976,28 @@ static void adapt_alpha(gd_buffer* b, int d) {
     }
     // misses per batch, for the copy-engine staging size (its pop finished long ago)
     b->m_est = (double)((volatile int64_t*)ss.h_meta)[0];
-    if (b->alpha_fixed || b->r_link <= 0) return;
+    if (b->alpha_fixed) return;
+    if (b->ce_mode && b->stage_chunk_rows > 0) {
+        // Chunked copy-engine staging: both paths share the link and the host memory
+        // system, so isolated rates do not add up.  Balance the two paths' measured
+        // durations instead (fixed point of alpha = r_zc / (r_zc + r_st) with the rates
+        // each path achieved while running concurrently with the other).
+        const double st_rows = (double)ss.h_meta[2], z_rows = (double)ss.h_meta[1];
+        float tz = 0, ts = 0;
+        if (z_rows >= 1024 && cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]) == cudaSuccess && tz > 0) {
+            const double r = z_rows * (double)b->R / tz;
+            b->r_zc = b->r_zc > 0 ? 0.7 * b->r_zc + 0.3 * r : r;
+        }
+        if (st_rows >= 1024 && cudaEventElapsedTime(&ts, b->ev_s0[d], b->ev_E[d]) == cudaSuccess && ts > 0) {
+            const double r = st_rows * (double)b->R / ts;
+            b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
+        }
+        cudaGetLastError();
+        if (b->r_zc > 0 && b->r_host > 0)
+            b->alpha = std::min(0.9, std::max(0.02, b->r_zc / (b->r_zc + b->r_host)));
+        return;
+    }
+    if (b->r_link <= 0) return;
     const double staged_rows = (double)ss.h_meta[2], zc_rows = (double)ss.h_meta[1];
     if (staged_rows >= 2048 && ss.cpu_ms > 0) {
         const double r = staged_rows * (double)b->R / ss.cpu_ms;
@@ -1187,6 +1210,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
             const int64_t ch = b->stage_chunk_rows, nch = cap > 0 ? cdiv(cap, ch) : 0;
             const int64_t maxch = cdiv(b->n_max, ch);
             const int t_ce = timed ? b->timer.begin(b->side_c) : -1;
+            GD_CUDA(cudaEventRecord(b->ev_s0[d], b->side_h));   // staged path starts (after its waits)
             if (nch == 0) ss->cpu_ms = 0;
             for (int64_t c = 0; c < nch; ++c) {
                 const int r = (int)(b->chunk_counter++ % kStageRing);

@@ -102,6 +102,7 @@ struct gd_buffer {
     std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
     std::vector<cudaEvent_t> ev_E, ev_P; // [D] staging slot d ready in HBM or pinned / staged pull done
     std::vector<cudaEvent_t> ev_H;       // [D] host gather of slot d done (copy-engine mode)
+    std::vector<cudaEvent_t> ev_s0;      // [D] staged path of slot d started (chunked mode, timing)
     cudaStream_t side_c = nullptr;       // C: copy-engine H2D of the staged share
     std::vector<cudaEvent_t> ev_z0, ev_z1, ev_p0, ev_p1;   // [D] timing of the two miss paths
     int64_t* trip_split = nullptr;       // [D] K0: misses [0, K0) zero-copy, [K0, M) staged
