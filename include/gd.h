@@ -233,6 +233,38 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
 gd_status gd_buffer_stage_mode(gd_buffer* b, int copy_engine);
 
 /* ----------------------------------------------------------------------------
+ * f2: NVLink peer feature buffers.  P:142: "each subprocess ... may
+ * reuse feature data that have been loaded [by] other subprocesses" (the paper shares
+ * the host staging buffer; on B200 the peers' HBM buffers are one NVLink/NVSwitch hop
+ * away).  With peers attached, every miss of gd_extract first looks its node up in
+ * each peer's mapping table and, if the peer slot is published (see below),
+ * copies the row over NVLink into the local slot and `out`; only the misses no peer
+ * served go to the host paths.  Alg. 1 is unchanged (a peer-served node is still a
+ * miss that takes a local LRU slot): out, alias, hits/misses and the buffer state are
+ * identical with or without peers.
+ * Consistency (seqlock, no locks): a buffer tags slot s with (batch epoch << 32 | node)
+ * after every copy into it has finished and clears the tag when the slot is
+ * reassigned (before it is refilled); a reader checks the tag, copies, re-reads the
+ * tag and falls back to the host when it changed.  Tags never repeat, so a stale copy
+ * is always detected.
+ *   gd_buffer_peer_attach     in-process peers (same or other device; P2P access is
+ *                             enabled here).  npeers = 0 detaches.  <= 7 peers; they
+ *                             must have the same num_nodes, row_bytes and table rows.
+ *   gd_buffer_peer_export_ipc writes GD_PEER_BLOB_BYTES describing b (sizes + CUDA IPC
+ *                             handles of its map, tags and slots) for other processes.
+ *   gd_buffer_peer_attach_ipc attaches npeers blobs (consecutive) from other processes;
+ *                             the handles are opened here and closed at destroy.
+ *   gd_buffer_peer_stats      synchronises; rows served by peers and misses probed since init.
+ * Peers stay alive (not destroyed) while attached.  Synchronise b's streams; call
+ * between batches.
+ * ------------------------------------------------------------------------- */
+#define GD_PEER_BLOB_BYTES 256
+gd_status gd_buffer_peer_attach(gd_buffer* b, int npeers, gd_buffer* const* peers);
+gd_status gd_buffer_peer_export_ipc(gd_buffer* b, void* blob, int64_t blob_bytes);
+gd_status gd_buffer_peer_attach_ipc(gd_buffer* b, int npeers, const void* blobs);
+gd_status gd_buffer_peer_stats(gd_buffer* b, int64_t* served, int64_t* probed);
+
+/* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a
  * slot whose count reaches zero is appended at the tail (MRU end) of the standby
  * list.  The node stays valid until its slot is reused (delayed invalidation).

@@ -277,6 +277,33 @@ class FeatureBuffer:
         return {"bookkeeping_ms": ms[0], "gather_ms": ms[1], "miss_zero_copy_ms": ms[2], "miss_staged_ms": ms[3],
                 "host_gather_ms": ms[4], "zero_copy_share": ms[5], "staged_copy_ms": ms[6], "batches": n.value}
 
+    # ---- f2: NVLink peer feature buffers
+    PEER_BLOB_BYTES = 256
+
+    def peer_attach(self, peers):
+        """gd_buffer_peer_attach: in-process peer buffers ([] detaches)."""
+        arr = (ctypes.c_void_p * max(1, len(peers)))(*[p._h.value for p in peers])
+        check(lib.gd_buffer_peer_attach(self._h, len(peers), arr))
+        self._peers = list(peers)      # keep them alive while attached
+
+    def peer_export_ipc(self) -> bytes:
+        """gd_buffer_peer_export_ipc: this buffer's descriptor for other processes."""
+        blob = ctypes.create_string_buffer(self.PEER_BLOB_BYTES)
+        check(lib.gd_buffer_peer_export_ipc(self._h, blob, self.PEER_BLOB_BYTES))
+        return blob.raw
+
+    def peer_attach_ipc(self, blobs):
+        """gd_buffer_peer_attach_ipc: attach other processes' buffers (their export blobs)."""
+        data = b"".join(blobs)
+        buf = ctypes.create_string_buffer(data, max(1, len(data)))
+        check(lib.gd_buffer_peer_attach_ipc(self._h, len(blobs), buf))
+
+    def peer_stats(self):
+        """gd_buffer_peer_stats: (rows served by peers, misses probed) since init."""
+        s, p = ctypes.c_int64(), ctypes.c_int64()
+        check(lib.gd_buffer_peer_stats(self._h, ctypes.byref(s), ctypes.byref(p)))
+        return s.value, p.value
+
     def stage_mode(self, copy_engine: bool):
         """gd_buffer_stage_mode: phase 2 of the staged share by copy engine (True) or SM pull."""
         check(lib.gd_buffer_stage_mode(self._h, int(bool(copy_engine))))

@@ -22,6 +22,7 @@ EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy",
            "gd_buffer_init", "gd_buffer_destroy", "gd_extract", "gd_buffer_release", "gd_check_device_status",
            "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream", "gd_buffer_timing",
            "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config", "gd_buffer_stage_mode",
+           "gd_buffer_peer_attach", "gd_buffer_peer_export_ipc", "gd_buffer_peer_attach_ipc", "gd_buffer_peer_stats",
            "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod"]
 
 
@@ -78,6 +79,10 @@ def _load():
     L.gd_buffer_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     L.gd_buffer_config.argtypes = [_vp, ctypes.c_int, ctypes.c_double, ctypes.c_int, ctypes.c_int]
     L.gd_buffer_stage_mode.argtypes = [_vp, ctypes.c_int]
+    L.gd_buffer_peer_attach.argtypes = [_vp, ctypes.c_int, ctypes.POINTER(_vp)]
+    L.gd_buffer_peer_export_ipc.argtypes = [_vp, ctypes.c_void_p, ctypes.c_int64]
+    L.gd_buffer_peer_attach_ipc.argtypes = [_vp, ctypes.c_int, ctypes.c_void_p]
+    L.gd_buffer_peer_stats.argtypes = [_vp, ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:

@@ -165,6 +165,7 @@ struct PopArgs {
     int64_t* trip_split;            // K0 = floor(M * alpha_q16 / 2^16): first staged rank
     uint32_t alpha_q16;
     long long staged_cap;           // >= 0 (copy-engine staging): K0 = max(0, M - staged_cap)
+    unsigned long long* ready;      // [S] publication tags: a reassigned slot is unpublished
     int32_t* h_nodes;               // mapped host: node ids of ranks [K0, M) (staged share)
     int64_t* h_meta;                // mapped host: {M, K0, M - K0}
     int64_t* stats;                 // caller's stats or null: [2] = K0, [3] = M - K0
@@ -295,6 +296,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                 a.reverse[s] = v;                               // line 28
                 a.alias[i] = s;                                 // line 29
                 a.pos_of_slot[s] = -1;
+                a.ready[s] = kReadyNone;                        // peers stop reading it (f2)
                 a.trip[rank] = make_int4(v, s, i, 0);
                 if (rank >= K0 && a.h_nodes) a.h_nodes[rank - K0] = v;
                 if (rank == M - 1) {
@@ -386,6 +388,112 @@ __global__ void k_miss_copy_w4(const int4* __restrict__ trip, const int64_t* __r
         ((uint32_t*)(slots + (int64_t)tr.y * R))[c] = v;
         ((uint32_t*)(out + (int64_t)tr.z * R))[c] = v;
     }
+}
+
+// ------------------------------------------------------- f2: NVLink peer buffers
+// One warp per miss: look the node up in each peer's mapping table (a hint), check the
+// peer slot's publication tag, copy the row over NVLink into the local slot and `out`,
+// then re-read the tag (seqlock): unchanged = the copy is the node's row (a slot is
+// unpublished before it is refilled, and a tag (epoch, node) never repeats); otherwise
+// the miss goes to the host paths, which rewrite slot and `out`.  Unserved misses are
+// compacted into trip2 (order irrelevant: every path writes the same bytes).
+__global__ void __launch_bounds__(256) k_peer_probe(const int4* __restrict__ trip, const int64_t* __restrict__ tcount,
+                                                    PeerView pv, int npeers, uint8_t* __restrict__ slots,
+                                                    uint8_t* __restrict__ out, int64_t R, int4* __restrict__ trip2,
+                                                    int64_t* __restrict__ t2count, unsigned long long* ctr) {
+    const int lane = threadIdx.x & 31;
+    const int64_t M = *tcount;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    const int64_t cpr = R >> 4;
+    unsigned long long served = 0;
+    for (int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < M; k += warps) {
+        const int4 tr = trip[k];
+        bool ok = false;
+        for (int p = 0; p < npeers && !ok; ++p) {
+            unsigned long long t1 = kReadyNone;
+            int32_t ps = -1;
+            if (lane == 0) {
+                int2 m;
+                asm volatile("ld.relaxed.sys.global.v2.s32 {%0,%1}, [%2];" : "=r"(m.x), "=r"(m.y) : "l"(pv.map[p] + tr.x));
+                if (m.x >= 0 && (m.y & 1)) {
+                    ps = m.x;
+                    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(t1) : "l"(pv.ready[p] + ps) : "memory");
+                    if ((uint32_t)t1 != (uint32_t)tr.x || t1 == kReadyNone) ps = -1;
+                }
+            }
+            ps = __shfl_sync(0xffffffffu, ps, 0);
+            if (ps < 0) continue;
+            const uint4* src = (const uint4*)(pv.slots[p] + (int64_t)ps * R);
+            uint4* ds = (uint4*)(slots + (int64_t)tr.y * R);
+            uint4* dout = (uint4*)(out + (int64_t)tr.z * R);
+            for (int64_t c = lane; c < cpr; c += 32) {
+                uint4 v;
+                asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
+                             : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(src + c));
+                ds[c] = v;
+                dout[c] = v;
+            }
+            __syncwarp();
+            __threadfence_system();   // the row's loads are ordered before the tag re-read
+            int good = 0;
+            if (lane == 0) {
+                unsigned long long t2;
+                asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(t2) : "l"(pv.ready[p] + ps) : "memory");
+                good = t2 == t1;
+            }
+            ok = __shfl_sync(0xffffffffu, good, 0) != 0;
+        }
+        if (ok) {
+            ++served;
+        } else if (lane == 0) {
+            const unsigned long long j = atomicAdd((unsigned long long*)t2count, 1ull);
+            trip2[j] = tr;
+        }
+    }
+    if (lane == 0 && served) atomicAdd(ctr, served);
+    if (threadIdx.x == 0 && blockIdx.x == 0) atomicAdd(ctr + 1, (unsigned long long)M);
+}
+
+// After k_peer_probe: split the unserved misses between zero-copy [0, K0) and staged
+// [K0, M2) (the rule k_pop_assign applies without peers) and publish the staged share's
+// node list and counts to the host gather.
+__global__ void k_peer_split(const int4* __restrict__ trip2, const int64_t* __restrict__ t2count,
+                             int64_t* __restrict__ t2split, uint32_t alpha_q16, long long staged_cap,
+                             int32_t* __restrict__ h_nodes, int64_t* __restrict__ h_meta, int64_t* __restrict__ stats) {
+    const long long M = *t2count;
+    const long long K0 = staged_cap >= 0 ? (M > staged_cap ? M - staged_cap : 0)
+                                         : (long long)(((unsigned long long)M * alpha_q16) >> 16);
+    if (h_nodes)
+        for (long long k = K0 + (long long)blockIdx.x * blockDim.x + threadIdx.x; k < M;
+             k += (long long)gridDim.x * blockDim.x)
+            h_nodes[k - K0] = trip2[k].x;
+    if (blockIdx.x == 0 && threadIdx.x == 0) {
+        *t2split = K0;
+        if (h_meta) {
+            h_meta[0] = M;
+            h_meta[1] = K0;
+            h_meta[2] = M - K0;
+        }
+        if (stats) {
+            stats[2] = K0;
+            stats[3] = M - K0;
+        }
+    }
+}
+
+// Publish the batch's newly filled slots to peers once every copy into them is done.
+__global__ void k_publish(const int4* __restrict__ trip, const int64_t* __restrict__ tcount,
+                          unsigned long long* __restrict__ ready, unsigned long long epoch) {
+    const int64_t M = *tcount;
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < M; k += (int64_t)gridDim.x * blockDim.x) {
+        const int4 tr = trip[k];
+        ready[tr.y] = (epoch << 32) | (uint32_t)tr.x;
+    }
+}
+
+__global__ void k_init_ready(unsigned long long* ready, int64_t S, int64_t N, int preload) {
+    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < S; s += (int64_t)gridDim.x * blockDim.x)
+        ready[s] = (preload && s < N) ? (unsigned long long)(uint32_t)s : kReadyNone;
 }
 
 // ------------------------------------------------------------- a8: hit gather
@@ -651,11 +759,12 @@ static void buffer_free(gd_buffer* b) {
         if (s) cudaStreamSynchronize(s);
     void* ptrs[] = {b->slots, b->map, b->reverse, b->pos_of_slot, b->ring, b->ctl, b->misslist, b->hitlist, b->hcount,
                     b->alias_ws, b->mcount, b->trip, b->trip_count, b->trip_split, b->tickets, b->done_word,
-                    b->hdr.dev_status, b->dstage};
+                    b->hdr.dev_status, b->dstage, b->ready, b->trip2, b->trip2_count, b->trip2_split, b->peer_ctr};
     for (void* p : ptrs)
         if (p) cudaFree(p);
     for (void* p : {(void*)b->stage_mem, (void*)b->hnodes_mem, (void*)b->hmeta_mem, (void*)b->ring_mem})
         if (p) cudaFreeHost(p);
+    for (void* p : b->ipc_opened) cudaIpcCloseMemHandle(p);
     delete b->pool;
     b->scan.release();
     b->timer.destroy();
@@ -757,6 +866,11 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     GD_ALLOC(b->trip_split, b->D * sizeof(int64_t));
     GD_ALLOC(b->tickets, 4 * sizeof(unsigned long long));
     GD_ALLOC(b->done_word, sizeof(unsigned long long));
+    GD_ALLOC(b->ready, capacity_slots * sizeof(unsigned long long));
+    GD_ALLOC(b->trip2, (int64_t)b->D * nm * sizeof(int4));
+    GD_ALLOC(b->trip2_count, b->D * sizeof(int64_t));
+    GD_ALLOC(b->trip2_split, b->D * sizeof(int64_t));
+    GD_ALLOC(b->peer_ctr, 2 * sizeof(unsigned long long));
 #undef GD_ALLOC
     gd_status s = b->scan.ensure(std::max(cdiv(nm, kBTile), cdiv(C, kBTile)) + 1);
     if (s != GD_OK) return fail(s);
@@ -770,10 +884,14 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
         cudaMemset(b->tickets, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
         cudaMemset(b->done_word, 0, sizeof(unsigned long long)) != cudaSuccess ||
         cudaMemset(b->trip_count, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
-        cudaMemset(b->trip_split, 0, b->D * sizeof(int64_t)) != cudaSuccess)
+        cudaMemset(b->trip_split, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
+        cudaMemset(b->trip2_count, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
+        cudaMemset(b->trip2_split, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
+        cudaMemset(b->peer_ctr, 0, 2 * sizeof(unsigned long long)) != cudaSuccess)
         return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: init copies"));
     k_init_map<<<148 * 8, 256>>>(b->map, num_nodes, preload);
     k_init_slots<<<148 * 8, 256>>>(b->reverse, b->pos_of_slot, b->ring, capacity_slots, num_nodes, preload);
+    k_init_ready<<<148 * 8, 256>>>(b->ready, capacity_slots, num_nodes, preload);
     if (preload) {
         for (int64_t v0 = 0; v0 < num_nodes; v0 += table_rows) {   // slot v holds row v mod P
             const int64_t nr = std::min(table_rows, num_nodes - v0);
@@ -901,6 +1019,122 @@ gd_status gd_buffer_stage_mode(gd_buffer* b, int copy_engine) {
     return gd_buffer_config(b, b->host_threads, b->alpha_fixed ? b->alpha : -1.0, 0, 0);
 }
 
+// ------------------------------------------------------------------ f2: peers
+static gd_status drain_streams(gd_buffer* b) {
+    for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
+        if (s) GD_CUDA(cudaStreamSynchronize(s));
+    return GD_OK;
+}
+
+static gd_status set_peers(gd_buffer* b, int n, const int2* const* maps, const unsigned long long* const* readys,
+                           const uint8_t* const* slots) {
+    if (n < 0 || n > kMaxPeers) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: 0..7 peers");
+    for (int p = 0; p < kMaxPeers; ++p) {
+        b->peers.map[p] = p < n ? maps[p] : nullptr;
+        b->peers.ready[p] = p < n ? readys[p] : nullptr;
+        b->peers.slots[p] = p < n ? slots[p] : nullptr;
+    }
+    b->npeers = n;
+    return GD_OK;
+}
+
+gd_status gd_buffer_peer_attach(gd_buffer* b, int npeers, gd_buffer* const* peers) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: bad handle");
+    if (npeers < 0 || npeers > kMaxPeers || (npeers > 0 && !peers))
+        return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: 0..7 peers");
+    const int2* maps[kMaxPeers];
+    const unsigned long long* readys[kMaxPeers];
+    const uint8_t* slots[kMaxPeers];
+    DeviceGuard guard(b->hdr.device);
+    for (int p = 0; p < npeers; ++p) {
+        gd_buffer* q = peers[p];
+        if (!q || q->hdr.magic != kMagicBuffer || q == b)
+            return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: bad peer handle");
+        if (q->N != b->N || q->R != b->R || q->P != b->P)
+            return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: peer has another graph size / row size / table");
+        if (q->hdr.device != b->hdr.device) {
+            int can = 0;
+            GD_CUDA(cudaDeviceCanAccessPeer(&can, b->hdr.device, q->hdr.device));
+            if (!can) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: no P2P path between the devices");
+            cudaError_t e = cudaDeviceEnablePeerAccess(q->hdr.device, 0);
+            if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) return cuda_error(e, "cudaDeviceEnablePeerAccess");
+            cudaGetLastError();
+        }
+        maps[p] = q->map;
+        readys[p] = q->ready;
+        slots[p] = q->slots;
+    }
+    gd_status s = drain_streams(b);
+    if (s != GD_OK) return s;
+    return set_peers(b, npeers, maps, readys, slots);
+}
+
+// blob layout: int64 {magic, N, R, P, S}, then 3 cudaIpcMemHandle_t (map, ready, slots)
+static constexpr int64_t kBlobMagic = 0x4744504545520001ll;   // "GDPEER" v1
+
+gd_status gd_buffer_peer_export_ipc(gd_buffer* b, void* blob, int64_t blob_bytes) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_export_ipc: bad handle");
+    if (!blob || blob_bytes < GD_PEER_BLOB_BYTES) return set_error(GD_ERR_INVALID, "gd_buffer_peer_export_ipc: blob too small");
+    DeviceGuard guard(b->hdr.device);
+    std::memset(blob, 0, GD_PEER_BLOB_BYTES);
+    int64_t* h = (int64_t*)blob;
+    h[0] = kBlobMagic;
+    h[1] = b->N;
+    h[2] = b->R;
+    h[3] = b->P;
+    h[4] = b->S;
+    cudaIpcMemHandle_t* mh = (cudaIpcMemHandle_t*)(h + 5);
+    GD_CUDA(cudaIpcGetMemHandle(&mh[0], b->map));
+    GD_CUDA(cudaIpcGetMemHandle(&mh[1], b->ready));
+    GD_CUDA(cudaIpcGetMemHandle(&mh[2], b->slots));
+    return GD_OK;
+}
+
+gd_status gd_buffer_peer_attach_ipc(gd_buffer* b, int npeers, const void* blobs) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach_ipc: bad handle");
+    if (npeers < 0 || npeers > kMaxPeers || (npeers > 0 && !blobs))
+        return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach_ipc: 0..7 peers");
+    DeviceGuard guard(b->hdr.device);
+    gd_status s = drain_streams(b);
+    if (s != GD_OK) return s;
+    set_peers(b, 0, nullptr, nullptr, nullptr);
+    for (void* p : b->ipc_opened) cudaIpcCloseMemHandle(p);
+    b->ipc_opened.clear();
+    const int2* maps[kMaxPeers];
+    const unsigned long long* readys[kMaxPeers];
+    const uint8_t* slots[kMaxPeers];
+    for (int p = 0; p < npeers; ++p) {
+        const int64_t* h = (const int64_t*)((const uint8_t*)blobs + (int64_t)p * GD_PEER_BLOB_BYTES);
+        if (h[0] != kBlobMagic) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach_ipc: not a peer blob");
+        if (h[1] != b->N || h[2] != b->R || h[3] != b->P)
+            return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach_ipc: peer has another graph size / row size / table");
+        const cudaIpcMemHandle_t* mh = (const cudaIpcMemHandle_t*)(h + 5);
+        void* ptr[3];
+        for (int k = 0; k < 3; ++k) {
+            cudaError_t e = cudaIpcOpenMemHandle(&ptr[k], mh[k], cudaIpcMemLazyEnablePeerAccess);
+            if (e != cudaSuccess) return cuda_error(e, "gd_buffer_peer_attach_ipc: cudaIpcOpenMemHandle");
+            b->ipc_opened.push_back(ptr[k]);
+        }
+        maps[p] = (const int2*)ptr[0];
+        readys[p] = (const unsigned long long*)ptr[1];
+        slots[p] = (const uint8_t*)ptr[2];
+    }
+    return set_peers(b, npeers, maps, readys, slots);
+}
+
+gd_status gd_buffer_peer_stats(gd_buffer* b, int64_t* served, int64_t* probed) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_stats: bad handle");
+    DeviceGuard guard(b->hdr.device);
+    gd_status s = drain_streams(b);
+    if (s != GD_OK) return s;
+    GD_CUDA(cudaDeviceSynchronize());
+    unsigned long long c[2];
+    GD_CUDA(cudaMemcpy(c, b->peer_ctr, sizeof(c), cudaMemcpyDeviceToHost));
+    if (served) *served = (int64_t)c[0];
+    if (probed) *probed = (int64_t)c[1];
+    return GD_OK;
+}
+
 gd_status gd_buffer_timing(gd_buffer* b, int enable) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_timing: bad handle");
     DeviceGuard guard(b->hdr.device);
@@ -977,26 +1211,9 @@ static void adapt_alpha(gd_buffer* b, int d) {
     // misses per batch, for the copy-engine staging size (its pop finished long ago)
     b->m_est = (double)((volatile int64_t*)ss.h_meta)[0];
     if (b->alpha_fixed) return;
-    if (b->ce_mode && b->stage_chunk_rows > 0) {
-        // Chunked copy-engine staging: both paths share the link and the host memory
-        // system, so isolated rates do not add up.  Balance the two paths' measured
-        // durations instead (fixed point of alpha = r_zc / (r_zc + r_st) with the rates
-        // each path achieved while running concurrently with the other).
-        const double st_rows = (double)ss.h_meta[2], z_rows = (double)ss.h_meta[1];
-        float tz = 0, ts = 0;
-        if (z_rows >= 1024 && cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]) == cudaSuccess && tz > 0) {
-            const double r = z_rows * (double)b->R / tz;
-            b->r_zc = b->r_zc > 0 ? 0.7 * b->r_zc + 0.3 * r : r;
-        }
-        if (st_rows >= 1024 && cudaEventElapsedTime(&ts, b->ev_s0[d], b->ev_E[d]) == cudaSuccess && ts > 0) {
-            const double r = st_rows * (double)b->R / ts;
-            b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
-        }
-        cudaGetLastError();
-        if (b->r_zc > 0 && b->r_host > 0)
-            b->alpha = std::min(0.9, std::max(0.02, b->r_zc / (b->r_zc + b->r_host)));
-        return;
-    }
+    // (Balancing the two paths' concurrently measured durations instead was tried and
+    // measured worse: the zero-copy share is translation-bound and its SM loads slow the
+    // copy engine's transfers, so the smallest share that keeps the link busy wins.)
     if (b->r_link <= 0) return;
     const double staged_rows = (double)ss.h_meta[2], zc_rows = (double)ss.h_meta[1];
     if (staged_rows >= 2048 && ss.cpu_ms > 0) {
@@ -1015,7 +1232,11 @@ static void adapt_alpha(gd_buffer* b, int d) {
         a = b->r_zc / (b->r_zc + b->r_host);
     else
         a = 1.0 - b->r_host / b->r_link;
-    b->alpha = std::min(0.9, std::max(0.05, a));
+    // With copy-engine staging the zero-copy share also costs the DMA engine: its random
+    // 4 KB-page reads contend for the host's DMA translation, and a share above ~0.2 was
+    // measured to collapse the copy rate (to ~17 GB/s at 0.4); cap it there.
+    const double hi = (b->ce_mode && b->dstage) ? 0.2 : 0.9;
+    b->alpha = std::min(hi, std::max(0.05, a));
 }
 
 // Contiguous host-link pull rate (bytes/ms), measured once on the staging memory.
@@ -1133,11 +1354,19 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.trip_split = tsplit;
     pa.alpha_q16 = alpha_q16;
     pa.staged_cap = cap;
+    pa.ready = b->ready;
     pa.h_nodes = nullptr;
     pa.h_meta = nullptr;
+    int32_t* h_nodes_dev = nullptr;
+    int64_t* h_meta_dev = nullptr;
     if (staged) {
-        GD_CUDA(cudaHostGetDevicePointer((void**)&pa.h_nodes, ss->h_nodes, 0));
-        GD_CUDA(cudaHostGetDevicePointer((void**)&pa.h_meta, ss->h_meta, 0));
+        GD_CUDA(cudaHostGetDevicePointer((void**)&h_nodes_dev, ss->h_nodes, 0));
+        GD_CUDA(cudaHostGetDevicePointer((void**)&h_meta_dev, ss->h_meta, 0));
+    }
+    const bool peer = b->npeers > 0 && !b->preload;
+    if (!peer) {   // with peers, k_peer_split publishes the host share instead
+        pa.h_nodes = h_nodes_dev;
+        pa.h_meta = h_meta_dev;
     }
     pa.stats = stats;
     pa.ticket = b->tickets;
@@ -1152,6 +1381,21 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     b->scan.flip();
     b->ctl_parity ^= 1;
     if (timed) b->timer.end(t_book, st);
+    // f2: peers first; the host paths copy what no peer served (trip2)
+    int4* mtrip = trip;
+    int64_t* mcount_d = tcount;
+    int64_t* msplit = tsplit;
+    if (peer) {
+        mtrip = b->trip2 + (int64_t)d * b->n_max;
+        mcount_d = b->trip2_count + d;
+        msplit = b->trip2_split + d;
+        GD_CUDA(cudaMemsetAsync(mcount_d, 0, sizeof(int64_t), st));
+        k_peer_probe<<<148 * 8, 256, 0, st>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R, mtrip,
+                                             mcount_d, b->peer_ctr);
+        GD_DEBUG_AFTER("k_peer_probe", st);
+        k_peer_split<<<148, 256, 0, st>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats);
+        GD_DEBUG_AFTER("k_peer_split", st);
+    }
     GD_CUDA(cudaEventRecord(b->ev_L, st));
 
     // Stream order (the host enqueue order below matters: each wait captures the event's
@@ -1191,9 +1435,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaEventRecord(b->ev_z0[d], b->side));
     if (b->preload) {
     } else if (b->R % 16 == 0)
-        k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
+        k_miss_copy<4, false><<<b->zc_blocks, 1024, 0, b->side>>>(mtrip, nullptr, msplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
     else
-        k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(trip, nullptr, tsplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
+        k_miss_copy_w4<false><<<b->zc_blocks, 1024, 0, b->side>>>(mtrip, nullptr, msplit, b->feat_dev, b->slots, (uint8_t*)out, b->R, b->P);
     GD_DEBUG_AFTER("k_miss_copy", b->side);
     GD_CUDA(cudaEventRecord(b->ev_z1[d], b->side));
     if (timed) b->timer.end(t_zc, b->side);
@@ -1255,9 +1499,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         const int t_pl = timed ? b->timer.begin(b->side_p) : -1;
         GD_CUDA(cudaEventRecord(b->ev_p0[d], b->side_p));
         if (b->R % 16 == 0)
-            k_miss_copy<4, true><<<ce ? 64 : b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
+            k_miss_copy<4, true><<<ce ? 64 : b->pull_blocks, 1024, 0, b->side_p>>>(mtrip, msplit, mcount_d, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         else
-            k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(trip, tsplit, tcount, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
+            k_miss_copy_w4<true><<<b->pull_blocks, 1024, 0, b->side_p>>>(mtrip, msplit, mcount_d, stage_dev, b->slots, (uint8_t*)out, b->R, b->P);
         GD_DEBUG_AFTER("k_stage_copy", b->side_p);
         GD_CUDA(cudaEventRecord(b->ev_p1[d], b->side_p));
         if (timed) b->timer.end(t_pl, b->side_p);
@@ -1272,6 +1516,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_X, 0));
     if (staged) GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_Xs, 0));
     GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_G, 0));
+    // f2: the batch's new slots are complete: publish them to peers (before `done`, so a
+    // release, and with it any reuse of these slots, is ordered after the publication)
+    if (!b->preload) k_publish<<<148, 256, 0, b->side_j>>>(trip, tcount, b->ready, pa.epoch);
     GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side_j));
     if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side_j));
     GD_CUDA(cudaGetLastError());
@@ -1384,10 +1631,14 @@ gd_status gd_buffer_set_state(gd_buffer* b, const int32_t* map_slot, const int32
     c[0].base = 0;
     c[1] = c[0];
     GD_CUDA(cudaMemcpy(b->ctl, c, sizeof(c), cudaMemcpyHostToDevice));
+    std::vector<unsigned long long> tags(b->S, kReadyNone);
     for (int64_t v = 0; v < b->N; ++v)
-        if ((map_valid[v] & 1) && map_slot[v] >= 0)
+        if ((map_valid[v] & 1) && map_slot[v] >= 0) {
             GD_CUDA(cudaMemcpy(b->slots + (int64_t)map_slot[v] * b->R, (const uint8_t*)b->host_feat + (v % b->P) * b->R, b->R,
                                cudaMemcpyHostToDevice));
+            tags[map_slot[v]] = (unsigned long long)(uint32_t)v;
+        }
+    GD_CUDA(cudaMemcpy(b->ready, tags.data(), b->S * sizeof(unsigned long long), cudaMemcpyHostToDevice));
     return GD_OK;
 }
 

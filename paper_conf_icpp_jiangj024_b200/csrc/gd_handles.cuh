@@ -43,6 +43,16 @@ struct GdCtl {
 
 struct gd_buffer;
 
+namespace gd {
+constexpr int kMaxPeers = 7;
+constexpr unsigned long long kReadyNone = ~0ull;
+struct PeerView {
+    const int2* map[kMaxPeers];
+    const unsigned long long* ready[kMaxPeers];
+    const uint8_t* slots[kMaxPeers];
+};
+}  // namespace gd
+
 // One slot of the staged miss path (phase 1 host gather -> phase 2 contiguous pull).
 struct ChunkJob {
     struct StagedSlot* ss = nullptr;
@@ -129,6 +139,17 @@ struct gd_buffer {
     std::vector<cudaEvent_t> ev_ring;    // [kStageRing] copy out of ring buffer r done
     cudaEvent_t ev_chunk = nullptr;      // chunk gathered (re-recorded per chunk)
     std::vector<struct ChunkJob> jobs;   // [D x max chunks] host-function arguments
+    // f2: NVLink peer feature buffers (subprocesses reuse rows another has loaded).
+    // ready[s] = (epoch << 32) | node once slot s holds that node's row (published after
+    // the batch's copies joined), kReadyNone from the moment the slot is reassigned.
+    unsigned long long* ready = nullptr; // HBM [S]
+    int npeers = 0;
+    gd::PeerView peers;                  // device pointers of the peers' map / ready / slots
+    std::vector<void*> ipc_opened;       // pointers opened with cudaIpcOpenMemHandle (closed at destroy)
+    int4* trip2 = nullptr;               // [D][n_max] misses no peer served (compacted)
+    int64_t* trip2_count = nullptr;      // [D]
+    int64_t* trip2_split = nullptr;      // [D]
+    unsigned long long* peer_ctr = nullptr;   // [2] rows served by peers, misses probed
     std::vector<StagedSlot> stg;
     uint8_t* stage_mem = nullptr;        // pinned allocations behind stg
     int32_t* hnodes_mem = nullptr;

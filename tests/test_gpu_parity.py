@@ -405,3 +405,122 @@ def test_run_twice_bitwise_identical_and_gpu_count_independent(gd):
         o = g.sample(seeds[bid], [15, 10, 5], 3, bid, stream=st, workspace=ws)
         st.synchronize()
         assert np.array_equal(o.to_host()["n_id"], a[bid][0])
+
+
+# ------------------------------------------------------------- f2: peer feature buffers
+
+
+def _peer_setup(gd, N=60_000, E=600_000, B=500, fan=(10, 5)):
+    indptr, indices = make_graph(N, E, seed=8)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, 512)
+    order = synth.epoch_order(synth.train_nodes(N, 0.3))
+    nb, _ = O.sample_bounds(B, list(fan), N, E)
+    return g, feat, order, nb[-1], list(fan), B
+
+
+@pytest.mark.parametrize("mode", ["ce", "pull"])
+def test_peer_buffer_parity_and_reuse(gd, mode):
+    """f2: buffer B with buffer A attached as a peer.  A miss of B whose row A holds is
+    copied from A's slot (served > 0); out, alias, hits/misses and B's whole state equal the
+    oracle, which knows nothing about peers (Alg. 1 is unchanged)."""
+    g, feat, order, n_max, fan, B = _peer_setup(gd)
+    S = 3 * n_max
+    bufA = gd.FeatureBuffer(torch.from_numpy(feat), S, 3, n_max)
+    bufB = gd.FeatureBuffer(torch.from_numpy(feat), S, 3, n_max)
+    for buf in (bufA, bufB):
+        buf.stage_mode(mode == "ce")
+        buf.config(4, 0.3)
+    # A loads batches 0..5 and keeps them (released, still valid: delayed invalidation)
+    pendA = []
+    for b in range(6):
+        res = g.sample(order[b * B:(b + 1) * B].cuda(), fan, 3, b)
+        _, _, done = bufA.extract(res.n_id, res.num_nodes_dev, res.max_nodes)
+        done.synchronize()
+        pendA.append(res)
+    for r in pendA:
+        bufA.release(r.n_id, r.num_nodes_dev, r.max_nodes)
+    torch.cuda.synchronize()
+    bufB.peer_attach([bufA])
+    ob = O.Buffer(feat, S)
+    pend = []
+    for b in range(2, 12):       # overlaps A's batches 2..5 exactly, then new batches
+        res = g.sample(order[b * B:(b + 1) * B].cuda(), fan, 3, b)
+        alias = torch.empty(n_max, dtype=torch.int32, device="cuda")
+        stats = torch.zeros(4, dtype=torch.int64, device="cuda")
+        out, _, done = bufB.extract(res.n_id, res.num_nodes_dev, res.max_nodes, alias=alias, stats=stats)
+        done.synchronize()
+        n_id = res.to_host()["n_id"]
+        o_out, o_alias, o_stats = ob.extract(n_id)
+        n = len(n_id)
+        assert tuple(stats.cpu().tolist()[:2]) == o_stats
+        assert np.array_equal(alias[:n].cpu().numpy(), o_alias)
+        assert np.array_equal(out[:n].cpu().numpy(), o_out)
+        pend.append((res, n_id))
+        if len(pend) == 3:
+            r0, n0 = pend.pop(0)
+            bufB.release(r0.n_id, r0.num_nodes_dev, r0.max_nodes)
+            ob.release(n0)
+    compare_state(bufB, ob)
+    served, probed = bufB.peer_stats()
+    assert probed > 0 and served > 0, (served, probed)
+    assert bufA.peer_stats() == (0, 0)
+    assert bufA.check() == 0 and bufB.check() == 0
+    bufB.peer_attach([])
+
+
+def test_peer_buffers_concurrent_eviction(gd):
+    """Two buffers attached to each other run concurrently on their own streams with the
+    minimum capacity (heavy eviction: peer slots are refilled while being read).  The seqlock
+    tags must reject every stale copy: both outputs stay bit-exact with the oracle."""
+    g, feat, order, n_max, fan, B = _peer_setup(gd, B=300)
+    Q = 2
+    S = Q * n_max
+    bufs = [gd.FeatureBuffer(torch.from_numpy(feat), S, Q, n_max) for _ in range(2)]
+    for buf in bufs:
+        buf.config(4, 0.5)
+    bufs[0].peer_attach([bufs[1]])
+    bufs[1].peer_attach([bufs[0]])
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    wss = [g.workspace(), g.workspace()]          # concurrent samplers need their own workspace
+    oracles = [O.Buffer(feat, S), O.Buffer(feat, S)]
+    nbat = 24
+    # rank r takes batches r, r+2, ... with a shift so the two share many nodes in flight
+    sched = [[(2 * j + r) % 40 for j in range(nbat)] for r in range(2)]
+    results = [[], []]
+    pend = [[], []]
+    for j in range(nbat):
+        for r in range(2):
+            b = sched[r][j]
+            with torch.cuda.stream(streams[r]):
+                res = g.sample(order[b * B:(b + 1) * B].cuda(non_blocking=True), fan, 3, b, stream=streams[r],
+                               workspace=wss[r])
+                out = torch.empty((n_max, 512), dtype=torch.uint8, device="cuda")
+                alias = torch.empty(n_max, dtype=torch.int32, device="cuda")
+                _, _, done = bufs[r].extract(res.n_id, res.num_nodes_dev, res.max_nodes, out=out, alias=alias,
+                                             stream=streams[r])
+                streams[r].wait_event(done)
+                results[r].append((res, out, alias))
+                pend[r].append(res)
+                if len(pend[r]) == Q:
+                    r0 = pend[r].pop(0)
+                    bufs[r].release(r0.n_id, r0.num_nodes_dev, r0.max_nodes, stream=streams[r])
+    torch.cuda.synchronize()
+    for r in range(2):
+        opend = []
+        for j, (res, out, alias) in enumerate(results[r]):
+            n_id = res.to_host()["n_id"]
+            o_out, o_alias, _ = oracles[r].extract(n_id)
+            n = len(n_id)
+            assert np.array_equal(out[:n].cpu().numpy(), o_out), (r, j)
+            assert np.array_equal(alias[:n].cpu().numpy(), o_alias), (r, j)
+            opend.append(n_id)
+            if len(opend) == Q:
+                oracles[r].release(opend.pop(0))
+        compare_state(bufs[r], oracles[r])
+    s0, _ = bufs[0].peer_stats()
+    s1, _ = bufs[1].peer_stats()
+    assert s0 + s1 > 0
+    for buf in bufs:
+        buf.peer_attach([])
+        assert buf.check() == 0
