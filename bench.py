@@ -49,6 +49,8 @@ def parse():
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the oracle cpu_baseline sample")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
+                   "peer (CUDA IPC); misses are served from peers' HBM before the host link")
     p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
     p.add_argument("--prewarm-max", type=int, default=400,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
@@ -332,6 +334,13 @@ def run_ours(args, rank, world, local_rank):
         if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
             buf.config(host_threads)
     barrier()
+    if args.peer and world > 1:
+        import torch.distributed as dist
+        blobs = [None] * world
+        dist.all_gather_object(blobs, buf.peer_export_ipc())
+        buf.peer_attach_ipc([bl for r, bl in enumerate(blobs) if r != rank][:7])
+        barrier()
+        log(f"peer buffers attached: {min(world - 1, 7)} per rank")
 
     # ---- buffer pre-warm (untimed): the feature buffer reaches steady state once the
     # cumulative misses exceed its capacity; stats are read every 8 batches
@@ -510,6 +519,12 @@ def run_ours(args, rank, world, local_rank):
                 if r["kernel"].startswith(kname):
                     r["traffic"] = tv
 
+    peer_info = None
+    if args.peer and world > 1:
+        served, probed = buf.peer_stats()
+        served_all, probed_all = sum_over_ranks(served, dev), sum_over_ranks(probed, dev)
+        peer_info = {"served_rows": int(served_all), "probed_misses": int(probed_all),
+                     "served_share": round(served_all / max(1, probed_all), 4), "peers_per_rank": min(world - 1, 7)}
     cpu = None
     log("cpu baseline ...")
     if want_cpu:
@@ -546,6 +561,7 @@ def run_ours(args, rank, world, local_rank):
         "sweep": sweep or None,
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
+        "peer": peer_info,
         "setup_s": round(time.time() - t_setup, 1),
     }
     if rank == 0:
