@@ -772,7 +772,7 @@ static void buffer_free(gd_buffer* b) {
                     &b->ev_s0})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
-    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk})
+    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk, b->ev_S})
         if (e) cudaEventDestroy(e);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
         if (s) cudaStreamDestroy(s);
@@ -907,7 +907,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_g, &b->side_c})
         if (cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
-    for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G})
+    for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G, &b->ev_S})
         if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
     for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_s0}) {
@@ -1389,12 +1389,6 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         mtrip = b->trip2 + (int64_t)d * b->n_max;
         mcount_d = b->trip2_count + d;
         msplit = b->trip2_split + d;
-        GD_CUDA(cudaMemsetAsync(mcount_d, 0, sizeof(int64_t), st));
-        k_peer_probe<<<148 * 8, 256, 0, st>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R, mtrip,
-                                             mcount_d, b->peer_ctr);
-        GD_DEBUG_AFTER("k_peer_probe", st);
-        k_peer_split<<<148, 256, 0, st>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats);
-        GD_DEBUG_AFTER("k_peer_split", st);
     }
     GD_CUDA(cudaEventRecord(b->ev_L, st));
 
@@ -1406,9 +1400,21 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaStreamWaitEvent(b->side_g, b->ev_X, 0));
     GD_CUDA(cudaStreamWaitEvent(b->side_g, b->ev_Xs, 0));
     GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_L, 0));
-    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
+    GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));   // (before the probe: it writes slots too)
+    if (peer) {
+        // f2 on stream Z (off the caller's stream, so the next batch's sampling does not
+        // wait for NVLink round trips): peers serve what they hold, the rest is split
+        // between the host paths.  H waits for the split (its node list).
+        GD_CUDA(cudaMemsetAsync(mcount_d, 0, sizeof(int64_t), b->side));
+        k_peer_probe<<<148 * 8, 256, 0, b->side>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R,
+                                                  mtrip, mcount_d, b->peer_ctr);
+        GD_DEBUG_AFTER("k_peer_probe", b->side);
+        k_peer_split<<<148, 256, 0, b->side>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats);
+        GD_DEBUG_AFTER("k_peer_split", b->side);
+        GD_CUDA(cudaEventRecord(b->ev_S, b->side));
+    }
     if (staged) {
-        GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_L, 0));
+        GD_CUDA(cudaStreamWaitEvent(b->side_h, peer ? b->ev_S : b->ev_L, 0));
         GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_P[d], 0));   // pull of batch - D left slot d
         GD_CUDA(cudaStreamWaitEvent(b->side_p, b->ev_G, 0));
     }

@@ -109,6 +109,7 @@ struct gd_buffer {
     cudaStream_t side_j = nullptr;       // J: joins Z, P and the hit gather into `done`
     cudaStream_t side_g = nullptr;       // G: hit gather (slots -> out)
     cudaEvent_t ev_L = nullptr, ev_X = nullptr, ev_Xs = nullptr, ev_G = nullptr;
+    cudaEvent_t ev_S = nullptr;          // f2: peer probe + split done (stream Z)
     std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
     std::vector<cudaEvent_t> ev_E, ev_P; // [D] staging slot d ready in HBM or pinned / staged pull done
     std::vector<cudaEvent_t> ev_H;       // [D] host gather of slot d done (copy-engine mode)

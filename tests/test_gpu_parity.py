@@ -438,6 +438,9 @@ def test_peer_buffer_parity_and_reuse(gd, mode):
         _, _, done = bufA.extract(res.n_id, res.num_nodes_dev, res.max_nodes)
         done.synchronize()
         pendA.append(res)
+        if len(pendA) == 3:
+            r = pendA.pop(0)
+            bufA.release(r.n_id, r.num_nodes_dev, r.max_nodes)
     for r in pendA:
         bufA.release(r.n_id, r.num_nodes_dev, r.max_nodes)
     torch.cuda.synchronize()
