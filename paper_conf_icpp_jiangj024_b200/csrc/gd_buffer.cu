@@ -434,7 +434,9 @@ __global__ void __launch_bounds__(256) k_peer_probe(const int4* __restrict__ tri
                 dout[c] = v;
             }
             __syncwarp();
-            __threadfence_system();   // the row's loads are ordered before the tag re-read
+            // load-load ordering only (the seqlock read side): the row's loads are ordered
+            // before the tag re-read; a full fence.sc would also drain this warp's stores
+            asm volatile("fence.acq_rel.sys;" ::: "memory");
             int good = 0;
             if (lane == 0) {
                 unsigned long long t2;
@@ -1406,7 +1408,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         // wait for NVLink round trips): peers serve what they hold, the rest is split
         // between the host paths.  H waits for the split (its node list).
         GD_CUDA(cudaMemsetAsync(mcount_d, 0, sizeof(int64_t), b->side));
-        k_peer_probe<<<148 * 8, 256, 0, b->side>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R,
+        k_peer_probe<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R,
                                                   mtrip, mcount_d, b->peer_ctr);
         GD_DEBUG_AFTER("k_peer_probe", b->side);
         k_peer_split<<<148, 256, 0, b->side>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats);
