@@ -401,31 +401,46 @@ __global__ void __launch_bounds__(256) k_peer_probe(const int4* __restrict__ tri
                                                     PeerView pv, int npeers, uint8_t* __restrict__ slots,
                                                     uint8_t* __restrict__ out, int64_t R, int4* __restrict__ trip2,
                                                     int64_t* __restrict__ t2count, unsigned long long* ctr) {
+    // A warp takes 32 misses: every lane looks its miss up in the peers (the round trips
+    // overlap), the warp copies the found rows one after another (16 B per lane), then
+    // every finder re-checks its tag; the unserved misses are appended with one atomic.
     const int lane = threadIdx.x & 31;
     const int64_t M = *tcount;
+    const int64_t gw = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
     const int64_t cpr = R >> 4;
     unsigned long long served = 0;
-    for (int64_t k = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); k < M; k += warps) {
-        const int4 tr = trip[k];
-        bool ok = false;
-        for (int p = 0; p < npeers && !ok; ++p) {
-            unsigned long long t1 = kReadyNone;
-            int32_t ps = -1;
-            if (lane == 0) {
+    for (int64_t k0 = gw * 32; k0 < M; k0 += warps * 32) {
+        const int64_t k = k0 + lane;
+        const bool have = k < M;
+        int4 tr = make_int4(0, 0, 0, 0);
+        int p_hit = -1, ps = -1;
+        unsigned long long t1 = kReadyNone;
+        if (have) {
+            tr = trip[k];
+            for (int p = 0; p < npeers && p_hit < 0; ++p) {
                 int2 m;
                 asm volatile("ld.relaxed.sys.global.v2.s32 {%0,%1}, [%2];" : "=r"(m.x), "=r"(m.y) : "l"(pv.map[p] + tr.x));
-                if (m.x >= 0 && (m.y & 1)) {
+                if (m.x < 0 || !(m.y & 1)) continue;
+                unsigned long long t;
+                asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(t) : "l"(pv.ready[p] + m.x) : "memory");
+                if (t != kReadyNone && (uint32_t)t == (uint32_t)tr.x) {
+                    p_hit = p;
                     ps = m.x;
-                    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(t1) : "l"(pv.ready[p] + ps) : "memory");
-                    if ((uint32_t)t1 != (uint32_t)tr.x || t1 == kReadyNone) ps = -1;
+                    t1 = t;
                 }
             }
-            ps = __shfl_sync(0xffffffffu, ps, 0);
-            if (ps < 0) continue;
-            const uint4* src = (const uint4*)(pv.slots[p] + (int64_t)ps * R);
-            uint4* ds = (uint4*)(slots + (int64_t)tr.y * R);
-            uint4* dout = (uint4*)(out + (int64_t)tr.z * R);
+        }
+        unsigned found = __ballot_sync(0xffffffffu, p_hit >= 0);
+        for (unsigned f = found; f; f &= f - 1) {
+            const int src_lane = __ffs(f) - 1;
+            const int pp = __shfl_sync(0xffffffffu, p_hit, src_lane);
+            const int sps = __shfl_sync(0xffffffffu, ps, src_lane);
+            const int dsl = __shfl_sync(0xffffffffu, tr.y, src_lane);
+            const int dpos = __shfl_sync(0xffffffffu, tr.z, src_lane);
+            const uint4* src = (const uint4*)(pv.slots[pp] + (int64_t)sps * R);
+            uint4* ds = (uint4*)(slots + (int64_t)dsl * R);
+            uint4* dout = (uint4*)(out + (int64_t)dpos * R);
             for (int64_t c = lane; c < cpr; c += 32) {
                 uint4 v;
                 asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];"
@@ -433,23 +448,25 @@ __global__ void __launch_bounds__(256) k_peer_probe(const int4* __restrict__ tri
                 ds[c] = v;
                 dout[c] = v;
             }
-            __syncwarp();
-            // load-load ordering only (the seqlock read side): the row's loads are ordered
-            // before the tag re-read; a full fence.sc would also drain this warp's stores
-            asm volatile("fence.acq_rel.sys;" ::: "memory");
-            int good = 0;
-            if (lane == 0) {
-                unsigned long long t2;
-                asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(t2) : "l"(pv.ready[p] + ps) : "memory");
-                good = t2 == t1;
-            }
-            ok = __shfl_sync(0xffffffffu, good, 0) != 0;
         }
-        if (ok) {
-            ++served;
-        } else if (lane == 0) {
-            const unsigned long long j = atomicAdd((unsigned long long*)t2count, 1ull);
-            trip2[j] = tr;
+        bool ok = false;
+        if (found) {
+            __syncwarp();
+            // load-load ordering (seqlock read side): the rows' loads before the tag re-reads
+            asm volatile("fence.acq_rel.sys;" ::: "memory");
+            if (p_hit >= 0) {
+                unsigned long long t2;
+                asm volatile("ld.relaxed.sys.global.u64 %0, [%1];" : "=l"(t2) : "l"(pv.ready[p_hit] + ps) : "memory");
+                ok = t2 == t1;
+            }
+        }
+        served += __popc(__ballot_sync(0xffffffffu, ok));
+        const unsigned rest = __ballot_sync(0xffffffffu, have && !ok);
+        if (rest) {
+            unsigned long long base = 0;
+            if (lane == 0) base = atomicAdd((unsigned long long*)t2count, (unsigned long long)__popc(rest));
+            base = __shfl_sync(0xffffffffu, base, 0);
+            if (have && !ok) trip2[base + __popc(rest & ((1u << lane) - 1u))] = tr;
         }
     }
     if (lane == 0 && served) atomicAdd(ctr, served);
