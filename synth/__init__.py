@@ -190,3 +190,57 @@ def segment(num_batches: int, rank: int, world: int) -> range:
     lo = num_batches * rank // world
     hi = num_batches * (rank + 1) // world
     return range(lo, hi)
+
+
+# ---------------------------------------------------------------- f4: train stage inputs
+# (3-layer GraphSAGE, hidden 256.)  Values are multiples of
+# 2^-23 in [-1, 1) (exact in fp32 and fp64), drawn with SplitMix64 like everything above.
+LABEL_SEED = 5
+WEIGHT_SEED = 6
+
+
+def _unit(key: torch.Tensor) -> torch.Tensor:
+    """SplitMix64(key) -> float64 in [-1, 1), a multiple of 2^-23."""
+    u = _lsr(splitmix64(key), 40).to(torch.float64)          # 24 random bits
+    return u / float(1 << 23) - 1.0
+
+
+def numeric_feature_rows(v0: int, v1: int, dim: int, seed: int = FEATURE_SEED, device="cpu") -> torch.Tensor:
+    """fp32 rows v0..v1-1 [v1-v0, dim] in [-1, 1) (the train stage needs finite features;
+    the extraction path copies bytes and does not care)."""
+    v = torch.arange(v0, v1, dtype=torch.int64, device=device)
+    c = torch.arange(dim, dtype=torch.int64, device=device)
+    return _unit((v[:, None] * dim + c[None, :]) ^ _mix_seed(seed, 31)).to(torch.float32)
+
+
+def numeric_feature_table(num_nodes: int, dim: int, seed: int = FEATURE_SEED, out: torch.Tensor | None = None,
+                          gen_device="cpu", chunk_rows: int = 1 << 20) -> torch.Tensor:
+    """The [N, dim*4] uint8 host table holding numeric_feature_rows (fp32 little endian)."""
+    if out is None:
+        out = torch.empty((num_nodes, dim * 4), dtype=torch.uint8)
+    for s in range(0, num_nodes, chunk_rows):
+        e = min(num_nodes, s + chunk_rows)
+        out[s:e].copy_(numeric_feature_rows(s, e, dim, seed, gen_device).view(torch.uint8), non_blocking=False)
+    return out
+
+
+def labels(nodes: torch.Tensor, num_classes: int, seed: int = LABEL_SEED) -> torch.Tensor:
+    """Synthetic class label of each node (the paper trains Friendster on random labels)."""
+    key = nodes.to(torch.int64) ^ _mix_seed(seed, 41)
+    return (_lsr(splitmix64(key), 33) % num_classes).to(torch.int32)
+
+
+def sage_init(dims, seed: int = WEIGHT_SEED):
+    """Initial parameters of an L-layer SAGE model with layer widths dims[0..L]: per layer
+    W [2*d_in, d_out] (rows 0..d_in-1 multiply the node's own features, rows d_in.. the
+    neighbour mean) uniform in +-1/sqrt(2 d_in), and b [d_out] uniform in +-0.1; float32
+    numpy arrays."""
+    out = []
+    for l in range(len(dims) - 1):
+        di, do = dims[l], dims[l + 1]
+        k = torch.arange(2 * di * do, dtype=torch.int64) ^ _mix_seed(seed, 50 + l)
+        W = (_unit(k) / np.sqrt(2 * di)).to(torch.float32).reshape(2 * di, do).numpy()
+        kb = torch.arange(do, dtype=torch.int64) ^ _mix_seed(seed, 80 + l)
+        b = (_unit(kb) * 0.1).to(torch.float32).numpy()
+        out.append((W, b))
+    return out
