@@ -265,6 +265,45 @@ gd_status gd_buffer_peer_attach_ipc(gd_buffer* b, int npeers, const void* blobs)
 gd_status gd_buffer_peer_stats(gd_buffer* b, int64_t* served, int64_t* probed);
 
 /* ----------------------------------------------------------------------------
+ * f4: the train stage on the extracted mini-batch.  GraphSAGE
+ * (three layers, hidden 256; mean aggregator with root weight, PyG SAGEConv,
+ * P:146) on the blocks of gd_sample, features = the rows gd_extract wrote (fp32).
+ * Layer j = 0..L-1 consumes hop h = L - j: a_i = [x_i | mean_{e in row i} x_col[e]],
+ * z = a W_j + b_j, relu between layers; loss = mean softmax cross entropy of the n_0
+ * seeds.  bf16 tensor-core GEMMs (cuBLAS), fp32 accumulation, fp32 master parameters.
+ *   gd_sage_create   dims[0..L] widths (dims[0] = feature dim, multiples of 4 for the
+ *                    inputs); init_w[j] host fp32 row-major [2 dims[j] x dims[j+1]] (rows
+ *                    0..dims[j]-1 multiply x_i, the rest the neighbour mean), init_b[j]
+ *                    [dims[j+1]]; max_nodes[0..L] = gd_sample_bounds of the blocks (the
+ *                    GEMMs run at these row counts with zero padding: no host sync).
+ *   gd_sage_step     forward + loss + backward for one batch, stream-ordered: rowptr[h-1]
+ *                    / col[h-1] the device block arrays of hop h (gd_sample_out), sizes the
+ *                    device sizes array, feats device fp32 [n_L x dims[0]], labels device
+ *                    int32 [n_0], loss a device float.  Writes the gradients.
+ *   gd_sage_grads    device pointer + length of the flat fp32 gradient buffer (layout
+ *                    [W_0 b_0 W_1 b_1 ...]) for a data-parallel all-reduce.
+ *   gd_sage_apply_sgd  p -= lr * grad_scale * g (grad_scale = 1/world after a SUM
+ *                    all-reduce), then refreshes the bf16 copies; stream-ordered.
+ *   gd_sage_get      synchronising debug copy of one layer's item (GD_SAGE_*) to host.
+ * ------------------------------------------------------------------------- */
+typedef struct gd_sage gd_sage;
+#define GD_SAGE_W 0     /* fp32 [2 d_in x d_out] */
+#define GD_SAGE_B 1     /* fp32 [d_out] */
+#define GD_SAGE_DW 2
+#define GD_SAGE_DB 3
+#define GD_SAGE_A16 4   /* bf16 [n_dst bound x 2 d_in], last forward */
+#define GD_SAGE_Z 5     /* fp32 [n_dst bound x d_out], last forward (z + b) */
+gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* const* init_w,
+                         const float* const* init_b, const int64_t* max_nodes, int device, gd_sage** out);
+gd_status gd_sage_destroy(gd_sage* s);
+gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* const* col,
+                       const int64_t* sizes, const float* feats, const int32_t* labels, float* loss,
+                       void* stream);
+gd_status gd_sage_grads(gd_sage* s, float** grads, int64_t* count);
+gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream);
+gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, int64_t bytes);
+
+/* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a
  * slot whose count reaches zero is appended at the tail (MRU end) of the standby
  * list.  The node stays valid until its slot is reused (delayed invalidation).

@@ -23,6 +23,7 @@ EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy",
            "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream", "gd_buffer_timing",
            "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config", "gd_buffer_stage_mode",
            "gd_buffer_peer_attach", "gd_buffer_peer_export_ipc", "gd_buffer_peer_attach_ipc", "gd_buffer_peer_stats",
+           "gd_sage_create", "gd_sage_destroy", "gd_sage_step", "gd_sage_grads", "gd_sage_apply_sgd", "gd_sage_get",
            "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod"]
 
 
@@ -83,6 +84,12 @@ def _load():
     L.gd_buffer_peer_export_ipc.argtypes = [_vp, ctypes.c_void_p, ctypes.c_int64]
     L.gd_buffer_peer_attach_ipc.argtypes = [_vp, ctypes.c_int, ctypes.c_void_p]
     L.gd_buffer_peer_stats.argtypes = [_vp, ctypes.POINTER(ctypes.c_int64), ctypes.POINTER(ctypes.c_int64)]
+    L.gd_sage_create.argtypes = [_i32, _vp, _vp, _vp, _vp, ctypes.c_int, ctypes.POINTER(_vp)]
+    L.gd_sage_destroy.argtypes = [_vp]
+    L.gd_sage_step.argtypes = [_vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp]
+    L.gd_sage_grads.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_i64)]
+    L.gd_sage_apply_sgd.argtypes = [_vp, ctypes.c_float, ctypes.c_float, _vp]
+    L.gd_sage_get.argtypes = [_vp, _i32, _i32, _vp, _i64]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:

@@ -1,0 +1,490 @@
+// gd_train.cu — f4: the train stage of the SET pipeline on B200.
+//
+// One GraphSAGE training step on the blocks gd_sample produced and the rows gd_extract
+// gathered (the trainer "adopts the node alias list to index required feature data
+// in device memory"; GraphSAGE, 3 layers, hidden 256; DDP gradient sync).
+// Layer j (j = 0..L-1) consumes hop h = L - j (outermost block first):
+//   a_i = [x_i | mean_{e in row i} x_col[e]]  (k_sage_agg: warp per dst row, fp32 sums,
+//                                              bf16 out, rows past n_dst zeroed)
+//   z   = a W + b                             (cuBLAS bf16 tensor-core GEMM, fp32 accumulate;
+//                                              k_bias_act adds b and applies relu)
+//   loss = mean softmax cross entropy of the seeds' logits (k_xent + k_loss_sum)
+// backward: dW = a^T dz, db = dz^T 1 (GEMMs), da = dz W^T, k_sage_scatter spreads da to
+// the layer's inputs (own row + neighbour mean, fp32 red.add), k_relu_grad masks by the
+// previous layer's activation.  GEMMs run at the host-side worst-case row counts
+// (gd_sample_bounds) with padded rows zero, so nothing synchronises the host.
+// Gradients live in one flat fp32 buffer (layout [W0 b0 W1 b1 ...]) that the caller may
+// all-reduce (NCCL) between gd_sage_step and gd_sage_apply_sgd.
+#include <cublas_v2.h>
+#include <cuda_bf16.h>
+
+#include <algorithm>
+#include <cstring>
+#include <vector>
+
+#include "gd_common.cuh"
+
+namespace gd {
+
+constexpr uint32_t kMagicSage = 0x47445341u;   // "GDSA"
+
+struct SageLayer {
+    int din = 0, dout = 0, hop = 0;
+    int64_t n_dst_max = 0, n_src_max = 0;
+    int64_t w_off = 0, b_off = 0, w16_off = 0;   // offsets into params / grads / W16
+    __nv_bfloat16* A16 = nullptr;   // [n_dst_max, 2 din]  (saved for backward)
+    float* Z = nullptr;             // [n_dst_max, dout]   pre-activation / logits
+    float* H = nullptr;             // [n_dst_max, dout]   relu(Z + b) (j < L-1)
+    __nv_bfloat16* dZ16 = nullptr;  // [n_dst_max, dout]
+    float* dA = nullptr;            // [n_dst_max, 2 din]  (j >= 1)
+    float* dX = nullptr;            // [n_src_max, din]    gradient wrt this layer's input (j >= 1)
+};
+
+}  // namespace gd
+
+struct gd_sage {
+    gd::HandleHdr hdr;
+    int L = 0;
+    std::vector<int> dims;
+    std::vector<int64_t> max_nodes;
+    std::vector<gd::SageLayer> layers;
+    float* params = nullptr;        // flat fp32 master parameters [W0 b0 W1 b1 ...]
+    float* grads = nullptr;         // same layout
+    __nv_bfloat16* W16 = nullptr;   // bf16 copies of the W's
+    int64_t nparams = 0, nw16 = 0;
+    float* loss_rows = nullptr;     // [n0_max]
+    __nv_bfloat16* ones16 = nullptr;
+    int64_t ones_n = 0;
+    cublasHandle_t cublas = nullptr;
+};
+
+namespace gd {
+
+// ------------------------------------------------------------------ kernels
+// a_i = [x_i | mean x_col] for i < n_dst, zero rows up to n_dst_max.  Warp per row; each
+// lane owns 4-column groups (float4) g = lane, lane + 32, ...; neighbour ids are loaded
+// 32 at a time and broadcast with shuffles.
+__global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, int din, const int64_t* __restrict__ rowptr,
+                                                  const int32_t* __restrict__ col, const int64_t* __restrict__ n_dst_p,
+                                                  int64_t n_dst_max, __nv_bfloat16* __restrict__ A16) {
+    const int lane = threadIdx.x & 31;
+    const int64_t n_dst = *n_dst_p;
+    const int groups = din >> 2;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst_max; i += warps) {
+        __nv_bfloat162* arow = (__nv_bfloat162*)(A16 + i * 2 * din);
+        if (i >= n_dst) {
+            for (int g = lane; g < groups; g += 32) {
+                const __nv_bfloat162 z = __floats2bfloat162_rn(0.f, 0.f);
+                arow[2 * g] = z;
+                arow[2 * g + 1] = z;
+                arow[(din >> 1) + 2 * g] = z;
+                arow[(din >> 1) + 2 * g + 1] = z;
+            }
+            continue;
+        }
+        const int64_t lo = rowptr[i], hi = rowptr[i + 1];
+        const float inv = hi > lo ? 1.0f / (float)(hi - lo) : 0.0f;
+        for (int g0 = 0; g0 < groups; g0 += 64) {          // up to 2 float4 per lane per pass
+            const int ga = g0 + lane, gb = g0 + 32 + lane;
+            float4 sa = make_float4(0.f, 0.f, 0.f, 0.f), sb = sa;
+            for (int64_t e0 = lo; e0 < hi; e0 += 32) {
+                const int m = (int)(hi - e0 < 32 ? hi - e0 : 32);
+                const int32_t c = lane < m ? col[e0 + lane] : 0;
+                for (int t = 0; t < m; ++t) {
+                    const int64_t u = __shfl_sync(0xffffffffu, c, t);
+                    const float4* xr = (const float4*)(x + u * din);
+                    if (ga < groups) {
+                        const float4 v = __ldg(xr + ga);
+                        sa.x += v.x; sa.y += v.y; sa.z += v.z; sa.w += v.w;
+                    }
+                    if (gb < groups) {
+                        const float4 v = __ldg(xr + gb);
+                        sb.x += v.x; sb.y += v.y; sb.z += v.z; sb.w += v.w;
+                    }
+                }
+            }
+            const float4* xi = (const float4*)(x + i * din);
+            if (ga < groups) {
+                const float4 s = __ldg(xi + ga);
+                arow[2 * ga] = __floats2bfloat162_rn(s.x, s.y);
+                arow[2 * ga + 1] = __floats2bfloat162_rn(s.z, s.w);
+                arow[(din >> 1) + 2 * ga] = __floats2bfloat162_rn(sa.x * inv, sa.y * inv);
+                arow[(din >> 1) + 2 * ga + 1] = __floats2bfloat162_rn(sa.z * inv, sa.w * inv);
+            }
+            if (gb < groups) {
+                const float4 s = __ldg(xi + gb);
+                arow[2 * gb] = __floats2bfloat162_rn(s.x, s.y);
+                arow[2 * gb + 1] = __floats2bfloat162_rn(s.z, s.w);
+                arow[(din >> 1) + 2 * gb] = __floats2bfloat162_rn(sb.x * inv, sb.y * inv);
+                arow[(din >> 1) + 2 * gb + 1] = __floats2bfloat162_rn(sb.z * inv, sb.w * inv);
+            }
+        }
+    }
+}
+
+// Z[i] += b; H[i] = relu(Z[i]) (relu = 1) for i < n; rows past n are zeroed.
+__global__ void k_bias_act(float* __restrict__ Z, float* __restrict__ H, const float* __restrict__ b, int dout,
+                           const int64_t* __restrict__ n_p, int64_t n_max, int relu) {
+    const int64_t n = *n_p;
+    const int64_t total = n_max * dout;
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = k / dout;
+        const int c = (int)(k - i * dout);
+        const float z = i < n ? Z[k] + b[c] : 0.f;
+        Z[k] = z;
+        if (relu) H[k] = z > 0.f ? z : 0.f;
+    }
+}
+
+// Softmax cross entropy, warp per seed row: loss_rows[i] = lse - z[label];
+// dZ16[i] = (softmax - onehot) / n0; rows past n0 zeroed.
+__global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, const int32_t* __restrict__ labels,
+                                              const int64_t* __restrict__ n_p, int64_t n_max,
+                                              __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows) {
+    const int lane = threadIdx.x & 31;
+    const int64_t n = *n_p;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_max; i += warps) {
+        const float* z = Z + i * C;
+        __nv_bfloat16* dz = dZ16 + i * C;
+        if (i >= n) {
+            for (int c = lane; c < C; c += 32) dz[c] = __float2bfloat16_rn(0.f);
+            continue;
+        }
+        float m = -INFINITY;
+        for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
+        for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
+        float s = 0.f;
+        for (int c = lane; c < C; c += 32) s += __expf(z[c] - m);
+        for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+        const int y = labels[i];
+        const float inv_n = 1.0f / (float)n;
+        for (int c = lane; c < C; c += 32) {
+            const float p = __expf(z[c] - m) / s;
+            dz[c] = __float2bfloat16_rn((p - (c == y ? 1.f : 0.f)) * inv_n);
+        }
+        if (lane == 0) loss_rows[i] = m + __logf(s) - z[y];
+    }
+}
+
+// loss = mean of loss_rows[0:n] (one block, fixed reduction order: deterministic).
+__global__ void k_loss_sum(const float* __restrict__ loss_rows, const int64_t* __restrict__ n_p, float* __restrict__ loss) {
+    __shared__ float sh[256];
+    const int64_t n = *n_p;
+    float s = 0.f;
+    for (int64_t i = threadIdx.x; i < n; i += blockDim.x) s += loss_rows[i];
+    sh[threadIdx.x] = s;
+    __syncthreads();
+    for (int w = blockDim.x / 2; w; w >>= 1) {
+        if ((int)threadIdx.x < w) sh[threadIdx.x] += sh[threadIdx.x + w];
+        __syncthreads();
+    }
+    if (threadIdx.x == 0) *loss = n > 0 ? sh[0] / (float)n : 0.f;
+}
+
+// dX (zeroed) += contributions of da: own row (first din columns) and neighbour mean
+// (last din columns / deg), warp per dst row, vector red.add.
+__global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ dA, int din,
+                                                      const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                                                      const int64_t* __restrict__ n_dst_p, float* __restrict__ dX) {
+    const int lane = threadIdx.x & 31;
+    const int64_t n_dst = *n_dst_p;
+    const int groups = din >> 2;
+    const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst; i += warps) {
+        const int64_t lo = rowptr[i], hi = rowptr[i + 1];
+        const float inv = hi > lo ? 1.0f / (float)(hi - lo) : 0.0f;
+        const float4* da = (const float4*)(dA + i * 2 * din);
+        for (int g = lane; g < groups; g += 32) {
+            const float4 own = da[g];
+            atomicAdd((float4*)(dX + i * din) + g, own);
+        }
+        if (hi == lo) continue;
+        for (int64_t e0 = lo; e0 < hi; e0 += 32) {
+            const int m = (int)(hi - e0 < 32 ? hi - e0 : 32);
+            const int32_t c = lane < m ? col[e0 + lane] : 0;
+            for (int t = 0; t < m; ++t) {
+                const int64_t u = __shfl_sync(0xffffffffu, c, t);
+                for (int g = lane; g < groups; g += 32) {
+                    float4 nb = da[groups + g];
+                    nb.x *= inv; nb.y *= inv; nb.z *= inv; nb.w *= inv;
+                    atomicAdd((float4*)(dX + u * din) + g, nb);
+                }
+            }
+        }
+    }
+}
+
+// dZ16 = bf16(dX * (H > 0)) for rows < n, zero rows up to n_max.
+__global__ void k_relu_grad(const float* __restrict__ dX, const float* __restrict__ H, int d,
+                            const int64_t* __restrict__ n_p, int64_t n_max, __nv_bfloat16* __restrict__ dZ16) {
+    const int64_t n = *n_p;
+    const int64_t total = n_max * d;
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t i = k / d;
+        dZ16[k] = __float2bfloat16_rn(i < n && H[k] > 0.f ? dX[k] : 0.f);
+    }
+}
+
+__global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float step) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+        p[k] = fmaf(-step, g[k], p[k]);
+}
+
+__global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst, int64_t n) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+        dst[k] = __float2bfloat16_rn(src[k]);
+}
+
+__global__ void k_fill_bf16(__nv_bfloat16* dst, int64_t n, float v) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
+        dst[k] = __float2bfloat16_rn(v);
+}
+
+// ------------------------------------------------------------------ GEMMs (row-major)
+static const char* cublas_msg(cublasStatus_t s) {
+    switch (s) {
+        case CUBLAS_STATUS_NOT_INITIALIZED: return "CUBLAS_STATUS_NOT_INITIALIZED";
+        case CUBLAS_STATUS_ALLOC_FAILED: return "CUBLAS_STATUS_ALLOC_FAILED";
+        case CUBLAS_STATUS_INVALID_VALUE: return "CUBLAS_STATUS_INVALID_VALUE";
+        case CUBLAS_STATUS_ARCH_MISMATCH: return "CUBLAS_STATUS_ARCH_MISMATCH";
+        case CUBLAS_STATUS_EXECUTION_FAILED: return "CUBLAS_STATUS_EXECUTION_FAILED";
+        case CUBLAS_STATUS_NOT_SUPPORTED: return "CUBLAS_STATUS_NOT_SUPPORTED";
+        default: return "cuBLAS error";
+    }
+}
+#define GD_CUBLAS(call)                                                                       \
+    do {                                                                                      \
+        cublasStatus_t s_ = (call);                                                           \
+        if (s_ != CUBLAS_STATUS_SUCCESS)                                                      \
+            return ::gd::set_error(GD_ERR_CUDA, std::string(#call ": ") + ::gd::cublas_msg(s_)); \
+    } while (0)
+
+// C[M x N] (row-major, fp32) = op(A) op(B) with bf16 operands, fp32 accumulate.  A row-major
+// [M x K] (transA: stored [K x M]), B row-major [K x N] (transB: stored [N x K]).  Column-
+// major cuBLAS computes C^T = op(B)^T op(A)^T.
+static gd_status gemm_rm(cublasHandle_t h, bool transA, bool transB, int64_t M, int64_t N, int64_t K,
+                         const __nv_bfloat16* A, const __nv_bfloat16* B, float* C) {
+    const float one = 1.f, zero = 0.f;
+    const int lda = (int)(transA ? M : K), ldb = (int)(transB ? K : N);
+    GD_CUBLAS(cublasGemmEx(h, transB ? CUBLAS_OP_T : CUBLAS_OP_N, transA ? CUBLAS_OP_T : CUBLAS_OP_N, (int)N, (int)M,
+                           (int)K, &one, B, CUDA_R_16BF, ldb, A, CUDA_R_16BF, lda, &zero, C, CUDA_R_32F, (int)N,
+                           CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT));
+    return GD_OK;
+}
+
+static unsigned grid_for(int64_t n, int per_block = 256) {
+    return (unsigned)std::max<int64_t>(1, std::min<int64_t>((n + per_block - 1) / per_block, 148 * 16));
+}
+
+static void sage_free(gd_sage* s) {
+    if (!s) return;
+    DeviceGuard guard(s->hdr.device);
+    cudaDeviceSynchronize();
+    for (auto& l : s->layers)
+        for (void* p : {(void*)l.A16, (void*)l.Z, (void*)l.H, (void*)l.dZ16, (void*)l.dA, (void*)l.dX})
+            if (p) cudaFree(p);
+    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->ones16})
+        if (p) cudaFree(p);
+    if (s->cublas) cublasDestroy(s->cublas);
+    s->hdr.magic = 0;
+    delete s;
+}
+
+}  // namespace gd
+
+using namespace gd;
+
+extern "C" {
+
+gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* const* init_w,
+                         const float* const* init_b, const int64_t* max_nodes, int device, gd_sage** out) {
+    if (!out || !dims || !init_w || !init_b || !max_nodes || num_layers < 1 || num_layers > GD_MAX_HOPS)
+        return set_error(GD_ERR_INVALID, "gd_sage_create: null pointer or num_layers outside 1..GD_MAX_HOPS");
+    for (int l = 0; l <= num_layers; ++l)
+        if (dims[l] <= 0 || dims[l] > 4096 || (l < num_layers && dims[l] % 4 != 0))
+            return set_error(GD_ERR_INVALID, "gd_sage_create: widths in 1..4096, input widths multiples of 4");
+    for (int l = 0; l <= num_layers; ++l)
+        if (max_nodes[l] < 1 || (l > 0 && max_nodes[l] < max_nodes[l - 1]))
+            return set_error(GD_ERR_INVALID, "gd_sage_create: max_nodes must be the gd_sample_bounds of the blocks");
+    *out = nullptr;
+    DeviceGuard guard(device);
+    gd_sage* s = new gd_sage();
+    s->hdr.magic = kMagicSage;
+    s->hdr.device = device;
+    s->hdr.dev_status = nullptr;
+    s->L = num_layers;
+    s->dims.assign(dims, dims + num_layers + 1);
+    s->max_nodes.assign(max_nodes, max_nodes + num_layers + 1);
+    auto fail = [&](gd_status st) { sage_free(s); return st; };
+    int64_t off = 0, off16 = 0;
+    s->layers.resize(num_layers);
+    for (int j = 0; j < num_layers; ++j) {
+        SageLayer& l = s->layers[j];
+        l.din = dims[j];
+        l.dout = dims[j + 1];
+        l.hop = num_layers - j;
+        l.n_dst_max = max_nodes[l.hop - 1];
+        l.n_src_max = max_nodes[l.hop];
+        l.w_off = off;
+        off += (int64_t)2 * l.din * l.dout;
+        l.b_off = off;
+        off += l.dout;
+        l.w16_off = off16;
+        off16 += (int64_t)2 * l.din * l.dout;
+    }
+    s->nparams = off;
+    s->nw16 = off16;
+#define SA(ptr, bytes)                                                                    \
+    do {                                                                                  \
+        cudaError_t e_ = cudaMalloc(&(ptr), (size_t)(bytes));                             \
+        if (e_ != cudaSuccess) return fail(cuda_error(e_, "gd_sage_create: cudaMalloc")); \
+    } while (0)
+    SA(s->params, off * sizeof(float));
+    SA(s->grads, off * sizeof(float));
+    SA(s->W16, off16 * sizeof(__nv_bfloat16));
+    SA(s->loss_rows, max_nodes[0] * sizeof(float));
+    int64_t ones = 1;
+    for (int j = 0; j < num_layers; ++j) {
+        SageLayer& l = s->layers[j];
+        SA(l.A16, l.n_dst_max * 2 * l.din * sizeof(__nv_bfloat16));
+        SA(l.Z, l.n_dst_max * l.dout * sizeof(float));
+        if (j < num_layers - 1) SA(l.H, l.n_dst_max * l.dout * sizeof(float));
+        SA(l.dZ16, l.n_dst_max * l.dout * sizeof(__nv_bfloat16));
+        if (j > 0) {
+            SA(l.dA, l.n_dst_max * 2 * l.din * sizeof(float));
+            SA(l.dX, l.n_src_max * l.din * sizeof(float));
+        }
+        ones = std::max(ones, l.n_dst_max);
+    }
+    SA(s->ones16, ones * sizeof(__nv_bfloat16));
+    s->ones_n = ones;
+#undef SA
+    for (int j = 0; j < num_layers; ++j) {
+        const SageLayer& l = s->layers[j];
+        if (!init_w[j] || !init_b[j]) return fail(set_error(GD_ERR_INVALID, "gd_sage_create: null initial parameter"));
+        cudaError_t e = cudaMemcpy(s->params + l.w_off, init_w[j], (size_t)2 * l.din * l.dout * sizeof(float),
+                                   cudaMemcpyHostToDevice);
+        if (e == cudaSuccess)
+            e = cudaMemcpy(s->params + l.b_off, init_b[j], (size_t)l.dout * sizeof(float), cudaMemcpyHostToDevice);
+        if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: parameter copy"));
+        k_to_bf16<<<grid_for(2 * l.din * l.dout), 256>>>(s->params + l.w_off, s->W16 + l.w16_off, (int64_t)2 * l.din * l.dout);
+    }
+    k_fill_bf16<<<grid_for(ones), 256>>>(s->ones16, ones, 1.0f);
+    if (cudaMemset(s->grads, 0, off * sizeof(float)) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
+    if (cublasCreate(&s->cublas) != CUBLAS_STATUS_SUCCESS)
+        return fail(set_error(GD_ERR_CUDA, "gd_sage_create: cublasCreate failed"));
+    cublasSetMathMode(s->cublas, CUBLAS_DEFAULT_MATH);
+    cudaError_t e = cudaDeviceSynchronize();
+    if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: init kernels"));
+    *out = s;
+    return GD_OK;
+}
+
+gd_status gd_sage_destroy(gd_sage* s) {
+    if (!s) return GD_OK;
+    if (s->hdr.magic != kMagicSage) return set_error(GD_ERR_INVALID, "gd_sage_destroy: bad handle");
+    sage_free(s);
+    return GD_OK;
+}
+
+gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* const* col, const int64_t* sizes,
+                       const float* feats, const int32_t* labels, float* loss, void* stream_v) {
+    if (!s || s->hdr.magic != kMagicSage) return set_error(GD_ERR_INVALID, "gd_sage_step: bad handle");
+    if (!rowptr || !col || !sizes || !feats || !labels || !loss)
+        return set_error(GD_ERR_INVALID, "gd_sage_step: null pointer");
+    for (int h = 0; h < s->L; ++h)
+        if (!rowptr[h] || !col[h]) return set_error(GD_ERR_INVALID, "gd_sage_step: null block pointer");
+    DeviceGuard guard(s->hdr.device);
+    cudaStream_t st = (cudaStream_t)stream_v;
+    GD_CUBLAS(cublasSetStream(s->cublas, st));
+    const int L = s->L;
+    // ---- forward
+    const float* x = feats;
+    for (int j = 0; j < L; ++j) {
+        SageLayer& l = s->layers[j];
+        const int h = l.hop;
+        k_sage_agg<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(x, l.din, rowptr[h - 1], col[h - 1], sizes + (h - 1),
+                                                               l.n_dst_max, l.A16);
+        GD_DEBUG_AFTER("k_sage_agg", st);
+        gd_status g = gemm_rm(s->cublas, false, false, l.n_dst_max, l.dout, 2 * l.din, l.A16, s->W16 + l.w16_off, l.Z);
+        if (g != GD_OK) return g;
+        k_bias_act<<<grid_for(l.n_dst_max * l.dout), 256, 0, st>>>(l.Z, l.H, s->params + l.b_off, l.dout, sizes + (h - 1),
+                                                                   l.n_dst_max, j < L - 1 ? 1 : 0);
+        GD_DEBUG_AFTER("k_bias_act", st);
+        x = l.H;
+    }
+    // ---- loss
+    SageLayer& top = s->layers[L - 1];
+    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, labels, sizes, top.n_dst_max, top.dZ16,
+                                                         s->loss_rows);
+    k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
+    GD_DEBUG_AFTER("k_xent", st);
+    // ---- backward
+    for (int j = L - 1; j >= 0; --j) {
+        SageLayer& l = s->layers[j];
+        const int h = l.hop;
+        gd_status g = gemm_rm(s->cublas, true, false, 2 * l.din, l.dout, l.n_dst_max, l.A16, l.dZ16, s->grads + l.w_off);
+        if (g != GD_OK) return g;
+        g = gemm_rm(s->cublas, true, false, l.dout, 1, l.n_dst_max, l.dZ16, s->ones16, s->grads + l.b_off);
+        if (g != GD_OK) return g;
+        if (j == 0) break;
+        g = gemm_rm(s->cublas, false, true, l.n_dst_max, 2 * l.din, l.dout, l.dZ16, s->W16 + l.w16_off, l.dA);
+        if (g != GD_OK) return g;
+        GD_CUDA(cudaMemsetAsync(l.dX, 0, (size_t)l.n_src_max * l.din * sizeof(float), st));
+        k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1],
+                                                                   sizes + (h - 1), l.dX);
+        GD_DEBUG_AFTER("k_sage_scatter", st);
+        SageLayer& prev = s->layers[j - 1];   // its output (H) is this layer's input
+        k_relu_grad<<<grid_for(prev.n_dst_max * prev.dout), 256, 0, st>>>(l.dX, prev.H, prev.dout, sizes + h,
+                                                                           prev.n_dst_max, prev.dZ16);
+        GD_DEBUG_AFTER("k_relu_grad", st);
+    }
+    GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
+gd_status gd_sage_grads(gd_sage* s, float** grads, int64_t* count) {
+    if (!s || s->hdr.magic != kMagicSage || !grads || !count) return set_error(GD_ERR_INVALID, "gd_sage_grads: bad argument");
+    *grads = s->grads;
+    *count = s->nparams;
+    return GD_OK;
+}
+
+gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream_v) {
+    if (!s || s->hdr.magic != kMagicSage) return set_error(GD_ERR_INVALID, "gd_sage_apply_sgd: bad handle");
+    DeviceGuard guard(s->hdr.device);
+    cudaStream_t st = (cudaStream_t)stream_v;
+    k_sgd<<<grid_for(s->nparams), 256, 0, st>>>(s->params, s->grads, s->nparams, lr * grad_scale);
+    for (const SageLayer& l : s->layers)
+        k_to_bf16<<<grid_for(2 * l.din * l.dout), 256, 0, st>>>(s->params + l.w_off, s->W16 + l.w16_off,
+                                                                (int64_t)2 * l.din * l.dout);
+    GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
+gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, int64_t bytes) {
+    if (!s || s->hdr.magic != kMagicSage || !host_out || layer < 0 || layer >= s->L)
+        return set_error(GD_ERR_INVALID, "gd_sage_get: bad argument");
+    DeviceGuard guard(s->hdr.device);
+    const SageLayer& l = s->layers[layer];
+    const void* src = nullptr;
+    int64_t n = 0;
+    switch (what) {
+        case GD_SAGE_W: src = s->params + l.w_off; n = (int64_t)2 * l.din * l.dout * 4; break;
+        case GD_SAGE_B: src = s->params + l.b_off; n = (int64_t)l.dout * 4; break;
+        case GD_SAGE_DW: src = s->grads + l.w_off; n = (int64_t)2 * l.din * l.dout * 4; break;
+        case GD_SAGE_DB: src = s->grads + l.b_off; n = (int64_t)l.dout * 4; break;
+        case GD_SAGE_A16: src = l.A16; n = l.n_dst_max * 2 * l.din * 2; break;
+        case GD_SAGE_Z: src = l.Z; n = l.n_dst_max * l.dout * 4; break;
+        default: return set_error(GD_ERR_INVALID, "gd_sage_get: unknown item");
+    }
+    if (bytes < n) return set_error(GD_ERR_INVALID, "gd_sage_get: host buffer too small");
+    GD_CUDA(cudaDeviceSynchronize());
+    GD_CUDA(cudaMemcpy(host_out, src, (size_t)n, cudaMemcpyDeviceToHost));
+    return GD_OK;
+}
+
+}  // extern "C"
