@@ -64,8 +64,8 @@ def forward(params, feats: np.ndarray, blocks, labels: np.ndarray):
     return loss, (cache, logits)
 
 
-def backward(params, cache_all, labels: np.ndarray):
-    """Gradients [(dW, db)] of the mean loss."""
+def backward(params, cache_all, labels: np.ndarray, return_dz: bool = False):
+    """Gradients [(dW, db)] of the mean loss (and, if asked, d loss / d z of every layer)."""
     cache, logits = cache_all
     L = len(params)
     n0 = logits.shape[0]
@@ -75,11 +75,13 @@ def backward(params, cache_all, labels: np.ndarray):
     dz[np.arange(n0), labels] -= 1.0
     dz /= n0                                           # d loss / d logits
     grads = [None] * L
+    dzs = [None] * L
     for j in range(L - 1, -1, -1):
         x, a, z, rowptr, col = cache[j]
         W = np.asarray(params[j][0], dtype=np.float64)
         if j < L - 1:
             dz = dz * (z > 0)                          # relu'
+        dzs[j] = dz
         grads[j] = (a.T @ dz, dz.sum(axis=0))
         if j == 0:
             break
@@ -93,7 +95,7 @@ def backward(params, cache_all, labels: np.ndarray):
             if hi > lo:
                 np.add.at(dx, col[lo:hi], da[i, d:] / (hi - lo))
         dz = dx                                        # d loss / d (previous layer output)
-    return grads
+    return (grads, dzs) if return_dz else grads
 
 
 def sgd(params, grads, lr: float):
