@@ -7,10 +7,12 @@ u = 2^-9 each) and accumulates in fp32, so an output entry obeys
 |z_gpu - z| <= (2u + u^2 + K 2^-24) (|a| |W|) <= 2^-7 (|a| |W|) for K <= 2^15; the
 aggregation rounds once to bf16: |a_gpu - a| <= 2^-8 |a| + 1e-6.  A gradient of layer j is
 the end of a chain of at most 2L GEMMs (forward through every layer, backward down to j), each
-adding <= 2^-7 relative to the magnitudes |A||B| it multiplies, so entrywise
-|dW_gpu - dW| <= 2^-4 (|a|^T |dz|) and |db_gpu - db| <= 2^-4 sum_i |dz_i| (6 x 2^-7 < 2^-4; the
-magnitudes, not the values, bound the error: sums of gradients cancel).  The loss is within
-2e-2 relative."""
+adding <= 2^-7 relative to the magnitudes |A||B| it multiplies, so
+||dW_gpu - dW|| <= 2^-4 || |a|^T |dz| || and ||db_gpu - db|| <= 2^-4 || sum_i |dz_i| || (6 x 2^-7
+< 2^-4; the magnitudes, not the values, bound the error: sums of gradients cancel).  The bound
+is normwise, not entrywise: where a pre-activation lies within rounding of 0 the two sides can
+take different relu branches (a decision made in different precisions), which moves single
+entries by up to their own size.  The loss is within 2e-2 relative."""
 import numpy as np
 import pytest
 import torch
@@ -105,8 +107,8 @@ def test_sage_step_parity(problem):
             a_j, dz_j = cache[0][j][1], dzs[j]
             mags = {"dW": np.abs(a_j).T @ np.abs(dz_j), "db": np.abs(dz_j).sum(axis=0)}
             for got, want, name in ((dW, grads[j][0], "dW"), (db, grads[j][1], "db")):
-                err = np.abs(got - want) / np.maximum(mags[name], 1e-30)
-                assert err.max() <= 2.0 ** -4 and cos(got, want) >= 0.99, (b, j, name, err.max(), cos(got, want))
+                err = np.linalg.norm(got - want) / max(1e-30, np.linalg.norm(mags[name]))
+                assert err <= 2.0 ** -4 and cos(got, want) >= 0.99, (b, j, name, err, cos(got, want))
     model.close()
 
 
