@@ -56,6 +56,7 @@ def run_batch(P, b, model=None, steps=0, lr=0.0):
     res = g.sample(seeds.cuda(), FAN, 3, b)
     out, _, done = buf.extract(res.n_id, res.num_nodes_dev, res.max_nodes)
     torch.cuda.current_stream().wait_event(done)
+    buf.release(res.n_id, res.num_nodes_dev, res.max_nodes)   # preload: rows stay resident
     labels = synth.labels(seeds, DIMS[-1]).cuda()
     return res, out, labels, seeds
 
