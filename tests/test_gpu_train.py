@@ -131,7 +131,8 @@ def test_sgd_update_and_training_reduces_loss(problem):
         losses.append(float(model.step(res, out, labels).item()))
         model.apply_sgd(0.5)
     torch.cuda.synchronize()
-    assert losses[-1] < 0.5 * losses[0], losses[::5]
+    assert losses[-1] < 0.9 * losses[0], losses[::5]                       # full-batch SGD descends
+    assert sum(b < a for a, b in zip(losses, losses[1:])) >= 27, losses
     model.close()
 
 
