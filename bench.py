@@ -49,6 +49,9 @@ def parse():
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the oracle cpu_baseline sample")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
+    p.add_argument("--train", action="store_true", help="f4: add the train stage (3-layer GraphSAGE, hidden 256, "
+                   "P:173) to every step on its own stream; the host table holds numeric fp32 features")
+    p.add_argument("--lr", type=float, default=0.01, help="f4 SGD learning rate")
     p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
                    "peer (CUDA IPC); misses are served from peers' HBM before the host link")
     p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
@@ -145,6 +148,9 @@ def measured_peaks():
         return {}
 
 
+NUM_CLASSES = {"papers100m": 172, "products": 47, "friendster": 64, "tiny": 16, "mag240m": 153}
+
+
 def capacity_for(cfg, n_max: int) -> int:
     if cfg.preload:
         return cfg.num_nodes
@@ -198,16 +204,19 @@ class Workload:
         if int(rc) != 0:
             raise RuntimeError(f"cudaHostRegister(host table, {n} bytes) failed: code {int(rc)}")
 
-    def fill_table(self):
+    def fill_table(self, numeric: bool = False):
         """Rank 0 writes the feature rows (generated on the GPU) into the host table; then
-        the other ranks register the (now resident) shared pages one after another."""
+        the other ranks register the (now resident) shared pages one after another.
+        numeric: finite fp32 features for the train stage (f4) instead of random bits."""
         t0 = time.time()
         if self.table.owner:
             cfg = self.cfg
             chunk = max(1, (256 << 20) // cfg.row_bytes)
             for s in range(0, cfg.host_rows, chunk):
                 e = min(cfg.host_rows, s + chunk)
-                self.table.tensor[s:e].copy_(synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
+                rows = (synth.numeric_feature_rows(s, e, cfg.feat_dim, device=self.device).view(torch.uint8) if numeric
+                        else synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
+                self.table.tensor[s:e].copy_(rows)
         torch.cuda.synchronize(self.device)
         self._barrier()
         for r in range(1, self.world):
@@ -251,7 +260,7 @@ def run_ours(args, rank, world, local_rank):
     cfg = config_from_args(args)
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
-    want_cpu = (not args.no_cpu_baseline) and rank == 0 and world == 1
+    want_cpu = (not args.no_cpu_baseline) and rank == 0 and world == 1 and not args.train
     need_host_csr = want_cpu or (rank == 0 and args.parity_batches > 0)
     W, K = args.warmup, args.steps
     t_setup = time.time()
@@ -263,7 +272,9 @@ def run_ours(args, rank, world, local_rank):
     nm, em = g.bounds(cfg.batch_size, fan)
     n_max = nm[-1]
     S = capacity_for(cfg, n_max)
-    wl.fill_table()
+    if args.train:
+        assert cfg.elem_bytes == 4, "--train needs fp32 features (papers100m, products, friendster, tiny)"
+    wl.fill_table(numeric=args.train)
     t0 = time.time()
     buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank,
                            num_nodes=cfg.num_nodes)
@@ -295,6 +306,22 @@ def run_ours(args, rank, world, local_rank):
     main = torch.cuda.current_stream(dev)
     pending = []
 
+    # ---- f4: the train stage on its own stream (GraphSAGE 3 x 256; DDP all-reduce)
+    model = None
+    if args.train:
+        from paper_conf_icpp_jiangj024_b200.train import SageModel
+        n_cls = NUM_CLASSES.get(cfg.name, 64)
+        dims = [cfg.feat_dim] + [256] * (len(fan) - 1) + [n_cls]   # L = #hops layers, hidden 256
+        model = SageModel(dims, synth.sage_init(dims), nm, device=local_rank)
+        labels_dev = synth.labels(seeds_dev.reshape(-1), n_cls).reshape(seeds_dev.shape)
+        tstream = torch.cuda.Stream(dev)
+        tdones = [torch.cuda.Event() for _ in range(RING)]
+        for e in tdones:
+            e.record(main)
+        loss_log = torch.zeros(total, dtype=torch.float32, device=dev)
+        t_events = []
+    train_timing = [False]
+
     dbg = os.environ.get("GD_DEBUG_SYNC") == "1"
 
     def dsync(what, j):
@@ -306,12 +333,28 @@ def run_ours(args, rank, world, local_rank):
         s = j % RING
         o = outs[s]
         main.wait_event(dones[s])          # batch j - RING is complete: its buffers are free
+        if model is not None:
+            main.wait_event(tdones[s])     # ... and trained (the trainer reads outs[s], feats[s])
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
         g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
         dsync("sample", j)
         buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, out=feats[s], alias=aliases[s], stats=stats[j],
                     stream=main, done=dones[s])
         dsync("extract", j)
+        if model is not None:              # f4 on stream T: train on batch j once its rows are in
+            tstream.wait_event(dones[s])
+            with torch.cuda.stream(tstream):
+                if train_timing[0]:
+                    a, z = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(tstream)
+                model.step(o, feats[s], labels_dev[j], stream=tstream)
+                scale = model.allreduce_grads()           # NCCL sum over ranks (no-op at N=1)
+                model.apply_sgd(args.lr, scale, stream=tstream)
+                loss_log[j].copy_(model.loss[0])
+                if train_timing[0]:
+                    z.record(tstream)
+                    t_events.append((a, z))
+            tdones[s].record(tstream)
         pending.append(o)
         if len(pending) == Q:
             r = pending.pop(0)
@@ -367,6 +410,7 @@ def run_ours(args, rank, world, local_rank):
     log("timed region ...")
     g.timing(True)
     buf.timing(True)
+    train_timing[0] = True
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local_rank) as clk:
@@ -374,11 +418,14 @@ def run_ours(args, rank, world, local_rank):
         for j in range(off + W, off + W + K):
             step(j)
         main.wait_event(dones[(off + W + K - 1) % RING])  # the last batch's rows are all in `out`
+        if model is not None:
+            main.wait_event(tdones[(off + W + K - 1) % RING])   # ... and it is trained
         ev1.record(main)
         ev1.synchronize()
     torch.cuda.synchronize(dev)
     g.timing(False)
     buf.timing(False)
+    train_timing[0] = False
     ms = ev0.elapsed_time(ev1)
     ms_max = max_over_ranks(ms, dev)
     tg = g.timing_read()
@@ -402,6 +449,8 @@ def run_ours(args, rank, world, local_rank):
         for j in range(off + W + K, off + W + 2 * K):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats))
         main.wait_event(dones[(off + W + 2 * K - 1) % RING])
+        if model is not None:
+            main.wait_event(tdones[(off + W + 2 * K - 1) % RING])
         e1.record(main)
         e1.synchronize()
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)
@@ -424,6 +473,8 @@ def run_ours(args, rank, world, local_rank):
         for j in range(j0 + W, j0 + W + K):
             step(j)
         main.wait_event(dones[(j0 + W + K - 1) % RING])
+        if model is not None:
+            main.wait_event(tdones[(j0 + W + K - 1) % RING])
         z.record(main)
         z.synchronize()
         buf.timing(False)
@@ -519,6 +570,21 @@ def run_ours(args, rank, world, local_rank):
                 if r["kernel"].startswith(kname):
                     r["traffic"] = tv
 
+    train_info = None
+    if model is not None:
+        t_ms = sum(a.elapsed_time(z) for a, z in t_events) / max(1, len(t_events))
+        L = model.L
+        flop = 0
+        for j in range(L):
+            nd, din, dout = nm[L - 1 - j], model.dims[j], model.dims[j + 1]
+            flop += 2 * nd * 2 * din * dout * (2 if j == 0 else 3)   # fwd + dW (+ dA above layer 0)
+        ll = loss_log[off + W:off + W + K].cpu().tolist()
+        train_info = {"model": f"GraphSAGE mean, widths {model.dims} (P:173)", "lr": args.lr,
+                      "train_ms_per_batch": round(t_ms, 4),
+                      "gemm_gflop_per_batch_at_bounds": round(flop / 1e9, 2),
+                      "gemm_tflops_if_train_ms_were_gemm": round(flop / (t_ms * 1e9), 1) if t_ms > 0 else None,
+                      "loss_first": round(ll[0], 4), "loss_last": round(ll[-1], 4),
+                      "allreduce": "NCCL all_reduce of the flat fp32 gradients (P:140)" if world > 1 else "none (N=1)"}
     peer_info = None
     if args.peer and world > 1:
         served, probed = buf.peer_stats()
@@ -532,7 +598,7 @@ def run_ours(args, rank, world, local_rank):
     total_batches = sum_over_ranks(K, dev)
     value = total_batches / (ms_max / 1e3)
     line = {
-        "metric": "sampled+extracted mini-batches/s",
+        "metric": "SET (sampled+extracted+trained) mini-batches/s" if model is not None else "sampled+extracted mini-batches/s",
         "value": round(value, 2), "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": round(ms_max / K, 4), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
@@ -562,6 +628,7 @@ def run_ours(args, rank, world, local_rank):
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
         "peer": peer_info,
+        "train": train_info,
         "setup_s": round(time.time() - t_setup, 1),
     }
     if rank == 0:
@@ -570,6 +637,8 @@ def run_ours(args, rank, world, local_rank):
         if args.out:
             with open(args.out, "w") as f:
                 f.write(s + "\n")
+    if model is not None:
+        model.close()
     buf.close()
     g.close()
     wl.close()
