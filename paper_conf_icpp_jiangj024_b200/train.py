@@ -80,11 +80,7 @@ class SageModel:
     def allreduce_grads(self, group=None) -> float:
         """Sum the flat gradients over the process group (NCCL on GPUs); returns the
         grad_scale (1 / world) for apply_sgd."""
-        import torch.distributed as dist
-        if not (dist.is_available() and dist.is_initialized()):
-            return 1.0
-        dist.all_reduce(self.grad_flat, group=group)
-        return 1.0 / dist.get_world_size(group)
+        return allreduce_flat(self.grad_flat, group)
 
     def get(self, what: int, layer: int) -> np.ndarray:
         di, do = self.dims[layer], self.dims[layer + 1]
@@ -107,6 +103,22 @@ class SageModel:
         a = np.zeros((n_dst_max, do), dtype=np.float32)
         check(lib.gd_sage_get(self._h, what, layer, a.ctypes.data_as(ctypes.c_void_p), a.nbytes))
         return a
+
+
+def allreduce_flat(flat: torch.Tensor, group=None) -> float:
+    """DDP's gradient step: SUM-all-reduce one flat gradient tensor in place and
+    return the scale (1 / world) that turns the sum into the mean."""
+    import torch.distributed as dist
+    if not (dist.is_available() and dist.is_initialized()):
+        return 1.0
+    dist.all_reduce(flat, group=group)
+    return 1.0 / dist.get_world_size(group)
+
+
+def flatten_params(pairs) -> np.ndarray:
+    """[(W_0, b_0), (W_1, b_1), ...] in the flat layout of gd_sage's parameter / gradient
+    buffers ([W_0 b_0 W_1 b_1 ...], row-major W)."""
+    return np.concatenate([np.concatenate([np.ravel(W), np.ravel(b)]) for W, b in pairs])
 
 
 def _device_view(ptr: int, n: int, device: int) -> torch.Tensor:

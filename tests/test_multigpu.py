@@ -44,6 +44,18 @@ def _worker(rank, world, port, shm_dir, q):
         out["table_row7"] = t.array[7].tolist()
         out["max"] = M.max_over_ranks(float(rank * 10 + 1))
         out["sum"] = M.sum_over_ranks(float(rank + 1))
+        # f4 data parallelism: each rank's oracle gradients on its own batch, summed
+        # by the same all-reduce helper the GPU path uses, scaled by 1/world = the mean
+        from paper_conf_icpp_jiangj024_b200 import train as T
+        from oracle import sage as S
+        sys.path.insert(0, os.path.join(ROOT, "tests"))
+        from test_oracle_sage import small_problem
+        mine = small_problem(B=5 + rank, seed=3 + rank)
+        loss, cache = S.forward(mine[0], mine[1], mine[2], mine[3])
+        flat = torch.from_numpy(T.flatten_params(S.backward(mine[0], cache, mine[3])))
+        scale = T.allreduce_flat(flat)
+        out["ddp_scale"] = scale
+        out["ddp_mean"] = (flat * scale).numpy()
         M.barrier()
         t.close(unlink=True)
         q.put((rank, out))
@@ -88,6 +100,24 @@ def test_shared_host_table_visible_to_all_ranks(results):
     expect = (np.arange(1000 * 64) % 251).astype(np.int64)
     assert results[0]["table_sum"] == results[1]["table_sum"] == int(expect.sum())
     assert results[1]["table_row7"] == expect.reshape(1000, 64)[7].tolist()
+
+
+def test_ddp_gradient_mean(results):
+    """The all-reduced flat gradient equals the mean of the per-rank oracle gradients."""
+    from oracle import sage as S
+    from paper_conf_icpp_jiangj024_b200 import train as T
+    import sys
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    from test_oracle_sage import small_problem
+    per = []
+    for rank in range(2):
+        p, f, bl, lab = small_problem(B=5 + rank, seed=3 + rank)
+        _, cache = S.forward(p, f, bl, lab)
+        per.append(T.flatten_params(S.backward(p, cache, lab)))
+    want = (per[0] + per[1]) / 2
+    for rank in range(2):
+        assert results[rank]["ddp_scale"] == 0.5
+        assert np.allclose(results[rank]["ddp_mean"], want, rtol=1e-12, atol=1e-15)
 
 
 def test_max_and_sum_over_ranks(results):
