@@ -7,12 +7,15 @@
 //   a_i = [x_i | mean_{e in row i} x_col[e]]  (k_sage_agg: warp per dst row, fp32 sums,
 //                                              bf16 out, rows past n_dst zeroed)
 //   z   = a W + b                             (cuBLAS bf16 tensor-core GEMM, fp32 accumulate;
-//                                              k_bias_act adds b and applies relu)
+//                                              k_bias_act adds b and applies relu; the top
+//                                              layer's b is added in k_xent)
 //   loss = mean softmax cross entropy of the seeds' logits (k_xent + k_loss_sum)
-// backward: dW = a^T dz, db = dz^T 1 (GEMMs), da = dz W^T, k_sage_scatter spreads da to
-// the layer's inputs (own row + neighbour mean, fp32 red.add), k_relu_grad masks by the
-// previous layer's activation.  GEMMs run at the host-side worst-case row counts
-// (gd_sample_bounds) with padded rows zero, so nothing synchronises the host.
+// backward: dW = a^T dz, da = dz W^T (GEMMs), db = column sums of dz (k_colsum_*,
+// deterministic), k_scatter_init + k_sage_scatter spread da to the layer's inputs (own row
+// by plain stores, neighbour mean by fp32 red.add), k_relu_grad masks by the previous
+// layer's activation.  GEMMs run at the host-side worst-case row counts (gd_sample_bounds)
+// with padded rows zero, so nothing synchronises the host; the elementwise kernels stop at
+// the device-resident row counts and re-zero only the rows the previous step wrote (hw).
 // Gradients live in one flat fp32 buffer (layout [W0 b0 W1 b1 ...]) that the caller may
 // all-reduce (NCCL) between gd_sage_step and gd_sage_apply_sgd.
 #include <cublas_v2.h>
@@ -53,25 +56,28 @@ struct gd_sage {
     __nv_bfloat16* W16 = nullptr;   // bf16 copies of the W's
     int64_t nparams = 0, nw16 = 0;
     float* loss_rows = nullptr;     // [n0_max]
-    __nv_bfloat16* ones16 = nullptr;
-    int64_t ones_n = 0;
+    int64_t* hw = nullptr;          // [L] rows of A16 / dZ16 of layer j that may be nonzero
+                                    // (the previous step's n_dst): padded rows are zeroed
+                                    // only up to it, not up to the bound
+    float* colsum_part = nullptr;   // [kColsumChunks x max dout] partial column sums (db)
     cublasHandle_t cublas = nullptr;
 };
 
 namespace gd {
 
 // ------------------------------------------------------------------ kernels
-// a_i = [x_i | mean x_col] for i < n_dst, zero rows up to n_dst_max.  Warp per row; each
+// a_i = [x_i | mean x_col] for i < n_dst, zero rows [n_dst, hw) (rows past hw are zero).  Warp per row; each
 // lane owns 4-column groups (float4) g = lane, lane + 32, ...; neighbour ids are loaded
 // 32 at a time and broadcast with shuffles.
 __global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, int din, const int64_t* __restrict__ rowptr,
                                                   const int32_t* __restrict__ col, const int64_t* __restrict__ n_dst_p,
-                                                  int64_t n_dst_max, __nv_bfloat16* __restrict__ A16) {
+                                                  const int64_t* __restrict__ hw_p, __nv_bfloat16* __restrict__ A16) {
     const int lane = threadIdx.x & 31;
     const int64_t n_dst = *n_dst_p;
+    const int64_t n_end = n_dst > *hw_p ? n_dst : *hw_p;   // rows [n_dst, hw) held the last batch
     const int groups = din >> 2;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst_max; i += warps) {
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
         __nv_bfloat162* arow = (__nv_bfloat162*)(A16 + i * 2 * din);
         if (i >= n_dst) {
             for (int g = lane; g < groups; g += 32) {
@@ -91,7 +97,27 @@ __global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, i
             for (int64_t e0 = lo; e0 < hi; e0 += 32) {
                 const int m = (int)(hi - e0 < 32 ? hi - e0 : 32);
                 const int32_t c = lane < m ? col[e0 + lane] : 0;
-                for (int t = 0; t < m; ++t) {
+                int t = 0;
+                for (; t + 4 <= m; t += 4) {      // 4 neighbour rows in flight per lane
+                    const float4* xr[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) xr[q] = (const float4*)(x + (int64_t)__shfl_sync(0xffffffffu, c, t + q) * din);
+                    if (ga < groups) {
+                        float4 v[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) v[q] = __ldg(xr[q] + ga);
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) { sa.x += v[q].x; sa.y += v[q].y; sa.z += v[q].z; sa.w += v[q].w; }
+                    }
+                    if (gb < groups) {
+                        float4 v[4];
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) v[q] = __ldg(xr[q] + gb);
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) { sb.x += v[q].x; sb.y += v[q].y; sb.z += v[q].z; sb.w += v[q].w; }
+                    }
+                }
+                for (; t < m; ++t) {
                     const int64_t u = __shfl_sync(0xffffffffu, c, t);
                     const float4* xr = (const float4*)(x + u * din);
                     if (ga < groups) {
@@ -123,37 +149,50 @@ __global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, i
     }
 }
 
-// Z[i] += b; H[i] = relu(Z[i]) (relu = 1) for i < n; rows past n are zeroed.
-__global__ void k_bias_act(float* __restrict__ Z, float* __restrict__ H, const float* __restrict__ b, int dout,
-                           const int64_t* __restrict__ n_p, int64_t n_max, int relu) {
+// Z[i] += b; H[i] = relu(Z[i]) for i < n (hidden layers, dout % 4 == 0).  Block (32, 8):
+// threadIdx.x walks a row's float4 columns, threadIdx.y rows; no index division.  Rows past
+// n are not touched (the GEMM produced 0 there from zero A16 rows, and nothing reads them).
+__global__ void __launch_bounds__(256) k_bias_act(float* __restrict__ Z, float* __restrict__ H, const float* __restrict__ b,
+                                                  int dout, const int64_t* __restrict__ n_p) {
     const int64_t n = *n_p;
-    const int64_t total = n_max * dout;
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t i = k / dout;
-        const int c = (int)(k - i * dout);
-        const float z = i < n ? Z[k] + b[c] : 0.f;
-        Z[k] = z;
-        if (relu) H[k] = z > 0.f ? z : 0.f;
+    const int dv = dout >> 2;
+    const float4* b4 = (const float4*)b;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n; i += (int64_t)gridDim.x * blockDim.y) {
+        float4* z4 = (float4*)(Z + i * dout);
+        float4* h4 = (float4*)(H + i * dout);
+        for (int c = threadIdx.x; c < dv; c += blockDim.x) {
+            float4 z = z4[c];
+            const float4 bb = __ldg(b4 + c);
+            z.x += bb.x; z.y += bb.y; z.z += bb.z; z.w += bb.w;
+            z4[c] = z;
+            h4[c] = make_float4(fmaxf(z.x, 0.f), fmaxf(z.y, 0.f), fmaxf(z.z, 0.f), fmaxf(z.w, 0.f));
+        }
     }
 }
 
-// Softmax cross entropy, warp per seed row: loss_rows[i] = lse - z[label];
-// dZ16[i] = (softmax - onehot) / n0; rows past n0 zeroed.
-__global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, const int32_t* __restrict__ labels,
-                                              const int64_t* __restrict__ n_p, int64_t n_max,
-                                              __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows) {
+// Softmax cross entropy of the logits z + b, warp per seed row: Z[i] = z + b,
+// loss_rows[i] = lse - z[label]; dZ16[i] = (softmax - onehot) / n0; rows [n0, hw) zeroed.
+__global__ void __launch_bounds__(256) k_xent(float* __restrict__ Z, const float* __restrict__ b, int C,
+                                              const int32_t* __restrict__ labels, const int64_t* __restrict__ n_p,
+                                              const int64_t* __restrict__ hw_p, __nv_bfloat16* __restrict__ dZ16,
+                                              float* __restrict__ loss_rows) {
     const int lane = threadIdx.x & 31;
     const int64_t n = *n_p;
+    const int64_t n_end = n > *hw_p ? n : *hw_p;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_max; i += warps) {
-        const float* z = Z + i * C;
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
+        float* z = Z + i * C;
         __nv_bfloat16* dz = dZ16 + i * C;
         if (i >= n) {
             for (int c = lane; c < C; c += 32) dz[c] = __float2bfloat16_rn(0.f);
             continue;
         }
         float m = -INFINITY;
-        for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
+        for (int c = lane; c < C; c += 32) {
+            const float v = z[c] + b[c];
+            z[c] = v;
+            m = fmaxf(m, v);
+        }
         for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
         float s = 0.f;
         for (int c = lane; c < C; c += 32) s += __expf(z[c] - m);
@@ -164,6 +203,7 @@ __global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C
             const float p = __expf(z[c] - m) / s;
             dz[c] = __float2bfloat16_rn((p - (c == y ? 1.f : 0.f)) * inv_n);
         }
+        __syncwarp();
         if (lane == 0) loss_rows[i] = m + __logf(s) - z[y];
     }
 }
@@ -183,8 +223,21 @@ __global__ void k_loss_sum(const float* __restrict__ loss_rows, const int64_t* _
     if (threadIdx.x == 0) *loss = n > 0 ? sh[0] / (float)n : 0.f;
 }
 
-// dX (zeroed) += contributions of da: own row (first din columns) and neighbour mean
-// (last din columns / deg), warp per dst row, vector red.add.
+// dX[i] = own-row part of da (first din columns) for i < n_dst, 0 for n_dst <= i < n_src:
+// plain stores, so neither a bound-sized memset nor atomics for the own rows.
+__global__ void __launch_bounds__(256) k_scatter_init(const float* __restrict__ dA, int din, const int64_t* __restrict__ n_dst_p,
+                                                      const int64_t* __restrict__ n_src_p, float* __restrict__ dX) {
+    const int64_t n_dst = *n_dst_p, n_src = *n_src_p;
+    const int dv = din >> 2;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n_src; i += (int64_t)gridDim.x * blockDim.y) {
+        float4* d4 = (float4*)(dX + i * din);
+        const float4* a4 = (const float4*)(dA + i * 2 * din);
+        for (int c = threadIdx.x; c < dv; c += blockDim.x) d4[c] = i < n_dst ? a4[c] : make_float4(0.f, 0.f, 0.f, 0.f);
+    }
+}
+
+// dX += neighbour-mean contributions of da (last din columns / deg), warp per dst row,
+// vector red.add (fp32; the summation order of a row's contributions is not fixed).
 __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ dA, int din,
                                                       const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                                                       const int64_t* __restrict__ n_dst_p, float* __restrict__ dX) {
@@ -194,37 +247,94 @@ __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ 
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
     for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst; i += warps) {
         const int64_t lo = rowptr[i], hi = rowptr[i + 1];
-        const float inv = hi > lo ? 1.0f / (float)(hi - lo) : 0.0f;
-        const float4* da = (const float4*)(dA + i * 2 * din);
-        for (int g = lane; g < groups; g += 32) {
-            const float4 own = da[g];
-            atomicAdd((float4*)(dX + i * din) + g, own);
-        }
         if (hi == lo) continue;
-        for (int64_t e0 = lo; e0 < hi; e0 += 32) {
-            const int m = (int)(hi - e0 < 32 ? hi - e0 : 32);
-            const int32_t c = lane < m ? col[e0 + lane] : 0;
-            for (int t = 0; t < m; ++t) {
-                const int64_t u = __shfl_sync(0xffffffffu, c, t);
-                for (int g = lane; g < groups; g += 32) {
-                    float4 nb = da[groups + g];
-                    nb.x *= inv; nb.y *= inv; nb.z *= inv; nb.w *= inv;
-                    atomicAdd((float4*)(dX + u * din) + g, nb);
+        const float inv = 1.0f / (float)(hi - lo);
+        const float4* da = (const float4*)(dA + i * 2 * din) + groups;
+        for (int g0 = 0; g0 < groups; g0 += 32) {
+            const int g = g0 + lane;
+            float4 nb = g < groups ? da[g] : make_float4(0.f, 0.f, 0.f, 0.f);
+            nb.x *= inv; nb.y *= inv; nb.z *= inv; nb.w *= inv;
+            for (int64_t e0 = lo; e0 < hi; e0 += 32) {
+                const int m = (int)(hi - e0 < 32 ? hi - e0 : 32);
+                const int32_t c = lane < m ? col[e0 + lane] : 0;
+                for (int t = 0; t < m; ++t) {
+                    const int64_t u = __shfl_sync(0xffffffffu, c, t);
+                    if (g < groups) atomicAdd((float4*)(dX + u * din) + g, nb);
                 }
             }
         }
     }
 }
 
-// dZ16 = bf16(dX * (H > 0)) for rows < n, zero rows up to n_max.
-__global__ void k_relu_grad(const float* __restrict__ dX, const float* __restrict__ H, int d,
-                            const int64_t* __restrict__ n_p, int64_t n_max, __nv_bfloat16* __restrict__ dZ16) {
+// dZ16 = bf16(dX * (H > 0)) for rows < n, zero rows [n, hw).  Block (32, 8) as k_bias_act.
+__global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX, const float* __restrict__ H, int d,
+                                                   const int64_t* __restrict__ n_p, const int64_t* __restrict__ hw_p,
+                                                   __nv_bfloat16* __restrict__ dZ16) {
     const int64_t n = *n_p;
-    const int64_t total = n_max * d;
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < total; k += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t i = k / d;
-        dZ16[k] = __float2bfloat16_rn(i < n && H[k] > 0.f ? dX[k] : 0.f);
+    const int64_t n_end = n > *hw_p ? n : *hw_p;
+    const int dv = d >> 2;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n_end; i += (int64_t)gridDim.x * blockDim.y) {
+        const float4* x4 = (const float4*)(dX + i * d);
+        const float4* h4 = (const float4*)(H + i * d);
+        __nv_bfloat162* o2 = (__nv_bfloat162*)(dZ16 + i * d);
+        for (int c = threadIdx.x; c < dv; c += blockDim.x) {
+            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
+            if (i < n) {
+                const float4 x = x4[c], h = h4[c];
+                v = make_float4(h.x > 0.f ? x.x : 0.f, h.y > 0.f ? x.y : 0.f, h.z > 0.f ? x.z : 0.f, h.w > 0.f ? x.w : 0.f);
+            }
+            o2[2 * c] = __floats2bfloat162_rn(v.x, v.y);
+            o2[2 * c + 1] = __floats2bfloat162_rn(v.z, v.w);
+        }
     }
+}
+
+// db = column sums of dZ16 rows < n, deterministic (fixed assignment and reduction order).
+// Pass 1: block (32, 8) sums a 32-column strip over row chunk blockIdx.y (thread (x, y) takes
+// rows y, y + 8, ... of the chunk), reduces the 8 row lanes in shared memory and writes
+// part[chunk][col].  Pass 2 does the same over the kColsumChunks partials.
+constexpr int kColsumChunks = 256;
+__global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __restrict__ dZ16, int d,
+                                                     const int64_t* __restrict__ n_p, float* __restrict__ part) {
+    __shared__ float sh[8][33];
+    const int64_t n = *n_p;
+    const int64_t per = (n + gridDim.y - 1) / gridDim.y;
+    const int64_t r0 = (int64_t)blockIdx.y * per, r1 = r0 + per < n ? r0 + per : n;
+    const int c = blockIdx.x * 32 + threadIdx.x;
+    float s = 0.f;
+    if (c < d) {
+        int64_t i = r0 + threadIdx.y;
+#pragma unroll 4
+        for (; i < r1; i += 8) s += __bfloat162float(dZ16[i * d + c]);
+    }
+    sh[threadIdx.y][threadIdx.x] = s;
+    __syncthreads();
+    if (threadIdx.y == 0 && c < d) {
+        float t = 0.f;
+        for (int y = 0; y < 8; ++y) t += sh[y][threadIdx.x];
+        part[(int64_t)blockIdx.y * d + c] = t;
+    }
+}
+
+__global__ void __launch_bounds__(256) k_colsum_final(const float* __restrict__ part, int d, int nchunk,
+                                                      float* __restrict__ out) {
+    __shared__ float sh[8][33];
+    const int c = blockIdx.x * 32 + threadIdx.x;
+    float s = 0.f;
+    if (c < d)
+        for (int k = threadIdx.y; k < nchunk; k += 8) s += part[(int64_t)k * d + c];
+    sh[threadIdx.y][threadIdx.x] = s;
+    __syncthreads();
+    if (threadIdx.y == 0 && c < d) {
+        float t = 0.f;
+        for (int y = 0; y < 8; ++y) t += sh[y][threadIdx.x];
+        out[c] = t;
+    }
+}
+
+__global__ void k_set_hw(int64_t* __restrict__ hw, const int64_t* __restrict__ sizes, int L) {
+    const int j = threadIdx.x;
+    if (j < L) hw[j] = sizes[L - 1 - j];      // layer j's dst rows = n_{hop-1}, hop = L - j
 }
 
 __global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float step) {
@@ -235,11 +345,6 @@ __global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_
 __global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst, int64_t n) {
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
         dst[k] = __float2bfloat16_rn(src[k]);
-}
-
-__global__ void k_fill_bf16(__nv_bfloat16* dst, int64_t n, float v) {
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
-        dst[k] = __float2bfloat16_rn(v);
 }
 
 // ------------------------------------------------------------------ GEMMs (row-major)
@@ -285,7 +390,7 @@ static void sage_free(gd_sage* s) {
     for (auto& l : s->layers)
         for (void* p : {(void*)l.A16, (void*)l.Z, (void*)l.H, (void*)l.dZ16, (void*)l.dA, (void*)l.dX})
             if (p) cudaFree(p);
-    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->ones16})
+    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->hw, (void*)s->colsum_part})
         if (p) cudaFree(p);
     if (s->cublas) cublasDestroy(s->cublas);
     s->hdr.magic = 0;
@@ -345,7 +450,7 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
     SA(s->grads, off * sizeof(float));
     SA(s->W16, off16 * sizeof(__nv_bfloat16));
     SA(s->loss_rows, max_nodes[0] * sizeof(float));
-    int64_t ones = 1;
+    int max_dout = 1;
     for (int j = 0; j < num_layers; ++j) {
         SageLayer& l = s->layers[j];
         SA(l.A16, l.n_dst_max * 2 * l.din * sizeof(__nv_bfloat16));
@@ -356,11 +461,22 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
             SA(l.dA, l.n_dst_max * 2 * l.din * sizeof(float));
             SA(l.dX, l.n_src_max * l.din * sizeof(float));
         }
-        ones = std::max(ones, l.n_dst_max);
+        max_dout = std::max(max_dout, l.dout);
     }
-    SA(s->ones16, ones * sizeof(__nv_bfloat16));
-    s->ones_n = ones;
+    SA(s->hw, num_layers * sizeof(int64_t));
+    SA(s->colsum_part, (size_t)kColsumChunks * max_dout * sizeof(float));
 #undef SA
+    // the GEMMs run at the bound row counts: padded rows of their bf16 operands start zero
+    // and every step re-zeroes only the rows the previous step wrote (hw)
+    for (int j = 0; j < num_layers; ++j) {
+        const SageLayer& l = s->layers[j];
+        cudaError_t e = cudaMemset(l.A16, 0, l.n_dst_max * 2 * l.din * sizeof(__nv_bfloat16));
+        if (e == cudaSuccess) e = cudaMemset(l.dZ16, 0, l.n_dst_max * l.dout * sizeof(__nv_bfloat16));
+        if (e == cudaSuccess) e = cudaMemset(l.Z, 0, l.n_dst_max * l.dout * sizeof(float));
+        if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: memset"));
+    }
+    if (cudaMemset(s->hw, 0, num_layers * sizeof(int64_t)) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
     for (int j = 0; j < num_layers; ++j) {
         const SageLayer& l = s->layers[j];
         if (!init_w[j] || !init_b[j]) return fail(set_error(GD_ERR_INVALID, "gd_sage_create: null initial parameter"));
@@ -371,7 +487,6 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: parameter copy"));
         k_to_bf16<<<grid_for(2 * l.din * l.dout), 256>>>(s->params + l.w_off, s->W16 + l.w16_off, (int64_t)2 * l.din * l.dout);
     }
-    k_fill_bf16<<<grid_for(ones), 256>>>(s->ones16, ones, 1.0f);
     if (cudaMemset(s->grads, 0, off * sizeof(float)) != cudaSuccess)
         return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
     if (cublasCreate(&s->cublas) != CUBLAS_STATUS_SUCCESS)
@@ -401,25 +516,28 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
     cudaStream_t st = (cudaStream_t)stream_v;
     GD_CUBLAS(cublasSetStream(s->cublas, st));
     const int L = s->L;
+    const dim3 rows_blk(32, 8);          // (float4 column, row) blocks of the row-wise kernels
     // ---- forward
     const float* x = feats;
     for (int j = 0; j < L; ++j) {
         SageLayer& l = s->layers[j];
         const int h = l.hop;
         k_sage_agg<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(x, l.din, rowptr[h - 1], col[h - 1], sizes + (h - 1),
-                                                               l.n_dst_max, l.A16);
+                                                               s->hw + j, l.A16);
         GD_DEBUG_AFTER("k_sage_agg", st);
         gd_status g = gemm_rm(s->cublas, false, false, l.n_dst_max, l.dout, 2 * l.din, l.A16, s->W16 + l.w16_off, l.Z);
         if (g != GD_OK) return g;
-        k_bias_act<<<grid_for(l.n_dst_max * l.dout), 256, 0, st>>>(l.Z, l.H, s->params + l.b_off, l.dout, sizes + (h - 1),
-                                                                   l.n_dst_max, j < L - 1 ? 1 : 0);
-        GD_DEBUG_AFTER("k_bias_act", st);
+        if (j < L - 1) {
+            k_bias_act<<<grid_for(l.n_dst_max * 8), rows_blk, 0, st>>>(l.Z, l.H, s->params + l.b_off, l.dout,
+                                                                       sizes + (h - 1));
+            GD_DEBUG_AFTER("k_bias_act", st);
+        }
         x = l.H;
     }
-    // ---- loss
+    // ---- loss (the top layer's bias is added here)
     SageLayer& top = s->layers[L - 1];
-    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, labels, sizes, top.n_dst_max, top.dZ16,
-                                                         s->loss_rows);
+    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, s->params + top.b_off, top.dout, labels, sizes,
+                                                         s->hw + (L - 1), top.dZ16, s->loss_rows);
     k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
     GD_DEBUG_AFTER("k_xent", st);
     // ---- backward
@@ -428,20 +546,23 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         const int h = l.hop;
         gd_status g = gemm_rm(s->cublas, true, false, 2 * l.din, l.dout, l.n_dst_max, l.A16, l.dZ16, s->grads + l.w_off);
         if (g != GD_OK) return g;
-        g = gemm_rm(s->cublas, true, false, l.dout, 1, l.n_dst_max, l.dZ16, s->ones16, s->grads + l.b_off);
-        if (g != GD_OK) return g;
+        const unsigned strips = (unsigned)((l.dout + 31) / 32);
+        k_colsum_part<<<dim3(strips, kColsumChunks), rows_blk, 0, st>>>(l.dZ16, l.dout, sizes + (h - 1), s->colsum_part);
+        k_colsum_final<<<strips, rows_blk, 0, st>>>(s->colsum_part, l.dout, kColsumChunks, s->grads + l.b_off);
+        GD_DEBUG_AFTER("k_colsum", st);
         if (j == 0) break;
         g = gemm_rm(s->cublas, false, true, l.n_dst_max, 2 * l.din, l.dout, l.dZ16, s->W16 + l.w16_off, l.dA);
         if (g != GD_OK) return g;
-        GD_CUDA(cudaMemsetAsync(l.dX, 0, (size_t)l.n_src_max * l.din * sizeof(float), st));
+        k_scatter_init<<<grid_for(l.n_src_max * 8), rows_blk, 0, st>>>(l.dA, l.din, sizes + (h - 1), sizes + h, l.dX);
         k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1],
                                                                    sizes + (h - 1), l.dX);
         GD_DEBUG_AFTER("k_sage_scatter", st);
         SageLayer& prev = s->layers[j - 1];   // its output (H) is this layer's input
-        k_relu_grad<<<grid_for(prev.n_dst_max * prev.dout), 256, 0, st>>>(l.dX, prev.H, prev.dout, sizes + h,
-                                                                           prev.n_dst_max, prev.dZ16);
+        k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H, prev.dout, sizes + h,
+                                                                       s->hw + (j - 1), prev.dZ16);
         GD_DEBUG_AFTER("k_relu_grad", st);
     }
+    k_set_hw<<<1, 32, 0, st>>>(s->hw, sizes, L);
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
