@@ -270,12 +270,14 @@ gd_status gd_buffer_peer_stats(gd_buffer* b, int64_t* served, int64_t* probed);
  * P:146) on the blocks of gd_sample, features = the rows gd_extract wrote (fp32).
  * Layer j = 0..L-1 consumes hop h = L - j: a_i = [x_i | mean_{e in row i} x_col[e]],
  * z = a W_j + b_j, relu between layers; loss = mean softmax cross entropy of the n_0
- * seeds.  bf16 tensor-core GEMMs (cuBLAS), fp32 accumulation, fp32 master parameters.
+ * seeds.  bf16 tensor-core GEMMs (hand-written tcgen05, csrc/gd_umma.cuh) over the
+ * device-resident row counts, fp32 accumulation, fp32 master parameters.
  *   gd_sage_create   dims[0..L] widths (dims[0] = feature dim, multiples of 4 for the
  *                    inputs); init_w[j] host fp32 row-major [2 dims[j] x dims[j+1]] (rows
  *                    0..dims[j]-1 multiply x_i, the rest the neighbour mean), init_b[j]
- *                    [dims[j+1]]; max_nodes[0..L] = gd_sample_bounds of the blocks (the
- *                    GEMMs run at these row counts with zero padding: no host sync).
+ *                    [dims[j+1]]; max_nodes[0..L] = gd_sample_bounds of the blocks (buffers
+ *                    are sized by them; kernels read the actual counts on the device: no
+ *                    host sync).
  *   gd_sage_step     forward + loss + backward for one batch, stream-ordered: rowptr[h-1]
  *                    / col[h-1] the device block arrays of hop h (gd_sample_out), sizes the
  *                    device sizes array, feats device fp32 [n_L x dims[0]], labels device
@@ -302,6 +304,21 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
 gd_status gd_sage_grads(gd_sage* s, float** grads, int64_t* count);
 gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream);
 gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, int64_t bytes);
+
+/* Test surface of the train stage's tensor-core GEMM (csrc/gd_umma.cuh; tcgen05.mma with
+ * the accumulator in TMEM), all pointers device, bf16 operands, fp32 C, stream-ordered:
+ *   mode 0 FWD  C[i, n] = sum_k A[i*lda + k] B[k*ldb + n] (+ bias[n]; H = relu(C))
+ *   mode 1 DA   C[i, n] = sum_k A[i*lda + k] B[n*ldb + k]
+ *   for i < *rows_dev (<= rows_max), k < k_valid (multiple of 8), n < n_store; B is valid
+ *   (and read) for n < n_valid (multiple of 8), zero beyond.
+ *   mode 2 DW   C[m, n] += sum_{i < *rows_dev} A[i*lda + m] B[i*ldb + n] for m < m_valid
+ *   (multiple of 8), n < n_store, the reduction split over `splits` CTAs per tile (fp32
+ *   red.add into C: the caller zeroes it).
+ * Row strides are multiples of 8 elements, base pointers 16-byte aligned (GD_ERR_INVALID). */
+gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb,
+                             float* C, int64_t ldc, float* H, const float* bias, const int64_t* rows_dev,
+                             int64_t rows_max, int64_t m_valid, int32_t k_valid, int32_t n_valid,
+                             int32_t n_store, int32_t splits, void* stream);
 
 /* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a

@@ -24,7 +24,7 @@ EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy",
            "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config", "gd_buffer_stage_mode",
            "gd_buffer_peer_attach", "gd_buffer_peer_export_ipc", "gd_buffer_peer_attach_ipc", "gd_buffer_peer_stats",
            "gd_sage_create", "gd_sage_destroy", "gd_sage_step", "gd_sage_grads", "gd_sage_apply_sgd", "gd_sage_get",
-           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod"]
+           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod", "gd_debug_umma_gemm"]
 
 
 class GdError(RuntimeError):
@@ -90,6 +90,8 @@ def _load():
     L.gd_sage_grads.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_i64)]
     L.gd_sage_apply_sgd.argtypes = [_vp, ctypes.c_float, ctypes.c_float, _vp]
     L.gd_sage_get.argtypes = [_vp, _i32, _i32, _vp, _i64]
+    L.gd_debug_umma_gemm.argtypes = [_i32, _vp, _i64, _vp, _i64, _vp, _i64, _vp, _vp, _vp, _i64, _i64, _i32, _i32,
+                                     _i32, _i32, _vp]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:

@@ -26,6 +26,7 @@
 #include <vector>
 
 #include "gd_common.cuh"
+#include "gd_umma.cuh"
 
 namespace gd {
 
@@ -605,6 +606,22 @@ gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, i
     if (bytes < n) return set_error(GD_ERR_INVALID, "gd_sage_get: host buffer too small");
     GD_CUDA(cudaDeviceSynchronize());
     GD_CUDA(cudaMemcpy(host_out, src, (size_t)n, cudaMemcpyDeviceToHost));
+    return GD_OK;
+}
+
+gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb, float* C, int64_t ldc,
+                             float* H, const float* bias, const int64_t* rows_dev, int64_t rows_max, int64_t m_valid,
+                             int32_t k_valid, int32_t n_valid, int32_t n_store, int32_t splits, void* stream) {
+    if (mode < 0 || mode > 2 || !A || !B || !C || !rows_dev || n_store < 1 || n_valid < 1)
+        return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: bad argument");
+    if ((lda | ldb) & 7 || (k_valid & 7) || (n_valid & 7) || (m_valid & 7) || ((uintptr_t)A | (uintptr_t)B) & 15)
+        return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: strides / extents must be multiples of 8, bases 16-byte aligned");
+    umma::Args a{};
+    a.A = (const __nv_bfloat16*)A; a.lda = lda;
+    a.B = (const __nv_bfloat16*)B; a.ldb = ldb;
+    a.C = C; a.ldc = ldc; a.H = H; a.bias = bias; a.rows_dev = rows_dev;
+    a.m_valid = m_valid; a.k_valid = k_valid; a.n_valid = n_valid; a.n_store = n_store;
+    GD_CUDA(umma::launch(mode, a, rows_max, mode == 2 ? n_store : n_store, splits, (cudaStream_t)stream));
     return GD_OK;
 }
 
