@@ -294,7 +294,8 @@ typedef struct gd_sage gd_sage;
 #define GD_SAGE_DW 2
 #define GD_SAGE_DB 3
 #define GD_SAGE_A16 4   /* bf16 [n_dst bound x 2 d_in], last forward */
-#define GD_SAGE_Z 5     /* fp32 [n_dst bound x d_out], last forward (z + b) */
+#define GD_SAGE_Z 5     /* fp32 [n_dst bound x d_out], last forward logits z + b (top layer only) */
+#define GD_SAGE_H 6     /* bf16 [n_dst bound x d_out], last forward relu(z + b) (hidden layers only) */
 gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* const* init_w,
                          const float* const* init_b, const int64_t* max_nodes, int device, gd_sage** out);
 gd_status gd_sage_destroy(gd_sage* s);
@@ -306,19 +307,20 @@ gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream
 gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, int64_t bytes);
 
 /* Test surface of the train stage's tensor-core GEMM (csrc/gd_umma.cuh; tcgen05.mma with
- * the accumulator in TMEM), all pointers device, bf16 operands, fp32 C, stream-ordered:
- *   mode 0 FWD  C[i, n] = sum_k A[i*lda + k] B[k*ldb + n] (+ bias[n]; H = relu(C))
+ * the accumulator in TMEM), all pointers device, bf16 operands, stream-ordered:
+ *   mode 0 FWD  C[i, n] = f(sum_k A[i*lda + k] B[k*ldb + n] + bias[n]), f = relu if `relu`
  *   mode 1 DA   C[i, n] = sum_k A[i*lda + k] B[n*ldb + k]
- *   for i < *rows_dev (<= rows_max), k < k_valid (multiple of 8), n < n_store; B is valid
- *   (and read) for n < n_valid (multiple of 8), zero beyond.
+ *   for i < *rows_dev (<= rows_max), k < k_valid (multiple of 8), n < n_store; C is bf16 if
+ *   c_bf16 else fp32, row stride ldc; bias nullable; B is valid (and read) for n < n_valid
+ *   (multiple of 8), zero beyond.
  *   mode 2 DW   C[m, n] += sum_{i < *rows_dev} A[i*lda + m] B[i*ldb + n] for m < m_valid
- *   (multiple of 8), n < n_store, the reduction split over `splits` CTAs per tile (fp32
- *   red.add into C: the caller zeroes it).
+ *   (multiple of 8), n < n_store, C fp32, the reduction split over `splits` CTAs per tile
+ *   (fp32 red.add into C: the caller zeroes it).
  * Row strides are multiples of 8 elements, base pointers 16-byte aligned (GD_ERR_INVALID). */
 gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb,
-                             float* C, int64_t ldc, float* H, const float* bias, const int64_t* rows_dev,
-                             int64_t rows_max, int64_t m_valid, int32_t k_valid, int32_t n_valid,
-                             int32_t n_store, int32_t splits, void* stream);
+                             void* C, int64_t ldc, int32_t c_bf16, int32_t relu, const float* bias,
+                             const int64_t* rows_dev, int64_t rows_max, int64_t m_valid, int32_t k_valid,
+                             int32_t n_valid, int32_t n_store, int32_t splits, void* stream);
 
 /* ----------------------------------------------------------------------------
  * Release stage: for node_ids in list order decrement the refcount; a

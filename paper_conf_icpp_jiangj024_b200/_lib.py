@@ -90,8 +90,8 @@ def _load():
     L.gd_sage_grads.argtypes = [_vp, ctypes.POINTER(_vp), ctypes.POINTER(_i64)]
     L.gd_sage_apply_sgd.argtypes = [_vp, ctypes.c_float, ctypes.c_float, _vp]
     L.gd_sage_get.argtypes = [_vp, _i32, _i32, _vp, _i64]
-    L.gd_debug_umma_gemm.argtypes = [_i32, _vp, _i64, _vp, _i64, _vp, _i64, _vp, _vp, _vp, _i64, _i64, _i32, _i32,
-                                     _i32, _i32, _vp]
+    L.gd_debug_umma_gemm.argtypes = [_i32, _vp, _i64, _vp, _i64, _vp, _i64, _i32, _i32, _vp, _vp, _i64, _i64, _i32,
+                                     _i32, _i32, _i32, _vp]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:

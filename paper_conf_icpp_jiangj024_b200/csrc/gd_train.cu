@@ -4,21 +4,20 @@
 // gathered (the trainer "adopts the node alias list to index required feature data
 // in device memory"; GraphSAGE, 3 layers, hidden 256; DDP gradient sync).
 // Layer j (j = 0..L-1) consumes hop h = L - j (outermost block first):
-//   a_i = [x_i | mean_{e in row i} x_col[e]]  (k_sage_agg: warp per dst row, fp32 sums,
-//                                              bf16 out, rows past n_dst zeroed)
-//   z   = a W + b                             (cuBLAS bf16 tensor-core GEMM, fp32 accumulate;
-//                                              k_bias_act adds b and applies relu; the top
-//                                              layer's b is added in k_xent)
+//   a_i = [x_i | mean_{e in row i} x_col[e]]  (k_sage_agg: warp per dst row, fp32 sums, bf16 out)
+//   z   = a W + b, h = relu(z)                (gd_umma.cuh FWD: tcgen05 GEMM, TMEM accumulator,
+//                                              bias + relu in the epilogue)
 //   loss = mean softmax cross entropy of the seeds' logits (k_xent + k_loss_sum)
-// backward: dW = a^T dz, da = dz W^T (GEMMs), db = column sums of dz (k_colsum_*,
-// deterministic), k_scatter_init + k_sage_scatter spread da to the layer's inputs (own row
-// by plain stores, neighbour mean by fp32 red.add), k_relu_grad masks by the previous
-// layer's activation.  GEMMs run at the host-side worst-case row counts (gd_sample_bounds)
-// with padded rows zero, so nothing synchronises the host; the elementwise kernels stop at
-// the device-resident row counts and re-zero only the rows the previous step wrote (hw).
+// backward: dW = a^T dz (umma DW, split over rows, red.add), da = dz W^T (umma DA), db =
+// column sums of dz (k_colsum_*, deterministic), k_scatter_init + k_sage_scatter spread da to
+// the layer's inputs (own row by plain stores, neighbour mean by fp32 red.add), k_relu_grad
+// masks by the previous layer's activation.  Every kernel, the GEMMs included, reads the
+// block sizes from device memory (gd_sample's `sizes`) and stops there: buffers are sized by
+// the host-side bounds (gd_sample_bounds), nothing synchronises the host, and no padded row
+// is read, multiplied or written.  Widths dout are stored at a stride dp = round_up(dout, 16)
+// (the MMA N granularity; pad columns of W16 and dZ16 are zero).
 // Gradients live in one flat fp32 buffer (layout [W0 b0 W1 b1 ...]) that the caller may
 // all-reduce (NCCL) between gd_sage_step and gd_sage_apply_sgd.
-#include <cublas_v2.h>
 #include <cuda_bf16.h>
 
 #include <algorithm>
@@ -33,13 +32,13 @@ namespace gd {
 constexpr uint32_t kMagicSage = 0x47445341u;   // "GDSA"
 
 struct SageLayer {
-    int din = 0, dout = 0, hop = 0;
+    int din = 0, dout = 0, dp = 0, hop = 0;     // dp = round_up(dout, 16): row stride of Z, H, dZ16, W16
     int64_t n_dst_max = 0, n_src_max = 0;
     int64_t w_off = 0, b_off = 0, w16_off = 0;   // offsets into params / grads / W16
     __nv_bfloat16* A16 = nullptr;   // [n_dst_max, 2 din]  (saved for backward)
-    float* Z = nullptr;             // [n_dst_max, dout]   pre-activation / logits
-    float* H = nullptr;             // [n_dst_max, dout]   relu(Z + b) (j < L-1)
-    __nv_bfloat16* dZ16 = nullptr;  // [n_dst_max, dout]
+    float* Z = nullptr;             // [n_dst_max, dp]     logits z + b (top layer)
+    __nv_bfloat16* H16 = nullptr;   // [n_dst_max, dp]     relu(z + b) (hidden layers: the next layer's input)
+    __nv_bfloat16* dZ16 = nullptr;  // [n_dst_max, dp]
     float* dA = nullptr;            // [n_dst_max, 2 din]  (j >= 1)
     float* dX = nullptr;            // [n_src_max, din]    gradient wrt this layer's input (j >= 1)
 };
@@ -54,42 +53,35 @@ struct gd_sage {
     std::vector<gd::SageLayer> layers;
     float* params = nullptr;        // flat fp32 master parameters [W0 b0 W1 b1 ...]
     float* grads = nullptr;         // same layout
-    __nv_bfloat16* W16 = nullptr;   // bf16 copies of the W's
+    __nv_bfloat16* W16 = nullptr;   // bf16 copies of the W's, [2 din x dp] each (pad columns 0)
     int64_t nparams = 0, nw16 = 0;
     float* loss_rows = nullptr;     // [n0_max]
-    int64_t* hw = nullptr;          // [L] rows of A16 / dZ16 of layer j that may be nonzero
-                                    // (the previous step's n_dst): padded rows are zeroed
-                                    // only up to it, not up to the bound
     float* colsum_part = nullptr;   // [kColsumChunks x max dout] partial column sums (db)
-    cublasHandle_t cublas = nullptr;
 };
 
 namespace gd {
 
 // ------------------------------------------------------------------ kernels
-// a_i = [x_i | mean x_col] for i < n_dst, zero rows [n_dst, hw) (rows past hw are zero).  Warp per row; each
-// lane owns 4-column groups (float4) g = lane, lane + 32, ...; neighbour ids are loaded
-// 32 at a time and broadcast with shuffles.
-__global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, int din, const int64_t* __restrict__ rowptr,
-                                                  const int32_t* __restrict__ col, const int64_t* __restrict__ n_dst_p,
-                                                  const int64_t* __restrict__ hw_p, __nv_bfloat16* __restrict__ A16) {
+// a_i = [x_i | mean x_col] for i < n_dst (x fp32 features or bf16 activations, rows at stride ldx).  Warp per row; each lane
+// owns 4-column groups (float4) g = lane, lane + 32, ...; neighbour ids are loaded 32 at a
+// time and broadcast with shuffles, 4 neighbour rows in flight per lane.
+__device__ __forceinline__ float4 load4(const float* __restrict__ row, int g) { return __ldg((const float4*)row + g); }
+__device__ __forceinline__ float4 load4(const __nv_bfloat16* __restrict__ row, int g) {
+    const uint2 u = __ldg((const uint2*)row + g);
+    const float2 a = __bfloat1622float2(*(const __nv_bfloat162*)&u.x), b = __bfloat1622float2(*(const __nv_bfloat162*)&u.y);
+    return make_float4(a.x, a.y, b.x, b.y);
+}
+
+template <typename T>
+__global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64_t ldx, int din,
+                                                  const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                                                  const int64_t* __restrict__ n_dst_p, __nv_bfloat16* __restrict__ A16) {
     const int lane = threadIdx.x & 31;
     const int64_t n_dst = *n_dst_p;
-    const int64_t n_end = n_dst > *hw_p ? n_dst : *hw_p;   // rows [n_dst, hw) held the last batch
     const int groups = din >> 2;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst; i += warps) {
         __nv_bfloat162* arow = (__nv_bfloat162*)(A16 + i * 2 * din);
-        if (i >= n_dst) {
-            for (int g = lane; g < groups; g += 32) {
-                const __nv_bfloat162 z = __floats2bfloat162_rn(0.f, 0.f);
-                arow[2 * g] = z;
-                arow[2 * g + 1] = z;
-                arow[(din >> 1) + 2 * g] = z;
-                arow[(din >> 1) + 2 * g + 1] = z;
-            }
-            continue;
-        }
         const int64_t lo = rowptr[i], hi = rowptr[i + 1];
         const float inv = hi > lo ? 1.0f / (float)(hi - lo) : 0.0f;
         for (int g0 = 0; g0 < groups; g0 += 64) {          // up to 2 float4 per lane per pass
@@ -100,47 +92,47 @@ __global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, i
                 const int32_t c = lane < m ? col[e0 + lane] : 0;
                 int t = 0;
                 for (; t + 4 <= m; t += 4) {      // 4 neighbour rows in flight per lane
-                    const float4* xr[4];
+                    const T* xr[4];
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) xr[q] = (const float4*)(x + (int64_t)__shfl_sync(0xffffffffu, c, t + q) * din);
+                    for (int q = 0; q < 4; ++q) xr[q] = x + (int64_t)__shfl_sync(0xffffffffu, c, t + q) * ldx;
                     if (ga < groups) {
                         float4 v[4];
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) v[q] = __ldg(xr[q] + ga);
+                        for (int q = 0; q < 4; ++q) v[q] = load4(xr[q], ga);
 #pragma unroll
                         for (int q = 0; q < 4; ++q) { sa.x += v[q].x; sa.y += v[q].y; sa.z += v[q].z; sa.w += v[q].w; }
                     }
                     if (gb < groups) {
                         float4 v[4];
 #pragma unroll
-                        for (int q = 0; q < 4; ++q) v[q] = __ldg(xr[q] + gb);
+                        for (int q = 0; q < 4; ++q) v[q] = load4(xr[q], gb);
 #pragma unroll
                         for (int q = 0; q < 4; ++q) { sb.x += v[q].x; sb.y += v[q].y; sb.z += v[q].z; sb.w += v[q].w; }
                     }
                 }
                 for (; t < m; ++t) {
                     const int64_t u = __shfl_sync(0xffffffffu, c, t);
-                    const float4* xr = (const float4*)(x + u * din);
+                    const T* xr = x + u * ldx;
                     if (ga < groups) {
-                        const float4 v = __ldg(xr + ga);
+                        const float4 v = load4(xr, ga);
                         sa.x += v.x; sa.y += v.y; sa.z += v.z; sa.w += v.w;
                     }
                     if (gb < groups) {
-                        const float4 v = __ldg(xr + gb);
+                        const float4 v = load4(xr, gb);
                         sb.x += v.x; sb.y += v.y; sb.z += v.z; sb.w += v.w;
                     }
                 }
             }
-            const float4* xi = (const float4*)(x + i * din);
+            const T* xi = x + i * ldx;
             if (ga < groups) {
-                const float4 s = __ldg(xi + ga);
+                const float4 s = load4(xi, ga);
                 arow[2 * ga] = __floats2bfloat162_rn(s.x, s.y);
                 arow[2 * ga + 1] = __floats2bfloat162_rn(s.z, s.w);
                 arow[(din >> 1) + 2 * ga] = __floats2bfloat162_rn(sa.x * inv, sa.y * inv);
                 arow[(din >> 1) + 2 * ga + 1] = __floats2bfloat162_rn(sa.z * inv, sa.w * inv);
             }
             if (gb < groups) {
-                const float4 s = __ldg(xi + gb);
+                const float4 s = load4(xi, gb);
                 arow[2 * gb] = __floats2bfloat162_rn(s.x, s.y);
                 arow[2 * gb + 1] = __floats2bfloat162_rn(s.z, s.w);
                 arow[(din >> 1) + 2 * gb] = __floats2bfloat162_rn(sb.x * inv, sb.y * inv);
@@ -150,61 +142,30 @@ __global__ void __launch_bounds__(256) k_sage_agg(const float* __restrict__ x, i
     }
 }
 
-// Z[i] += b; H[i] = relu(Z[i]) for i < n (hidden layers, dout % 4 == 0).  Block (32, 8):
-// threadIdx.x walks a row's float4 columns, threadIdx.y rows; no index division.  Rows past
-// n are not touched (the GEMM produced 0 there from zero A16 rows, and nothing reads them).
-__global__ void __launch_bounds__(256) k_bias_act(float* __restrict__ Z, float* __restrict__ H, const float* __restrict__ b,
-                                                  int dout, const int64_t* __restrict__ n_p) {
-    const int64_t n = *n_p;
-    const int dv = dout >> 2;
-    const float4* b4 = (const float4*)b;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n; i += (int64_t)gridDim.x * blockDim.y) {
-        float4* z4 = (float4*)(Z + i * dout);
-        float4* h4 = (float4*)(H + i * dout);
-        for (int c = threadIdx.x; c < dv; c += blockDim.x) {
-            float4 z = z4[c];
-            const float4 bb = __ldg(b4 + c);
-            z.x += bb.x; z.y += bb.y; z.z += bb.z; z.w += bb.w;
-            z4[c] = z;
-            h4[c] = make_float4(fmaxf(z.x, 0.f), fmaxf(z.y, 0.f), fmaxf(z.z, 0.f), fmaxf(z.w, 0.f));
-        }
-    }
-}
-
-// Softmax cross entropy of the logits z + b, warp per seed row: Z[i] = z + b,
-// loss_rows[i] = lse - z[label]; dZ16[i] = (softmax - onehot) / n0; rows [n0, hw) zeroed.
-__global__ void __launch_bounds__(256) k_xent(float* __restrict__ Z, const float* __restrict__ b, int C,
-                                              const int32_t* __restrict__ labels, const int64_t* __restrict__ n_p,
-                                              const int64_t* __restrict__ hw_p, __nv_bfloat16* __restrict__ dZ16,
+// Softmax cross entropy of the logits (z + b, from the FWD epilogue, row stride dp), warp
+// per seed row: loss_rows[i] = lse - z[label]; dZ16[i] = (softmax - onehot) / n0 for the C
+// classes, 0 in the pad columns [C, dp).
+__global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, int dp, const int32_t* __restrict__ labels,
+                                              const int64_t* __restrict__ n_p, __nv_bfloat16* __restrict__ dZ16,
                                               float* __restrict__ loss_rows) {
     const int lane = threadIdx.x & 31;
     const int64_t n = *n_p;
-    const int64_t n_end = n > *hw_p ? n : *hw_p;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
-        float* z = Z + i * C;
-        __nv_bfloat16* dz = dZ16 + i * C;
-        if (i >= n) {
-            for (int c = lane; c < C; c += 32) dz[c] = __float2bfloat16_rn(0.f);
-            continue;
-        }
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n; i += warps) {
+        const float* z = Z + i * dp;
+        __nv_bfloat16* dz = dZ16 + i * dp;
         float m = -INFINITY;
-        for (int c = lane; c < C; c += 32) {
-            const float v = z[c] + b[c];
-            z[c] = v;
-            m = fmaxf(m, v);
-        }
+        for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
         for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
         float s = 0.f;
         for (int c = lane; c < C; c += 32) s += __expf(z[c] - m);
         for (int o = 16; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
         const int y = labels[i];
         const float inv_n = 1.0f / (float)n;
-        for (int c = lane; c < C; c += 32) {
-            const float p = __expf(z[c] - m) / s;
-            dz[c] = __float2bfloat16_rn((p - (c == y ? 1.f : 0.f)) * inv_n);
+        for (int c = lane; c < dp; c += 32) {
+            const float p = c < C ? __expf(z[c] - m) / s : 0.f;
+            dz[c] = __float2bfloat16_rn(c < C ? (p - (c == y ? 1.f : 0.f)) * inv_n : 0.f);
         }
-        __syncwarp();
         if (lane == 0) loss_rows[i] = m + __logf(s) - z[y];
     }
 }
@@ -267,25 +228,21 @@ __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ 
     }
 }
 
-// dZ16 = bf16(dX * (H > 0)) for rows < n, zero rows [n, hw).  Block (32, 8) as k_bias_act.
-__global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX, const float* __restrict__ H, int d,
-                                                   const int64_t* __restrict__ n_p, const int64_t* __restrict__ hw_p,
-                                                   __nv_bfloat16* __restrict__ dZ16) {
+// dZ16 = bf16(dX * (H > 0)) for rows < n (dX at stride d, H16 and dZ16 at stride dp; pad
+// columns stay zero).  Block (32, 8): threadIdx.x walks a row's float4 columns, threadIdx.y
+// rows; no index division.
+__global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX, const __nv_bfloat16* __restrict__ H16, int d, int dp,
+                                                   const int64_t* __restrict__ n_p, __nv_bfloat16* __restrict__ dZ16) {
     const int64_t n = *n_p;
-    const int64_t n_end = n > *hw_p ? n : *hw_p;
     const int dv = d >> 2;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n_end; i += (int64_t)gridDim.x * blockDim.y) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n; i += (int64_t)gridDim.x * blockDim.y) {
         const float4* x4 = (const float4*)(dX + i * d);
-        const float4* h4 = (const float4*)(H + i * d);
-        __nv_bfloat162* o2 = (__nv_bfloat162*)(dZ16 + i * d);
+        const __nv_bfloat16* hrow = H16 + i * dp;
+        __nv_bfloat162* o2 = (__nv_bfloat162*)(dZ16 + i * dp);
         for (int c = threadIdx.x; c < dv; c += blockDim.x) {
-            float4 v = make_float4(0.f, 0.f, 0.f, 0.f);
-            if (i < n) {
-                const float4 x = x4[c], h = h4[c];
-                v = make_float4(h.x > 0.f ? x.x : 0.f, h.y > 0.f ? x.y : 0.f, h.z > 0.f ? x.z : 0.f, h.w > 0.f ? x.w : 0.f);
-            }
-            o2[2 * c] = __floats2bfloat162_rn(v.x, v.y);
-            o2[2 * c + 1] = __floats2bfloat162_rn(v.z, v.w);
+            const float4 x = x4[c], h = load4(hrow, c);
+            o2[2 * c] = __floats2bfloat162_rn(h.x > 0.f ? x.x : 0.f, h.y > 0.f ? x.y : 0.f);
+            o2[2 * c + 1] = __floats2bfloat162_rn(h.z > 0.f ? x.z : 0.f, h.w > 0.f ? x.w : 0.f);
         }
     }
 }
@@ -295,7 +252,7 @@ __global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX,
 // rows y, y + 8, ... of the chunk), reduces the 8 row lanes in shared memory and writes
 // part[chunk][col].  Pass 2 does the same over the kColsumChunks partials.
 constexpr int kColsumChunks = 256;
-__global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __restrict__ dZ16, int d,
+__global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __restrict__ dZ16, int d, int ld,
                                                      const int64_t* __restrict__ n_p, float* __restrict__ part) {
     __shared__ float sh[8][33];
     const int64_t n = *n_p;
@@ -306,7 +263,7 @@ __global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __rest
     if (c < d) {
         int64_t i = r0 + threadIdx.y;
 #pragma unroll 4
-        for (; i < r1; i += 8) s += __bfloat162float(dZ16[i * d + c]);
+        for (; i < r1; i += 8) s += __bfloat162float(dZ16[i * ld + c]);
     }
     sh[threadIdx.y][threadIdx.x] = s;
     __syncthreads();
@@ -333,51 +290,26 @@ __global__ void __launch_bounds__(256) k_colsum_final(const float* __restrict__ 
     }
 }
 
-__global__ void k_set_hw(int64_t* __restrict__ hw, const int64_t* __restrict__ sizes, int L) {
-    const int j = threadIdx.x;
-    if (j < L) hw[j] = sizes[L - 1 - j];      // layer j's dst rows = n_{hop-1}, hop = L - j
-}
-
 __global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float step) {
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
         p[k] = fmaf(-step, g[k], p[k]);
 }
 
-__global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst, int64_t n) {
-    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
-        dst[k] = __float2bfloat16_rn(src[k]);
-}
-
-// ------------------------------------------------------------------ GEMMs (row-major)
-static const char* cublas_msg(cublasStatus_t s) {
-    switch (s) {
-        case CUBLAS_STATUS_NOT_INITIALIZED: return "CUBLAS_STATUS_NOT_INITIALIZED";
-        case CUBLAS_STATUS_ALLOC_FAILED: return "CUBLAS_STATUS_ALLOC_FAILED";
-        case CUBLAS_STATUS_INVALID_VALUE: return "CUBLAS_STATUS_INVALID_VALUE";
-        case CUBLAS_STATUS_ARCH_MISMATCH: return "CUBLAS_STATUS_ARCH_MISMATCH";
-        case CUBLAS_STATUS_EXECUTION_FAILED: return "CUBLAS_STATUS_EXECUTION_FAILED";
-        case CUBLAS_STATUS_NOT_SUPPORTED: return "CUBLAS_STATUS_NOT_SUPPORTED";
-        default: return "cuBLAS error";
+// W16[r, c] = bf16(W[r, c]) for c < d, 0 for d <= c < dp (rows of W at stride d).
+__global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst, int64_t rows, int d, int dp) {
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < rows * dp; k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = k / dp;
+        const int c = (int)(k - r * dp);
+        dst[k] = __float2bfloat16_rn(c < d ? src[r * d + c] : 0.f);
     }
 }
-#define GD_CUBLAS(call)                                                                       \
-    do {                                                                                      \
-        cublasStatus_t s_ = (call);                                                           \
-        if (s_ != CUBLAS_STATUS_SUCCESS)                                                      \
-            return ::gd::set_error(GD_ERR_CUDA, std::string(#call ": ") + ::gd::cublas_msg(s_)); \
-    } while (0)
 
-// C[M x N] (row-major, fp32) = op(A) op(B) with bf16 operands, fp32 accumulate.  A row-major
-// [M x K] (transA: stored [K x M]), B row-major [K x N] (transB: stored [N x K]).  Column-
-// major cuBLAS computes C^T = op(B)^T op(A)^T.
-static gd_status gemm_rm(cublasHandle_t h, bool transA, bool transB, int64_t M, int64_t N, int64_t K,
-                         const __nv_bfloat16* A, const __nv_bfloat16* B, float* C) {
-    const float one = 1.f, zero = 0.f;
-    const int lda = (int)(transA ? M : K), ldb = (int)(transB ? K : N);
-    GD_CUBLAS(cublasGemmEx(h, transB ? CUBLAS_OP_T : CUBLAS_OP_N, transA ? CUBLAS_OP_T : CUBLAS_OP_N, (int)N, (int)M,
-                           (int)K, &one, B, CUDA_R_16BF, ldb, A, CUDA_R_16BF, lda, &zero, C, CUDA_R_32F, (int)N,
-                           CUBLAS_COMPUTE_32F, CUBLAS_GEMM_DEFAULT));
-    return GD_OK;
+// ------------------------------------------------------------------ GEMMs (gd_umma.cuh)
+static umma::Args gemm_args(const __nv_bfloat16* A, int64_t lda, const __nv_bfloat16* B, int64_t ldb, void* C, int64_t ldc,
+                            const int64_t* rows_dev) {
+    umma::Args a{};
+    a.A = A; a.lda = lda; a.B = B; a.ldb = ldb; a.C = C; a.ldc = ldc; a.rows_dev = rows_dev;
+    return a;
 }
 
 static unsigned grid_for(int64_t n, int per_block = 256) {
@@ -389,11 +321,10 @@ static void sage_free(gd_sage* s) {
     DeviceGuard guard(s->hdr.device);
     cudaDeviceSynchronize();
     for (auto& l : s->layers)
-        for (void* p : {(void*)l.A16, (void*)l.Z, (void*)l.H, (void*)l.dZ16, (void*)l.dA, (void*)l.dX})
+        for (void* p : {(void*)l.A16, (void*)l.Z, (void*)l.H16, (void*)l.dZ16, (void*)l.dA, (void*)l.dX})
             if (p) cudaFree(p);
-    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->hw, (void*)s->colsum_part})
+    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->colsum_part})
         if (p) cudaFree(p);
-    if (s->cublas) cublasDestroy(s->cublas);
     s->hdr.magic = 0;
     delete s;
 }
@@ -430,6 +361,7 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         SageLayer& l = s->layers[j];
         l.din = dims[j];
         l.dout = dims[j + 1];
+        l.dp = (l.dout + 15) / 16 * 16;
         l.hop = num_layers - j;
         l.n_dst_max = max_nodes[l.hop - 1];
         l.n_src_max = max_nodes[l.hop];
@@ -438,7 +370,7 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         l.b_off = off;
         off += l.dout;
         l.w16_off = off16;
-        off16 += (int64_t)2 * l.din * l.dout;
+        off16 += (int64_t)2 * l.din * l.dp;
     }
     s->nparams = off;
     s->nw16 = off16;
@@ -455,29 +387,22 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
     for (int j = 0; j < num_layers; ++j) {
         SageLayer& l = s->layers[j];
         SA(l.A16, l.n_dst_max * 2 * l.din * sizeof(__nv_bfloat16));
-        SA(l.Z, l.n_dst_max * l.dout * sizeof(float));
-        if (j < num_layers - 1) SA(l.H, l.n_dst_max * l.dout * sizeof(float));
-        SA(l.dZ16, l.n_dst_max * l.dout * sizeof(__nv_bfloat16));
+        if (j == num_layers - 1) SA(l.Z, l.n_dst_max * l.dp * sizeof(float));
+        else SA(l.H16, l.n_dst_max * l.dp * sizeof(__nv_bfloat16));
+        SA(l.dZ16, l.n_dst_max * l.dp * sizeof(__nv_bfloat16));
         if (j > 0) {
             SA(l.dA, l.n_dst_max * 2 * l.din * sizeof(float));
             SA(l.dX, l.n_src_max * l.din * sizeof(float));
         }
         max_dout = std::max(max_dout, l.dout);
     }
-    SA(s->hw, num_layers * sizeof(int64_t));
     SA(s->colsum_part, (size_t)kColsumChunks * max_dout * sizeof(float));
 #undef SA
-    // the GEMMs run at the bound row counts: padded rows of their bf16 operands start zero
-    // and every step re-zeroes only the rows the previous step wrote (hw)
-    for (int j = 0; j < num_layers; ++j) {
+    for (int j = 0; j < num_layers; ++j) {      // pad columns of dZ16 (the DA GEMM's K) start and stay zero
         const SageLayer& l = s->layers[j];
-        cudaError_t e = cudaMemset(l.A16, 0, l.n_dst_max * 2 * l.din * sizeof(__nv_bfloat16));
-        if (e == cudaSuccess) e = cudaMemset(l.dZ16, 0, l.n_dst_max * l.dout * sizeof(__nv_bfloat16));
-        if (e == cudaSuccess) e = cudaMemset(l.Z, 0, l.n_dst_max * l.dout * sizeof(float));
+        cudaError_t e = cudaMemset(l.dZ16, 0, l.n_dst_max * l.dp * sizeof(__nv_bfloat16));
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: memset"));
     }
-    if (cudaMemset(s->hw, 0, num_layers * sizeof(int64_t)) != cudaSuccess)
-        return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
     for (int j = 0; j < num_layers; ++j) {
         const SageLayer& l = s->layers[j];
         if (!init_w[j] || !init_b[j]) return fail(set_error(GD_ERR_INVALID, "gd_sage_create: null initial parameter"));
@@ -486,13 +411,10 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         if (e == cudaSuccess)
             e = cudaMemcpy(s->params + l.b_off, init_b[j], (size_t)l.dout * sizeof(float), cudaMemcpyHostToDevice);
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: parameter copy"));
-        k_to_bf16<<<grid_for(2 * l.din * l.dout), 256>>>(s->params + l.w_off, s->W16 + l.w16_off, (int64_t)2 * l.din * l.dout);
+        k_to_bf16<<<grid_for(2 * l.din * l.dp), 256>>>(s->params + l.w_off, s->W16 + l.w16_off, 2 * l.din, l.dout, l.dp);
     }
     if (cudaMemset(s->grads, 0, off * sizeof(float)) != cudaSuccess)
         return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
-    if (cublasCreate(&s->cublas) != CUBLAS_STATUS_SUCCESS)
-        return fail(set_error(GD_ERR_CUDA, "gd_sage_create: cublasCreate failed"));
-    cublasSetMathMode(s->cublas, CUBLAS_DEFAULT_MATH);
     cudaError_t e = cudaDeviceSynchronize();
     if (e != cudaSuccess) return fail(cuda_error(e, "gd_sage_create: init kernels"));
     *out = s;
@@ -515,55 +437,78 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         if (!rowptr[h] || !col[h]) return set_error(GD_ERR_INVALID, "gd_sage_step: null block pointer");
     DeviceGuard guard(s->hdr.device);
     cudaStream_t st = (cudaStream_t)stream_v;
-    GD_CUBLAS(cublasSetStream(s->cublas, st));
     const int L = s->L;
     const dim3 rows_blk(32, 8);          // (float4 column, row) blocks of the row-wise kernels
     // ---- forward
-    const float* x = feats;
+    const void* x = feats;
+    int64_t ldx = s->dims[0];
     for (int j = 0; j < L; ++j) {
         SageLayer& l = s->layers[j];
         const int h = l.hop;
-        k_sage_agg<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(x, l.din, rowptr[h - 1], col[h - 1], sizes + (h - 1),
-                                                               s->hw + j, l.A16);
+        const int64_t* n_dst = sizes + (h - 1);
+        if (j == 0)
+            k_sage_agg<float><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const float*)x, ldx, l.din, rowptr[h - 1],
+                                                                          col[h - 1], n_dst, l.A16);
+        else
+            k_sage_agg<__nv_bfloat16><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const __nv_bfloat16*)x, ldx, l.din,
+                                                                                  rowptr[h - 1], col[h - 1], n_dst, l.A16);
         GD_DEBUG_AFTER("k_sage_agg", st);
-        gd_status g = gemm_rm(s->cublas, false, false, l.n_dst_max, l.dout, 2 * l.din, l.A16, s->W16 + l.w16_off, l.Z);
-        if (g != GD_OK) return g;
-        if (j < L - 1) {
-            k_bias_act<<<grid_for(l.n_dst_max * 8), rows_blk, 0, st>>>(l.Z, l.H, s->params + l.b_off, l.dout,
-                                                                       sizes + (h - 1));
-            GD_DEBUG_AFTER("k_bias_act", st);
-        }
-        x = l.H;
+        const bool hidden = j < L - 1;   // hidden: h = relu(z + b) in bf16 (the next layer's input); top: logits
+        umma::Args a = gemm_args(l.A16, 2 * l.din, s->W16 + l.w16_off, l.dp, hidden ? (void*)l.H16 : (void*)l.Z, l.dp, n_dst);
+        a.c_bf16 = hidden;
+        a.relu = hidden;
+        a.bias = s->params + l.b_off;
+        a.k_valid = 2 * l.din;
+        a.n_valid = l.dp;
+        a.n_store = l.dout;
+        GD_CUDA(umma::launch(umma::FWD, a, l.n_dst_max, l.dout, 1, st));
+        GD_DEBUG_AFTER("k_umma_gemm<FWD>", st);
+        x = l.H16;
+        ldx = l.dp;
     }
-    // ---- loss (the top layer's bias is added here)
+    // ---- loss
     SageLayer& top = s->layers[L - 1];
-    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, s->params + top.b_off, top.dout, labels, sizes,
-                                                         s->hw + (L - 1), top.dZ16, s->loss_rows);
+    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, top.dp, labels, sizes, top.dZ16, s->loss_rows);
     k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
     GD_DEBUG_AFTER("k_xent", st);
     // ---- backward
+    GD_CUDA(cudaMemsetAsync(s->grads, 0, (size_t)s->nparams * sizeof(float), st));   // dW accumulates by red.add
     for (int j = L - 1; j >= 0; --j) {
         SageLayer& l = s->layers[j];
         const int h = l.hop;
-        gd_status g = gemm_rm(s->cublas, true, false, 2 * l.din, l.dout, l.n_dst_max, l.A16, l.dZ16, s->grads + l.w_off);
-        if (g != GD_OK) return g;
+        const int64_t* n_dst = sizes + (h - 1);
+        {   // dW = a^T dz, the rows split over ~1 CTA per SM
+            umma::Args a = gemm_args(l.A16, 2 * l.din, l.dZ16, l.dp, s->grads + l.w_off, l.dout, n_dst);
+            a.m_valid = 2 * l.din;
+            a.n_valid = l.dp;
+            a.n_store = l.dout;
+            const int64_t tiles = ((2 * l.din + umma::BM - 1) / umma::BM) * ((l.dout + 255) / 256);
+            const int64_t kblocks = (l.n_dst_max + umma::BK - 1) / umma::BK;
+            const int splits = (int)std::max<int64_t>(1, std::min<int64_t>(kblocks, 148 / tiles));
+            GD_CUDA(umma::launch(umma::DW, a, l.n_dst_max, l.dout, splits, st));
+            GD_DEBUG_AFTER("k_umma_gemm<DW>", st);
+        }
         const unsigned strips = (unsigned)((l.dout + 31) / 32);
-        k_colsum_part<<<dim3(strips, kColsumChunks), rows_blk, 0, st>>>(l.dZ16, l.dout, sizes + (h - 1), s->colsum_part);
+        k_colsum_part<<<dim3(strips, kColsumChunks), rows_blk, 0, st>>>(l.dZ16, l.dout, l.dp, n_dst, s->colsum_part);
         k_colsum_final<<<strips, rows_blk, 0, st>>>(s->colsum_part, l.dout, kColsumChunks, s->grads + l.b_off);
         GD_DEBUG_AFTER("k_colsum", st);
         if (j == 0) break;
-        g = gemm_rm(s->cublas, false, true, l.n_dst_max, 2 * l.din, l.dout, l.dZ16, s->W16 + l.w16_off, l.dA);
-        if (g != GD_OK) return g;
-        k_scatter_init<<<grid_for(l.n_src_max * 8), rows_blk, 0, st>>>(l.dA, l.din, sizes + (h - 1), sizes + h, l.dX);
-        k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1],
-                                                                   sizes + (h - 1), l.dX);
+        {   // da = dz W^T
+            umma::Args a = gemm_args(l.dZ16, l.dp, s->W16 + l.w16_off, l.dp, l.dA, 2 * l.din, n_dst);
+            a.k_valid = l.dp;
+            a.n_valid = 2 * l.din;
+            a.n_store = 2 * l.din;
+            GD_CUDA(umma::launch(umma::DA, a, l.n_dst_max, 2 * l.din, 1, st));
+            GD_DEBUG_AFTER("k_umma_gemm<DA>", st);
+        }
+        k_scatter_init<<<grid_for(l.n_src_max * 8), rows_blk, 0, st>>>(l.dA, l.din, n_dst, sizes + h, l.dX);
+        k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1], n_dst, l.dX);
         GD_DEBUG_AFTER("k_sage_scatter", st);
-        SageLayer& prev = s->layers[j - 1];   // its output (H) is this layer's input
-        k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H, prev.dout, sizes + h,
-                                                                       s->hw + (j - 1), prev.dZ16);
+        SageLayer& prev = s->layers[j - 1];   // its output (H16) is this layer's input
+        k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H16, prev.dout, prev.dp, sizes + h,
+                                                                       prev.dZ16);
         GD_DEBUG_AFTER("k_relu_grad", st);
     }
-    k_set_hw<<<1, 32, 0, st>>>(s->hw, sizes, L);
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
@@ -581,8 +526,8 @@ gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream
     cudaStream_t st = (cudaStream_t)stream_v;
     k_sgd<<<grid_for(s->nparams), 256, 0, st>>>(s->params, s->grads, s->nparams, lr * grad_scale);
     for (const SageLayer& l : s->layers)
-        k_to_bf16<<<grid_for(2 * l.din * l.dout), 256, 0, st>>>(s->params + l.w_off, s->W16 + l.w16_off,
-                                                                (int64_t)2 * l.din * l.dout);
+        k_to_bf16<<<grid_for(2 * l.din * l.dp), 256, 0, st>>>(s->params + l.w_off, s->W16 + l.w16_off, 2 * l.din, l.dout,
+                                                              l.dp);
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
@@ -601,27 +546,36 @@ gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, i
         case GD_SAGE_DB: src = s->grads + l.b_off; n = (int64_t)l.dout * 4; break;
         case GD_SAGE_A16: src = l.A16; n = l.n_dst_max * 2 * l.din * 2; break;
         case GD_SAGE_Z: src = l.Z; n = l.n_dst_max * l.dout * 4; break;
+        case GD_SAGE_H: src = l.H16; n = l.n_dst_max * l.dout * 2; break;
         default: return set_error(GD_ERR_INVALID, "gd_sage_get: unknown item");
     }
+    if (!src) return set_error(GD_ERR_INVALID, "gd_sage_get: Z exists for the top layer, H for hidden layers");
     if (bytes < n) return set_error(GD_ERR_INVALID, "gd_sage_get: host buffer too small");
     GD_CUDA(cudaDeviceSynchronize());
-    GD_CUDA(cudaMemcpy(host_out, src, (size_t)n, cudaMemcpyDeviceToHost));
+    if (what == GD_SAGE_Z || what == GD_SAGE_H) {   // stored at row stride dp
+        const size_t e = what == GD_SAGE_Z ? 4 : 2;
+        GD_CUDA(cudaMemcpy2D(host_out, (size_t)l.dout * e, src, (size_t)l.dp * e, (size_t)l.dout * e, (size_t)l.n_dst_max,
+                             cudaMemcpyDeviceToHost));
+    }
+    else
+        GD_CUDA(cudaMemcpy(host_out, src, (size_t)n, cudaMemcpyDeviceToHost));
     return GD_OK;
 }
 
-gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb, float* C, int64_t ldc,
-                             float* H, const float* bias, const int64_t* rows_dev, int64_t rows_max, int64_t m_valid,
-                             int32_t k_valid, int32_t n_valid, int32_t n_store, int32_t splits, void* stream) {
-    if (mode < 0 || mode > 2 || !A || !B || !C || !rows_dev || n_store < 1 || n_valid < 1)
+gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb, void* C, int64_t ldc,
+                             int32_t c_bf16, int32_t relu, const float* bias, const int64_t* rows_dev, int64_t rows_max,
+                             int64_t m_valid, int32_t k_valid, int32_t n_valid, int32_t n_store, int32_t splits,
+                             void* stream) {
+    if (mode < 0 || mode > 2 || !A || !B || !C || !rows_dev || n_store < 1 || n_valid < 1 || (mode == 2 && c_bf16))
         return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: bad argument");
     if ((lda | ldb) & 7 || (k_valid & 7) || (n_valid & 7) || (m_valid & 7) || ((uintptr_t)A | (uintptr_t)B) & 15)
         return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: strides / extents must be multiples of 8, bases 16-byte aligned");
-    umma::Args a{};
-    a.A = (const __nv_bfloat16*)A; a.lda = lda;
-    a.B = (const __nv_bfloat16*)B; a.ldb = ldb;
-    a.C = C; a.ldc = ldc; a.H = H; a.bias = bias; a.rows_dev = rows_dev;
+    umma::Args a = gemm_args((const __nv_bfloat16*)A, lda, (const __nv_bfloat16*)B, ldb, C, ldc, rows_dev);
+    a.c_bf16 = c_bf16;
+    a.relu = relu;
+    a.bias = bias;
     a.m_valid = m_valid; a.k_valid = k_valid; a.n_valid = n_valid; a.n_store = n_store;
-    GD_CUDA(umma::launch(mode, a, rows_max, mode == 2 ? n_store : n_store, splits, (cudaStream_t)stream));
+    GD_CUDA(umma::launch(mode, a, rows_max, n_store, splits, (cudaStream_t)stream));
     return GD_OK;
 }
 

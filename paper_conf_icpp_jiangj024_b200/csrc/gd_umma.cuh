@@ -8,12 +8,15 @@
 // GEMM run at the host-side bound, no padded rows are read, multiplied or written.
 //
 // Tile: UMMA M = 128 rows (one TMEM lane per output row), N = BN <= 256 columns (TMEM columns),
-// K = 64 per pipeline stage (4 MMAs of K = 16).  The 128 threads of the CTA stage operands with
-// cp.async (16-byte chunks, zero-filled past the valid range) into the no-swizzle canonical
-// UMMA layouts, 2 stages deep; thread 0 issues the MMAs and tcgen05.commit's them to the
-// stage's mbarrier, which releases the stage for the next load.  The epilogue reads the
-// accumulator with tcgen05.ld (warp w owns TMEM lanes 32w..32w+31 = rows), adds the bias,
-// stores fp32 (FWD: also relu into H) or red.adds the split-K partial (DW).
+// K = 64 per pipeline stage (4 MMAs of K = 16).  CTAs are persistent over the tiles.  The 128
+// threads of a CTA stage operands with cp.async (16-byte chunks, zero-filled past the valid
+// range) into the no-swizzle canonical UMMA layouts, 4 stages deep and across tile
+// boundaries; thread 0 issues the MMAs and tcgen05.commit's them to the stage's mbarrier,
+// which releases the stage for the next load.  The epilogue reads the
+// accumulator with tcgen05.ld (warp w owns TMEM lanes 32w..32w+31 = rows, 32 columns per
+// load), adds the bias and applies relu (FWD), transposes the 32 x 32 block through shared
+// memory (the drained stage buffers) and writes whole rows per instruction: fp32 or bf16
+// stores, or fp32 red.add of the split-K partial (DW).
 //
 // Shared-memory image of one operand tile (R rows of the M/N dimension x 64 of K), both majors:
 //   K-major  (row-major global, K contiguous):  byte(r, k8) = (r / 8) * 1024 + k8 * 128 + (r % 8) * 16
@@ -25,12 +28,14 @@
 #include <cuda_bf16.h>
 #include <stdint.h>
 
+#include <algorithm>
+
 namespace gd {
 namespace umma {
 
 constexpr int BM = 128;
 constexpr int BK = 64;
-constexpr int STAGES = 2;
+constexpr int STAGES = 4;
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 enum Mode { FWD = 0, DA = 1, DW = 2 };
@@ -38,8 +43,9 @@ enum Mode { FWD = 0, DA = 1, DW = 2 };
 struct Args {
     const __nv_bfloat16* A; int64_t lda;
     const __nv_bfloat16* B; int64_t ldb;
-    float* C; int64_t ldc;
-    float* H;                    // FWD: relu(C) (nullable)
+    void* C; int64_t ldc;        // fp32, or bf16 when c_bf16 (FWD / DA); fp32 for DW
+    int c_bf16;
+    int relu;                    // FWD: C = relu(acc + bias)
     const float* bias;           // FWD: [n_store] (nullable)
     const int64_t* rows_dev;     // device row count: M (FWD, DA) or the reduction length (DW)
     int64_t m_valid;             // DW: output rows (A's contiguous width); FWD/DA: unused
@@ -83,32 +89,120 @@ __host__ __device__ constexpr uint32_t instr_desc(int bn) {
            | ((uint32_t)(BM >> 4) << 24); // M / 16
 }
 
-// Stage one operand tile (R rows along M/N starting at r0, BK along K starting at k0).
+// Stage one operand tile (R rows along M/N starting at r0, BK along K starting at k0).  Chunks
+// are assigned so that every 8 consecutive lanes write 8 distinct 16-byte bank slots (the low
+// 7 address bits are (r % 8) * 16, resp. (k % 8) * 16: conflict-free cp.async writes) while
+// each warp still reads whole 32-byte sectors of global memory:
+//   K-major:  idx = (r / 8) * 64 + k8 * 8 + r % 8            (8 rows x 4 chunks of 16 B per warp)
+//   MN-major: idx = (r8 / 2) * 128 + (k / 8) * 16 + (r8 % 2) * 8 + k % 8
+//                                                          (8 K-rows x 2 adjacent chunks per 16 lanes)
 template <bool MN_MAJOR>
 __device__ __forceinline__ void load_tile(uint32_t s, const __nv_bfloat16* __restrict__ g, int64_t ld, int R, int64_t r0,
                                           int64_t r_valid, int64_t k0, int64_t k_end) {
-    if (!MN_MAJOR) {
-        const int total = R * 8;
-        for (int idx = threadIdx.x; idx < total; idx += blockDim.x) {
-            const int r = idx >> 3, k8 = idx & 7;
-            const int64_t gr = r0 + r, gk = k0 + k8 * 8;
-            const bool v = gr < r_valid && gk < k_end;
-            cp_async16(s + (r >> 3) * 1024 + k8 * 128 + (r & 7) * 16, v ? g + gr * ld + gk : g, v);
+    const int total = R * 8;   // 16-byte chunks in an R x 64 bf16 tile
+    for (int idx = threadIdx.x; idx < total; idx += blockDim.x) {
+        int r, k;              // K-major: row r, chunk k (of 8 elements); MN-major: 8-group r, K-row k
+        uint32_t off;
+        if (!MN_MAJOR) {
+            r = ((idx >> 6) << 3) + (idx & 7);
+            k = (idx >> 3) & 7;
+            off = (uint32_t)idx * 16;   // (r / 8) * 1024 + k * 128 + (r % 8) * 16
+        } else {
+            r = ((idx >> 7) << 1) | ((idx >> 3) & 1);
+            k = (((idx >> 4) & 7) << 3) + (idx & 7);
+            off = (uint32_t)(r * 1024 + (k >> 3) * 128 + (k & 7) * 16);
         }
-    } else {
-        const int r8n = R >> 3;
-        const int total = r8n * BK;
-        for (int idx = threadIdx.x; idx < total; idx += blockDim.x) {
-            const int r8 = idx % r8n, k = idx / r8n;
-            const int64_t gr = r0 + r8 * 8, gk = k0 + k;
-            const bool v = gr < r_valid && gk < k_end;
-            cp_async16(s + r8 * 1024 + (k >> 3) * 128 + (k & 7) * 16, v ? g + gk * ld + gr : g, v);
-        }
+        const int64_t gr = r0 + (MN_MAJOR ? r * 8 : r), gk = k0 + (MN_MAJOR ? k : k * 8);
+        const bool v = gr < r_valid && gk < k_end;
+        cp_async16(s + off, v ? (MN_MAJOR ? g + gk * ld + gr : g + gr * ld + gk) : g, v);
     }
 }
 
+// Epilogue of one unit: warp w reads TMEM lanes 32w.. (= tile rows rbase..rbase+31), 32
+// columns per load (bn is a multiple of 16 and the allocation a power of two >= 32, so a load
+// past bn stays inside it; those columns are not stored), transposes the 32 x 32 block
+// through its 4 KB of shared memory and writes (or red.adds) one 32-column row segment per
+// instruction.
 template <int MODE>
-__global__ void __launch_bounds__(128) k_umma_gemm(Args a) {
+__device__ __forceinline__ void epilogue(const Args& a, uint32_t tmem, float* st, int64_t rbase, int64_t n0, int64_t m_valid,
+                                         int bn, int warp, int lane) {
+    for (int c0 = 0; c0 < bn; c0 += 32) {
+        uint32_t r[32];
+        const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
+        asm volatile(
+            "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+            "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
+            : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+              "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
+              "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
+              "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+            : "r"(taddr));
+        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+#pragma unroll
+        for (int j = 0; j < 32; ++j) st[lane * 33 + j] = __uint_as_float(r[j]);
+        __syncwarp();
+        const int64_t cg = n0 + c0 + lane;              // this lane's output column
+        const bool col_ok = c0 + lane < bn && cg < a.n_store;
+        const float b = (MODE == FWD && a.bias && col_ok) ? __ldg(a.bias + cg) : 0.f;
+        for (int rr = 0; rr < 32; ++rr) {
+            const int64_t row = rbase + rr;
+            if (row >= m_valid) break;
+            float v = st[rr * 33 + lane];
+            if (!col_ok) continue;
+            if (MODE == DW) {
+                atomicAdd((float*)a.C + row * a.ldc + cg, v);
+            } else {
+                v += b;
+                if (MODE == FWD && a.relu) v = fmaxf(v, 0.f);
+                if (a.c_bf16) ((__nv_bfloat16*)a.C)[row * a.ldc + cg] = __float2bfloat16_rn(v);
+                else ((float*)a.C)[row * a.ldc + cg] = v;
+            }
+        }
+        __syncwarp();
+    }
+}
+
+// One unit of work: an output tile (m0, n0) and its reduction range [k_begin, k_end).
+struct Unit {
+    int64_t u, m0, n0, k_begin, k_end;
+    int nkb, kb;
+};
+
+// Units: FWD / DA: (m-tile, n-tile) over the device row count, full K.  DW: (m-tile, n-tile,
+// split) with split z taking a BK-aligned slice of the device row count (empty slices skipped).
+template <int MODE>
+__device__ __forceinline__ bool unit_at(Unit& c, int64_t u, const Args& a, int64_t rows, int nt, int splits) {
+    for (;; u += gridDim.x) {
+        if (MODE == DW) {
+            const int64_t mt = (a.m_valid + BM - 1) / BM;
+            if (u >= mt * nt * splits) return false;
+            const int64_t z = u % splits, rest = u / splits;
+            c.n0 = (rest % nt) * a.bn;
+            c.m0 = (rest / nt) * BM;
+            int64_t per = (rows + splits - 1) / splits;
+            per = (per + BK - 1) / BK * BK;
+            c.k_begin = z * per;
+            c.k_end = c.k_begin + per < rows ? c.k_begin + per : rows;
+            if (c.k_begin >= c.k_end) continue;
+        } else {
+            if (u >= (rows + BM - 1) / BM * nt) return false;
+            c.m0 = (u / nt) * BM;
+            c.n0 = (u % nt) * a.bn;
+            c.k_begin = 0;
+            c.k_end = a.k_valid;
+        }
+        c.u = u;
+        c.kb = 0;
+        c.nkb = (int)((c.k_end - c.k_begin + BK - 1) / BK);
+        return true;
+    }
+}
+
+// Persistent CTAs (grid <= resident CTAs); the load cursor runs STAGES-1 k-blocks ahead of the
+// MMA cursor across unit boundaries, so the next unit's operands stream in during a unit's
+// epilogue.
+template <int MODE>
+__global__ void __launch_bounds__(128) k_umma_gemm(Args a, int nt, int splits) {
     constexpr bool A_MN = MODE == DW;
     constexpr bool B_MN = MODE != DA;
     extern __shared__ __align__(1024) uint8_t smem[];
@@ -116,33 +210,18 @@ __global__ void __launch_bounds__(128) k_umma_gemm(Args a) {
     const int b_stage = bn * BK * 2;
     uint8_t* sA = smem;
     uint8_t* sB = smem + STAGES * A_STAGE;
-    uint64_t* mbar = (uint64_t*)(sB + STAGES * b_stage);
+    float* stage_out = (float*)(sB + STAGES * b_stage);          // 4 warps x 32 x 33 fp32
+    uint64_t* mbar = (uint64_t*)(stage_out + 4 * 32 * 33);
     uint32_t* tmem_slot = (uint32_t*)(mbar + STAGES);
 
-    // ---- work range (device-resident sizes: tiles past them leave at once)
-    const int64_t rows = *a.rows_dev;
-    int64_t m0, m_valid, k_begin, k_end;
-    if (MODE == DW) {
-        m0 = (int64_t)blockIdx.x * BM;
-        m_valid = a.m_valid;
-        int64_t per = (rows + gridDim.z - 1) / gridDim.z;
-        per = (per + BK - 1) / BK * BK;
-        k_begin = (int64_t)blockIdx.z * per;
-        k_end = k_begin + per < rows ? k_begin + per : rows;
-        if (k_begin >= k_end) return;
-    } else {
-        m0 = (int64_t)blockIdx.x * BM;
-        m_valid = rows;
-        k_begin = 0;
-        k_end = a.k_valid;
-        if (m0 >= rows) return;
-    }
-    const int64_t n0 = (int64_t)blockIdx.y * bn;
-    const int nkb = (int)((k_end - k_begin + BK - 1) / BK);
+    const int64_t rows = *a.rows_dev;   // device-resident size
+    Unit cm, ld;
+    if (!unit_at<MODE>(cm, blockIdx.x, a, rows, nt, splits)) return;
+    ld = cm;
+    const int64_t m_valid = MODE == DW ? a.m_valid : rows;
     uint32_t ncols = 32;
     while ((int)ncols < bn) ncols <<= 1;
 
-    // ---- setup: TMEM accumulator (warp 0), stage barriers (thread 0)
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
@@ -160,36 +239,37 @@ __global__ void __launch_bounds__(128) k_umma_gemm(Args a) {
     const uint32_t tmem = *tmem_slot;
     const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
 
-    auto load_stage = [&](int kb) {
-        const int s = kb % STAGES;
-        const int64_t k0 = k_begin + (int64_t)kb * BK;
-        load_tile<A_MN>(smem_u32(sA + s * A_STAGE), a.A, a.lda, BM, m0, m_valid, k0, k_end);
-        load_tile<B_MN>(smem_u32(sB + s * b_stage), a.B, a.ldb, bn, n0, a.n_valid, k0, k_end);
+    bool ld_ok = true;
+    auto issue_load = [&](uint32_t it) {
+        const int s = (int)(it % STAGES);
+        const int64_t k0 = ld.k_begin + (int64_t)ld.kb * BK;
+        load_tile<A_MN>(smem_u32(sA + s * A_STAGE), a.A, a.lda, BM, ld.m0, m_valid, k0, ld.k_end);
+        load_tile<B_MN>(smem_u32(sB + s * b_stage), a.B, a.ldb, bn, ld.n0, a.n_valid, k0, ld.k_end);
+        if (++ld.kb == ld.nkb) ld_ok = unit_at<MODE>(ld, ld.u + gridDim.x, a, rows, nt, splits);
     };
-
-    // ---- main loop: loads of stage kb+1 overlap the MMAs of stage kb
+    uint32_t it_ld = 0, it_cm = 0;
     for (int s = 0; s < STAGES - 1; ++s) {
-        if (s < nkb) load_stage(s);
+        if (ld_ok) issue_load(it_ld++);
         asm volatile("cp.async.commit_group;\n" ::: "memory");
     }
-    for (int kb = 0; kb < nkb; ++kb) {
-        const int pf = kb + STAGES - 1;
-        if (pf < nkb) {
-            if (kb >= 1) mbar_wait(smem_u32(mbar + (kb - 1) % STAGES), ((kb - 1) / STAGES) & 1);  // MMAs of kb-1 done
-            load_stage(pf);
+    for (;;) {
+        if (ld_ok) {
+            if (it_ld >= STAGES)   // the stage's previous occupant (item it_ld - STAGES) was multiplied
+                mbar_wait(smem_u32(mbar + it_ld % STAGES), ((it_ld / STAGES) - 1) & 1);
+            issue_load(it_ld++);
         }
         asm volatile("cp.async.commit_group;\n" ::: "memory");
-        asm volatile("cp.async.wait_group %0;\n" ::"n"(STAGES - 1) : "memory");
-        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");   // generic-proxy writes -> tensor core
+        asm volatile("cp.async.wait_group %0;\n" ::"n"(STAGES - 1) : "memory");   // item it_cm landed
+        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");            // generic writes -> tensor core
         __syncthreads();
+        const int s = (int)(it_cm % STAGES);
         if (threadIdx.x == 0) {
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-            const int s = kb % STAGES;
             const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
 #pragma unroll
             for (int ks = 0; ks < BK / 16; ++ks) {
                 const uint64_t ad = smem_desc(a0 + ks * 256), bd = smem_desc(b0 + ks * 256);
-                const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
+                const uint32_t acc = (cm.kb > 0 || ks > 0) ? 1u : 0u;
                 asm volatile(
                     "{\n\t.reg .pred p;\n\t"
                     "setp.ne.b32 p, %4, 0;\n\t"
@@ -201,92 +281,50 @@ __global__ void __launch_bounds__(128) k_umma_gemm(Args a) {
                              smem_u32(mbar + s))
                          : "memory");
         }
-    }
-    mbar_wait(smem_u32(mbar + (nkb - 1) % STAGES), ((nkb - 1) / STAGES) & 1);
-    asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-
-    // ---- epilogue: warp w reads TMEM lanes 32w.. (= tile rows), 16 columns per load
-    const int64_t row = m0 + warp * 32 + lane;
-    const bool row_ok = row < m_valid;
-    for (int c0 = 0; c0 < bn; c0 += 16) {
-        uint32_t r[16];
-        const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
-        asm volatile(
-            "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];\n"
-            : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
-              "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15])
-            : "r"(taddr));
-        asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
-        const int64_t cg = n0 + c0;
-        if (!row_ok || cg >= a.n_store) continue;
-        float v[16];
-#pragma unroll
-        for (int j = 0; j < 16; ++j) v[j] = __uint_as_float(r[j]);
-        const bool full = cg + 16 <= a.n_store && (a.ldc & 3) == 0;
-        if (MODE == DW) {
-            float* dst = a.C + row * a.ldc + cg;
-            if (full) {
-#pragma unroll
-                for (int j = 0; j < 16; j += 4) atomicAdd((float4*)(dst + j), make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]));
-            } else {
-                for (int j = 0; j < 16 && cg + j < a.n_store; ++j) atomicAdd(dst + j, v[j]);
-            }
-        } else {
-            if (a.bias) {
-#pragma unroll
-                for (int j = 0; j < 16; ++j) v[j] += cg + j < a.n_store ? __ldg(a.bias + cg + j) : 0.f;
-            }
-            float* dst = a.C + row * a.ldc + cg;
-            float* hdst = a.H ? a.H + row * a.ldc + cg : nullptr;
-            if (full) {
-#pragma unroll
-                for (int j = 0; j < 16; j += 4) {
-                    *(float4*)(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
-                    if (hdst)
-                        *(float4*)(hdst + j) = make_float4(fmaxf(v[j], 0.f), fmaxf(v[j + 1], 0.f), fmaxf(v[j + 2], 0.f),
-                                                           fmaxf(v[j + 3], 0.f));
-                }
-            } else {
-                for (int j = 0; j < 16 && cg + j < a.n_store; ++j) {
-                    dst[j] = v[j];
-                    if (hdst) hdst[j] = fmaxf(v[j], 0.f);
-                }
-            }
+        if (cm.kb == cm.nkb - 1) {
+            mbar_wait(smem_u32(mbar + s), (it_cm / STAGES) & 1);   // the unit's accumulator is complete
+            asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+            epilogue<MODE>(a, tmem, stage_out + warp * (32 * 33), cm.m0 + warp * 32, cm.n0, m_valid, bn, warp, lane);
+            asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
         }
+        ++it_cm;
+        if (++cm.kb == cm.nkb && !unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
     }
-    asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
     __syncthreads();
     if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(ncols));
 }
 
-inline int smem_bytes(int bn) { return STAGES * (A_STAGE + bn * BK * 2) + 64; }
+inline int smem_bytes(int bn) { return STAGES * (A_STAGE + bn * BK * 2) + 4 * 32 * 33 * 4 + 64; }
 
 // Host launcher.  rows_max: host bound of *rows_dev (grid sizing).  n_total: output columns
-// to cover (FWD/DA: n_store rounded up; DW: n_store).  splits: DW reduction CTAs per tile.
+// (split into <= 256-wide tiles).  splits: DW reduction slices per tile.
 inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_total, int splits, cudaStream_t st) {
     Args a = a0;
-    const int nt = (n_total + 255) / 256;                        // N tiles of <= 256 columns
+    const int nt = (n_total + 255) / 256;
     int bn = (n_total + nt - 1) / nt;
     bn = (bn + 15) / 16 * 16;
     a.bn = bn;
+    if (splits < 1) splits = 1;
     const int smem = smem_bytes(bn);
-    dim3 grid;
-    if (mode == DW) grid = dim3((unsigned)((a.m_valid + BM - 1) / BM), (unsigned)nt, (unsigned)(splits < 1 ? 1 : splits));
-    else grid = dim3((unsigned)((rows_max + BM - 1) / BM), (unsigned)nt, 1);
-    if (grid.x == 0) return cudaSuccess;
+    int ncols = 32;
+    while (ncols < bn) ncols <<= 1;
+    const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / ncols));
+    const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
+    if (units <= 0) return cudaSuccess;
+    const unsigned grid = (unsigned)std::min<int64_t>(units, (int64_t)148 * per_sm);
     cudaError_t e = cudaSuccess;
     switch (mode) {
         case FWD:
             e = cudaFuncSetAttribute(k_umma_gemm<FWD>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<FWD><<<grid, 128, smem, st>>>(a);
+            if (e == cudaSuccess) k_umma_gemm<FWD><<<grid, 128, smem, st>>>(a, nt, splits);
             break;
         case DA:
             e = cudaFuncSetAttribute(k_umma_gemm<DA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<DA><<<grid, 128, smem, st>>>(a);
+            if (e == cudaSuccess) k_umma_gemm<DA><<<grid, 128, smem, st>>>(a, nt, splits);
             break;
         default:
             e = cudaFuncSetAttribute(k_umma_gemm<DW>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<DW><<<grid, 128, smem, st>>>(a);
+            if (e == cudaSuccess) k_umma_gemm<DW><<<grid, 128, smem, st>>>(a, nt, splits);
             break;
     }
     return e != cudaSuccess ? e : cudaGetLastError();

@@ -14,7 +14,7 @@ import torch
 
 from ._lib import check, lib
 
-GD_SAGE_W, GD_SAGE_B, GD_SAGE_DW, GD_SAGE_DB, GD_SAGE_A16, GD_SAGE_Z = range(6)
+GD_SAGE_W, GD_SAGE_B, GD_SAGE_DW, GD_SAGE_DB, GD_SAGE_A16, GD_SAGE_Z, GD_SAGE_H = range(7)
 
 
 def _stream_ptr(stream, device):
@@ -96,8 +96,8 @@ class SageModel:
 
     def get_activation(self, what: int, layer: int, n_dst_max: int) -> np.ndarray:
         di, do = self.dims[layer], self.dims[layer + 1]
-        if what == GD_SAGE_A16:     # bf16 -> float32 (bf16 is the top half of an fp32)
-            raw = np.zeros((n_dst_max, 2 * di), dtype=np.uint16)
+        if what in (GD_SAGE_A16, GD_SAGE_H):     # bf16 -> float32 (bf16 is the top half of an fp32)
+            raw = np.zeros((n_dst_max, 2 * di if what == GD_SAGE_A16 else do), dtype=np.uint16)
             check(lib.gd_sage_get(self._h, what, layer, raw.ctypes.data_as(ctypes.c_void_p), raw.nbytes))
             return (raw.astype(np.uint32) << 16).view(np.float32)
         a = np.zeros((n_dst_max, do), dtype=np.float32)

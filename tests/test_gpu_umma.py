@@ -28,10 +28,11 @@ def vp(t):
 
 
 def run(lib, mode, A, lda, B, ldb, C, ldc, rows, rows_max, m_valid, k_valid, n_valid, n_store, splits=1,
-        H=None, bias=None):
+        relu=0, bias=None):
     rows_dev = torch.tensor([rows], dtype=torch.int64, device="cuda")
-    lib.check(lib.lib.gd_debug_umma_gemm(mode, vp(A), lda, vp(B), ldb, vp(C), ldc, vp(H), vp(bias), vp(rows_dev),
-                                         rows_max, m_valid, k_valid, n_valid, n_store, splits,
+    c_bf16 = int(C.dtype == torch.bfloat16)
+    lib.check(lib.lib.gd_debug_umma_gemm(mode, vp(A), lda, vp(B), ldb, vp(C), ldc, c_bf16, relu, vp(bias),
+                                         vp(rows_dev), rows_max, m_valid, k_valid, n_valid, n_store, splits,
                                          ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)))
     torch.cuda.synchronize()
 
@@ -55,13 +56,17 @@ def test_fwd(lib, rows, rows_max, K, N):
     W[:, :N] = bf((K, N), g)
     bias = torch.randn(N, generator=g).cuda()
     C = torch.full((rows_max, Np), 7.0, device="cuda")
-    H = torch.full((rows_max, Np), 7.0, device="cuda")
-    run(lib, 0, A, K, W, Np, C, Np, rows, rows_max, 0, K, Np, N, H=H, bias=bias)
+    H = torch.full((rows_max, Np), 7.0, device="cuda", dtype=torch.bfloat16)
+    run(lib, 0, A, K, W, Np, C, Np, rows, rows_max, 0, K, Np, N, bias=bias)
+    run(lib, 0, A, K, W, Np, H, Np, rows, rows_max, 0, K, Np, N, relu=1, bias=bias)
     Af, Wf = A[:rows].float(), W[:, :N].float()
     ref = Af @ Wf + bias
-    close(C[:rows, :N], ref, Af.abs() @ Wf.abs())
-    close(H[:rows, :N], ref.clamp_min(0), Af.abs() @ Wf.abs())
+    mag = Af.abs() @ Wf.abs() + bias.abs()
+    close(C[:rows, :N], ref, mag)
+    # bf16 output: one more rounding of the result (unit roundoff 2^-8 relative)
+    close(H[:rows, :N].float(), ref.clamp_min(0), mag + 2.0 ** 6 * ref.abs(), tol=2.0 ** -14)
     assert bool((C[rows:] == 7.0).all()) and bool((C[:, N:] == 7.0).all())   # nothing past the device count / n_store
+    assert bool((H[rows:].float() == 7.0).all())
 
 
 @pytest.mark.parametrize("rows,rows_max,K,N", [(1000, 1100, 256, 512), (300, 300, 48, 200), (129, 256, 256, 256)])

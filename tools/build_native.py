@@ -58,10 +58,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         if verbose and out:
             print(out)
     tmp = LIB + ".tmp"
-    # cuBLAS (f4's plain GEMMs) is linked dynamically: torch has usually loaded its own
-    # libcublas.so.12 already, which then satisfies this SONAME; the rpath is the fallback.
-    subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-o", tmp, *objs,
-                           "-L/usr/local/cuda/lib64", "-lcublas", "-Xlinker", "-rpath=/usr/local/cuda/lib64"])
+    subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", "-Xcompiler", "-fPIC", "-o", tmp, *objs])
     os.replace(tmp, LIB)
     return LIB
 
