@@ -576,12 +576,13 @@ def run_ours(args, rank, world, local_rank):
         L = model.L
         flop = 0
         for j in range(L):
-            nd, din, dout = nm[L - 1 - j], model.dims[j], model.dims[j + 1]
+            nd, din, dout = sz[L - 1 - j], model.dims[j], model.dims[j + 1]   # mean actual dst rows
             flop += 2 * nd * 2 * din * dout * (2 if j == 0 else 3)   # fwd + dW (+ dA above layer 0)
         ll = loss_log[off + W:off + W + K].cpu().tolist()
         train_info = {"model": f"GraphSAGE mean, widths {model.dims} (P:173)", "lr": args.lr,
                       "train_ms_per_batch": round(t_ms, 4),
-                      "gemm_gflop_per_batch_at_bounds": round(flop / 1e9, 2),
+                      "gemm": "hand-written tcgen05 (gd_umma.cuh) over the device-resident row counts",
+                      "gemm_gflop_per_batch": round(flop / 1e9, 2),
                       "gemm_tflops_if_train_ms_were_gemm": round(flop / (t_ms * 1e9), 1) if t_ms > 0 else None,
                       "loss_first": round(ll[0], 4), "loss_last": round(ll[-1], 4),
                       "allreduce": "NCCL all_reduce of the flat fp32 gradients (P:140)" if world > 1 else "none (N=1)"}

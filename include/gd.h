@@ -315,7 +315,8 @@ gd_status gd_sage_get(gd_sage* s, int32_t what, int32_t layer, void* host_out, i
  *   (multiple of 8), zero beyond.
  *   mode 2 DW   C[m, n] += sum_{i < *rows_dev} A[i*lda + m] B[i*ldb + n] for m < m_valid
  *   (multiple of 8), n < n_store, C fp32, the reduction split over `splits` CTAs per tile
- *   (fp32 red.add into C: the caller zeroes it).
+ *   (fp32 red.add into C: the caller zeroes it); rows [*rows_dev, round_up(*rows_dev, 64))
+ *   of A and B (below rows_max) must be zero (64-row blocks are reduced whole).
  * Row strides are multiples of 8 elements, base pointers 16-byte aligned (GD_ERR_INVALID). */
 gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const void* B, int64_t ldb,
                              void* C, int64_t ldc, int32_t c_bf16, int32_t relu, const float* bias,

@@ -62,6 +62,13 @@ struct gd_sage {
 namespace gd {
 
 // ------------------------------------------------------------------ kernels
+// rows [n, round_up(n, 64)) of the GEMM operands A16 / dZ16 are zeroed by their producers
+// (gd_umma.cuh: the DW GEMM reduces over whole 64-row blocks)
+__device__ __forceinline__ int64_t pad64(int64_t n, int64_t n_alloc) {
+    const int64_t p = (n + 63) / 64 * 64;
+    return p < n_alloc ? p : n_alloc;
+}
+
 // a_i = [x_i | mean x_col] for i < n_dst (x fp32 features or bf16 activations, rows at stride ldx).  Warp per row; each lane
 // owns 4-column groups (float4) g = lane, lane + 32, ...; neighbour ids are loaded 32 at a
 // time and broadcast with shuffles, 4 neighbour rows in flight per lane.
@@ -75,13 +82,19 @@ __device__ __forceinline__ float4 load4(const __nv_bfloat16* __restrict__ row, i
 template <typename T>
 __global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64_t ldx, int din,
                                                   const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
-                                                  const int64_t* __restrict__ n_dst_p, __nv_bfloat16* __restrict__ A16) {
+                                                  const int64_t* __restrict__ n_dst_p, int64_t n_alloc,
+                                                  __nv_bfloat16* __restrict__ A16) {
     const int lane = threadIdx.x & 31;
     const int64_t n_dst = *n_dst_p;
+    const int64_t n_end = pad64(n_dst, n_alloc);
     const int groups = din >> 2;
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_dst; i += warps) {
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
         __nv_bfloat162* arow = (__nv_bfloat162*)(A16 + i * 2 * din);
+        if (i >= n_dst) {   // zero pad rows up to a multiple of 64 (the DW GEMM reduces whole 64-row blocks)
+            for (int c = lane; c < din; c += 32) arow[c] = __floats2bfloat162_rn(0.f, 0.f);
+            continue;
+        }
         const int64_t lo = rowptr[i], hi = rowptr[i + 1];
         const float inv = hi > lo ? 1.0f / (float)(hi - lo) : 0.0f;
         for (int g0 = 0; g0 < groups; g0 += 64) {          // up to 2 float4 per lane per pass
@@ -146,14 +159,19 @@ __global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64
 // per seed row: loss_rows[i] = lse - z[label]; dZ16[i] = (softmax - onehot) / n0 for the C
 // classes, 0 in the pad columns [C, dp).
 __global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, int dp, const int32_t* __restrict__ labels,
-                                              const int64_t* __restrict__ n_p, __nv_bfloat16* __restrict__ dZ16,
-                                              float* __restrict__ loss_rows) {
+                                              const int64_t* __restrict__ n_p, int64_t n_alloc,
+                                              __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows) {
     const int lane = threadIdx.x & 31;
     const int64_t n = *n_p;
+    const int64_t n_end = pad64(n, n_alloc);
     const int64_t warps = (int64_t)gridDim.x * (blockDim.x >> 5);
-    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n; i += warps) {
+    for (int64_t i = (int64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); i < n_end; i += warps) {
         const float* z = Z + i * dp;
         __nv_bfloat16* dz = dZ16 + i * dp;
+        if (i >= n) {
+            for (int c = lane; c < dp; c += 32) dz[c] = __float2bfloat16_rn(0.f);
+            continue;
+        }
         float m = -INFINITY;
         for (int c = lane; c < C; c += 32) m = fmaxf(m, z[c]);
         for (int o = 16; o; o >>= 1) m = fmaxf(m, __shfl_xor_sync(0xffffffffu, m, o));
@@ -232,13 +250,20 @@ __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ 
 // columns stay zero).  Block (32, 8): threadIdx.x walks a row's float4 columns, threadIdx.y
 // rows; no index division.
 __global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX, const __nv_bfloat16* __restrict__ H16, int d, int dp,
-                                                   const int64_t* __restrict__ n_p, __nv_bfloat16* __restrict__ dZ16) {
+                                                   const int64_t* __restrict__ n_p, int64_t n_alloc,
+                                                   __nv_bfloat16* __restrict__ dZ16) {
     const int64_t n = *n_p;
+    const int64_t n_end = pad64(n, n_alloc);
     const int dv = d >> 2;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n; i += (int64_t)gridDim.x * blockDim.y) {
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n_end; i += (int64_t)gridDim.x * blockDim.y) {
         const float4* x4 = (const float4*)(dX + i * d);
         const __nv_bfloat16* hrow = H16 + i * dp;
         __nv_bfloat162* o2 = (__nv_bfloat162*)(dZ16 + i * dp);
+        if (i >= n) {
+            for (int c = threadIdx.x; c < dv; c += blockDim.x)
+                o2[2 * c] = o2[2 * c + 1] = __floats2bfloat162_rn(0.f, 0.f);
+            continue;
+        }
         for (int c = threadIdx.x; c < dv; c += blockDim.x) {
             const float4 x = x4[c], h = load4(hrow, c);
             o2[2 * c] = __floats2bfloat162_rn(h.x > 0.f ? x.x : 0.f, h.y > 0.f ? x.y : 0.f);
@@ -448,10 +473,11 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         const int64_t* n_dst = sizes + (h - 1);
         if (j == 0)
             k_sage_agg<float><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const float*)x, ldx, l.din, rowptr[h - 1],
-                                                                          col[h - 1], n_dst, l.A16);
+                                                                          col[h - 1], n_dst, l.n_dst_max, l.A16);
         else
             k_sage_agg<__nv_bfloat16><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const __nv_bfloat16*)x, ldx, l.din,
-                                                                                  rowptr[h - 1], col[h - 1], n_dst, l.A16);
+                                                                                  rowptr[h - 1], col[h - 1], n_dst,
+                                                                                  l.n_dst_max, l.A16);
         GD_DEBUG_AFTER("k_sage_agg", st);
         const bool hidden = j < L - 1;   // hidden: h = relu(z + b) in bf16 (the next layer's input); top: logits
         umma::Args a = gemm_args(l.A16, 2 * l.din, s->W16 + l.w16_off, l.dp, hidden ? (void*)l.H16 : (void*)l.Z, l.dp, n_dst);
@@ -468,7 +494,8 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
     }
     // ---- loss
     SageLayer& top = s->layers[L - 1];
-    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, top.dp, labels, sizes, top.dZ16, s->loss_rows);
+    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, top.dp, labels, sizes, top.n_dst_max, top.dZ16,
+                                                         s->loss_rows);
     k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
     GD_DEBUG_AFTER("k_xent", st);
     // ---- backward
@@ -506,7 +533,7 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         GD_DEBUG_AFTER("k_sage_scatter", st);
         SageLayer& prev = s->layers[j - 1];   // its output (H16) is this layer's input
         k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H16, prev.dout, prev.dp, sizes + h,
-                                                                       prev.dZ16);
+                                                                       prev.n_dst_max, prev.dZ16);
         GD_DEBUG_AFTER("k_relu_grad", st);
     }
     GD_CUDA(cudaGetLastError());

@@ -1,31 +1,42 @@
-// gd_umma.cuh — hand-written sm_100a tensor-core GEMM (tcgen05.mma, accumulator in TMEM) for
-// the f4 train stage.  The three GEMMs of a GraphSAGE layer are
-//   FWD  Z[i, n]  = sum_k A16[i, k] W16[k, n] (+ b[n]; H = relu(Z))    i < n_dst (device count)
-//   DA   dA[i, n] = sum_k dZ16[i, k] W16[n, k]                          i < n_dst
-//   DW   dW[m, n] += sum_i A16[i, m] dZ16[i, n]                         i < n_dst, split over i
-// all with bf16 operands and fp32 accumulation.  The row count lives in device memory (it is
-// the sampled block size), so tiles past it exit before touching memory: unlike a library
-// GEMM run at the host-side bound, no padded rows are read, multiplied or written.
+// gd_umma.cuh — hand-written sm_100a tensor-core GEMM (TMA -> shared memory -> tcgen05.mma,
+// accumulator in TMEM) for the f4 train stage.  The three GEMMs of a GraphSAGE layer:
+//   FWD  H[i, n]  = f(sum_k A16[i, k] W16[k, n] + b[n])   f = relu (hidden, bf16 out) or id (logits)
+//   DA   dA[i, n] = sum_k dZ16[i, k] W16[n, k]
+//   DW   dW[m, n] += sum_i A16[i, m] dZ16[i, n]           (split over i, fp32 red.add)
+// for i < n_dst, all with bf16 operands and fp32 accumulation.  The row count n_dst lives in
+// device memory (it is the sampled block size), so work past it is skipped on the device:
+// unlike a library GEMM run at the host-side bound, no padded rows are multiplied or written.
 //
-// Tile: UMMA M = 128 rows (one TMEM lane per output row), N = BN <= 256 columns (TMEM columns),
-// K = 64 per pipeline stage (4 MMAs of K = 16).  CTAs are persistent over the tiles.  The 128
-// threads of a CTA stage operands with cp.async (16-byte chunks, zero-filled past the valid
-// range) into the no-swizzle canonical UMMA layouts, 4 stages deep and across tile
-// boundaries; thread 0 issues the MMAs and tcgen05.commit's them to the stage's mbarrier,
-// which releases the stage for the next load.  The epilogue reads the
-// accumulator with tcgen05.ld (warp w owns TMEM lanes 32w..32w+31 = rows, 32 columns per
-// load), adds the bias and applies relu (FWD), transposes the 32 x 32 block through shared
-// memory (the drained stage buffers) and writes whole rows per instruction: fp32 or bf16
-// stores, or fp32 red.add of the split-K partial (DW).
+// Tile: UMMA M = 128 rows (one TMEM lane per output row), N = bn <= 256 columns (TMEM
+// columns), K = 64 per pipeline stage (4 MMAs of K = 16).  CTAs are persistent over the tiles
+// ("units"; DW units are (tile, row slice) pairs) and warp-specialised (288 threads):
+//   warp 0, lane 0: producer + MMA issuer.  It keeps STAGES-1 k-blocks of TMA loads in flight
+//     ahead of the MMAs, across unit boundaries (TMA completes a stage's "full" mbarrier with
+//     its byte count; the tcgen05.commit of the MMAs that read a stage arrives on its "empty"
+//     mbarrier, which lets the stage be refilled), and accumulates unit u into TMEM buffer
+//     u % 2, committing the unit's last k-block to acc_full[u % 2].
+//   warps 1-8: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per thread)
+//     of the finished buffer, alternate 32-column chunks per warp pair (tcgen05.ld, 32
+//     columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
+//     (fp32 / bf16 stores, or fp32 vector red.add for DW), then arrives on acc_empty[u % 2].
+//     The next unit's MMAs run meanwhile in the other buffer.
 //
-// Shared-memory image of one operand tile (R rows of the M/N dimension x 64 of K), both majors:
-//   K-major  (row-major global, K contiguous):  byte(r, k8) = (r / 8) * 1024 + k8 * 128 + (r % 8) * 16
-//   MN-major (M/N contiguous):                 byte(r8, k) = r8 * 1024 + (k / 8) * 128 + (k % 8) * 16
-// i.e. 8 x 16-byte core matrices, K-adjacent ones 128 B apart (LBO), M/N-adjacent 8-groups
-// 1024 B apart (SBO); one MMA (K = 16) covers two K groups, so the k-th MMA of a stage starts
-// 256 B further.
+// Operand tiles use the 128-byte-swizzled canonical UMMA layouts that TMA writes directly
+// (SWIZZLE_128B, tile bases 1024-byte aligned):
+//   K-major  (K contiguous in global):  box {64 (K), R rows}: row r at r * 128 B, 8-row groups
+//            1024 B apart (SBO); the k-th MMA (K = 16) of a stage starts 32 B further.
+//   MN-major (M/N contiguous in global): boxes {64 (M/N), 64 (K)}: K-row k at k * 128 B, 8-row
+//            K groups 1024 B apart (SBO), 64-wide M/N blocks 8 KB apart (LBO); the k-th MMA
+//            starts 2048 B further.
+// Out-of-bounds box elements (past the tensor extents) are zero-filled by TMA.  Rows between
+// the device count and the host bound hold stale data: FWD / DA never store those rows, and
+// DW (which reduces over rows) requires the producers of A16 / dZ16 to zero rows
+// [n, round_up(n, 64)) (k_sage_agg, k_xent and k_relu_grad do).
 #pragma once
+#include <cuda.h>
+#include <cudaTypedefs.h>
 #include <cuda_bf16.h>
+#include <cuda_runtime.h>
 #include <stdint.h>
 
 #include <algorithm>
@@ -50,16 +61,12 @@ struct Args {
     const int64_t* rows_dev;     // device row count: M (FWD, DA) or the reduction length (DW)
     int64_t m_valid;             // DW: output rows (A's contiguous width); FWD/DA: unused
     int k_valid;                 // FWD/DA: reduction length (multiple of 8)
-    int n_valid;                 // B's valid extent along N (multiple of 8; zero-filled past it)
+    int n_valid;                 // B's extent along N (multiple of 8; zero-filled past it)
     int n_store;                 // output columns written
-    int bn;                      // N tile (multiple of 16, <= 256)
+    int bn;                      // N tile (multiple of 16, <= 256; multiple of 64 when B is MN-major)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
-
-__device__ __forceinline__ void cp_async16(uint32_t dst, const void* src, bool valid) {
-    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(dst), "l"(src), "r"(valid ? 16 : 0) : "memory");
-}
 
 __device__ __forceinline__ void mbar_wait(uint32_t addr, uint32_t parity) {
     asm volatile(
@@ -71,13 +78,17 @@ __device__ __forceinline__ void mbar_wait(uint32_t addr, uint32_t parity) {
         : "memory");
 }
 
-__device__ __forceinline__ uint64_t smem_desc(uint32_t addr) {
-    uint64_t d = 0;
-    d |= (uint64_t)((addr >> 4) & 0x3FFF);            // start address
-    d |= (uint64_t)(128 >> 4) << 16;                   // LBO: K-adjacent core matrices
-    d |= (uint64_t)(1024 >> 4) << 32;                  // SBO: M/N-adjacent 8-row groups
-    d |= (uint64_t)1 << 46;                            // descriptor version (sm_100)
-    return d;                                          // base offset 0, layout SWIZZLE_NONE
+__device__ __forceinline__ void tma2d(uint32_t dst, const CUtensorMap* map, int32_t c0, int32_t c1, uint32_t bar) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];\n" ::"r"(dst),
+        "l"((uint64_t)map), "r"(c0), "r"(c1), "r"(bar)
+        : "memory");
+}
+
+// UMMA shared-memory descriptor, SWIZZLE_128B (layout type 2), version 1 (sm_100).
+__device__ __forceinline__ uint64_t smem_desc_sw128(uint32_t addr, uint32_t lbo, uint32_t sbo) {
+    return (uint64_t)((addr >> 4) & 0x3FFF) | ((uint64_t)((lbo >> 4) & 0x3FFF) << 16) |
+           ((uint64_t)((sbo >> 4) & 0x3FFF) << 32) | ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
 }
 
 template <bool A_MN, bool B_MN>
@@ -89,46 +100,18 @@ __host__ __device__ constexpr uint32_t instr_desc(int bn) {
            | ((uint32_t)(BM >> 4) << 24); // M / 16
 }
 
-// Stage one operand tile (R rows along M/N starting at r0, BK along K starting at k0).  Chunks
-// are assigned so that every 8 consecutive lanes write 8 distinct 16-byte bank slots (the low
-// 7 address bits are (r % 8) * 16, resp. (k % 8) * 16: conflict-free cp.async writes) while
-// each warp still reads whole 32-byte sectors of global memory:
-//   K-major:  idx = (r / 8) * 64 + k8 * 8 + r % 8            (8 rows x 4 chunks of 16 B per warp)
-//   MN-major: idx = (r8 / 2) * 128 + (k / 8) * 16 + (r8 % 2) * 8 + k % 8
-//                                                          (8 K-rows x 2 adjacent chunks per 16 lanes)
-template <bool MN_MAJOR>
-__device__ __forceinline__ void load_tile(uint32_t s, const __nv_bfloat16* __restrict__ g, int64_t ld, int R, int64_t r0,
-                                          int64_t r_valid, int64_t k0, int64_t k_end) {
-    const int total = R * 8;   // 16-byte chunks in an R x 64 bf16 tile
-    for (int idx = threadIdx.x; idx < total; idx += blockDim.x) {
-        int r, k;              // K-major: row r, chunk k (of 8 elements); MN-major: 8-group r, K-row k
-        uint32_t off;
-        if (!MN_MAJOR) {
-            r = ((idx >> 6) << 3) + (idx & 7);
-            k = (idx >> 3) & 7;
-            off = (uint32_t)idx * 16;   // (r / 8) * 1024 + k * 128 + (r % 8) * 16
-        } else {
-            r = ((idx >> 7) << 1) | ((idx >> 3) & 1);
-            k = (((idx >> 4) & 7) << 3) + (idx & 7);
-            off = (uint32_t)(r * 1024 + (k >> 3) * 128 + (k & 7) * 16);
-        }
-        const int64_t gr = r0 + (MN_MAJOR ? r * 8 : r), gk = k0 + (MN_MAJOR ? k : k * 8);
-        const bool v = gr < r_valid && gk < k_end;
-        cp_async16(s + off, v ? (MN_MAJOR ? g + gk * ld + gr : g + gr * ld + gk) : g, v);
-    }
-}
-
-// Epilogue of one unit: warp w reads TMEM lanes 32w.. (= tile rows rbase..rbase+31), 32
-// columns per load (bn is a multiple of 16 and the allocation a power of two >= 32, so a load
-// past bn stays inside it; those columns are not stored), transposes the 32 x 32 block
-// through its 4 KB of shared memory and writes (or red.adds) one 32-column row segment per
-// instruction.
-template <int MODE>
-__device__ __forceinline__ void epilogue(const Args& a, uint32_t tmem, float* st, int64_t rbase, int64_t n0, int64_t m_valid,
-                                         int bn, int warp, int lane) {
-    for (int c0 = 0; c0 < bn; c0 += 32) {
+// Epilogue of one unit for one epilogue warp: TMEM lanes 32q.. (q = CTA warp % 4, the
+// tcgen05.ld lane rule) are tile rows rbase..rbase+31, one row per thread; the warp takes the
+// 32-column chunks c0 = 32 h, 32 h + 64, ... (h = which of the two warps of the quarter).  A
+// thread holds 32 consecutive columns of its row after one tcgen05.ld and writes them as
+// 16-byte vectors (bf16: 4 stores, fp32: 8) or vector red.adds (DW), scalar at a ragged edge.
+template <int MODE, bool OUT_BF16, bool RELU>
+__device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t rbase, int64_t n0, int64_t m_valid, int bn,
+                                         int h, int lane, bool vec_ok) {
+    const int64_t row = rbase + lane;
+    const bool row_ok = row < m_valid;
+    for (int c0 = 32 * h; c0 < bn; c0 += 64) {
         uint32_t r[32];
-        const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16) + (uint32_t)c0;
         asm volatile(
             "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
             "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];\n"
@@ -136,29 +119,51 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tmem, float* st
               "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]),
               "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]),
               "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
-            : "r"(taddr));
+            : "r"(tacc + (uint32_t)c0));
         asm volatile("tcgen05.wait::ld.sync.aligned;\n" ::: "memory");
+        const int64_t cg = n0 + c0;
+        if (!row_ok || cg >= a.n_store) continue;
+        float v[32];
 #pragma unroll
-        for (int j = 0; j < 32; ++j) st[lane * 33 + j] = __uint_as_float(r[j]);
-        __syncwarp();
-        const int64_t cg = n0 + c0 + lane;              // this lane's output column
-        const bool col_ok = c0 + lane < bn && cg < a.n_store;
-        const float b = (MODE == FWD && a.bias && col_ok) ? __ldg(a.bias + cg) : 0.f;
-        for (int rr = 0; rr < 32; ++rr) {
-            const int64_t row = rbase + rr;
-            if (row >= m_valid) break;
-            float v = st[rr * 33 + lane];
-            if (!col_ok) continue;
-            if (MODE == DW) {
-                atomicAdd((float*)a.C + row * a.ldc + cg, v);
-            } else {
-                v += b;
-                if (MODE == FWD && a.relu) v = fmaxf(v, 0.f);
-                if (a.c_bf16) ((__nv_bfloat16*)a.C)[row * a.ldc + cg] = __float2bfloat16_rn(v);
-                else ((float*)a.C)[row * a.ldc + cg] = v;
+        for (int j = 0; j < 32; ++j) {
+            v[j] = __uint_as_float(r[j]);
+            if (MODE == FWD) {
+                if (a.bias) v[j] += cg + j < a.n_store ? __ldg(a.bias + cg + j) : 0.f;
+                if (RELU) v[j] = fmaxf(v[j], 0.f);
             }
         }
-        __syncwarp();
+        const bool full = vec_ok && cg + 32 <= a.n_store;
+        if (MODE == DW) {
+            float* dst = (float*)a.C + row * a.ldc + cg;
+            if (full) {
+#pragma unroll
+                for (int j = 0; j < 32; j += 4) atomicAdd((float4*)(dst + j), make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]));
+            } else {
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) atomicAdd(dst + j, v[j]);
+            }
+        } else if (OUT_BF16) {
+            __nv_bfloat16* dst = (__nv_bfloat16*)a.C + row * a.ldc + cg;
+            if (full) {
+#pragma unroll
+                for (int j = 0; j < 32; j += 8) {
+                    uint4 w;
+                    __nv_bfloat162 p0 = __floats2bfloat162_rn(v[j], v[j + 1]), p1 = __floats2bfloat162_rn(v[j + 2], v[j + 3]);
+                    __nv_bfloat162 p2 = __floats2bfloat162_rn(v[j + 4], v[j + 5]), p3 = __floats2bfloat162_rn(v[j + 6], v[j + 7]);
+                    w.x = *(uint32_t*)&p0; w.y = *(uint32_t*)&p1; w.z = *(uint32_t*)&p2; w.w = *(uint32_t*)&p3;
+                    *(uint4*)(dst + j) = w;
+                }
+            } else {
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = __float2bfloat16_rn(v[j]);
+            }
+        } else {
+            float* dst = (float*)a.C + row * a.ldc + cg;
+            if (full) {
+#pragma unroll
+                for (int j = 0; j < 32; j += 4) *(float4*)(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
+            } else {
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = v[j];
+            }
+        }
     }
 }
 
@@ -198,135 +203,203 @@ __device__ __forceinline__ bool unit_at(Unit& c, int64_t u, const Args& a, int64
     }
 }
 
-// Persistent CTAs (grid <= resident CTAs); the load cursor runs STAGES-1 k-blocks ahead of the
-// MMA cursor across unit boundaries, so the next unit's operands stream in during a unit's
-// epilogue.
-template <int MODE>
-__global__ void __launch_bounds__(128) k_umma_gemm(Args a, int nt, int splits) {
+template <int MODE, bool OUT_BF16, bool RELU>
+__global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
+                                                   const __grid_constant__ CUtensorMap tmB, Args a, int nt, int splits,
+                                                   int vec_ok) {
     constexpr bool A_MN = MODE == DW;
     constexpr bool B_MN = MODE != DA;
-    extern __shared__ __align__(1024) uint8_t smem[];
+    extern __shared__ uint8_t smem_raw[];
+    // SWIZZLE_128B tiles need 1024-byte aligned bases
+    uint8_t* smem = smem_raw + ((1024 - (smem_u32(smem_raw) & 1023)) & 1023);
     const int bn = a.bn;
     const int b_stage = bn * BK * 2;
     uint8_t* sA = smem;
     uint8_t* sB = smem + STAGES * A_STAGE;
-    float* stage_out = (float*)(sB + STAGES * b_stage);          // 4 warps x 32 x 33 fp32
-    uint64_t* mbar = (uint64_t*)(stage_out + 4 * 32 * 33);
-    uint32_t* tmem_slot = (uint32_t*)(mbar + STAGES);
+    uint64_t* full = (uint64_t*)(sB + STAGES * b_stage);
+    uint64_t* empty = full + STAGES;
+    uint64_t* acc_full = empty + STAGES;                          // [2] accumulator buffer ready
+    uint64_t* acc_empty = acc_full + 2;                           // [2] accumulator buffer drained
+    uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
 
     const int64_t rows = *a.rows_dev;   // device-resident size
-    Unit cm, ld;
+    Unit cm;
     if (!unit_at<MODE>(cm, blockIdx.x, a, rows, nt, splits)) return;
-    ld = cm;
     const int64_t m_valid = MODE == DW ? a.m_valid : rows;
-    uint32_t ncols = 32;
-    while ((int)ncols < bn) ncols <<= 1;
+    uint32_t nc = 32;                   // columns of one accumulator buffer
+    while ((int)nc < bn) nc <<= 1;
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     if (warp == 0) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;\n" ::"r"(smem_u32(tmem_slot)),
-                     "r"(ncols));
+                     "r"(2 * nc));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;\n");
     }
     if (threadIdx.x == 0) {
-        for (int s = 0; s < STAGES; ++s)
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(mbar + s)));
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmA) : "memory");
+        asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmB) : "memory");
+        for (int s = 0; s < 2 * STAGES + 2; ++s)
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(full + s)));
+        for (int s = 0; s < 2; ++s)
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;\n" ::"r"(smem_u32(acc_empty + s)));   // one per epilogue warp
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
     __syncthreads();
     asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
     const uint32_t tmem = *tmem_slot;
-    const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
 
-    bool ld_ok = true;
-    auto issue_load = [&](uint32_t it) {
-        const int s = (int)(it % STAGES);
-        const int64_t k0 = ld.k_begin + (int64_t)ld.kb * BK;
-        load_tile<A_MN>(smem_u32(sA + s * A_STAGE), a.A, a.lda, BM, ld.m0, m_valid, k0, ld.k_end);
-        load_tile<B_MN>(smem_u32(sB + s * b_stage), a.B, a.ldb, bn, ld.n0, a.n_valid, k0, ld.k_end);
-        if (++ld.kb == ld.nkb) ld_ok = unit_at<MODE>(ld, ld.u + gridDim.x, a, rows, nt, splits);
-    };
-    uint32_t it_ld = 0, it_cm = 0;
-    for (int s = 0; s < STAGES - 1; ++s) {
-        if (ld_ok) issue_load(it_ld++);
-        asm volatile("cp.async.commit_group;\n" ::: "memory");
-    }
-    for (;;) {
-        if (ld_ok) {
-            if (it_ld >= STAGES)   // the stage's previous occupant (item it_ld - STAGES) was multiplied
-                mbar_wait(smem_u32(mbar + it_ld % STAGES), ((it_ld / STAGES) - 1) & 1);
-            issue_load(it_ld++);
-        }
-        asm volatile("cp.async.commit_group;\n" ::: "memory");
-        asm volatile("cp.async.wait_group %0;\n" ::"n"(STAGES - 1) : "memory");   // item it_cm landed
-        asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");            // generic writes -> tensor core
-        __syncthreads();
-        const int s = (int)(it_cm % STAGES);
-        if (threadIdx.x == 0) {
-            asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-            const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
+    if (warp == 0) {
+        if (lane == 0) {
+            // ===== producer (TMA) + MMA issuer
+            const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
+            const uint32_t stage_bytes = (uint32_t)(A_STAGE + b_stage);
+            Unit ld = cm;
+            bool ld_ok = true;
+            uint32_t it_ld = 0, it_cm = 0, u_local = 0;
+            auto issue_load = [&]() {
+                const int s = (int)(it_ld % STAGES);
+                if (it_ld >= STAGES) mbar_wait(smem_u32(empty + s), ((it_ld / STAGES) - 1) & 1);   // stage's MMAs done
+                const uint32_t fb = smem_u32(full + s);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(fb), "r"(stage_bytes) : "memory");
+                const int32_t k0 = (int32_t)(ld.k_begin + (int64_t)ld.kb * BK);
+                const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
+                if (!A_MN) tma2d(a0, &tmA, k0, (int32_t)ld.m0, fb);
+                else
+                    for (int j = 0; j < BM / 64; ++j) tma2d(a0 + j * 8192, &tmA, (int32_t)ld.m0 + 64 * j, k0, fb);
+                if (!B_MN) tma2d(b0, &tmB, k0, (int32_t)ld.n0, fb);
+                else
+                    for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
+                ++it_ld;
+                if (++ld.kb == ld.nkb) ld_ok = unit_at<MODE>(ld, ld.u + gridDim.x, a, rows, nt, splits);
+            };
+            for (int s = 0; s < STAGES - 1 && ld_ok; ++s) issue_load();
+            for (;;) {
+                const int s = (int)(it_cm % STAGES);
+                const uint32_t buf = u_local & 1;
+                if (cm.kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
+                    mbar_wait(smem_u32(acc_empty + buf), ((u_local >> 1) - 1) & 1);
+                mbar_wait(smem_u32(full + s), (it_cm / STAGES) & 1);            // operands landed
+                asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+                const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
 #pragma unroll
-            for (int ks = 0; ks < BK / 16; ++ks) {
-                const uint64_t ad = smem_desc(a0 + ks * 256), bd = smem_desc(b0 + ks * 256);
-                const uint32_t acc = (cm.kb > 0 || ks > 0) ? 1u : 0u;
-                asm volatile(
-                    "{\n\t.reg .pred p;\n\t"
-                    "setp.ne.b32 p, %4, 0;\n\t"
-                    "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem),
-                    "l"(ad), "l"(bd), "r"(idesc), "r"(acc)
-                    : "memory");
+                for (int ks = 0; ks < BK / 16; ++ks) {
+                    const uint64_t ad = A_MN ? smem_desc_sw128(a0 + ks * 2048, 8192, 1024) : smem_desc_sw128(a0 + ks * 32, 16, 1024);
+                    const uint64_t bd = B_MN ? smem_desc_sw128(b0 + ks * 2048, 8192, 1024) : smem_desc_sw128(b0 + ks * 32, 16, 1024);
+                    const uint32_t acc = (cm.kb > 0 || ks > 0) ? 1u : 0u;
+                    asm volatile(
+                        "{\n\t.reg .pred p;\n\t"
+                        "setp.ne.b32 p, %4, 0;\n\t"
+                        "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n}\n" ::"r"(tmem + buf * nc),
+                        "l"(ad), "l"(bd), "r"(idesc), "r"(acc)
+                        : "memory");
+                }
+                asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                                 smem_u32(empty + s))
+                             : "memory");
+                const bool last = cm.kb == cm.nkb - 1;
+                if (last)
+                    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
+                                     smem_u32(acc_full + buf))
+                                 : "memory");
+                if (ld_ok) issue_load();   // refill the stage the previous k-block used (MMAs stay queued)
+                ++it_cm;
+                if (last) ++u_local;
+                if (++cm.kb == cm.nkb && !unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
             }
-            asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
-                             smem_u32(mbar + s))
-                         : "memory");
         }
-        if (cm.kb == cm.nkb - 1) {
-            mbar_wait(smem_u32(mbar + s), (it_cm / STAGES) & 1);   // the unit's accumulator is complete
+    } else {
+        // ===== epilogue warps 1..8: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
+        // column half h = (warp - 1) / 4
+        const int q = warp & 3, h = (warp - 1) >> 2;
+        for (uint32_t u_local = 0;; ++u_local) {
+            const uint32_t buf = u_local & 1;
+            mbar_wait(smem_u32(acc_full + buf), (u_local >> 1) & 1);
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-            epilogue<MODE>(a, tmem, stage_out + warp * (32 * 33), cm.m0 + warp * 32, cm.n0, m_valid, bn, warp, lane);
+            epilogue<MODE, OUT_BF16, RELU>(a, tmem + buf * nc + ((uint32_t)(q * 32) << 16), cm.m0 + q * 32, cm.n0, m_valid, bn,
+                                           h, lane, vec_ok != 0);
             asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
+            __syncwarp();
+            if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_empty + buf)) : "memory");
+            if (!unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
         }
-        ++it_cm;
-        if (++cm.kb == cm.nkb && !unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
     }
     __syncthreads();
-    if (warp == 0) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(ncols));
+    if (warp == 0) {
+        asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
+        asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * nc));
+    }
 }
 
-inline int smem_bytes(int bn) { return STAGES * (A_STAGE + bn * BK * 2) + 4 * 32 * 33 * 4 + 64; }
+inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 16; }
 
-// Host launcher.  rows_max: host bound of *rows_dev (grid sizing).  n_total: output columns
-// (split into <= 256-wide tiles).  splits: DW reduction slices per tile.
+// 2-D bf16 tensor map, SWIZZLE_128B, box {64, box_outer}; inner = contiguous extent, outer =
+// rows, ld = row stride in elements.  Out-of-bounds box elements read as zero.
+inline cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t ld, uint32_t box_outer) {
+    static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+    if (!encode) {
+        cudaDriverEntryPointQueryResult q;
+        cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&encode, cudaEnableDefault, &q);
+        if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !encode) return e != cudaSuccess ? e : cudaErrorNotSupported;
+    }
+    const cuuint64_t dims[2] = {inner, outer < 1 ? 1 : outer};
+    const cuuint64_t strides[1] = {ld * 2};
+    const cuuint32_t box[2] = {64, box_outer};
+    const cuuint32_t es[2] = {1, 1};
+    const CUresult r = encode(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS ? cudaSuccess : cudaErrorInvalidValue;
+}
+
+// Host launcher.  rows_max: host bound of *rows_dev (grid sizing, tensor extents).  n_total:
+// output columns (split into <= 256-wide tiles).  splits: DW reduction slices per tile.
 inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_total, int splits, cudaStream_t st) {
     Args a = a0;
+    const bool b_mn = mode != DA;
     const int nt = (n_total + 255) / 256;
     int bn = (n_total + nt - 1) / nt;
-    bn = (bn + 15) / 16 * 16;
+    bn = b_mn ? (bn + 63) / 64 * 64 : (bn + 15) / 16 * 16;
     a.bn = bn;
     if (splits < 1) splits = 1;
+    CUtensorMap tmA, tmB;
+    cudaError_t e;
+    if (mode == FWD) {
+        e = make_map(&tmA, a.A, a.k_valid, rows_max, a.lda, BM);
+        if (e == cudaSuccess) e = make_map(&tmB, a.B, a.n_valid, a.k_valid, a.ldb, 64);
+    } else if (mode == DA) {
+        e = make_map(&tmA, a.A, a.k_valid, rows_max, a.lda, BM);
+        if (e == cudaSuccess) e = make_map(&tmB, a.B, a.k_valid, a.n_valid, a.ldb, bn);
+    } else {
+        e = make_map(&tmA, a.A, a.m_valid, rows_max, a.lda, 64);
+        if (e == cudaSuccess) e = make_map(&tmB, a.B, a.n_valid, rows_max, a.ldb, 64);
+    }
+    if (e != cudaSuccess) return e;
     const int smem = smem_bytes(bn);
     int ncols = 32;
     while (ncols < bn) ncols <<= 1;
-    const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / ncols));
+    const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / (2 * ncols)));   // two accumulator buffers
     const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
     if (units <= 0) return cudaSuccess;
     const unsigned grid = (unsigned)std::min<int64_t>(units, (int64_t)148 * per_sm);
-    cudaError_t e = cudaSuccess;
-    switch (mode) {
-        case FWD:
-            e = cudaFuncSetAttribute(k_umma_gemm<FWD>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<FWD><<<grid, 128, smem, st>>>(a, nt, splits);
-            break;
-        case DA:
-            e = cudaFuncSetAttribute(k_umma_gemm<DA>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<DA><<<grid, 128, smem, st>>>(a, nt, splits);
-            break;
-        default:
-            e = cudaFuncSetAttribute(k_umma_gemm<DW>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-            if (e == cudaSuccess) k_umma_gemm<DW><<<grid, 128, smem, st>>>(a, nt, splits);
-            break;
+    const int vec_ok = mode == FWD && a.c_bf16 ? (a.ldc % 8 == 0) : (a.ldc % 4 == 0);
+#define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
+    do {                                                                                              \
+        e = cudaFuncSetAttribute(k_umma_gemm<M, BF, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
+        if (e == cudaSuccess) k_umma_gemm<M, BF, RL><<<grid, 288, smem, st>>>(tmA, tmB, a, nt, splits, vec_ok); \
+    } while (0)
+    if (mode == FWD) {
+        if (a.c_bf16 && a.relu) GD_UMMA_LAUNCH(FWD, true, true);
+        else if (a.c_bf16) GD_UMMA_LAUNCH(FWD, true, false);
+        else if (a.relu) GD_UMMA_LAUNCH(FWD, false, true);
+        else GD_UMMA_LAUNCH(FWD, false, false);
+    } else if (mode == DA) {
+        if (a.c_bf16) GD_UMMA_LAUNCH(DA, true, false);
+        else GD_UMMA_LAUNCH(DA, false, false);
+    } else {
+        GD_UMMA_LAUNCH(DW, false, false);
     }
+#undef GD_UMMA_LAUNCH
     return e != cudaSuccess ? e : cudaGetLastError();
 }
 

@@ -86,11 +86,16 @@ def test_da(lib, rows, rows_max, K, N):
 def test_dw(lib, rows, Mv, N, splits):
     g = torch.Generator().manual_seed(5 * rows + Mv + N)
     Np = (N + 15) // 16 * 16
-    A = bf((max(rows, 1) + 64, Mv), g)            # [rows x 2 din], rows past `rows` must be ignored
+    A = bf((max(rows, 1) + 64, Mv), g)            # [rows x 2 din]
     B = torch.zeros(max(rows, 1) + 64, Np, dtype=torch.bfloat16, device="cuda")
     B[:, :N] = bf((max(rows, 1) + 64, N), g)
+    pad = (rows + 63) // 64 * 64                  # the DW contract: rows [rows, round_up(rows, 64)) are zero
+    A[rows:pad] = 0
+    B[rows:pad] = 0
+    A[pad:] = float("nan")                        # rows past that are never read
+    B[pad:] = float("nan")
     C = torch.zeros(Mv, N, device="cuda")
-    run(lib, 2, A, Mv, B, Np, C, N, rows, rows, Mv, 0, Np, N, splits=splits)
+    run(lib, 2, A, Mv, B, Np, C, N, rows, A.shape[0], Mv, 0, Np, N, splits=splits)
     Af, Bf = A[:rows].float(), B[:rows, :N].float()
     ref = Af.T @ Bf
     close(C, ref, Af.abs().T @ Bf.abs(), tol=2.0 ** -12)
