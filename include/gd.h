@@ -102,7 +102,10 @@ typedef struct {
  * sampled node IDs is made"; "3-hop random neighborhood sampling").
  *
  *   seeds      host or device int32[num_seeds], distinct, in [0, N) (the
- *              mini-batch's training nodes).  n_id[0:num_seeds] = seeds.
+ *              mini-batch's training nodes).  n_id[0:num_seeds] = seeds.  Pinned
+ *              host memory is read by the kernel through its mapping (no copy-engine
+ *              transfer to queue behind the miss stream's H2D copies); pageable host
+ *              memory is copied first.
  *   fanouts    host int32[num_hops]; f in [0, GD_MAX_FANOUT] or -1 (whole row).
  *   rng_seed   64-bit key of the counter-based Philox4x32-10 stream (R1).
  *   batch_id   global mini-batch index; part of the Philox counter, so results

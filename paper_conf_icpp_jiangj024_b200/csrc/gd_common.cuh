@@ -56,6 +56,8 @@ void debug_after(const char* what, cudaStream_t s);
 // Pointer kind: true if `p` is device-accessible memory of the current context
 // (device / managed), false for host memory (pageable or pinned).
 bool is_device_pointer(const void* p);
+// Device address of page-locked (mapped) host memory, nullptr for anything else.
+const void* mapped_host_pointer(const void* p);
 
 // ------------------------------------------------------------ event timing (host)
 // Pairs of events recorded around kernel groups; summed on read (which syncs).

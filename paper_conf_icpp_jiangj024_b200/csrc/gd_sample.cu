@@ -591,7 +591,12 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     if ((s = w.scan.ensure(tiles)) != GD_OK) return s;
 
     const int32_t* seeds_d = seeds;
-    if (num_seeds > 0 && !is_device_pointer(seeds)) {
+    // pinned host seeds are read by k_seed_intake through the mapping (a few KB): a copy-engine
+    // transfer would queue behind the miss stream's bulk H2D copies and stall this stream
+    const int32_t* mapped = (num_seeds > 0 && !is_device_pointer(seeds)) ? (const int32_t*)mapped_host_pointer(seeds) : nullptr;
+    if (mapped) {
+        seeds_d = mapped;
+    } else if (num_seeds > 0 && !is_device_pointer(seeds)) {   // pageable host memory: staged copy
         if (num_seeds > w.seeds_cap) {
             if (w.seeds_ws) cudaFree(w.seeds_ws);
             w.seeds_ws = nullptr;

@@ -10,8 +10,10 @@ is used only for start-up barriers and the off-path max-over-ranks of the timing
 """
 from __future__ import annotations
 
+import ctypes
 import mmap
 import os
+import platform
 
 import numpy as np
 import torch
@@ -59,6 +61,49 @@ def sum_over_ranks(x: float, device=None) -> float:
     t = torch.tensor([float(x)], dtype=torch.float64, device=device)
     dist.all_reduce(t, op=dist.ReduceOp.SUM)
     return float(t.item())
+
+
+def _parse_list(text: str):
+    out = []
+    for part in text.strip().split(","):
+        if part:
+            lo, _, hi = part.partition("-")
+            out.extend(range(int(lo), int(hi or lo) + 1))
+    return out
+
+
+def numa_nodes():
+    """Online NUMA node ids (empty if unknown)."""
+    try:
+        with open("/sys/devices/system/node/online") as f:
+            return _parse_list(f.read())
+    except OSError:
+        return []
+
+
+def set_interleave(enable: bool) -> bool:
+    """Interleave this thread's future page allocations over all online NUMA nodes
+    (set_mempolicy(MPOL_INTERLEAVE)), or restore the default policy.  Used while rank 0
+    faults the shared host table in, so that on a multi-socket box the random row reads of
+    all GPUs' miss streams spread over every socket's memory controllers.
+    Returns False (and changes nothing) on a single-node host or where the syscall is
+    unavailable."""
+    nodes = numa_nodes()
+    if len(nodes) < 2 and enable:
+        return False
+    nr = {"x86_64": 238, "aarch64": 237}.get(platform.machine())
+    if nr is None:
+        return False
+    try:
+        libc = ctypes.CDLL(None, use_errno=True)
+        mask = (ctypes.c_ulong * 16)()
+        for n in nodes:
+            mask[n // 64] |= 1 << (n % 64)
+        mode = 3 if enable else 0                      # MPOL_INTERLEAVE / MPOL_DEFAULT
+        rc = libc.syscall(nr, mode, mask if enable else None, ctypes.c_ulong(1024 if enable else 0))
+        return rc == 0
+    except (OSError, AttributeError):
+        return False
 
 
 class HostTable:

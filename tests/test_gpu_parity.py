@@ -68,9 +68,15 @@ def test_sample_parity_tiny(tiny, gd, fanouts):
 def test_sample_parity_host_seeds_and_no_eid(tiny, gd):
     cfg, g, indptr, indices, order = tiny
     seeds = synth.batch_seeds(order, cfg.batch_size, 3).pin_memory()
-    res = g.sample(seeds, (5, 5), 77, 3)          # host seeds, eid not requested
+    res = g.sample(seeds, (5, 5), 77, 3)          # pinned host seeds (read through the mapping), no eid
     torch.cuda.synchronize()
-    compare_sample(res, O.sample(indptr, indices, seeds.numpy(), [5, 5], 77, 3), 2)
+    ref = O.sample(indptr, indices, seeds.numpy(), [5, 5], 77, 3)
+    compare_sample(res, ref, 2)
+    pageable = seeds.clone()                      # pageable host seeds: staged copy
+    assert not pageable.is_pinned()
+    res2 = g.sample(pageable, (5, 5), 77, 3)
+    torch.cuda.synchronize()
+    compare_sample(res2, ref, 2)
 
 
 def test_sample_parity_multi_tile(gd):

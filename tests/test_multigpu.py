@@ -131,3 +131,16 @@ def test_single_process_fallbacks():
     assert list(M.segment(7, 0, 1)) == list(range(7))
     assert M.batch_schedule(3, 0, 1, 7) == [(0, 0), (1, 0), (2, 0), (0, 1), (1, 1), (2, 1), (0, 2)]
     assert M.batch_schedule(1, 1, 4, 3) == []       # more ranks than batches: an empty segment
+
+
+def test_numa_helpers():
+    """NUMA interleave of the shared host table (bench.py, world > 1): node-list parsing and a
+    policy call that never raises (False on single-node hosts)."""
+    from paper_conf_icpp_jiangj024_b200 import multigpu as mg
+    assert mg._parse_list("0-1,3\n") == [0, 1, 3]
+    assert mg._parse_list("0") == [0]
+    nodes = mg.numa_nodes()
+    assert all(isinstance(n, int) for n in nodes)
+    ok = mg.set_interleave(True)
+    assert ok == (len(nodes) >= 2) or not ok
+    mg.set_interleave(False)
