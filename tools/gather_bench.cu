@@ -139,16 +139,16 @@ float timeit(F f) {
 }
 
 int main() {
-    const int64_t S = 11100000, R = 512, H = 150000;
+    const int64_t S = 11100000, R = 512, H = 337000;
     uint8_t *src, *out;
     int2* hl;
     CK(cudaMalloc(&src, S * R));
-    CK(cudaMalloc(&out, 400000 * R));
+    CK(cudaMalloc(&out, 1000000 * R));
     CK(cudaMemset(src, 1, S * R));
     std::vector<int2> h(H);
     std::mt19937_64 g(3);
-    std::vector<int> pos(400000);
-    for (int i = 0; i < 400000; ++i) pos[i] = i;
+    std::vector<int> pos(1000000);
+    for (int i = 0; i < 1000000; ++i) pos[i] = i;
     std::shuffle(pos.begin(), pos.end(), g);
     std::sort(pos.begin(), pos.begin() + H);
     for (int64_t i = 0; i < H; ++i) h[i] = make_int2(pos[i], (int)(g() % S));
@@ -171,6 +171,10 @@ int main() {
     rep("warp u2 g1184x256", [&] { k_warp<2><<<1184, 256>>>(hl, H, src, out, R); });
     rep("warp u4 g1184x256", [&] { k_warp<4><<<1184, 256>>>(hl, H, src, out, R); });
     rep("warp u4 g592x256", [&] { k_warp<4><<<592, 256>>>(hl, H, src, out, R); });
+    rep("warp u8 g592x256", [&] { k_warp<8><<<592, 256>>>(hl, H, src, out, R); });
+    rep("warp u8 g1184x256", [&] { k_warp<8><<<1184, 256>>>(hl, H, src, out, R); });
+    rep("warp u4 g2368x256", [&] { k_warp<4><<<2368, 256>>>(hl, H, src, out, R); });
+    rep("warp u2 g2368x256", [&] { k_warp<2><<<2368, 256>>>(hl, H, src, out, R); });
     for (int st : {2, 4}) {
         for (int G : {148, 296, 592}) {
             size_t sm = (size_t)128 * st * R;
