@@ -635,11 +635,14 @@ def run_ours(args, rank, world, local_rank):
                     kern["staged_copy_engine_ms_per_batch"])
     dominant = roof_miss if misses > 0 and miss_busy >= kern["gather_ms_per_batch"] else roof_gather
     traffic = load_traffic(cfg.name)
-    if traffic:
-        for r in (roof_gather, roof_miss):
-            for kname, tv in traffic.items():
-                if r["kernel"].startswith(kname):
-                    r["traffic"] = tv
+    if traffic:                            # per-launch DRAM bytes of the committed ncu launch list
+        for kname, tv in traffic.items():
+            base = kname.replace("gd::", "").split("<")[0]
+            if base == roof_gather["kernel"] and isinstance(tv, (int, float)):
+                roof_gather["traffic"] = tv
+                roof_gather["traffic_source"] = f"profiles/traffic.json[{cfg.name}][{kname}] (ncu, per launch)"
+    roof_miss["traffic_note"] = ("host-link bound: the bytes that bound it cross PCIe (R per miss); DRAM traffic of "
+                                 "the miss kernels is in profiles/r01_<config>_launches.md")
 
     train_info = None
     if model is not None:
