@@ -21,6 +21,8 @@
 #include <cuda_bf16.h>
 
 #include <algorithm>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -57,6 +59,9 @@ struct gd_sage {
     int64_t nparams = 0, nw16 = 0;
     float* loss_rows = nullptr;     // [n0_max]
     float* colsum_part = nullptr;   // [kColsumChunks x max dout] partial column sums (db)
+    unsigned int* gemm_counter = nullptr;   // work counter of the (stream-ordered) GEMM launches
+    gd::EventTimer timer;                   // GD_SAGE_TIMING=1: per-phase stream times, printed at destroy
+    std::vector<const char*> phase;         // name of each timer pair
 };
 
 namespace gd {
@@ -331,9 +336,9 @@ __global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restri
 
 // ------------------------------------------------------------------ GEMMs (gd_umma.cuh)
 static umma::Args gemm_args(const __nv_bfloat16* A, int64_t lda, const __nv_bfloat16* B, int64_t ldb, void* C, int64_t ldc,
-                            const int64_t* rows_dev) {
+                            const int64_t* rows_dev, unsigned int* counter) {
     umma::Args a{};
-    a.A = A; a.lda = lda; a.B = B; a.ldb = ldb; a.C = C; a.ldc = ldc; a.rows_dev = rows_dev;
+    a.A = A; a.lda = lda; a.B = B; a.ldb = ldb; a.C = C; a.ldc = ldc; a.rows_dev = rows_dev; a.counter = counter;
     return a;
 }
 
@@ -345,10 +350,29 @@ static void sage_free(gd_sage* s) {
     if (!s) return;
     DeviceGuard guard(s->hdr.device);
     cudaDeviceSynchronize();
+    if (s->timer.on && !s->phase.empty()) {   // summary of the per-phase live times on the train stream
+        std::vector<std::pair<const char*, double>> acc;
+        int steps = 0;
+        for (size_t i = 0; i < s->phase.size(); ++i) {
+            float ms = 0;
+            const auto pr = s->timer.pairs[i];
+            if (pr.second < 0) continue;
+            cudaEventElapsedTime(&ms, s->timer.pool[pr.first], s->timer.pool[pr.second]);
+            size_t k = 0;
+            while (k < acc.size() && std::strcmp(acc[k].first, s->phase[i]) != 0) ++k;
+            if (k == acc.size()) acc.push_back({s->phase[i], 0.0});
+            acc[k].second += ms;
+            if (std::strcmp(s->phase[i], "agg0") == 0) ++steps;
+        }
+        std::fprintf(stderr, "[gd_sage] live ms per step over %d steps:", steps);
+        for (auto& p : acc) std::fprintf(stderr, " %s %.4f", p.first, p.second / std::max(1, steps));
+        std::fprintf(stderr, "\n");
+    }
+    s->timer.destroy();
     for (auto& l : s->layers)
         for (void* p : {(void*)l.A16, (void*)l.Z, (void*)l.H16, (void*)l.dZ16, (void*)l.dA, (void*)l.dX})
             if (p) cudaFree(p);
-    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->colsum_part})
+    for (void* p : {(void*)s->params, (void*)s->grads, (void*)s->W16, (void*)s->loss_rows, (void*)s->colsum_part, (void*)s->gemm_counter})
         if (p) cudaFree(p);
     s->hdr.magic = 0;
     delete s;
@@ -422,6 +446,8 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         max_dout = std::max(max_dout, l.dout);
     }
     SA(s->colsum_part, (size_t)kColsumChunks * max_dout * sizeof(float));
+    SA(s->gemm_counter, sizeof(unsigned int));
+    if (const char* e = std::getenv("GD_SAGE_TIMING")) s->timer.on = std::atoi(e) != 0;
 #undef SA
     for (int j = 0; j < num_layers; ++j) {      // pad columns of dZ16 (the DA GEMM's K) start and stay zero
         const SageLayer& l = s->layers[j];
@@ -464,6 +490,19 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
     cudaStream_t st = (cudaStream_t)stream_v;
     const int L = s->L;
     const dim3 rows_blk(32, 8);          // (float4 column, row) blocks of the row-wise kernels
+    int tph = -1;                        // GD_SAGE_TIMING: one event pair per phase
+    auto ph_begin = [&]() { tph = s->timer.on ? s->timer.begin(st) : -1; };
+    auto ph_end = [&](const char* name) {
+        if (tph >= 0) {
+            s->timer.end(tph, st);
+            s->phase.push_back(name);
+        }
+    };
+    static const char* kAgg[] = {"agg0", "agg1", "agg2", "agg3", "agg4", "agg5", "agg6", "agg7"};
+    static const char* kFwd[] = {"fwd0", "fwd1", "fwd2", "fwd3", "fwd4", "fwd5", "fwd6", "fwd7"};
+    static const char* kDw[] = {"dw0", "dw1", "dw2", "dw3", "dw4", "dw5", "dw6", "dw7"};
+    static const char* kDa[] = {"da0", "da1", "da2", "da3", "da4", "da5", "da6", "da7"};
+    static const char* kSc[] = {"scatter0", "scatter1", "scatter2", "scatter3", "scatter4", "scatter5", "scatter6", "scatter7"};
     // ---- forward
     const void* x = feats;
     int64_t ldx = s->dims[0];
@@ -471,6 +510,7 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         SageLayer& l = s->layers[j];
         const int h = l.hop;
         const int64_t* n_dst = sizes + (h - 1);
+        ph_begin();
         if (j == 0)
             k_sage_agg<float><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const float*)x, ldx, l.din, rowptr[h - 1],
                                                                           col[h - 1], n_dst, l.n_dst_max, l.A16);
@@ -479,8 +519,11 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
                                                                                   rowptr[h - 1], col[h - 1], n_dst,
                                                                                   l.n_dst_max, l.A16);
         GD_DEBUG_AFTER("k_sage_agg", st);
+        ph_end(kAgg[j]);
+        ph_begin();
         const bool hidden = j < L - 1;   // hidden: h = relu(z + b) in bf16 (the next layer's input); top: logits
-        umma::Args a = gemm_args(l.A16, 2 * l.din, s->W16 + l.w16_off, l.dp, hidden ? (void*)l.H16 : (void*)l.Z, l.dp, n_dst);
+        umma::Args a = gemm_args(l.A16, 2 * l.din, s->W16 + l.w16_off, l.dp, hidden ? (void*)l.H16 : (void*)l.Z, l.dp, n_dst,
+                                 s->gemm_counter);
         a.c_bf16 = hidden;
         a.relu = hidden;
         a.bias = s->params + l.b_off;
@@ -489,23 +532,27 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         a.n_store = l.dout;
         GD_CUDA(umma::launch(umma::FWD, a, l.n_dst_max, l.dout, 1, st));
         GD_DEBUG_AFTER("k_umma_gemm<FWD>", st);
+        ph_end(kFwd[j]);
         x = l.H16;
         ldx = l.dp;
     }
     // ---- loss
     SageLayer& top = s->layers[L - 1];
+    ph_begin();
     k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, top.dp, labels, sizes, top.n_dst_max, top.dZ16,
                                                          s->loss_rows);
     k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
     GD_DEBUG_AFTER("k_xent", st);
+    ph_end("loss");
     // ---- backward
     GD_CUDA(cudaMemsetAsync(s->grads, 0, (size_t)s->nparams * sizeof(float), st));   // dW accumulates by red.add
     for (int j = L - 1; j >= 0; --j) {
         SageLayer& l = s->layers[j];
         const int h = l.hop;
         const int64_t* n_dst = sizes + (h - 1);
+        ph_begin();
         {   // dW = a^T dz, the rows split over ~1 CTA per SM
-            umma::Args a = gemm_args(l.A16, 2 * l.din, l.dZ16, l.dp, s->grads + l.w_off, l.dout, n_dst);
+            umma::Args a = gemm_args(l.A16, 2 * l.din, l.dZ16, l.dp, s->grads + l.w_off, l.dout, n_dst, s->gemm_counter);
             a.m_valid = 2 * l.din;
             a.n_valid = l.dp;
             a.n_store = l.dout;
@@ -519,15 +566,19 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         k_colsum_part<<<dim3(strips, kColsumChunks), rows_blk, 0, st>>>(l.dZ16, l.dout, l.dp, n_dst, s->colsum_part);
         k_colsum_final<<<strips, rows_blk, 0, st>>>(s->colsum_part, l.dout, kColsumChunks, s->grads + l.b_off);
         GD_DEBUG_AFTER("k_colsum", st);
+        ph_end(kDw[j]);
         if (j == 0) break;
+        ph_begin();
         {   // da = dz W^T
-            umma::Args a = gemm_args(l.dZ16, l.dp, s->W16 + l.w16_off, l.dp, l.dA, 2 * l.din, n_dst);
+            umma::Args a = gemm_args(l.dZ16, l.dp, s->W16 + l.w16_off, l.dp, l.dA, 2 * l.din, n_dst, s->gemm_counter);
             a.k_valid = l.dp;
             a.n_valid = 2 * l.din;
             a.n_store = 2 * l.din;
             GD_CUDA(umma::launch(umma::DA, a, l.n_dst_max, 2 * l.din, 1, st));
             GD_DEBUG_AFTER("k_umma_gemm<DA>", st);
         }
+        ph_end(kDa[j]);
+        ph_begin();
         k_scatter_init<<<grid_for(l.n_src_max * 8), rows_blk, 0, st>>>(l.dA, l.din, n_dst, sizes + h, l.dX);
         k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1], n_dst, l.dX);
         GD_DEBUG_AFTER("k_sage_scatter", st);
@@ -535,6 +586,7 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H16, prev.dout, prev.dp, sizes + h,
                                                                        prev.n_dst_max, prev.dZ16);
         GD_DEBUG_AFTER("k_relu_grad", st);
+        ph_end(kSc[j]);
     }
     GD_CUDA(cudaGetLastError());
     return GD_OK;
@@ -597,12 +649,17 @@ gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const voi
         return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: bad argument");
     if ((lda | ldb) & 7 || (k_valid & 7) || (n_valid & 7) || (m_valid & 7) || ((uintptr_t)A | (uintptr_t)B) & 15)
         return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: strides / extents must be multiples of 8, bases 16-byte aligned");
-    umma::Args a = gemm_args((const __nv_bfloat16*)A, lda, (const __nv_bfloat16*)B, ldb, C, ldc, rows_dev);
+    cudaStream_t st = (cudaStream_t)stream;
+    unsigned int* counter = nullptr;
+    GD_CUDA(cudaMallocAsync((void**)&counter, sizeof(unsigned int), st));
+    umma::Args a = gemm_args((const __nv_bfloat16*)A, lda, (const __nv_bfloat16*)B, ldb, C, ldc, rows_dev, counter);
     a.c_bf16 = c_bf16;
     a.relu = relu;
     a.bias = bias;
     a.m_valid = m_valid; a.k_valid = k_valid; a.n_valid = n_valid; a.n_store = n_store;
-    GD_CUDA(umma::launch(mode, a, rows_max, n_store, splits, (cudaStream_t)stream));
+    const cudaError_t e = umma::launch(mode, a, rows_max, n_store, splits, st);
+    cudaFreeAsync(counter, st);
+    GD_CUDA(e);
     return GD_OK;
 }
 

@@ -9,7 +9,10 @@
 //
 // Tile: UMMA M = 128 rows (one TMEM lane per output row), N = bn <= 256 columns (TMEM
 // columns), K = 64 per pipeline stage (4 MMAs of K = 16).  CTAs are persistent over the tiles
-// ("units"; DW units are (tile, row slice) pairs) and warp-specialised (288 threads):
+// ("units"; DW units are (tile, row slice) pairs), fetched from a per-launch atomic counter
+// (a CTA that only gets an SM after the others finished finds no work and leaves, so SMs held
+// by concurrent kernels of the SET pipeline do not stretch the grid), and warp-specialised
+// (288 threads):
 //   warp 0, lane 0: producer + MMA issuer.  It keeps STAGES-1 k-blocks of TMA loads in flight
 //     ahead of the MMAs, across unit boundaries (TMA completes a stage's "full" mbarrier with
 //     its byte count; the tcgen05.commit of the MMAs that read a stage arrives on its "empty"
@@ -64,6 +67,7 @@ struct Args {
     int n_valid;                 // B's extent along N (multiple of 8; zero-filled past it)
     int n_store;                 // output columns written
     int bn;                      // N tile (multiple of 16, <= 256; multiple of 64 when B is MN-major)
+    unsigned int* counter;       // device work counter, zero at launch (units are fetched dynamically)
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -174,32 +178,41 @@ struct Unit {
 };
 
 // Units: FWD / DA: (m-tile, n-tile) over the device row count, full K.  DW: (m-tile, n-tile,
-// split) with split z taking a BK-aligned slice of the device row count (empty slices skipped).
+// split) with split z taking a BK-aligned slice of the device row count.  decode: 1 = a unit
+// with work, 0 = an empty DW slice, -1 = past the last unit.
 template <int MODE>
-__device__ __forceinline__ bool unit_at(Unit& c, int64_t u, const Args& a, int64_t rows, int nt, int splits) {
-    for (;; u += gridDim.x) {
-        if (MODE == DW) {
-            const int64_t mt = (a.m_valid + BM - 1) / BM;
-            if (u >= mt * nt * splits) return false;
-            const int64_t z = u % splits, rest = u / splits;
-            c.n0 = (rest % nt) * a.bn;
-            c.m0 = (rest / nt) * BM;
-            int64_t per = (rows + splits - 1) / splits;
-            per = (per + BK - 1) / BK * BK;
-            c.k_begin = z * per;
-            c.k_end = c.k_begin + per < rows ? c.k_begin + per : rows;
-            if (c.k_begin >= c.k_end) continue;
-        } else {
-            if (u >= (rows + BM - 1) / BM * nt) return false;
-            c.m0 = (u / nt) * BM;
-            c.n0 = (u % nt) * a.bn;
-            c.k_begin = 0;
-            c.k_end = a.k_valid;
-        }
-        c.u = u;
-        c.kb = 0;
-        c.nkb = (int)((c.k_end - c.k_begin + BK - 1) / BK);
-        return true;
+__device__ __forceinline__ int decode_unit(Unit& c, int64_t u, const Args& a, int64_t rows, int nt, int splits) {
+    if (MODE == DW) {
+        const int64_t mt = (a.m_valid + BM - 1) / BM;
+        if (u >= mt * nt * splits) return -1;
+        const int64_t z = u % splits, rest = u / splits;
+        c.n0 = (rest % nt) * a.bn;
+        c.m0 = (rest / nt) * BM;
+        int64_t per = (rows + splits - 1) / splits;
+        per = (per + BK - 1) / BK * BK;
+        c.k_begin = z * per;
+        c.k_end = c.k_begin + per < rows ? c.k_begin + per : rows;
+        if (c.k_begin >= c.k_end) return 0;
+    } else {
+        if (u >= (rows + BM - 1) / BM * nt) return -1;
+        c.m0 = (u / nt) * BM;
+        c.n0 = (u % nt) * a.bn;
+        c.k_begin = 0;
+        c.k_end = a.k_valid;
+    }
+    c.u = u;
+    c.kb = 0;
+    c.nkb = (int)((c.k_end - c.k_begin + BK - 1) / BK);
+    return 1;
+}
+
+// Next unit with work from the launch's shared counter (CTAs that start late, e.g. on SMs
+// other streams' kernels held, find the work taken and leave instead of delaying the grid).
+template <int MODE>
+__device__ __forceinline__ bool fetch_unit(Unit& c, const Args& a, int64_t rows, int nt, int splits) {
+    for (;;) {
+        const int r = decode_unit<MODE>(c, (int64_t)atomicAdd(a.counter, 1u), a, rows, nt, splits);
+        if (r != 0) return r > 0;
     }
 }
 
@@ -221,10 +234,15 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
     uint64_t* acc_full = empty + STAGES;                          // [2] accumulator buffer ready
     uint64_t* acc_empty = acc_full + 2;                           // [2] accumulator buffer drained
     uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
+    int64_t* ep_unit = (int64_t*)(tmem_slot + 2);                 // [2] unit id of each accumulator buffer (-1: end)
 
     const int64_t rows = *a.rows_dev;   // device-resident size
     Unit cm;
-    if (!unit_at<MODE>(cm, blockIdx.x, a, rows, nt, splits)) return;
+    __shared__ int64_t first_unit;
+    if (threadIdx.x == 0) first_unit = fetch_unit<MODE>(cm, a, rows, nt, splits) ? cm.u : -1;
+    __syncthreads();
+    if (first_unit < 0) return;         // no work left for this CTA
+    decode_unit<MODE>(cm, first_unit, a, rows, nt, splits);
     const int64_t m_valid = MODE == DW ? a.m_valid : rows;
     uint32_t nc = 32;                   // columns of one accumulator buffer
     while ((int)nc < bn) nc <<= 1;
@@ -238,8 +256,10 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
     if (threadIdx.x == 0) {
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmB) : "memory");
-        for (int s = 0; s < 2 * STAGES + 2; ++s)
+        for (int s = 0; s < 2 * STAGES; ++s)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(full + s)));
+        for (int s = 0; s < 2; ++s)   // tcgen05.commit + the issuer's arrive after publishing the unit id
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 2;\n" ::"r"(smem_u32(acc_full + s)));
         for (int s = 0; s < 2; ++s)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;\n" ::"r"(smem_u32(acc_empty + s)));   // one per epilogue warp
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
@@ -256,6 +276,8 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
             const uint32_t stage_bytes = (uint32_t)(A_STAGE + b_stage);
             Unit ld = cm;
             bool ld_ok = true;
+            int64_t uq[8];                 // units fetched by the load cursor, not yet reached by the MMAs
+            uint32_t uq_head = 0, uq_tail = 0;
             uint32_t it_ld = 0, it_cm = 0, u_local = 0;
             auto issue_load = [&]() {
                 const int s = (int)(it_ld % STAGES);
@@ -271,7 +293,10 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
                 else
                     for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
                 ++it_ld;
-                if (++ld.kb == ld.nkb) ld_ok = unit_at<MODE>(ld, ld.u + gridDim.x, a, rows, nt, splits);
+                if (++ld.kb == ld.nkb) {
+                    ld_ok = fetch_unit<MODE>(ld, a, rows, nt, splits);
+                    if (ld_ok) uq[uq_tail++ & 7] = ld.u;
+                }
             };
             for (int s = 0; s < STAGES - 1 && ld_ok; ++s) issue_load();
             for (;;) {
@@ -298,15 +323,27 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
                                  smem_u32(empty + s))
                              : "memory");
                 const bool last = cm.kb == cm.nkb - 1;
-                if (last)
+                if (last) {
                     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                      smem_u32(acc_full + buf))
                                  : "memory");
+                    ep_unit[buf] = cm.u;   // published by the release-arrive below
+                    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
+                }
                 if (ld_ok) issue_load();   // refill the stage the previous k-block used (MMAs stay queued)
                 ++it_cm;
                 if (last) ++u_local;
-                if (++cm.kb == cm.nkb && !unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
+                if (++cm.kb == cm.nkb) {
+                    if (uq_head == uq_tail) break;
+                    decode_unit<MODE>(cm, uq[uq_head++ & 7], a, rows, nt, splits);
+                }
             }
+            // end marker for the epilogue warps in the next buffer
+            const uint32_t buf = u_local & 1;
+            if (u_local >= 2) mbar_wait(smem_u32(acc_empty + buf), ((u_local >> 1) - 1) & 1);
+            ep_unit[buf] = -1;
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
         }
     } else {
         // ===== epilogue warps 1..8: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
@@ -315,13 +352,15 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
         for (uint32_t u_local = 0;; ++u_local) {
             const uint32_t buf = u_local & 1;
             mbar_wait(smem_u32(acc_full + buf), (u_local >> 1) & 1);
+            const int64_t u = *(volatile int64_t*)(ep_unit + buf);
+            if (u < 0) break;
+            decode_unit<MODE>(cm, u, a, rows, nt, splits);
             asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
             epilogue<MODE, OUT_BF16, RELU>(a, tmem + buf * nc + ((uint32_t)(q * 32) << 16), cm.m0 + q * 32, cm.n0, m_valid, bn,
                                            h, lane, vec_ok != 0);
             asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
             __syncwarp();
             if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_empty + buf)) : "memory");
-            if (!unit_at<MODE>(cm, cm.u + gridDim.x, a, rows, nt, splits)) break;
         }
     }
     __syncthreads();
@@ -331,7 +370,7 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
     }
 }
 
-inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 16; }
+inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 8 + 16; }
 
 // 2-D bf16 tensor map, SWIZZLE_128B, box {64, box_outer}; inner = contiguous extent, outer =
 // rows, ld = row stride in elements.  Out-of-bounds box elements read as zero.
@@ -354,6 +393,7 @@ inline cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, ui
 
 // Host launcher.  rows_max: host bound of *rows_dev (grid sizing, tensor extents).  n_total:
 // output columns (split into <= 256-wide tiles).  splits: DW reduction slices per tile.
+// a.counter: a device word the launch may use (zeroed here, on the stream).
 inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_total, int splits, cudaStream_t st) {
     Args a = a0;
     const bool b_mn = mode != DA;
@@ -381,6 +421,9 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
     const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / (2 * ncols)));   // two accumulator buffers
     const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
     if (units <= 0) return cudaSuccess;
+    if (!a.counter) return cudaErrorInvalidValue;
+    e = cudaMemsetAsync(a.counter, 0, sizeof(unsigned int), st);
+    if (e != cudaSuccess) return e;
     const unsigned grid = (unsigned)std::min<int64_t>(units, (int64_t)148 * per_sm);
     const int vec_ok = mode == FWD && a.c_bf16 ? (a.ldc % 8 == 0) : (a.ldc % 4 == 0);
 #define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
