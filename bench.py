@@ -311,6 +311,13 @@ def run_ours(args, rank, world, local_rank):
     sizes_log = torch.zeros((total, 2 * len(fan) + 1), dtype=torch.int64, device=dev)
     main = torch.cuda.current_stream(dev)
     pending = []
+    # GD_RELEASE_STREAM=1: releases on their own stream; release(j - Q) is ordered after extract(j)'s bookkeeping
+    # and before extract(j + 1)'s (the sequential order of Alg. 1, so the buffer state is the
+    # oracle's), and overlaps sample(j + 1), which does not touch the buffer
+    rel_stream = torch.cuda.Stream(dev) if os.environ.get("GD_RELEASE_STREAM", "0") == "1" else main
+    ev_bk = torch.cuda.Event()      # extract(j)'s bookkeeping enqueued on main
+    ev_rel = torch.cuda.Event()     # release(j - Q) done
+    rel_live = [False]
 
     # ---- f4: the train stage on its own stream (GraphSAGE 3 x 256; DDP all-reduce)
     model = None
@@ -347,6 +354,8 @@ def run_ours(args, rank, world, local_rank):
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
         g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
         dsync("sample", j)
+        if rel_live[0]:
+            main.wait_event(ev_rel)        # the previous step's release precedes this lookup
         buf.extract(o.n_id, o.num_nodes_dev, o.max_nodes, out=feats[s], alias=aliases[s], stats=stats[j],
                     stream=main, done=dones[s])
         dsync("extract", j)
@@ -367,7 +376,13 @@ def run_ours(args, rank, world, local_rank):
         pending.append(o)
         if len(pending) == Q:
             r = pending.pop(0)
-            buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
+            if rel_stream is not main:
+                ev_bk.record(main)
+                rel_stream.wait_event(ev_bk)
+            buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=rel_stream)
+            if rel_stream is not main:
+                ev_rel.record(rel_stream)
+                rel_live[0] = True
             dsync("release", j)
         sizes_log[j].copy_(o.sizes, non_blocking=True)
         if host_out is not None:               # e2e: this step's result -> pinned host memory (D2H on the
@@ -435,6 +450,8 @@ def run_ours(args, rank, world, local_rank):
         for j in range(off + W, off + W + K):
             step(j)
         main.wait_event(dones[(off + W + K - 1) % RING])  # the last batch's rows are all in `out`
+        if rel_live[0]:
+            main.wait_event(ev_rel)                          # ... and the last release is done
         if model is not None:
             main.wait_event(tdones[(off + W + K - 1) % RING])   # ... and it is trained
         ev1.record(main)
@@ -451,6 +468,23 @@ def run_ours(args, rank, world, local_rank):
     sz = sizes_log[off + W:off + W + K].double().mean(0).cpu().tolist()
     hits, misses, miss_zc, miss_staged = (int(x) for x in st)
     barrier()
+
+    # ---- the timed configuration's output rows, checked by their closed form (P5):
+    # out[i] == table row (n_id[i] mod P) for the last Q + 1 batches of the timed region
+    # (extracted back to back, no host sync between them)
+    rows_check = {"batches": 0, "rows": 0, "ok": True}
+    torch.cuda.synchronize(dev)
+    for j in range(max(off + W, off + W + K - RING), off + W + K):
+        s_ = j % RING
+        dones[s_].synchronize()
+        n_j = int(sizes_log[j][len(fan)].item())
+        ids = outs[s_].n_id[:n_j].long().cpu() % cfg.host_rows
+        want = wl.table.tensor.index_select(0, ids)
+        got = feats[s_][:n_j].view(torch.uint8).reshape(n_j, cfg.row_bytes).cpu()
+        rows_check["ok"] &= bool(torch.equal(got, want))
+        rows_check["batches"] += 1
+        rows_check["rows"] += n_j
+    log(f"pipelined rows check: {rows_check}")
 
     # ---- e2e through the public API with host inputs / host-read results
     log(f"timed: {ms:.2f} ms for {K} steps; e2e ...")
@@ -474,6 +508,8 @@ def run_ours(args, rank, world, local_rank):
             h_ev[k].synchronize()
             seen[1] += int(h_sizes[k][len(fan)]) + int(h_stats[k][0]) + int(h_stats[k][1])
         main.wait_event(dones[(off + W + 2 * K - 1) % RING])
+        if rel_live[0]:
+            main.wait_event(ev_rel)
         if model is not None:
             main.wait_event(tdones[(off + W + 2 * K - 1) % RING])
         e1.record(main)
@@ -699,6 +735,7 @@ def run_ours(args, rank, world, local_rank):
                       "hits": hits / K, "misses": misses / K,
                       "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
         "parity": parity,
+        "rows_check": rows_check,
         "sweep": sweep or None,
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},

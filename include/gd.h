@@ -175,9 +175,10 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  *   loop 2: misses, in list order, take successive LRU standby slots; a slot's
  *           previous node is invalidated (R9); map / reverse / alias updated;
  *   the missed rows stream from the pinned host table into their slots and into
- *   `out` on the library's side stream (asynchronous extraction),
+ *   `out` on the library's side streams (asynchronous extraction),
  *   overlapping the caller's next gd_sample; hit rows are gathered from the slots
- *   into `out` on `stream` (the trainer's alias indexing, materialised).
+ *   into `out` on a side stream too (the trainer's alias indexing, P:96,
+ *   materialised).  Only the bookkeeping (loops 1 and 2) runs on `stream`.
  *
  *   node_ids  device int32[n], distinct, in [0, N) (normally gd_sample's n_id).
  *   n_dev     device int64*: n (normally &sizes[K]); n <= n_max.
@@ -191,6 +192,9 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  *             for the misses or the hit gather.  node_ids, *n_dev and alias
  *             must stay unmodified until `done`.
  * GD_ERR_CAPACITY if this would exceed max_inflight unreleased batches.
+ * The call does not synchronise the device; it blocks the calling thread only when
+ * that thread is max_inflight + 2 batches ahead of the staged miss path's host gather
+ * (whose per-batch host arguments are then reused).
  * ------------------------------------------------------------------------- */
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,
                      void* out, int32_t* alias, int64_t* stats, void* stream, void* done);
@@ -330,7 +334,10 @@ gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const voi
  * Release stage: for node_ids in list order decrement the refcount; a
  * slot whose count reaches zero is appended at the tail (MRU end) of the standby
  * list.  The node stays valid until its slot is reused (delayed invalidation).
- * Arguments as in gd_extract.  Stream-ordered; no host sync.
+ * Arguments as in gd_extract.  Stream-ordered; no host sync.  It does not wait for the
+ * batch's `done`: a slot it frees is refilled only by a later batch's miss copies, which
+ * wait for every earlier batch's hit gather.  Issue it after the gd_extract calls it must
+ * follow in Alg. 1 order, on `stream` or on a stream ordered after them by events.
  * ------------------------------------------------------------------------- */
 gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev,
                             int64_t n_max, void* stream);

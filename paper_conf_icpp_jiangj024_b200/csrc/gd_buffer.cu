@@ -1324,6 +1324,11 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // every stream is done with trip / host-list slot d (batch - D)
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));
     if (staged) {
+        // The host-side arguments of slot d (StagedSlot, chunk jobs) are rewritten below at
+        // enqueue time; the host-gather callbacks of batch - D read them when stream H reaches
+        // them, so they must have run first.  This bounds how far the caller's thread runs
+        // ahead of the host gather (D batches), not the device.
+        if (b->batch_counter >= b->D) GD_CUDA(cudaEventSynchronize(b->ev_H[d]));
         adapt_alpha(b, (int)((b->batch_counter + b->D - 2) % b->D));
         ss->batch = b->batch_counter;
     }

@@ -196,6 +196,57 @@ def test_extract_parity_tiny_evict(tiny, gd, Q):
     run_schedule(gd, g, ip, ix, feat, S, Q, seeds, list(cfg.fanouts))
 
 
+@pytest.mark.parametrize("own_stream", [False, True])
+def test_release_on_its_own_stream_matches_oracle(tiny, gd, own_stream):
+    """bench.py's schedule: release(j - Q) on a second stream, ordered after extract(j)'s
+    bookkeeping and before extract(j + 1)'s by events, overlapping sample(j + 1); no host
+    sync until the end.  Outputs and the final buffer state equal the sequential oracle's."""
+    cfg, g, ip, ix, order = tiny
+    feat = table_np(cfg.num_nodes, cfg.row_bytes)
+    fan = list(cfg.fanouts)
+    Q = 4
+    nb, _ = O.sample_bounds(cfg.batch_size, fan, cfg.num_nodes, cfg.num_edges)
+    n_max = nb[-1]
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), Q * n_max, Q, n_max)
+    main = torch.cuda.current_stream()
+    rel = torch.cuda.Stream() if own_stream else main
+    ev_bk, ev_rel = torch.cuda.Event(), torch.cuda.Event()
+    nbat = 24
+    seeds = [synth.batch_seeds(order, cfg.batch_size, b).cuda() for b in range(nbat)]
+    res, outs, aliases, stats, pending, rel_live = [], [], [], [], [], False
+    for b in range(nbat):
+        r = g.sample(seeds[b], fan, 3, b, stream=main)
+        if rel_live:
+            main.wait_event(ev_rel)
+        a = torch.empty(n_max, dtype=torch.int32, device="cuda")
+        st = torch.zeros(4, dtype=torch.int64, device="cuda")
+        out, _, done = buf.extract(r.n_id, r.num_nodes_dev, r.max_nodes, alias=a, stats=st, stream=main)
+        res.append(r), outs.append(out), aliases.append(a), stats.append(st)
+        pending.append(r)
+        if len(pending) == Q:
+            r0 = pending.pop(0)
+            ev_bk.record(main)
+            rel.wait_event(ev_bk)
+            buf.release(r0.n_id, r0.num_nodes_dev, r0.max_nodes, stream=rel)
+            ev_rel.record(rel)
+            rel_live = True
+    torch.cuda.synchronize()
+    ob = O.Buffer(feat, Q * n_max)
+    opend = []
+    for b in range(nbat):
+        n_id = res[b].to_host()["n_id"]
+        o_out, o_alias, o_stats = ob.extract(n_id)
+        n = len(n_id)
+        assert tuple(stats[b].cpu().tolist()[:2]) == o_stats, b
+        assert np.array_equal(aliases[b][:n].cpu().numpy(), o_alias), b
+        assert np.array_equal(outs[b][:n].cpu().numpy(), o_out), b
+        opend.append(n_id)
+        if len(opend) == Q:
+            ob.release(opend.pop(0))
+    compare_state(buf, ob)
+    assert buf.check() == 0
+
+
 # phase 2 of the staged share: SM pull of the pinned slot, or copy engine with the
 # default 8 MB chunk ring, with 64 KB chunks (many chunks per batch, ring reuse), or
 # with one chunk per batch (GD_STAGE_CHUNK_KB=0)
