@@ -173,7 +173,8 @@ class Workload:
         self.cfg = cfg
         t0 = time.time()
         indptr, indices = synth.chung_lu_csr(cfg.num_nodes, cfg.num_edges, device=device)
-        torch.cuda.synchronize(device)
+        if device.type == "cuda":
+            torch.cuda.synchronize(device)
         self.t_graph = time.time() - t0
         deg = (indptr[1:] - indptr[:-1])
         self.deg_stats = {"max": int(deg.max()), "mean": float(cfg.num_edges / cfg.num_nodes),
@@ -189,8 +190,9 @@ class Workload:
         # others register afterwards, one at a time (concurrent first-touch pinning of the
         # same tmpfs pages by several processes fails).
         self.rank, self.world, self.device = rank, world, device
-        self._barrier = barrier
-        if rank == 0:
+        self._barrier = barrier if world > 1 else (lambda: None)   # world 1: also under torchrun (reference arm)
+        self.registered = False
+        if rank == 0 and device.type == "cuda":
             from paper_conf_icpp_jiangj024_b200.multigpu import set_interleave
             self.interleaved = world > 1 and set_interleave(True)   # the pages fault in here
             try:
@@ -202,13 +204,13 @@ class Workload:
         train, nb = train_batches(cfg, device)
         self.train, self.num_batches = train, nb
         self._orders = {}
-        self._barrier = barrier
 
     def _register(self):
         n = self.cfg.host_rows * self.cfg.row_bytes
         rc = torch.cuda.cudart().cudaHostRegister(self.table.tensor.data_ptr(), n, 3)
         if int(rc) != 0:
             raise RuntimeError(f"cudaHostRegister(host table, {n} bytes) failed: code {int(rc)}")
+        self.registered = True
 
     def fill_table(self, numeric: bool = False):
         """Rank 0 writes the feature rows (generated on the GPU) into the host table; then
@@ -223,7 +225,8 @@ class Workload:
                 rows = (synth.numeric_feature_rows(s, e, cfg.feat_dim, device=self.device).view(torch.uint8) if numeric
                         else synth.feature_rows(s, e, cfg.row_bytes, device=self.device))
                 self.table.tensor[s:e].copy_(rows)
-        torch.cuda.synchronize(self.device)
+        if self.device.type == "cuda":
+            torch.cuda.synchronize(self.device)
         self._barrier()
         for r in range(1, self.world):
             if self.rank == r:
@@ -232,7 +235,8 @@ class Workload:
         self.t_fill = time.time() - t0
 
     def close(self):
-        torch.cuda.cudart().cudaHostUnregister(self.table.tensor.data_ptr())
+        if self.registered:
+            torch.cuda.cudart().cudaHostUnregister(self.table.tensor.data_ptr())
         self.table.close()
 
     def seeds(self, b, epoch):
@@ -879,10 +883,12 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
         import torch.distributed as dist
-        if os.environ.get("GD_BENCH_SAME_DEVICE") == "1":
-            # test mode for 1-GPU boxes: every rank on cuda:0, gloo (NCCL refuses shared GPUs)
+        if os.environ.get("GD_BENCH_SAME_DEVICE") == "1" or not torch.cuda.is_available():
+            # test modes: every rank on cuda:0 (1-GPU boxes; NCCL refuses shared GPUs) or CPU-only
+            # (the reference arm's multi-rank launch), both over gloo
             local_rank = 0
-            torch.cuda.set_device(0)
+            if torch.cuda.is_available():
+                torch.cuda.set_device(0)
             dist.init_process_group("gloo")
         else:
             torch.cuda.set_device(local_rank)

@@ -144,3 +144,24 @@ def test_numa_helpers():
     ok = mg.set_interleave(True)
     assert ok == (len(nodes) >= 2) or not ok
     mg.set_interleave(False)
+
+
+def test_reference_arm_under_torchrun_world2():
+    """bench.py --impl reference launched like the driver's N>1 runs (torchrun, 2 ranks,
+    127.0.0.1): rank 0 alone runs the oracle and prints one JSON line, the other rank exits 0
+    without work (CPU here: gloo).  Rank 0's single-rank workload must not enter collectives."""
+    import json
+    import subprocess
+    import sys
+    env = dict(os.environ, CUDA_VISIBLE_DEVICES="", OMP_NUM_THREADS="1")
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(_free_port()),
+           os.path.join(ROOT, "bench.py"), "--impl", "reference", "--config", "tiny", "--gpus", "2",
+           "--steps", "3", "--warmup", "1"]
+    p = subprocess.run(cmd, cwd=ROOT, env=env, capture_output=True, text=True, timeout=600)
+    assert p.returncode == 0, p.stderr[-3000:]
+    lines = [json.loads(x) for x in p.stdout.splitlines() if x.startswith("{")]
+    assert len(lines) == 1, p.stdout
+    rec = lines[0]
+    assert rec["impl"] == "reference" and rec["n_gpus"] == 2 and rec["value"] > 0
+    assert rec["e2e"]["h2d_bytes_per_step"] == 0 and rec["cpu_baseline"]["kind"] == "oracle"
