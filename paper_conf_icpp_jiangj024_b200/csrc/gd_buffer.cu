@@ -78,6 +78,7 @@ struct LookupArgs {
 };
 
 __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t n = *a.n_dev;
     const int64_t tile = blockIdx.x;
@@ -192,6 +193,7 @@ __device__ __forceinline__ void ticket_finish(unsigned long long* ticket) {
 }
 
 __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const long long M = *a.mcount;
     const GdCtl c = *a.ctl_in;
@@ -612,6 +614,7 @@ struct ReleaseArgs {
 };
 
 __global__ void __launch_bounds__(kBThreads) k_release(ReleaseArgs a) {
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t n = *a.n_dev;
     const int64_t tile = blockIdx.x;
@@ -686,6 +689,7 @@ struct CompactArgs {
 };
 
 __global__ void __launch_bounds__(kBThreads) k_compact(CompactArgs a) {
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const GdCtl c = *a.ctl_in;
     const bool need = (c.tail + a.n_max > c.base + a.C);
@@ -1358,7 +1362,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     la.st_clear = b->scan.other();
     la.st_clear_n = b->scan.cap;
     la.status = b->hdr.dev_status;
-    k_lookup<<<(unsigned)lt, kBThreads, 0, st>>>(la);
+    GD_CUDA(launch_chain(k_lookup, dim3((unsigned)lt), dim3(kBThreads), 0, st, la));
     GD_DEBUG_AFTER("k_lookup", st);
     b->scan.flip();
 
@@ -1400,7 +1404,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.st_clear = b->scan.other();
     pa.st_clear_n = b->scan.cap;
     pa.status = b->hdr.dev_status;
-    k_pop_assign<<<148 * 2, kBThreads, 0, st>>>(pa);
+    GD_CUDA(launch_chain(k_pop_assign, dim3(148 * 2), dim3(kBThreads), 0, st, pa));
     GD_DEBUG_AFTER("k_pop_assign", st);
     b->scan.flip();
     b->ctl_parity ^= 1;
@@ -1578,7 +1582,7 @@ gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t
     ca.st = b->scan.use();
     ca.st_clear = b->scan.other();
     ca.st_clear_n = b->scan.cap;
-    k_compact<<<148 * 2, kBThreads, 0, st>>>(ca);
+    GD_CUDA(launch_chain(k_compact, dim3(148 * 2), dim3(kBThreads), 0, st, ca));
     GD_DEBUG_AFTER("k_compact", st);
     b->scan.flip();
     b->ctl_parity ^= 1;
@@ -1596,7 +1600,7 @@ gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t
     ra.st_clear = b->scan.other();
     ra.st_clear_n = b->scan.cap;
     ra.status = b->hdr.dev_status;
-    k_release<<<(unsigned)std::max<int64_t>(1, cdiv(n_max, kBTile)), kBThreads, 0, st>>>(ra);
+    GD_CUDA(launch_chain(k_release, dim3((unsigned)std::max<int64_t>(1, cdiv(n_max, kBTile))), dim3(kBThreads), 0, st, ra));
     GD_DEBUG_AFTER("k_release", st);
     b->scan.flip();
     b->ctl_parity ^= 1;

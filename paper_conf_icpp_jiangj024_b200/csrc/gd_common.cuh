@@ -59,6 +59,35 @@ bool is_device_pointer(const void* p);
 // Device address of page-locked (mapped) host memory, nullptr for anything else.
 const void* mapped_host_pointer(const void* p);
 
+// ------------------------------------------------------------ programmatic dependent launch
+// Kernels of a stream-ordered chain (sampling hops, bookkeeping) start with GD_PDL_ENTRY():
+// wait for the preceding kernel's completion and memory flush (griddepcontrol.wait; a no-op
+// without the launch attribute), then let the next kernel of the chain be scheduled
+// (griddepcontrol.launch_dependents), so its launch overlaps this kernel's tail instead of
+// following it.  Nothing may touch memory before the wait.
+#define GD_PDL_ENTRY()                                        \
+    do {                                                      \
+        asm volatile("griddepcontrol.wait;" ::: "memory");    \
+        asm volatile("griddepcontrol.launch_dependents;");    \
+    } while (0)
+
+bool pdl_enabled();   // GD_PDL=0 turns the launch attribute off
+
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_chain(void (*k)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, Args... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = pdl_enabled() ? 1 : 0;
+    return cudaLaunchKernelEx(&cfg, k, args...);
+}
+
 // ------------------------------------------------------------ event timing (host)
 // Pairs of events recorded around kernel groups; summed on read (which syncs).
 struct EventTimer {

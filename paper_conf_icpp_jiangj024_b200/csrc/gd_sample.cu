@@ -75,6 +75,7 @@ __global__ void __launch_bounds__(kThreads) k_seed_intake(const int32_t* __restr
                                                           int64_t N, uint32_t* hk, uint32_t* hv,
                                                           uint32_t mask, int32_t* n_id, int64_t* sizes,
                                                           unsigned int* status) {
+    GD_PDL_ENTRY();
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) sizes[0] = B;
     if (i >= B) return;
@@ -112,6 +113,7 @@ __device__ __forceinline__ void emit_edge(const SampleHopArgs& a, int64_t start,
 template <int G, int NPB>
 __global__ void __launch_bounds__(kThreads) k_sample_hop(SampleHopArgs a) {
     static_assert(NPB <= kThreads && (32 % G) == 0, "tile shape");
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t n_prev = a.sizes[a.hop - 1];
     const int64_t tile = blockIdx.x;
@@ -297,7 +299,7 @@ template <int G, int ITERS>
 static void launch_hop_t(const SampleHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
     constexpr int NPB = kWarps * ITERS * (32 / G);
     const unsigned nt = (unsigned)std::max<int64_t>(1, (n_frontier_max + NPB - 1) / NPB);
-    k_sample_hop<G, NPB><<<nt, kThreads, 0, st>>>(a);
+    launch_chain(k_sample_hop<G, NPB>, dim3(nt), dim3(kThreads), 0, st, a);
 }
 
 template <int G>
@@ -338,6 +340,7 @@ struct RelabelArgs {
 };
 
 __global__ void __launch_bounds__(kThreads) k_relabel_hop(RelabelArgs a) {
+    GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t e_h = a.sizes[a.K + a.hop];
     const int64_t n_prev = a.sizes[a.hop - 1];
@@ -402,6 +405,7 @@ struct ColResolveArgs {
 };
 
 __global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
+    GD_PDL_ENTRY();
     const int hop = blockIdx.y;
     const int64_t e_h = a.sizes[a.K + 1 + hop];
     int32_t* col = a.col[hop];
@@ -613,8 +617,8 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     const uint32_t mask = (uint32_t)(w.hcap - 1);
     const int tslot = g->timer.on ? g->timer.begin(st) : -1;
     GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 2 * w.hcap * sizeof(uint32_t), st));
-    k_seed_intake<<<(unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads)), kThreads, 0, st>>>(
-        seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status);
+    GD_CUDA(launch_chain(k_seed_intake, dim3((unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads))), dim3(kThreads),
+                         0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status));
 
     for (int h = 1; h <= num_hops; ++h) {
         SampleHopArgs a;
@@ -654,7 +658,7 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         r.st_clear = w.scan.other();
         r.st_clear_n = w.scan.cap;
         const int64_t et = std::max<int64_t>(1, ceil_div(emax[h - 1], kEdgesPerTile));
-        k_relabel_hop<<<(unsigned)et, kThreads, 0, st>>>(r);
+        GD_CUDA(launch_chain(k_relabel_hop, dim3((unsigned)et), dim3(kThreads), 0, st, r));
         GD_DEBUG_AFTER("k_relabel_hop", st);
         w.scan.flip();
     }
@@ -669,7 +673,7 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     c.hvals = hv;
     dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
               (unsigned)num_hops);
-    k_col_resolve<<<grid, kThreads, 0, st>>>(c);
+    GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
         GD_DEBUG_AFTER("k_col_resolve", st);
     if (tslot >= 0) g->timer.end(tslot, st);
     GD_CUDA(cudaGetLastError());
