@@ -89,6 +89,7 @@ __global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64
                                                   const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                                                   const int64_t* __restrict__ n_dst_p, int64_t n_alloc,
                                                   __nv_bfloat16* __restrict__ A16) {
+    GD_PDL_ENTRY();
     const int lane = threadIdx.x & 31;
     const int64_t n_dst = *n_dst_p;
     const int64_t n_end = pad64(n_dst, n_alloc);
@@ -166,6 +167,7 @@ __global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64
 __global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, int dp, const int32_t* __restrict__ labels,
                                               const int64_t* __restrict__ n_p, int64_t n_alloc,
                                               __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows) {
+    GD_PDL_ENTRY();
     const int lane = threadIdx.x & 31;
     const int64_t n = *n_p;
     const int64_t n_end = pad64(n, n_alloc);
@@ -195,6 +197,7 @@ __global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C
 
 // loss = mean of loss_rows[0:n] (one block, fixed reduction order: deterministic).
 __global__ void k_loss_sum(const float* __restrict__ loss_rows, const int64_t* __restrict__ n_p, float* __restrict__ loss) {
+    GD_PDL_ENTRY();
     __shared__ float sh[256];
     const int64_t n = *n_p;
     float s = 0.f;
@@ -212,6 +215,7 @@ __global__ void k_loss_sum(const float* __restrict__ loss_rows, const int64_t* _
 // plain stores, so neither a bound-sized memset nor atomics for the own rows.
 __global__ void __launch_bounds__(256) k_scatter_init(const float* __restrict__ dA, int din, const int64_t* __restrict__ n_dst_p,
                                                       const int64_t* __restrict__ n_src_p, float* __restrict__ dX) {
+    GD_PDL_ENTRY();
     const int64_t n_dst = *n_dst_p, n_src = *n_src_p;
     const int dv = din >> 2;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.y + threadIdx.y; i < n_src; i += (int64_t)gridDim.x * blockDim.y) {
@@ -226,6 +230,7 @@ __global__ void __launch_bounds__(256) k_scatter_init(const float* __restrict__ 
 __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ dA, int din,
                                                       const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                                                       const int64_t* __restrict__ n_dst_p, float* __restrict__ dX) {
+    GD_PDL_ENTRY();
     const int lane = threadIdx.x & 31;
     const int64_t n_dst = *n_dst_p;
     const int groups = din >> 2;
@@ -257,6 +262,7 @@ __global__ void __launch_bounds__(256) k_sage_scatter(const float* __restrict__ 
 __global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX, const __nv_bfloat16* __restrict__ H16, int d, int dp,
                                                    const int64_t* __restrict__ n_p, int64_t n_alloc,
                                                    __nv_bfloat16* __restrict__ dZ16) {
+    GD_PDL_ENTRY();
     const int64_t n = *n_p;
     const int64_t n_end = pad64(n, n_alloc);
     const int dv = d >> 2;
@@ -284,6 +290,7 @@ __global__ void __launch_bounds__(256) k_relu_grad(const float* __restrict__ dX,
 constexpr int kColsumChunks = 256;
 __global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __restrict__ dZ16, int d, int ld,
                                                      const int64_t* __restrict__ n_p, float* __restrict__ part) {
+    GD_PDL_ENTRY();
     __shared__ float sh[8][33];
     const int64_t n = *n_p;
     const int64_t per = (n + gridDim.y - 1) / gridDim.y;
@@ -306,6 +313,7 @@ __global__ void __launch_bounds__(256) k_colsum_part(const __nv_bfloat16* __rest
 
 __global__ void __launch_bounds__(256) k_colsum_final(const float* __restrict__ part, int d, int nchunk,
                                                       float* __restrict__ out) {
+    GD_PDL_ENTRY();
     __shared__ float sh[8][33];
     const int c = blockIdx.x * 32 + threadIdx.x;
     float s = 0.f;
@@ -321,12 +329,14 @@ __global__ void __launch_bounds__(256) k_colsum_final(const float* __restrict__ 
 }
 
 __global__ void k_sgd(float* __restrict__ p, const float* __restrict__ g, int64_t n, float step) {
+    GD_PDL_ENTRY();
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n; k += (int64_t)gridDim.x * blockDim.x)
         p[k] = fmaf(-step, g[k], p[k]);
 }
 
 // W16[r, c] = bf16(W[r, c]) for c < d, 0 for d <= c < dp (rows of W at stride d).
 __global__ void k_to_bf16(const float* __restrict__ src, __nv_bfloat16* __restrict__ dst, int64_t rows, int d, int dp) {
+    GD_PDL_ENTRY();
     for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < rows * dp; k += (int64_t)gridDim.x * blockDim.x) {
         const int64_t r = k / dp;
         const int c = (int)(k - r * dp);
@@ -446,9 +456,11 @@ gd_status gd_sage_create(int32_t num_layers, const int32_t* dims, const float* c
         max_dout = std::max(max_dout, l.dout);
     }
     SA(s->colsum_part, (size_t)kColsumChunks * max_dout * sizeof(float));
-    SA(s->gemm_counter, sizeof(unsigned int));
+    SA(s->gemm_counter, 2 * sizeof(unsigned int));
     if (const char* e = std::getenv("GD_SAGE_TIMING")) s->timer.on = std::atoi(e) != 0;
 #undef SA
+    if (cudaMemset(s->gemm_counter, 0, 2 * sizeof(unsigned int)) != cudaSuccess)
+        return fail(cuda_error(cudaGetLastError(), "gd_sage_create: memset"));
     for (int j = 0; j < num_layers; ++j) {      // pad columns of dZ16 (the DA GEMM's K) start and stay zero
         const SageLayer& l = s->layers[j];
         cudaError_t e = cudaMemset(l.dZ16, 0, l.n_dst_max * l.dp * sizeof(__nv_bfloat16));
@@ -512,12 +524,12 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         const int64_t* n_dst = sizes + (h - 1);
         ph_begin();
         if (j == 0)
-            k_sage_agg<float><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const float*)x, ldx, l.din, rowptr[h - 1],
-                                                                          col[h - 1], n_dst, l.n_dst_max, l.A16);
+            GD_CUDA(launch_chain(k_sage_agg<float>, dim3(grid_for(l.n_dst_max * 32)), dim3(256), 0, st, (const float*)x, ldx, l.din, rowptr[h - 1],
+                                                                          col[h - 1], n_dst, l.n_dst_max, l.A16));
         else
-            k_sage_agg<__nv_bfloat16><<<grid_for(l.n_dst_max * 32), 256, 0, st>>>((const __nv_bfloat16*)x, ldx, l.din,
+            GD_CUDA(launch_chain(k_sage_agg<__nv_bfloat16>, dim3(grid_for(l.n_dst_max * 32)), dim3(256), 0, st, (const __nv_bfloat16*)x, ldx, l.din,
                                                                                   rowptr[h - 1], col[h - 1], n_dst,
-                                                                                  l.n_dst_max, l.A16);
+                                                                                  l.n_dst_max, l.A16));
         GD_DEBUG_AFTER("k_sage_agg", st);
         ph_end(kAgg[j]);
         ph_begin();
@@ -539,9 +551,9 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
     // ---- loss
     SageLayer& top = s->layers[L - 1];
     ph_begin();
-    k_xent<<<grid_for(top.n_dst_max * 32), 256, 0, st>>>(top.Z, top.dout, top.dp, labels, sizes, top.n_dst_max, top.dZ16,
-                                                         s->loss_rows);
-    k_loss_sum<<<1, 256, 0, st>>>(s->loss_rows, sizes, loss);
+    GD_CUDA(launch_chain(k_xent, dim3(grid_for(top.n_dst_max * 32)), dim3(256), 0, st, top.Z, top.dout, top.dp, labels, sizes, top.n_dst_max, top.dZ16,
+                                                         s->loss_rows));
+    GD_CUDA(launch_chain(k_loss_sum, dim3(1), dim3(256), 0, st, s->loss_rows, sizes, loss));
     GD_DEBUG_AFTER("k_xent", st);
     ph_end("loss");
     // ---- backward
@@ -563,8 +575,8 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
             GD_DEBUG_AFTER("k_umma_gemm<DW>", st);
         }
         const unsigned strips = (unsigned)((l.dout + 31) / 32);
-        k_colsum_part<<<dim3(strips, kColsumChunks), rows_blk, 0, st>>>(l.dZ16, l.dout, l.dp, n_dst, s->colsum_part);
-        k_colsum_final<<<strips, rows_blk, 0, st>>>(s->colsum_part, l.dout, kColsumChunks, s->grads + l.b_off);
+        GD_CUDA(launch_chain(k_colsum_part, dim3(dim3(strips, kColsumChunks)), dim3(rows_blk), 0, st, l.dZ16, l.dout, l.dp, n_dst, s->colsum_part));
+        GD_CUDA(launch_chain(k_colsum_final, dim3(strips), dim3(rows_blk), 0, st, s->colsum_part, l.dout, kColsumChunks, s->grads + l.b_off));
         GD_DEBUG_AFTER("k_colsum", st);
         ph_end(kDw[j]);
         if (j == 0) break;
@@ -579,12 +591,12 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
         }
         ph_end(kDa[j]);
         ph_begin();
-        k_scatter_init<<<grid_for(l.n_src_max * 8), rows_blk, 0, st>>>(l.dA, l.din, n_dst, sizes + h, l.dX);
-        k_sage_scatter<<<grid_for(l.n_dst_max * 32), 256, 0, st>>>(l.dA, l.din, rowptr[h - 1], col[h - 1], n_dst, l.dX);
+        GD_CUDA(launch_chain(k_scatter_init, dim3(grid_for(l.n_src_max * 8)), dim3(rows_blk), 0, st, l.dA, l.din, n_dst, sizes + h, l.dX));
+        GD_CUDA(launch_chain(k_sage_scatter, dim3(grid_for(l.n_dst_max * 32)), dim3(256), 0, st, l.dA, l.din, rowptr[h - 1], col[h - 1], n_dst, l.dX));
         GD_DEBUG_AFTER("k_sage_scatter", st);
         SageLayer& prev = s->layers[j - 1];   // its output (H16) is this layer's input
-        k_relu_grad<<<grid_for(prev.n_dst_max * 8), rows_blk, 0, st>>>(l.dX, prev.H16, prev.dout, prev.dp, sizes + h,
-                                                                       prev.n_dst_max, prev.dZ16);
+        GD_CUDA(launch_chain(k_relu_grad, dim3(grid_for(prev.n_dst_max * 8)), dim3(rows_blk), 0, st, l.dX, prev.H16, prev.dout, prev.dp, sizes + h,
+                                                                       prev.n_dst_max, prev.dZ16));
         GD_DEBUG_AFTER("k_relu_grad", st);
         ph_end(kSc[j]);
     }
@@ -603,10 +615,10 @@ gd_status gd_sage_apply_sgd(gd_sage* s, float lr, float grad_scale, void* stream
     if (!s || s->hdr.magic != kMagicSage) return set_error(GD_ERR_INVALID, "gd_sage_apply_sgd: bad handle");
     DeviceGuard guard(s->hdr.device);
     cudaStream_t st = (cudaStream_t)stream_v;
-    k_sgd<<<grid_for(s->nparams), 256, 0, st>>>(s->params, s->grads, s->nparams, lr * grad_scale);
+    GD_CUDA(launch_chain(k_sgd, dim3(grid_for(s->nparams)), dim3(256), 0, st, s->params, s->grads, s->nparams, lr * grad_scale));
     for (const SageLayer& l : s->layers)
-        k_to_bf16<<<grid_for(2 * l.din * l.dp), 256, 0, st>>>(s->params + l.w_off, s->W16 + l.w16_off, 2 * l.din, l.dout,
-                                                              l.dp);
+        GD_CUDA(launch_chain(k_to_bf16, dim3(grid_for(2 * l.din * l.dp)), dim3(256), 0, st, s->params + l.w_off, s->W16 + l.w16_off, 2 * l.din, l.dout,
+                                                              l.dp));
     GD_CUDA(cudaGetLastError());
     return GD_OK;
 }
@@ -651,7 +663,8 @@ gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const voi
         return set_error(GD_ERR_INVALID, "gd_debug_umma_gemm: strides / extents must be multiples of 8, bases 16-byte aligned");
     cudaStream_t st = (cudaStream_t)stream;
     unsigned int* counter = nullptr;
-    GD_CUDA(cudaMallocAsync((void**)&counter, sizeof(unsigned int), st));
+    GD_CUDA(cudaMallocAsync((void**)&counter, 2 * sizeof(unsigned int), st));
+    GD_CUDA(cudaMemsetAsync(counter, 0, 2 * sizeof(unsigned int), st));
     umma::Args a = gemm_args((const __nv_bfloat16*)A, lda, (const __nv_bfloat16*)B, ldb, C, ldc, rows_dev, counter);
     a.c_bf16 = c_bf16;
     a.relu = relu;

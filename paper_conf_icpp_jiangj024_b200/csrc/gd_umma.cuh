@@ -44,6 +44,8 @@
 
 #include <algorithm>
 
+#include "gd_common.cuh"   // GD_PDL_ENTRY, launch_chain
+
 namespace gd {
 namespace umma {
 
@@ -67,7 +69,8 @@ struct Args {
     int n_valid;                 // B's extent along N (multiple of 8; zero-filled past it)
     int n_store;                 // output columns written
     int bn;                      // N tile (multiple of 16, <= 256; multiple of 64 when B is MN-major)
-    unsigned int* counter;       // device work counter, zero at launch (units are fetched dynamically)
+    unsigned int* counter;       // device words {work, exits}: zero at launch; the last CTA to
+                                 // leave re-zeroes them, so back-to-back launches need no memset
 };
 
 __device__ __forceinline__ uint32_t smem_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -216,12 +219,24 @@ __device__ __forceinline__ bool fetch_unit(Unit& c, const Args& a, int64_t rows,
     }
 }
 
+// The last CTA of the grid to leave re-zeroes the work counter (every CTA has fetched its
+// last unit by then), so the next launch starts from zero without a memset between kernels.
+__device__ __forceinline__ void cta_exit(unsigned int* counter) {
+    __threadfence();
+    if (atomicAdd(counter + 1, 1u) == gridDim.x - 1) {
+        counter[0] = 0u;
+        counter[1] = 0u;
+        __threadfence();
+    }
+}
+
 template <int MODE, bool OUT_BF16, bool RELU>
 __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
                                                    const __grid_constant__ CUtensorMap tmB, Args a, int nt, int splits,
                                                    int vec_ok) {
     constexpr bool A_MN = MODE == DW;
     constexpr bool B_MN = MODE != DA;
+    GD_PDL_ENTRY();   // the operands are the previous kernel's outputs
     extern __shared__ uint8_t smem_raw[];
     // SWIZZLE_128B tiles need 1024-byte aligned bases
     uint8_t* smem = smem_raw + ((1024 - (smem_u32(smem_raw) & 1023)) & 1023);
@@ -241,7 +256,10 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
     __shared__ int64_t first_unit;
     if (threadIdx.x == 0) first_unit = fetch_unit<MODE>(cm, a, rows, nt, splits) ? cm.u : -1;
     __syncthreads();
-    if (first_unit < 0) return;         // no work left for this CTA
+    if (first_unit < 0) {               // no work left for this CTA
+        if (threadIdx.x == 0) cta_exit(a.counter);
+        return;
+    }
     decode_unit<MODE>(cm, first_unit, a, rows, nt, splits);
     const int64_t m_valid = MODE == DW ? a.m_valid : rows;
     uint32_t nc = 32;                   // columns of one accumulator buffer
@@ -276,6 +294,9 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
             const uint32_t stage_bytes = (uint32_t)(A_STAGE + b_stage);
             Unit ld = cm;
             bool ld_ok = true;
+            // the next unit id is fetched one unit ahead, so the atomic's round trip hides
+            // behind the current unit's loads instead of stalling the producer
+            unsigned int next_u = atomicAdd(a.counter, 1u);
             int64_t uq[8];                 // units fetched by the load cursor, not yet reached by the MMAs
             uint32_t uq_head = 0, uq_tail = 0;
             uint32_t it_ld = 0, it_cm = 0, u_local = 0;
@@ -294,8 +315,14 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
                     for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
                 ++it_ld;
                 if (++ld.kb == ld.nkb) {
-                    ld_ok = fetch_unit<MODE>(ld, a, rows, nt, splits);
-                    if (ld_ok) uq[uq_tail++ & 7] = ld.u;
+                    int r;
+                    while ((r = decode_unit<MODE>(ld, (int64_t)next_u, a, rows, nt, splits)) == 0)   // empty DW slice
+                        next_u = atomicAdd(a.counter, 1u);
+                    ld_ok = r > 0;
+                    if (ld_ok) {
+                        uq[uq_tail++ & 7] = ld.u;
+                        next_u = atomicAdd(a.counter, 1u);
+                    }
                 }
             };
             for (int s = 0; s < STAGES - 1 && ld_ok; ++s) issue_load();
@@ -368,6 +395,7 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
         asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
         asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;\n" ::"r"(tmem), "r"(2 * nc));
     }
+    if (threadIdx.x == 0) cta_exit(a.counter);
 }
 
 inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 8 + 16; }
@@ -393,7 +421,7 @@ inline cudaError_t make_map(CUtensorMap* m, const void* base, uint64_t inner, ui
 
 // Host launcher.  rows_max: host bound of *rows_dev (grid sizing, tensor extents).  n_total:
 // output columns (split into <= 256-wide tiles).  splits: DW reduction slices per tile.
-// a.counter: a device word the launch may use (zeroed here, on the stream).
+// a.counter: two device words, zero before the first launch (each launch leaves them zero).
 inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_total, int splits, cudaStream_t st) {
     Args a = a0;
     const bool b_mn = mode != DA;
@@ -422,14 +450,12 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
     const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
     if (units <= 0) return cudaSuccess;
     if (!a.counter) return cudaErrorInvalidValue;
-    e = cudaMemsetAsync(a.counter, 0, sizeof(unsigned int), st);
-    if (e != cudaSuccess) return e;
     const unsigned grid = (unsigned)std::min<int64_t>(units, (int64_t)148 * per_sm);
     const int vec_ok = mode == FWD && a.c_bf16 ? (a.ldc % 8 == 0) : (a.ldc % 4 == 0);
 #define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
     do {                                                                                              \
         e = cudaFuncSetAttribute(k_umma_gemm<M, BF, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        if (e == cudaSuccess) k_umma_gemm<M, BF, RL><<<grid, 288, smem, st>>>(tmA, tmB, a, nt, splits, vec_ok); \
+        if (e == cudaSuccess) e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(288), smem, st, tmA, tmB, a, nt, splits, vec_ok); \
     } while (0)
     if (mode == FWD) {
         if (a.c_bf16 && a.relu) GD_UMMA_LAUNCH(FWD, true, true);
