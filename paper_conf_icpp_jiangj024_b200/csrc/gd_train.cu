@@ -163,11 +163,15 @@ __global__ void __launch_bounds__(256) k_sage_agg(const T* __restrict__ x, int64
 
 // Softmax cross entropy of the logits (z + b, from the FWD epilogue, row stride dp), warp
 // per seed row: loss_rows[i] = lse - z[label]; dZ16[i] = (softmax - onehot) / n0 for the C
-// classes, 0 in the pad columns [C, dp).
+// classes, 0 in the pad columns [C, dp).  Also zeroes the gradient buffer (the DW GEMMs
+// red.add into it), so no memset breaks the train stream's dependent-launch chain.
 __global__ void __launch_bounds__(256) k_xent(const float* __restrict__ Z, int C, int dp, const int32_t* __restrict__ labels,
                                               const int64_t* __restrict__ n_p, int64_t n_alloc,
-                                              __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows) {
+                                              __nv_bfloat16* __restrict__ dZ16, float* __restrict__ loss_rows,
+                                              float* __restrict__ grads, int64_t nparams) {
     GD_PDL_ENTRY();
+    for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < nparams; k += (int64_t)gridDim.x * blockDim.x)
+        grads[k] = 0.f;
     const int lane = threadIdx.x & 31;
     const int64_t n = *n_p;
     const int64_t n_end = pad64(n, n_alloc);
@@ -551,13 +555,12 @@ gd_status gd_sage_step(gd_sage* s, const int64_t* const* rowptr, const int32_t* 
     // ---- loss
     SageLayer& top = s->layers[L - 1];
     ph_begin();
-    GD_CUDA(launch_chain(k_xent, dim3(grid_for(top.n_dst_max * 32)), dim3(256), 0, st, top.Z, top.dout, top.dp, labels, sizes, top.n_dst_max, top.dZ16,
-                                                         s->loss_rows));
+    GD_CUDA(launch_chain(k_xent, dim3(grid_for(top.n_dst_max * 32)), dim3(256), 0, st, top.Z, top.dout, top.dp, labels, sizes,
+                         top.n_dst_max, top.dZ16, s->loss_rows, s->grads, s->nparams));
     GD_CUDA(launch_chain(k_loss_sum, dim3(1), dim3(256), 0, st, s->loss_rows, sizes, loss));
     GD_DEBUG_AFTER("k_xent", st);
     ph_end("loss");
     // ---- backward
-    GD_CUDA(cudaMemsetAsync(s->grads, 0, (size_t)s->nparams * sizeof(float), st));   // dW accumulates by red.add
     for (int j = L - 1; j >= 0; --j) {
         SageLayer& l = s->layers[j];
         const int h = l.hop;
