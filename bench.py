@@ -476,16 +476,26 @@ def run_ours(args, rank, world, local_rank):
     # ---- the timed configuration's output rows, checked by their closed form (P5):
     # out[i] == table row (n_id[i] mod P) for the last Q + 1 batches of the timed region
     # (extracted back to back, no host sync between them)
-    rows_check = {"batches": 0, "rows": 0, "ok": True}
+    # (and, when the host CSR is at hand, their sampled node lists against the oracle's)
+    rows_check = {"batches": 0, "rows": 0, "ok": True, "n_id_vs_oracle": None}
     torch.cuda.synchronize(dev)
     for j in range(max(off + W, off + W + K - RING), off + W + K):
         s_ = j % RING
         dones[s_].synchronize()
         n_j = int(sizes_log[j][len(fan)].item())
-        ids = outs[s_].n_id[:n_j].long().cpu() % cfg.host_rows
+        n_id_j = outs[s_].n_id[:n_j].cpu()
+        ids = n_id_j.long() % cfg.host_rows
         want = wl.table.tensor.index_select(0, ids)
         got = feats[s_][:n_j].view(torch.uint8).reshape(n_j, cfg.row_bytes).cpu()
         rows_check["ok"] &= bool(torch.equal(got, want))
+        if wl.host_indptr is not None:
+            from oracle import oracle as O
+            b_, ep_ = sched[j % len(sched)]
+            ref = O.sample(wl.host_indptr, wl.host_indices, wl.seeds(b_, ep_).cpu().numpy(), fan, synth.RNG_SEED,
+                           batch_ids[j])
+            same = bool(np.array_equal(n_id_j.numpy(), ref.n_id))
+            rows_check["n_id_vs_oracle"] = same if rows_check["n_id_vs_oracle"] is None else (
+                rows_check["n_id_vs_oracle"] and same)
         rows_check["batches"] += 1
         rows_check["rows"] += n_j
     log(f"pipelined rows check: {rows_check}")
