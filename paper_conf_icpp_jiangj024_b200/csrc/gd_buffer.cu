@@ -32,6 +32,7 @@ constexpr int kBItems = 8;
 constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
 constexpr int kStageRing = 4;    // pinned chunk buffers of the copy-engine staging ring
+constexpr int kJobRing = 1024;   // host-function argument slots of the staged chunks
 constexpr int kTimedPairs = 5;   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
@@ -792,7 +793,7 @@ static void buffer_free(gd_buffer* b) {
     b->scan.release();
     b->timer.destroy();
     for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_ring,
-                    &b->ev_s0})
+                    &b->ev_s0, &b->ev_job})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
     for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk, b->ev_S})
@@ -1018,7 +1019,11 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
                 for (auto& e : b->ev_ring) GD_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
                 GD_CUDA(cudaEventCreateWithFlags(&b->ev_chunk, cudaEventDisableTiming));
             }
-            b->jobs.assign((size_t)b->D * cdiv(b->n_max, rows), ChunkJob());
+            if (b->ev_job.empty()) {
+                b->ev_job.assign(kJobRing, nullptr);
+                for (auto& e : b->ev_job) GD_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+            }
+            b->jobs.assign((size_t)kJobRing, ChunkJob());
         }
     }
     b->host_threads = host_threads;
@@ -1328,11 +1333,6 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // every stream is done with trip / host-list slot d (batch - D)
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));
     if (staged) {
-        // The host-side arguments of slot d (StagedSlot, chunk jobs) are rewritten below at
-        // enqueue time; the host-gather callbacks of batch - D read them when stream H reaches
-        // them, so they must have run first.  This bounds how far the caller's thread runs
-        // ahead of the host gather (D batches), not the device.
-        if (b->batch_counter >= b->D) GD_CUDA(cudaEventSynchronize(b->ev_H[d]));
         adapt_alpha(b, (int)((b->batch_counter + b->D - 2) % b->D));
         ss->batch = b->batch_counter;
     }
@@ -1486,13 +1486,19 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
             // is done, gathers into it; C copies it to dstage[d] at rank offset lo
             stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
             const int64_t ch = b->stage_chunk_rows, nch = cap > 0 ? cdiv(cap, ch) : 0;
-            const int64_t maxch = cdiv(b->n_max, ch);
             const int t_ce = timed ? b->timer.begin(b->side_c) : -1;
             GD_CUDA(cudaEventRecord(b->ev_s0[d], b->side_h));   // staged path starts (after its waits)
             if (nch == 0) ss->cpu_ms = 0;
             for (int64_t c = 0; c < nch; ++c) {
                 const int r = (int)(b->chunk_counter++ % kStageRing);
-                ChunkJob* j = &b->jobs[(size_t)d * maxch + c];
+                // The callback reads its arguments when stream H reaches it, possibly many
+                // batches after this enqueue: each chunk gets its own argument slot, reused
+                // only after its previous callback ran (a host wait that needs the caller to
+                // be kJobRing chunks ahead of the host gather).
+                const uint64_t jk = b->job_counter++;
+                const size_t js = (size_t)(jk % kJobRing);
+                if (jk >= (uint64_t)kJobRing) GD_CUDA(cudaEventSynchronize(b->ev_job[js]));
+                ChunkJob* j = &b->jobs[js];
                 j->ss = ss;
                 j->lo = c * ch;
                 j->hi = std::min<int64_t>(cap, (c + 1) * ch);
@@ -1500,8 +1506,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
                 j->first = c == 0;
                 GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_ring[r], 0));
                 GD_CUDA(cudaLaunchHostFunc(b->side_h, chunk_gather_cb, j));
-                GD_CUDA(cudaEventRecord(b->ev_chunk, b->side_h));
-                GD_CUDA(cudaStreamWaitEvent(b->side_c, b->ev_chunk, 0));
+                GD_CUDA(cudaEventRecord(b->ev_job[js], b->side_h));
+                GD_CUDA(cudaStreamWaitEvent(b->side_c, b->ev_job[js], 0));
                 GD_CUDA(cudaMemcpyAsync((void*)(stage_dev + j->lo * b->R), j->buf, (size_t)(j->hi - j->lo) * b->R,
                                         cudaMemcpyHostToDevice, b->side_c));
                 GD_CUDA(cudaEventRecord(b->ev_ring[r], b->side_c));

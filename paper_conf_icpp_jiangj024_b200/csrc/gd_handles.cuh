@@ -137,9 +137,14 @@ struct gd_buffer {
     int64_t stage_chunk_rows = 0;
     uint8_t* ring_mem = nullptr;         // pinned [kStageRing x stage_chunk_rows x R]
     uint64_t chunk_counter = 0;
+    // host-function arguments of the staged chunks: a ring indexed by a global job counter, so
+    // a pending callback's arguments are never rewritten by a later batch's enqueue (slot k is
+    // reused only after ev_job[k], recorded after its callback, has fired)
+    std::vector<cudaEvent_t> ev_job;
+    uint64_t job_counter = 0;
     std::vector<cudaEvent_t> ev_ring;    // [kStageRing] copy out of ring buffer r done
     cudaEvent_t ev_chunk = nullptr;      // chunk gathered (re-recorded per chunk)
-    std::vector<struct ChunkJob> jobs;   // [D x max chunks] host-function arguments
+    std::vector<struct ChunkJob> jobs;   // [kJobRing] host-function arguments (see ev_job)
     // f2: NVLink peer feature buffers (subprocesses reuse rows another has loaded).
     // ready[s] = (epoch << 32) | node once slot s holds that node's row (published after
     // the batch's copies joined), kReadyNone from the moment the slot is reassigned.
