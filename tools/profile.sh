@@ -15,6 +15,6 @@ timeout 1200 ncu --metrics $METRICS --clock-control none --kernel-name-base func
 echo "launches rc=$?"
 for K in "$@"; do
   timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base function \
-      -k regex:"^$K\$" -s 8 -c 1 -o $OUT/prof_${K}_$CFG -f python bench.py $ARGS > $OUT/ncu_${K}_$CFG.log 2>&1
+      -k regex:"^$K\$" -s ${SKIP:-8} -c 1 -o $OUT/prof_${K}_$CFG -f python bench.py $ARGS > $OUT/ncu_${K}_$CFG.log 2>&1
   echo "$K rc=$?"
 done
