@@ -13,8 +13,11 @@
 struct gd_workspace {
     uint32_t magic = 0x47445753u;   // "GDWS"
     int device = 0;
-    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident)
+    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident); all empty
+                                    // between calls (each call clears the slots it used)
     int64_t hcap = 0;               // power of two >= 1.25 x max_nodes[K]
+    int32_t* slot_of = nullptr;     // [slot_cap] hash slot of n_id[i] (for that clearing)
+    int64_t slot_cap = 0;
     int32_t* seeds_ws = nullptr;    // staging for host seed arrays
     int64_t seeds_cap = 0;
     gd::ScanState scan;

@@ -74,7 +74,7 @@ __device__ __forceinline__ uint32_t hash_insert(uint32_t* __restrict__ hk, uint3
 __global__ void __launch_bounds__(kThreads) k_seed_intake(const int32_t* __restrict__ seeds, int64_t B,
                                                           int64_t N, uint32_t* hk, uint32_t* hv,
                                                           uint32_t mask, int32_t* n_id, int64_t* sizes,
-                                                          unsigned int* status) {
+                                                          int32_t* slot_of, unsigned int* status) {
     GD_PDL_ENTRY();
     const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     if (i == 0) sizes[0] = B;
@@ -90,6 +90,7 @@ __global__ void __launch_bounds__(kThreads) k_seed_intake(const int32_t* __restr
         const uint32_t old = atomicCAS(hk + h, kEmpty, (uint32_t)v);
         if (old == kEmpty) {
             hv[h] = (uint32_t)i;   // finalised local id = position
+            slot_of[i] = (int32_t)h;
             return;
         }
         if (old == (uint32_t)v) {
@@ -334,6 +335,7 @@ struct RelabelArgs {
     int K;
     uint32_t* hkeys;
     uint32_t* hvals;
+    int32_t* slot_of;
     unsigned long long* st;
     unsigned long long* st_clear;
     int64_t st_clear_n;
@@ -393,6 +395,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_hop(RelabelArgs a) {
             const int64_t local = n_prev + rank;
             a.n_id[local] = (int32_t)a.hkeys[slot[k]];
             a.hvals[slot[k]] = (uint32_t)local;
+            a.slot_of[local] = (int32_t)slot[k];
         }
     }
 }
@@ -412,6 +415,20 @@ __global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
     for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_h;
          e += (int64_t)gridDim.x * blockDim.x)
         col[e] = (int32_t)__ldg(a.hvals + col[e]);
+}
+
+// Empties exactly the hash slots this call used: every claimed key is a node of n_id (a seed
+// or a neighbour, appended at its first occurrence), whose slot k_seed_intake /
+// k_relabel_hop recorded.  Replaces a memset of the whole table per call.
+__global__ void __launch_bounds__(kThreads) k_hash_clear(const int32_t* __restrict__ slot_of, const int64_t* __restrict__ n_p,
+                                                         uint32_t* hk, uint32_t* hv) {
+    GD_PDL_ENTRY();
+    const int64_t n = *n_p;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+        const int32_t s = slot_of[i];
+        hk[s] = kEmpty;
+        hv[s] = kEmpty;
+    }
 }
 
 __global__ void k_validate_csr(const int64_t* indptr, const int32_t* indices, int64_t N, int64_t E,
@@ -519,6 +536,7 @@ gd_status gd_graph_destroy(gd_graph* g) {
     if (g->indptr) cudaFree(g->indptr);
     if (g->indices) cudaFree(g->indices);
     if (g->ws.hash) cudaFree(g->ws.hash);
+    if (g->ws.slot_of) cudaFree(g->ws.slot_of);
     if (g->ws.seeds_ws) cudaFree(g->ws.seeds_ws);
     if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
     g->ws.scan.release();
@@ -541,6 +559,7 @@ gd_status gd_workspace_destroy(gd_workspace* w) {
     if (w->magic != 0x47445753u) return set_error(GD_ERR_INVALID, "gd_workspace_destroy: bad handle");
     DeviceGuard guard(w->device);
     if (w->hash) cudaFree(w->hash);
+    if (w->slot_of) cudaFree(w->slot_of);
     if (w->seeds_ws) cudaFree(w->seeds_ws);
     w->scan.release();
     w->magic = 0;
@@ -585,7 +604,16 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         w.hash = nullptr;
         w.hcap = 0;
         GD_CUDA(cudaMalloc(&w.hash, 2 * want * sizeof(uint32_t)));
+        GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 2 * want * sizeof(uint32_t), st));   // empty; calls keep it so
         w.hcap = want;
+    }
+    if (nmax[num_hops] > w.slot_cap) {
+        if (w.slot_of) cudaFree(w.slot_of);
+        w.slot_of = nullptr;
+        w.slot_cap = 0;
+        GD_CUDA(cudaMalloc(&w.slot_of, std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t)));
+        GD_CUDA(cudaMemsetAsync(w.slot_of, 0, std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t), st));
+        w.slot_cap = nmax[num_hops];
     }
     int64_t tiles = 1;
     for (int h = 0; h < num_hops; ++h) {
@@ -616,9 +644,8 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     uint32_t* hv = w.hash + w.hcap;
     const uint32_t mask = (uint32_t)(w.hcap - 1);
     const int tslot = g->timer.on ? g->timer.begin(st) : -1;
-    GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 2 * w.hcap * sizeof(uint32_t), st));
     GD_CUDA(launch_chain(k_seed_intake, dim3((unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads))), dim3(kThreads),
-                         0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, g->hdr.dev_status));
+                         0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, w.slot_of, g->hdr.dev_status));
 
     for (int h = 1; h <= num_hops; ++h) {
         SampleHopArgs a;
@@ -654,6 +681,7 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         r.K = num_hops;
         r.hkeys = hk;
         r.hvals = hv;
+        r.slot_of = w.slot_of;
         r.st = w.scan.use();
         r.st_clear = w.scan.other();
         r.st_clear_n = w.scan.cap;
@@ -674,6 +702,8 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
               (unsigned)num_hops);
     GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
+    GD_CUDA(launch_chain(k_hash_clear, dim3((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(nmax[num_hops], kThreads)))),
+                         dim3(kThreads), 0, st, (const int32_t*)w.slot_of, (const int64_t*)(out->sizes + num_hops), hk, hv));
         GD_DEBUG_AFTER("k_col_resolve", st);
     if (tslot >= 0) g->timer.end(tslot, st);
     GD_CUDA(cudaGetLastError());
