@@ -58,6 +58,8 @@ def parse():
     p.add_argument("--prewarm-max", type=int, default=400,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
+    p.add_argument("--window", type=int, default=0, help="also report batches/s per window of this many timed steps "
+                   "(device events on the caller's stream; sustained-rate evidence)")
     p.add_argument("--pipeline-sweep", default="", help="f1: 'samplers:reorder,...' SET pipeline runs "
                    "(concurrent sampler streams, out-of-order extraction), results under 'pipeline'")
     p.add_argument("--miss-sweep", default="", help="tuning: 'threads:share:zc_blocks:pull_blocks,...' timed "
@@ -451,8 +453,13 @@ def run_ours(args, rank, world, local_rank):
     ev1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local_rank) as clk:
         ev0.record(main)
+        win_ev = []
         for j in range(off + W, off + W + K):
             step(j)
+            if args.window and (j - off - W + 1) % args.window == 0:
+                e_ = torch.cuda.Event(enable_timing=True)
+                e_.record(main)
+                win_ev.append(e_)
         main.wait_event(dones[(off + W + K - 1) % RING])  # the last batch's rows are all in `out`
         if rel_live[0]:
             main.wait_event(ev_rel)                          # ... and the last release is done
@@ -466,6 +473,10 @@ def run_ours(args, rank, world, local_rank):
     train_timing[0] = False
     ms = ev0.elapsed_time(ev1)
     ms_max = max_over_ranks(ms, dev)
+    windows = None
+    if win_ev:   # caller-stream progress per window (the miss stream trails it by < Q batches)
+        marks = [ev0] + win_ev
+        windows = [round(args.window / (a_.elapsed_time(b_) / 1e3), 1) for a_, b_ in zip(marks, marks[1:])]
     tg = g.timing_read()
     tb = buf.timing_read()
     st = stats[off + W:off + W + K].sum(0).cpu().tolist()
@@ -753,6 +764,7 @@ def run_ours(args, rank, world, local_rank):
                       "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
         "parity": parity,
         "rows_check": rows_check,
+        "windows": windows,
         "sweep": sweep or None,
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
