@@ -12,14 +12,14 @@
 // ("units"; DW units are (tile, row slice) pairs), fetched from a per-launch atomic counter
 // (a CTA that only gets an SM after the others finished finds no work and leaves, so SMs held
 // by concurrent kernels of the SET pipeline do not stretch the grid), and warp-specialised
-// (288 threads):
+// (32 x (1 + EPI_WARPS) threads):
 //   warp 0, lane 0: producer + MMA issuer.  It keeps STAGES-1 k-blocks of TMA loads in flight
 //     ahead of the MMAs, across unit boundaries (TMA completes a stage's "full" mbarrier with
 //     its byte count; the tcgen05.commit of the MMAs that read a stage arrives on its "empty"
 //     mbarrier, which lets the stage be refilled), and accumulates unit u into TMEM buffer
 //     u % 2, committing the unit's last k-block to acc_full[u % 2].
-//   warps 1-8: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per thread)
-//     of the finished buffer, alternate 32-column chunks per warp pair (tcgen05.ld, 32
+//   warps 1..EPI_WARPS: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per thread)
+//     of the finished buffer, every (EPI_WARPS / 4)-th 32-column chunk (tcgen05.ld, 32
 //     columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
 //     (fp32 / bf16 stores, or fp32 vector red.add for DW), then arrives on acc_empty[u % 2].
 //     The next unit's MMAs run meanwhile in the other buffer.
@@ -52,6 +52,8 @@ namespace umma {
 constexpr int BM = 128;
 constexpr int BK = 64;
 constexpr int STAGES = 4;
+constexpr int EPI_WARPS = 8;                  // epilogue warps (2 per TMEM lane quarter; 16 measured no faster)
+constexpr int THREADS = 32 * (1 + EPI_WARPS);
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 enum Mode { FWD = 0, DA = 1, DW = 2 };
@@ -117,7 +119,7 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
                                          int h, int lane, bool vec_ok) {
     const int64_t row = rbase + lane;
     const bool row_ok = row < m_valid;
-    for (int c0 = 32 * h; c0 < bn; c0 += 64) {
+    for (int c0 = 32 * h; c0 < bn; c0 += 32 * (EPI_WARPS / 4)) {
         uint32_t r[32];
         asm volatile(
             "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
@@ -231,7 +233,7 @@ __device__ __forceinline__ void cta_exit(unsigned int* counter) {
 }
 
 template <int MODE, bool OUT_BF16, bool RELU>
-__global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
+__global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
                                                    const __grid_constant__ CUtensorMap tmB, Args a, int nt, int splits,
                                                    int vec_ok) {
     constexpr bool A_MN = MODE == DW;
@@ -279,7 +281,7 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
         for (int s = 0; s < 2; ++s)   // tcgen05.commit + the issuer's arrive after publishing the unit id
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 2;\n" ::"r"(smem_u32(acc_full + s)));
         for (int s = 0; s < 2; ++s)
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;\n" ::"r"(smem_u32(acc_empty + s)));   // one per epilogue warp
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(acc_empty + s)), "r"(EPI_WARPS));   // one per epilogue warp
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
@@ -373,7 +375,7 @@ __global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUten
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
         }
     } else {
-        // ===== epilogue warps 1..8: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
+        // ===== epilogue warps 1..EPI_WARPS: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
         // column half h = (warp - 1) / 4
         const int q = warp & 3, h = (warp - 1) >> 2;
         for (uint32_t u_local = 0;; ++u_local) {
@@ -455,7 +457,7 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
 #define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
     do {                                                                                              \
         e = cudaFuncSetAttribute(k_umma_gemm<M, BF, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        if (e == cudaSuccess) e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(288), smem, st, tmA, tmB, a, nt, splits, vec_ok); \
+        if (e == cudaSuccess) e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(THREADS), smem, st, tmA, tmB, a, nt, splits, vec_ok); \
     } while (0)
     if (mode == FWD) {
         if (a.c_bf16 && a.relu) GD_UMMA_LAUNCH(FWD, true, true);
