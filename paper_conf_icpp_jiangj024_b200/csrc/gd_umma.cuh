@@ -51,7 +51,8 @@ namespace umma {
 
 constexpr int BM = 128;
 constexpr int BK = 64;
-constexpr int STAGES = 4;
+constexpr int STAGES = 4;                     // stages when both operands stream
+constexpr int MAX_STAGES = 12;                // stages when B is resident (only A streams)
 constexpr int EPI_WARPS = 8;                  // epilogue warps (2 per TMEM lane quarter; 16 measured no faster)
 constexpr int THREADS = 32 * (1 + EPI_WARPS);
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
@@ -148,7 +149,9 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) atomicAdd((float4*)(dst + j), make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]));
             } else {
-                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) atomicAdd(dst + j, v[j]);
+#pragma unroll
+                for (int j = 0; j < 32; ++j)   // compile-time indices keep v[] in registers
+                    if (cg + j < a.n_store) atomicAdd(dst + j, v[j]);
             }
         } else if (OUT_BF16) {
             __nv_bfloat16* dst = (__nv_bfloat16*)a.C + row * a.ldc + cg;
@@ -162,7 +165,9 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
                     *(uint4*)(dst + j) = w;
                 }
             } else {
-                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = __float2bfloat16_rn(v[j]);
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                    if (cg + j < a.n_store) dst[j] = __float2bfloat16_rn(v[j]);
             }
         } else {
             float* dst = (float*)a.C + row * a.ldc + cg;
@@ -170,7 +175,9 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) *(float4*)(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
             } else {
-                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = v[j];
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                    if (cg + j < a.n_store) dst[j] = v[j];
             }
         }
     }
@@ -235,7 +242,9 @@ __device__ __forceinline__ void cta_exit(unsigned int* counter) {
 template <int MODE, bool OUT_BF16, bool RELU>
 __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
                                                    const __grid_constant__ CUtensorMap tmB, Args a, int nt, int splits,
-                                                   int vec_ok) {
+                                                   int vec_ok, int ns, int nbres) {
+    // ns: pipeline stages; nbres > 0: B (all nbres k-blocks of the single N tile) is loaded
+    // once per CTA and stays resident, only A streams (FWD with W small enough)
     constexpr bool A_MN = MODE == DW;
     constexpr bool B_MN = MODE != DA;
     GD_PDL_ENTRY();   // the operands are the previous kernel's outputs
@@ -245,10 +254,11 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     const int bn = a.bn;
     const int b_stage = bn * BK * 2;
     uint8_t* sA = smem;
-    uint8_t* sB = smem + STAGES * A_STAGE;
-    uint64_t* full = (uint64_t*)(sB + STAGES * b_stage);
-    uint64_t* empty = full + STAGES;
-    uint64_t* acc_full = empty + STAGES;                          // [2] accumulator buffer ready
+    uint8_t* sB = smem + ns * A_STAGE;                            // [ns] streamed B stages or [nbres] resident B
+    uint64_t* full = (uint64_t*)(sB + (nbres > 0 ? nbres : ns) * b_stage);
+    uint64_t* empty = full + MAX_STAGES;
+    uint64_t* bres_full = empty + MAX_STAGES;                     // resident B landed
+    uint64_t* acc_full = bres_full + 1;                           // [2] accumulator buffer ready
     uint64_t* acc_empty = acc_full + 2;                           // [2] accumulator buffer drained
     uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
     int64_t* ep_unit = (int64_t*)(tmem_slot + 2);                 // [2] unit id of each accumulator buffer (-1: end)
@@ -276,7 +286,7 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     if (threadIdx.x == 0) {
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmB) : "memory");
-        for (int s = 0; s < 2 * STAGES; ++s)
+        for (int s = 0; s < 2 * MAX_STAGES + 1; ++s)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(full + s)));
         for (int s = 0; s < 2; ++s)   // tcgen05.commit + the issuer's arrive after publishing the unit id
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 2;\n" ::"r"(smem_u32(acc_full + s)));
@@ -293,7 +303,16 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
         if (lane == 0) {
             // ===== producer (TMA) + MMA issuer
             const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
-            const uint32_t stage_bytes = (uint32_t)(A_STAGE + b_stage);
+            const uint32_t stage_bytes = (uint32_t)(A_STAGE + (nbres > 0 ? 0 : b_stage));
+            if (nbres > 0) {   // the whole B of the (single) N tile, once
+                const uint32_t rb = smem_u32(bres_full);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(rb),
+                             "r"((uint32_t)(nbres * b_stage))
+                             : "memory");
+                for (int kb = 0; kb < nbres; ++kb)
+                    for (int j = 0; j < bn / 64; ++j)
+                        tma2d(smem_u32(sB + kb * b_stage) + j * 8192, &tmB, (int32_t)cm.n0 + 64 * j, kb * BK, rb);
+            }
             Unit ld = cm;
             bool ld_ok = true;
             // the next unit id is fetched one unit ahead, so the atomic's round trip hides
@@ -303,8 +322,8 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
             uint32_t uq_head = 0, uq_tail = 0;
             uint32_t it_ld = 0, it_cm = 0, u_local = 0;
             auto issue_load = [&]() {
-                const int s = (int)(it_ld % STAGES);
-                if (it_ld >= STAGES) mbar_wait(smem_u32(empty + s), ((it_ld / STAGES) - 1) & 1);   // stage's MMAs done
+                const int s = (int)(it_ld % ns);
+                if (it_ld >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it_ld / ns) - 1) & 1);   // stage's MMAs done
                 const uint32_t fb = smem_u32(full + s);
                 asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(fb), "r"(stage_bytes) : "memory");
                 const int32_t k0 = (int32_t)(ld.k_begin + (int64_t)ld.kb * BK);
@@ -312,9 +331,11 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                 if (!A_MN) tma2d(a0, &tmA, k0, (int32_t)ld.m0, fb);
                 else
                     for (int j = 0; j < BM / 64; ++j) tma2d(a0 + j * 8192, &tmA, (int32_t)ld.m0 + 64 * j, k0, fb);
-                if (!B_MN) tma2d(b0, &tmB, k0, (int32_t)ld.n0, fb);
-                else
-                    for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
+                if (nbres == 0) {
+                    if (!B_MN) tma2d(b0, &tmB, k0, (int32_t)ld.n0, fb);
+                    else
+                        for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
+                }
                 ++it_ld;
                 if (++ld.kb == ld.nkb) {
                     int r;
@@ -327,15 +348,17 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                     }
                 }
             };
-            for (int s = 0; s < STAGES - 1 && ld_ok; ++s) issue_load();
+            for (int s = 0; s < ns - 1 && ld_ok; ++s) issue_load();
+            if (nbres > 0) mbar_wait(smem_u32(bres_full), 0);
             for (;;) {
-                const int s = (int)(it_cm % STAGES);
+                const int s = (int)(it_cm % ns);
                 const uint32_t buf = u_local & 1;
                 if (cm.kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
                     mbar_wait(smem_u32(acc_empty + buf), ((u_local >> 1) - 1) & 1);
-                mbar_wait(smem_u32(full + s), (it_cm / STAGES) & 1);            // operands landed
+                mbar_wait(smem_u32(full + s), (it_cm / ns) & 1);                 // operands landed
                 asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-                const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
+                const uint32_t a0 = smem_u32(sA + s * A_STAGE);
+                const uint32_t b0 = smem_u32(sB + (nbres > 0 ? cm.kb : s) * b_stage);
 #pragma unroll
                 for (int ks = 0; ks < BK / 16; ++ks) {
                     const uint64_t ad = A_MN ? smem_desc_sw128(a0 + ks * 2048, 8192, 1024) : smem_desc_sw128(a0 + ks * 32, 16, 1024);
@@ -400,7 +423,12 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     if (threadIdx.x == 0) cta_exit(a.counter);
 }
 
-inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 8 + 16; }
+constexpr int SMEM_MAX = 227 * 1024;
+constexpr int SMEM_FIXED = 1024 + (2 * MAX_STAGES + 5) * 8 + 8 + 16;   // alignment slack, barriers, TMEM slot, unit ids
+// streamed: ns stages of A + B; resident: nbres B k-blocks once + ns stages of A
+inline int smem_bytes(int bn, int ns, int nbres) {
+    return SMEM_FIXED + ns * A_STAGE + (nbres > 0 ? nbres : ns) * bn * BK * 2;
+}
 
 // 2-D bf16 tensor map, SWIZZLE_128B, box {64, box_outer}; inner = contiguous extent, outer =
 // rows, ld = row stride in elements.  Out-of-bounds box elements read as zero.
@@ -445,10 +473,18 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
         if (e == cudaSuccess) e = make_map(&tmB, a.B, a.n_valid, rows_max, a.ldb, 64);
     }
     if (e != cudaSuccess) return e;
-    const int smem = smem_bytes(bn);
+    // FWD with a single N tile keeps all of W (= B, K x bn) in shared memory when it fits
+    // next to >= 6 A stages: only A streams, with up to MAX_STAGES k-blocks in flight
+    const int kblocks = (a.k_valid + BK - 1) / BK;
+    int ns = STAGES, nbres = 0;
+    if (mode == FWD && nt == 1 && SMEM_FIXED + kblocks * bn * BK * 2 + 6 * A_STAGE <= SMEM_MAX) {
+        nbres = kblocks;
+        ns = std::min(MAX_STAGES, (SMEM_MAX - SMEM_FIXED - kblocks * bn * BK * 2) / A_STAGE);
+    }
+    const int smem = smem_bytes(bn, ns, nbres);
     int ncols = 32;
     while (ncols < bn) ncols <<= 1;
-    const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / (2 * ncols)));   // two accumulator buffers
+    const int per_sm = std::max(1, std::min(SMEM_MAX / smem, 512 / (2 * ncols)));   // two accumulator buffers
     const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
     if (units <= 0) return cudaSuccess;
     if (!a.counter) return cudaErrorInvalidValue;
@@ -457,7 +493,9 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
 #define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
     do {                                                                                              \
         e = cudaFuncSetAttribute(k_umma_gemm<M, BF, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        if (e == cudaSuccess) e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(THREADS), smem, st, tmA, tmB, a, nt, splits, vec_ok); \
+        if (e == cudaSuccess)                                                                         \
+            e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(THREADS), smem, st, tmA, tmB, a, nt, splits, vec_ok, \
+                             ns, nbres);                                                              \
     } while (0)
     if (mode == FWD) {
         if (a.c_bf16 && a.relu) GD_UMMA_LAUNCH(FWD, true, true);
