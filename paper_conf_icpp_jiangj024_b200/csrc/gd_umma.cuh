@@ -12,15 +12,17 @@
 // ("units"; DW units are (tile, row slice) pairs), fetched from a per-launch atomic counter
 // (a CTA that only gets an SM after the others finished finds no work and leaves, so SMs held
 // by concurrent kernels of the SET pipeline do not stretch the grid), and warp-specialised
-// (32 x (1 + EPI_WARPS) threads):
-//   warp 0, lane 0: producer + MMA issuer.  It keeps STAGES-1 k-blocks of TMA loads in flight
-//     ahead of the MMAs, across unit boundaries (TMA completes a stage's "full" mbarrier with
-//     its byte count; the tcgen05.commit of the MMAs that read a stage arrives on its "empty"
-//     mbarrier, which lets the stage be refilled), and accumulates unit u into TMEM buffer
-//     u % 2, committing the unit's last k-block to acc_full[u % 2].
-//   warps 1..EPI_WARPS: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per thread)
-//     of the finished buffer, every (EPI_WARPS / 4)-th 32-column chunk (tcgen05.ld, 32
-//     columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
+// (32 x (2 + EPI_WARPS) threads):
+//   warp 0, lane 0: TMA producer.  It keeps up to ns k-blocks of TMA loads in flight, across
+//     unit boundaries: it publishes each stage's (unit, k-block) in shared memory and arms the
+//     stage's "full" mbarrier, which TMA completes with its byte count; it refills a stage once
+//     the tcgen05.commit of the MMAs that read it has arrived on the stage's "empty" mbarrier.
+//   warp 1, lane 0: MMA issuer.  It waits for "full", issues the stage's 4 MMAs into TMEM
+//     buffer u % 2 (unit u), commits them to "empty", and commits a unit's last k-block to
+//     acc_full[u % 2] (after publishing u).  Loads and MMAs never wait on each other's thread.
+//   warps 2..EPI_WARPS+1: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per
+//     thread) of the finished buffer, every (EPI_WARPS / 4)-th 32-column chunk (tcgen05.ld,
+//     32 columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
 //     (fp32 / bf16 stores, or fp32 vector red.add for DW), then arrives on acc_empty[u % 2].
 //     The next unit's MMAs run meanwhile in the other buffer.
 //
@@ -54,7 +56,7 @@ constexpr int BK = 64;
 constexpr int STAGES = 4;                     // stages when both operands stream
 constexpr int MAX_STAGES = 12;                // stages when B is resident (only A streams)
 constexpr int EPI_WARPS = 8;                  // epilogue warps (2 per TMEM lane quarter; 16 measured no faster)
-constexpr int THREADS = 32 * (1 + EPI_WARPS);
+constexpr int THREADS = 32 * (2 + EPI_WARPS);     // warp 0: TMA producer, warp 1: MMA issuer, then epilogue
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 enum Mode { FWD = 0, DA = 1, DW = 2 };
@@ -262,6 +264,9 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     uint64_t* acc_empty = acc_full + 2;                           // [2] accumulator buffer drained
     uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
     int64_t* ep_unit = (int64_t*)(tmem_slot + 2);                 // [2] unit id of each accumulator buffer (-1: end)
+    int64_t* st_unit = ep_unit + 2;                               // [MAX_STAGES] unit id of the k-block in stage s (-1: end)
+    int32_t* st_kb = (int32_t*)(st_unit + MAX_STAGES);            // [MAX_STAGES] its k-block index and the unit's count
+    int32_t* st_nkb = st_kb + MAX_STAGES;
 
     const int64_t rows = *a.rows_dev;   // device-resident size
     Unit cm;
@@ -301,8 +306,7 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
 
     if (warp == 0) {
         if (lane == 0) {
-            // ===== producer (TMA) + MMA issuer
-            const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
+            // ===== TMA producer: runs up to ns stages ahead of the MMAs, across units
             const uint32_t stage_bytes = (uint32_t)(A_STAGE + (nbres > 0 ? 0 : b_stage));
             if (nbres > 0) {   // the whole B of the (single) N tile, once
                 const uint32_t rb = smem_u32(bres_full);
@@ -314,16 +318,16 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                         tma2d(smem_u32(sB + kb * b_stage) + j * 8192, &tmB, (int32_t)cm.n0 + 64 * j, kb * BK, rb);
             }
             Unit ld = cm;
-            bool ld_ok = true;
             // the next unit id is fetched one unit ahead, so the atomic's round trip hides
-            // behind the current unit's loads instead of stalling the producer
+            // behind the current unit's loads
             unsigned int next_u = atomicAdd(a.counter, 1u);
-            int64_t uq[8];                 // units fetched by the load cursor, not yet reached by the MMAs
-            uint32_t uq_head = 0, uq_tail = 0;
-            uint32_t it_ld = 0, it_cm = 0, u_local = 0;
-            auto issue_load = [&]() {
-                const int s = (int)(it_ld % ns);
-                if (it_ld >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it_ld / ns) - 1) & 1);   // stage's MMAs done
+            uint32_t it = 0;
+            for (;;) {
+                const int s = (int)(it % ns);
+                if (it >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it / ns) - 1) & 1);   // stage's MMAs done
+                st_unit[s] = ld.u;   // published by the (release) arrive below
+                st_kb[s] = ld.kb;
+                st_nkb[s] = ld.nkb;
                 const uint32_t fb = smem_u32(full + s);
                 asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(fb), "r"(stage_bytes) : "memory");
                 const int32_t k0 = (int32_t)(ld.k_begin + (int64_t)ld.kb * BK);
@@ -336,34 +340,44 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                     else
                         for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
                 }
-                ++it_ld;
+                ++it;
                 if (++ld.kb == ld.nkb) {
                     int r;
                     while ((r = decode_unit<MODE>(ld, (int64_t)next_u, a, rows, nt, splits)) == 0)   // empty DW slice
                         next_u = atomicAdd(a.counter, 1u);
-                    ld_ok = r > 0;
-                    if (ld_ok) {
-                        uq[uq_tail++ & 7] = ld.u;
-                        next_u = atomicAdd(a.counter, 1u);
-                    }
+                    if (r < 0) break;
+                    next_u = atomicAdd(a.counter, 1u);
                 }
-            };
-            for (int s = 0; s < ns - 1 && ld_ok; ++s) issue_load();
+            }
+            // end marker in the next stage (a plain arrive completes its phase)
+            const int s = (int)(it % ns);
+            if (it >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it / ns) - 1) & 1);
+            st_unit[s] = -1;
+            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(full + s)) : "memory");
+        }
+    } else if (warp == 1) {
+        if (lane == 0) {
+            // ===== MMA issuer: one thread, accumulating unit u into TMEM buffer u % 2
+            const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
             if (nbres > 0) mbar_wait(smem_u32(bres_full), 0);
+            uint32_t it = 0, u_local = 0;
             for (;;) {
-                const int s = (int)(it_cm % ns);
+                const int s = (int)(it % ns);
+                mbar_wait(smem_u32(full + s), (it / ns) & 1);                    // operands landed
+                const int64_t u = *(volatile int64_t*)(st_unit + s);
+                if (u < 0) break;
+                const int kb = *(volatile int32_t*)(st_kb + s), nkb = *(volatile int32_t*)(st_nkb + s);
                 const uint32_t buf = u_local & 1;
-                if (cm.kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
+                if (kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
                     mbar_wait(smem_u32(acc_empty + buf), ((u_local >> 1) - 1) & 1);
-                mbar_wait(smem_u32(full + s), (it_cm / ns) & 1);                 // operands landed
                 asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
                 const uint32_t a0 = smem_u32(sA + s * A_STAGE);
-                const uint32_t b0 = smem_u32(sB + (nbres > 0 ? cm.kb : s) * b_stage);
+                const uint32_t b0 = smem_u32(sB + (nbres > 0 ? kb : s) * b_stage);
 #pragma unroll
                 for (int ks = 0; ks < BK / 16; ++ks) {
                     const uint64_t ad = A_MN ? smem_desc_sw128(a0 + ks * 2048, 8192, 1024) : smem_desc_sw128(a0 + ks * 32, 16, 1024);
                     const uint64_t bd = B_MN ? smem_desc_sw128(b0 + ks * 2048, 8192, 1024) : smem_desc_sw128(b0 + ks * 32, 16, 1024);
-                    const uint32_t acc = (cm.kb > 0 || ks > 0) ? 1u : 0u;
+                    const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
                     asm volatile(
                         "{\n\t.reg .pred p;\n\t"
                         "setp.ne.b32 p, %4, 0;\n\t"
@@ -374,21 +388,15 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                  smem_u32(empty + s))
                              : "memory");
-                const bool last = cm.kb == cm.nkb - 1;
-                if (last) {
+                if (kb == nkb - 1) {
                     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                      smem_u32(acc_full + buf))
                                  : "memory");
-                    ep_unit[buf] = cm.u;   // published by the release-arrive below
+                    ep_unit[buf] = u;   // published by the release-arrive below
                     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
+                    ++u_local;
                 }
-                if (ld_ok) issue_load();   // refill the stage the previous k-block used (MMAs stay queued)
-                ++it_cm;
-                if (last) ++u_local;
-                if (++cm.kb == cm.nkb) {
-                    if (uq_head == uq_tail) break;
-                    decode_unit<MODE>(cm, uq[uq_head++ & 7], a, rows, nt, splits);
-                }
+                ++it;
             }
             // end marker for the epilogue warps in the next buffer
             const uint32_t buf = u_local & 1;
@@ -398,9 +406,9 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
         }
     } else {
-        // ===== epilogue warps 1..EPI_WARPS: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
-        // column half h = (warp - 1) / 4
-        const int q = warp & 3, h = (warp - 1) >> 2;
+        // ===== epilogue warps 2..EPI_WARPS+1: TMEM lane quarter q = warp % 4 (tcgen05.ld lane
+        // rule), column group h = (warp - 2) / 4
+        const int q = warp & 3, h = (warp - 2) >> 2;
         for (uint32_t u_local = 0;; ++u_local) {
             const uint32_t buf = u_local & 1;
             mbar_wait(smem_u32(acc_full + buf), (u_local >> 1) & 1);
@@ -424,7 +432,7 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
 }
 
 constexpr int SMEM_MAX = 227 * 1024;
-constexpr int SMEM_FIXED = 1024 + (2 * MAX_STAGES + 5) * 8 + 8 + 16;   // alignment slack, barriers, TMEM slot, unit ids
+constexpr int SMEM_FIXED = 1024 + (2 * MAX_STAGES + 5) * 8 + 8 + 16 + MAX_STAGES * 16;   // alignment, barriers, TMEM slot, unit ids
 // streamed: ns stages of A + B; resident: nbres B k-blocks once + ns stages of A
 inline int smem_bytes(int bn, int ns, int nbres) {
     return SMEM_FIXED + ns * A_STAGE + (nbres > 0 ? nbres : ns) * bn * BK * 2;
