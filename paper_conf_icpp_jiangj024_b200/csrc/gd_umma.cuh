@@ -12,17 +12,15 @@
 // ("units"; DW units are (tile, row slice) pairs), fetched from a per-launch atomic counter
 // (a CTA that only gets an SM after the others finished finds no work and leaves, so SMs held
 // by concurrent kernels of the SET pipeline do not stretch the grid), and warp-specialised
-// (32 x (2 + EPI_WARPS) threads):
-//   warp 0, lane 0: TMA producer.  It keeps up to ns k-blocks of TMA loads in flight, across
-//     unit boundaries: it publishes each stage's (unit, k-block) in shared memory and arms the
-//     stage's "full" mbarrier, which TMA completes with its byte count; it refills a stage once
-//     the tcgen05.commit of the MMAs that read it has arrived on the stage's "empty" mbarrier.
-//   warp 1, lane 0: MMA issuer.  It waits for "full", issues the stage's 4 MMAs into TMEM
-//     buffer u % 2 (unit u), commits them to "empty", and commits a unit's last k-block to
-//     acc_full[u % 2] (after publishing u).  Loads and MMAs never wait on each other's thread.
-//   warps 2..EPI_WARPS+1: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per
-//     thread) of the finished buffer, every (EPI_WARPS / 4)-th 32-column chunk (tcgen05.ld,
-//     32 columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
+// (288 threads):
+//   warp 0, lane 0: producer + MMA issuer.  It keeps STAGES-1 k-blocks of TMA loads in flight
+//     ahead of the MMAs, across unit boundaries (TMA completes a stage's "full" mbarrier with
+//     its byte count; the tcgen05.commit of the MMAs that read a stage arrives on its "empty"
+//     mbarrier, which lets the stage be refilled), and accumulates unit u into TMEM buffer
+//     u % 2, committing the unit's last k-block to acc_full[u % 2].
+//   warps 1-8: epilogue.  Warp w drains TMEM lanes 32 (w % 4).. (one output row per thread)
+//     of the finished buffer, alternate 32-column chunks per warp pair (tcgen05.ld, 32
+//     columns per load), adds the bias / applies relu and writes 16-byte vectors of its row
 //     (fp32 / bf16 stores, or fp32 vector red.add for DW), then arrives on acc_empty[u % 2].
 //     The next unit's MMAs run meanwhile in the other buffer.
 //
@@ -53,10 +51,7 @@ namespace umma {
 
 constexpr int BM = 128;
 constexpr int BK = 64;
-constexpr int STAGES = 4;                     // stages when both operands stream
-constexpr int MAX_STAGES = 12;                // stages when B is resident (only A streams)
-constexpr int EPI_WARPS = 8;                  // epilogue warps (2 per TMEM lane quarter; 16 measured no faster)
-constexpr int THREADS = 32 * (2 + EPI_WARPS);     // warp 0: TMA producer, warp 1: MMA issuer, then epilogue
+constexpr int STAGES = 4;
 constexpr int A_STAGE = BM * BK * 2;   // 16 KB
 
 enum Mode { FWD = 0, DA = 1, DW = 2 };
@@ -122,7 +117,7 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
                                          int h, int lane, bool vec_ok) {
     const int64_t row = rbase + lane;
     const bool row_ok = row < m_valid;
-    for (int c0 = 32 * h; c0 < bn; c0 += 32 * (EPI_WARPS / 4)) {
+    for (int c0 = 32 * h; c0 < bn; c0 += 64) {
         uint32_t r[32];
         asm volatile(
             "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
@@ -151,9 +146,7 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) atomicAdd((float4*)(dst + j), make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]));
             } else {
-#pragma unroll
-                for (int j = 0; j < 32; ++j)   // compile-time indices keep v[] in registers
-                    if (cg + j < a.n_store) atomicAdd(dst + j, v[j]);
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) atomicAdd(dst + j, v[j]);
             }
         } else if (OUT_BF16) {
             __nv_bfloat16* dst = (__nv_bfloat16*)a.C + row * a.ldc + cg;
@@ -167,9 +160,7 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
                     *(uint4*)(dst + j) = w;
                 }
             } else {
-#pragma unroll
-                for (int j = 0; j < 32; ++j)
-                    if (cg + j < a.n_store) dst[j] = __float2bfloat16_rn(v[j]);
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = __float2bfloat16_rn(v[j]);
             }
         } else {
             float* dst = (float*)a.C + row * a.ldc + cg;
@@ -177,9 +168,7 @@ __device__ __forceinline__ void epilogue(const Args& a, uint32_t tacc, int64_t r
 #pragma unroll
                 for (int j = 0; j < 32; j += 4) *(float4*)(dst + j) = make_float4(v[j], v[j + 1], v[j + 2], v[j + 3]);
             } else {
-#pragma unroll
-                for (int j = 0; j < 32; ++j)
-                    if (cg + j < a.n_store) dst[j] = v[j];
+                for (int j = 0; j < 32 && cg + j < a.n_store; ++j) dst[j] = v[j];
             }
         }
     }
@@ -242,11 +231,9 @@ __device__ __forceinline__ void cta_exit(unsigned int* counter) {
 }
 
 template <int MODE, bool OUT_BF16, bool RELU>
-__global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
+__global__ void __launch_bounds__(288) k_umma_gemm(const __grid_constant__ CUtensorMap tmA,
                                                    const __grid_constant__ CUtensorMap tmB, Args a, int nt, int splits,
-                                                   int vec_ok, int ns, int nbres) {
-    // ns: pipeline stages; nbres > 0: B (all nbres k-blocks of the single N tile) is loaded
-    // once per CTA and stays resident, only A streams (FWD with W small enough)
+                                                   int vec_ok) {
     constexpr bool A_MN = MODE == DW;
     constexpr bool B_MN = MODE != DA;
     GD_PDL_ENTRY();   // the operands are the previous kernel's outputs
@@ -256,17 +243,13 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     const int bn = a.bn;
     const int b_stage = bn * BK * 2;
     uint8_t* sA = smem;
-    uint8_t* sB = smem + ns * A_STAGE;                            // [ns] streamed B stages or [nbres] resident B
-    uint64_t* full = (uint64_t*)(sB + (nbres > 0 ? nbres : ns) * b_stage);
-    uint64_t* empty = full + MAX_STAGES;
-    uint64_t* bres_full = empty + MAX_STAGES;                     // resident B landed
-    uint64_t* acc_full = bres_full + 1;                           // [2] accumulator buffer ready
+    uint8_t* sB = smem + STAGES * A_STAGE;
+    uint64_t* full = (uint64_t*)(sB + STAGES * b_stage);
+    uint64_t* empty = full + STAGES;
+    uint64_t* acc_full = empty + STAGES;                          // [2] accumulator buffer ready
     uint64_t* acc_empty = acc_full + 2;                           // [2] accumulator buffer drained
     uint32_t* tmem_slot = (uint32_t*)(acc_empty + 2);
     int64_t* ep_unit = (int64_t*)(tmem_slot + 2);                 // [2] unit id of each accumulator buffer (-1: end)
-    int64_t* st_unit = ep_unit + 2;                               // [MAX_STAGES] unit id of the k-block in stage s (-1: end)
-    int32_t* st_kb = (int32_t*)(st_unit + MAX_STAGES);            // [MAX_STAGES] its k-block index and the unit's count
-    int32_t* st_nkb = st_kb + MAX_STAGES;
 
     const int64_t rows = *a.rows_dev;   // device-resident size
     Unit cm;
@@ -291,12 +274,12 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     if (threadIdx.x == 0) {
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmA) : "memory");
         asm volatile("prefetch.tensormap [%0];\n" ::"l"((uint64_t)&tmB) : "memory");
-        for (int s = 0; s < 2 * MAX_STAGES + 1; ++s)
+        for (int s = 0; s < 2 * STAGES; ++s)
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(smem_u32(full + s)));
         for (int s = 0; s < 2; ++s)   // tcgen05.commit + the issuer's arrive after publishing the unit id
             asm volatile("mbarrier.init.shared::cta.b64 [%0], 2;\n" ::"r"(smem_u32(acc_full + s)));
         for (int s = 0; s < 2; ++s)
-            asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(acc_empty + s)), "r"(EPI_WARPS));   // one per epilogue warp
+            asm volatile("mbarrier.init.shared::cta.b64 [%0], 8;\n" ::"r"(smem_u32(acc_empty + s)));   // one per epilogue warp
         asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
     }
     asm volatile("tcgen05.fence::before_thread_sync;\n" ::: "memory");
@@ -306,28 +289,20 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
 
     if (warp == 0) {
         if (lane == 0) {
-            // ===== TMA producer: runs up to ns stages ahead of the MMAs, across units
-            const uint32_t stage_bytes = (uint32_t)(A_STAGE + (nbres > 0 ? 0 : b_stage));
-            if (nbres > 0) {   // the whole B of the (single) N tile, once
-                const uint32_t rb = smem_u32(bres_full);
-                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(rb),
-                             "r"((uint32_t)(nbres * b_stage))
-                             : "memory");
-                for (int kb = 0; kb < nbres; ++kb)
-                    for (int j = 0; j < bn / 64; ++j)
-                        tma2d(smem_u32(sB + kb * b_stage) + j * 8192, &tmB, (int32_t)cm.n0 + 64 * j, kb * BK, rb);
-            }
+            // ===== producer (TMA) + MMA issuer
+            const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
+            const uint32_t stage_bytes = (uint32_t)(A_STAGE + b_stage);
             Unit ld = cm;
+            bool ld_ok = true;
             // the next unit id is fetched one unit ahead, so the atomic's round trip hides
-            // behind the current unit's loads
+            // behind the current unit's loads instead of stalling the producer
             unsigned int next_u = atomicAdd(a.counter, 1u);
-            uint32_t it = 0;
-            for (;;) {
-                const int s = (int)(it % ns);
-                if (it >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it / ns) - 1) & 1);   // stage's MMAs done
-                st_unit[s] = ld.u;   // published by the (release) arrive below
-                st_kb[s] = ld.kb;
-                st_nkb[s] = ld.nkb;
+            int64_t uq[8];                 // units fetched by the load cursor, not yet reached by the MMAs
+            uint32_t uq_head = 0, uq_tail = 0;
+            uint32_t it_ld = 0, it_cm = 0, u_local = 0;
+            auto issue_load = [&]() {
+                const int s = (int)(it_ld % STAGES);
+                if (it_ld >= STAGES) mbar_wait(smem_u32(empty + s), ((it_ld / STAGES) - 1) & 1);   // stage's MMAs done
                 const uint32_t fb = smem_u32(full + s);
                 asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(fb), "r"(stage_bytes) : "memory");
                 const int32_t k0 = (int32_t)(ld.k_begin + (int64_t)ld.kb * BK);
@@ -335,49 +310,35 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                 if (!A_MN) tma2d(a0, &tmA, k0, (int32_t)ld.m0, fb);
                 else
                     for (int j = 0; j < BM / 64; ++j) tma2d(a0 + j * 8192, &tmA, (int32_t)ld.m0 + 64 * j, k0, fb);
-                if (nbres == 0) {
-                    if (!B_MN) tma2d(b0, &tmB, k0, (int32_t)ld.n0, fb);
-                    else
-                        for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
-                }
-                ++it;
+                if (!B_MN) tma2d(b0, &tmB, k0, (int32_t)ld.n0, fb);
+                else
+                    for (int j = 0; j < bn / 64; ++j) tma2d(b0 + j * 8192, &tmB, (int32_t)ld.n0 + 64 * j, k0, fb);
+                ++it_ld;
                 if (++ld.kb == ld.nkb) {
                     int r;
                     while ((r = decode_unit<MODE>(ld, (int64_t)next_u, a, rows, nt, splits)) == 0)   // empty DW slice
                         next_u = atomicAdd(a.counter, 1u);
-                    if (r < 0) break;
-                    next_u = atomicAdd(a.counter, 1u);
+                    ld_ok = r > 0;
+                    if (ld_ok) {
+                        uq[uq_tail++ & 7] = ld.u;
+                        next_u = atomicAdd(a.counter, 1u);
+                    }
                 }
-            }
-            // end marker in the next stage (a plain arrive completes its phase)
-            const int s = (int)(it % ns);
-            if (it >= (uint32_t)ns) mbar_wait(smem_u32(empty + s), ((it / ns) - 1) & 1);
-            st_unit[s] = -1;
-            asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(full + s)) : "memory");
-        }
-    } else if (warp == 1) {
-        if (lane == 0) {
-            // ===== MMA issuer: one thread, accumulating unit u into TMEM buffer u % 2
-            const uint32_t idesc = instr_desc<A_MN, B_MN>(bn);
-            if (nbres > 0) mbar_wait(smem_u32(bres_full), 0);
-            uint32_t it = 0, u_local = 0;
+            };
+            for (int s = 0; s < STAGES - 1 && ld_ok; ++s) issue_load();
             for (;;) {
-                const int s = (int)(it % ns);
-                mbar_wait(smem_u32(full + s), (it / ns) & 1);                    // operands landed
-                const int64_t u = *(volatile int64_t*)(st_unit + s);
-                if (u < 0) break;
-                const int kb = *(volatile int32_t*)(st_kb + s), nkb = *(volatile int32_t*)(st_nkb + s);
+                const int s = (int)(it_cm % STAGES);
                 const uint32_t buf = u_local & 1;
-                if (kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
+                if (cm.kb == 0 && u_local >= 2)   // the epilogue of unit u_local - 2 drained this buffer
                     mbar_wait(smem_u32(acc_empty + buf), ((u_local >> 1) - 1) & 1);
+                mbar_wait(smem_u32(full + s), (it_cm / STAGES) & 1);            // operands landed
                 asm volatile("tcgen05.fence::after_thread_sync;\n" ::: "memory");
-                const uint32_t a0 = smem_u32(sA + s * A_STAGE);
-                const uint32_t b0 = smem_u32(sB + (nbres > 0 ? kb : s) * b_stage);
+                const uint32_t a0 = smem_u32(sA + s * A_STAGE), b0 = smem_u32(sB + s * b_stage);
 #pragma unroll
                 for (int ks = 0; ks < BK / 16; ++ks) {
                     const uint64_t ad = A_MN ? smem_desc_sw128(a0 + ks * 2048, 8192, 1024) : smem_desc_sw128(a0 + ks * 32, 16, 1024);
                     const uint64_t bd = B_MN ? smem_desc_sw128(b0 + ks * 2048, 8192, 1024) : smem_desc_sw128(b0 + ks * 32, 16, 1024);
-                    const uint32_t acc = (kb > 0 || ks > 0) ? 1u : 0u;
+                    const uint32_t acc = (cm.kb > 0 || ks > 0) ? 1u : 0u;
                     asm volatile(
                         "{\n\t.reg .pred p;\n\t"
                         "setp.ne.b32 p, %4, 0;\n\t"
@@ -388,15 +349,21 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
                 asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                  smem_u32(empty + s))
                              : "memory");
-                if (kb == nkb - 1) {
+                const bool last = cm.kb == cm.nkb - 1;
+                if (last) {
                     asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n" ::"r"(
                                      smem_u32(acc_full + buf))
                                  : "memory");
-                    ep_unit[buf] = u;   // published by the release-arrive below
+                    ep_unit[buf] = cm.u;   // published by the release-arrive below
                     asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
-                    ++u_local;
                 }
-                ++it;
+                if (ld_ok) issue_load();   // refill the stage the previous k-block used (MMAs stay queued)
+                ++it_cm;
+                if (last) ++u_local;
+                if (++cm.kb == cm.nkb) {
+                    if (uq_head == uq_tail) break;
+                    decode_unit<MODE>(cm, uq[uq_head++ & 7], a, rows, nt, splits);
+                }
             }
             // end marker for the epilogue warps in the next buffer
             const uint32_t buf = u_local & 1;
@@ -406,9 +373,9 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
             asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];\n" ::"r"(smem_u32(acc_full + buf)) : "memory");
         }
     } else {
-        // ===== epilogue warps 2..EPI_WARPS+1: TMEM lane quarter q = warp % 4 (tcgen05.ld lane
-        // rule), column group h = (warp - 2) / 4
-        const int q = warp & 3, h = (warp - 2) >> 2;
+        // ===== epilogue warps 1..8: TMEM lane quarter q = warp % 4 (tcgen05.ld lane rule),
+        // column half h = (warp - 1) / 4
+        const int q = warp & 3, h = (warp - 1) >> 2;
         for (uint32_t u_local = 0;; ++u_local) {
             const uint32_t buf = u_local & 1;
             mbar_wait(smem_u32(acc_full + buf), (u_local >> 1) & 1);
@@ -431,12 +398,7 @@ __global__ void __launch_bounds__(THREADS) k_umma_gemm(const __grid_constant__ C
     if (threadIdx.x == 0) cta_exit(a.counter);
 }
 
-constexpr int SMEM_MAX = 227 * 1024;
-constexpr int SMEM_FIXED = 1024 + (2 * MAX_STAGES + 5) * 8 + 8 + 16 + MAX_STAGES * 16;   // alignment, barriers, TMEM slot, unit ids
-// streamed: ns stages of A + B; resident: nbres B k-blocks once + ns stages of A
-inline int smem_bytes(int bn, int ns, int nbres) {
-    return SMEM_FIXED + ns * A_STAGE + (nbres > 0 ? nbres : ns) * bn * BK * 2;
-}
+inline int smem_bytes(int bn) { return 1024 + STAGES * (A_STAGE + bn * BK * 2) + (2 * STAGES + 4) * 8 + 8 + 16; }
 
 // 2-D bf16 tensor map, SWIZZLE_128B, box {64, box_outer}; inner = contiguous extent, outer =
 // rows, ld = row stride in elements.  Out-of-bounds box elements read as zero.
@@ -481,18 +443,10 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
         if (e == cudaSuccess) e = make_map(&tmB, a.B, a.n_valid, rows_max, a.ldb, 64);
     }
     if (e != cudaSuccess) return e;
-    // FWD with a single N tile keeps all of W (= B, K x bn) in shared memory when it fits
-    // next to >= 6 A stages: only A streams, with up to MAX_STAGES k-blocks in flight
-    const int kblocks = (a.k_valid + BK - 1) / BK;
-    int ns = STAGES, nbres = 0;
-    if (mode == FWD && nt == 1 && SMEM_FIXED + kblocks * bn * BK * 2 + 6 * A_STAGE <= SMEM_MAX) {
-        nbres = kblocks;
-        ns = std::min(MAX_STAGES, (SMEM_MAX - SMEM_FIXED - kblocks * bn * BK * 2) / A_STAGE);
-    }
-    const int smem = smem_bytes(bn, ns, nbres);
+    const int smem = smem_bytes(bn);
     int ncols = 32;
     while (ncols < bn) ncols <<= 1;
-    const int per_sm = std::max(1, std::min(SMEM_MAX / smem, 512 / (2 * ncols)));   // two accumulator buffers
+    const int per_sm = std::max(1, std::min(227 * 1024 / smem, 512 / (2 * ncols)));   // two accumulator buffers
     const int64_t units = mode == DW ? (a.m_valid + BM - 1) / BM * nt * splits : (rows_max + BM - 1) / BM * nt;
     if (units <= 0) return cudaSuccess;
     if (!a.counter) return cudaErrorInvalidValue;
@@ -501,9 +455,7 @@ inline cudaError_t launch(int mode, const Args& a0, int64_t rows_max, int n_tota
 #define GD_UMMA_LAUNCH(M, BF, RL)                                                                     \
     do {                                                                                              \
         e = cudaFuncSetAttribute(k_umma_gemm<M, BF, RL>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem); \
-        if (e == cudaSuccess)                                                                         \
-            e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(THREADS), smem, st, tmA, tmB, a, nt, splits, vec_ok, \
-                             ns, nbres);                                                              \
+        if (e == cudaSuccess) e = launch_chain(k_umma_gemm<M, BF, RL>, dim3(grid), dim3(288), smem, st, tmA, tmB, a, nt, splits, vec_ok); \
     } while (0)
     if (mode == FWD) {
         if (a.c_bf16 && a.relu) GD_UMMA_LAUNCH(FWD, true, true);
