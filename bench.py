@@ -348,11 +348,14 @@ def run_ours(args, rank, world, local_rank):
             log(f"  step {j}: {what} ok")
 
     last_o = [None]
+    HOST_BOUND = os.environ.get("GD_HOST_BOUND", "1") == "1"   # GD_HOST_BOUND=0: unbounded host lookahead
 
     def step(j, host_inputs=False, host_out=None):
         s = j % RING
         o = outs[s]
         last_o[0] = o
+        if HOST_BOUND:
+            dones[s].synchronize()         # the host, too, stays at most RING batches ahead (bounded queue)
         main.wait_event(dones[s])          # batch j - RING is complete: its buffers are free
         if model is not None:
             main.wait_event(tdones[s])     # ... and trained (the trainer reads outs[s], feats[s])
