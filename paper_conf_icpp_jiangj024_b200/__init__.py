@@ -64,6 +64,9 @@ class SampleOut:
         return self.sizes[self.K:self.K + 1]
 
     def cstruct(self) -> SampleOutC:
+        c = getattr(self, "_cs", None)   # the arrays never move: build the struct once
+        if c is not None:
+            return c
         c = SampleOutC()
         c.n_id = self.n_id.data_ptr()
         for h in range(self.K):
@@ -71,6 +74,7 @@ class SampleOut:
             c.col[h] = self.col[h].data_ptr()
             c.eid[h] = self.eid[h].data_ptr() if self.eid is not None else None
         c.sizes = self.sizes.data_ptr()
+        self._cs = c
         return c
 
     def to_host(self):
@@ -132,7 +136,12 @@ class Graph:
         if out is None:
             out = self.alloc_out(seeds.numel(), fanouts, with_eid)
         K = len(fanouts)
-        f = (ctypes.c_int32 * K)(*fanouts)
+        key = tuple(fanouts)
+        f = self._fan_cache.get(key) if hasattr(self, "_fan_cache") else None
+        if f is None:
+            if not hasattr(self, "_fan_cache"):
+                self._fan_cache = {}
+            f = self._fan_cache[key] = (ctypes.c_int32 * K)(*fanouts)
         cs = out.cstruct()
         if workspace is None:
             check(lib.gd_sample(self._h, _ptr(seeds), seeds.numel(), f, K, ctypes.c_uint64(rng_seed),
