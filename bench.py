@@ -316,10 +316,10 @@ def run_ours(args, rank, world, local_rank):
     sizes_log = torch.zeros((total, 2 * len(fan) + 1), dtype=torch.int64, device=dev)
     main = torch.cuda.current_stream(dev)
     pending = []
-    # GD_RELEASE_STREAM=1: releases on their own stream; release(j - Q) is ordered after extract(j)'s bookkeeping
+    # releases on their own stream (GD_RELEASE_STREAM=0: on main); release(j - Q) is ordered after extract(j)'s bookkeeping
     # and before extract(j + 1)'s (the sequential order of Alg. 1, so the buffer state is the
     # oracle's), and overlaps sample(j + 1), which does not touch the buffer
-    rel_stream = torch.cuda.Stream(dev) if os.environ.get("GD_RELEASE_STREAM", "0") == "1" else main
+    rel_stream = torch.cuda.Stream(dev) if os.environ.get("GD_RELEASE_STREAM", "1") == "1" else main
     ev_bk = torch.cuda.Event()      # extract(j)'s bookkeeping enqueued on main
     ev_rel = torch.cuda.Event()     # release(j - Q) done
     rel_live = [False]
