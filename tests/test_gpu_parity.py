@@ -196,13 +196,18 @@ def test_extract_parity_tiny_evict(tiny, gd, Q):
     run_schedule(gd, g, ip, ix, feat, S, Q, seeds, list(cfg.fanouts))
 
 
-@pytest.mark.parametrize("own_stream", [False, True])
-def test_release_on_its_own_stream_matches_oracle(tiny, gd, own_stream):
+@pytest.mark.parametrize("own_stream,row_bytes,chunk_kb", [(False, None, None), (True, None, None), (True, 1024, "16"),
+                                                        (False, 1536, "24")])
+def test_release_on_its_own_stream_matches_oracle(tiny, gd, own_stream, row_bytes, chunk_kb, monkeypatch):
     """bench.py's schedule: release(j - Q) on a second stream, ordered after extract(j)'s
     bookkeeping and before extract(j + 1)'s by events, overlapping sample(j + 1); no host
-    sync until the end.  Outputs and the final buffer state equal the sequential oracle's."""
+    sync until the end.  Outputs and the final buffer state equal the sequential oracle's.
+    The small-chunk cases give the staged copy-engine path many chunks per batch, so the
+    host-callback argument ring (1024 slots) wraps during the run."""
+    if chunk_kb is not None:
+        monkeypatch.setenv("GD_STAGE_CHUNK_KB", chunk_kb)
     cfg, g, ip, ix, order = tiny
-    feat = table_np(cfg.num_nodes, cfg.row_bytes)
+    feat = table_np(cfg.num_nodes, row_bytes or cfg.row_bytes)
     fan = list(cfg.fanouts)
     Q = 4
     nb, _ = O.sample_bounds(cfg.batch_size, fan, cfg.num_nodes, cfg.num_edges)
