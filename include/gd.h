@@ -294,6 +294,11 @@ gd_status gd_buffer_peer_stats(gd_buffer* b, int64_t* served, int64_t* probed);
  *   gd_sage_apply_sgd  p -= lr * grad_scale * g (grad_scale = 1/world after a SUM
  *                    all-reduce), then refreshes the bf16 copies; stream-ordered.
  *   gd_sage_get      synchronising debug copy of one layer's item (GD_SAGE_*) to host.
+ *                    Activation items are valid for the rows of the last step's device
+ *                    count; the rows up to the next multiple of 64 are zero, rows past that
+ *                    hold earlier steps' data.
+ * Environment: GD_SAGE_TIMING=1 records one event pair per phase of every step on the
+ * train stream and prints the mean live time per phase at gd_sage_destroy.
  * ------------------------------------------------------------------------- */
 typedef struct gd_sage gd_sage;
 #define GD_SAGE_W 0     /* fp32 [2 d_in x d_out] */
