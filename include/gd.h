@@ -78,7 +78,9 @@ gd_status gd_graph_create(const int64_t* indptr, const int32_t* indices, int64_t
                           int64_t num_edges, int device, int validate, gd_graph** out);
 gd_status gd_graph_destroy(gd_graph* g);
 
-/* Host-only worst-case sizes of one gd_sample call (no device work):
+/* Host-only worst-case sizes of one gd_sample call (no device work).  The last entry,
+ * max_nodes[K], is the paper's M_b, "the maximum number of nodes in a mini-batch" that sizes
+ * the feature buffer's N_e x M_b reservation; the rest size gd_sample_out.
  *   max_nodes[0] = num_seeds,
  *   max_edges[h-1] = f_h < 0 ? num_edges : min(num_edges, max_nodes[h-1] * f_h),
  *   max_nodes[h]   = min(num_nodes, max_nodes[h-1] + max_edges[h-1]),  h = 1..num_hops.
@@ -192,9 +194,12 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  *             for the misses or the hit gather.  node_ids, *n_dev and alias
  *             must stay unmodified until `done`.
  * GD_ERR_CAPACITY if this would exceed max_inflight unreleased batches.
+ * stats[0..1] are written on `stream` (after loop 1); stats[2..3] are final only at
+ * `done` (with peers attached they are written on a side stream after the peer probe; rows
+ * served by peers count in neither, see gd_buffer_peer_stats).
  * The call does not synchronise the device; it blocks the calling thread only when
- * that thread is max_inflight + 2 batches ahead of the staged miss path's host gather
- * (whose per-batch host arguments are then reused).
+ * 1024 staged chunk jobs (8 MB each by default) enqueued by earlier calls are still
+ * waiting for their host-gather callbacks (their argument slots are then reused).
  * ------------------------------------------------------------------------- */
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,
                      void* out, int32_t* alias, int64_t* stats, void* stream, void* done);
@@ -211,7 +216,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  *                    and host gather rate r_host and the contiguous pull rate r_link of
  *                    the host link (calibrated when this call enables adaptation):
  *                    r_zc / (r_zc + r_host) if r_zc + r_host <= r_link, else
- *                    1 - r_host / r_link; clamped to [0.05, 0.9].
+ *                    1 - r_host / r_link; clamped to [0.05, 0.9] (to [0.05, 0.2] with
+ *                    copy-engine staging, [0.05, 0.3] once >= 8 host-rate samples show the
+ *                    host gather below 0.6 r_link; back to 0.2 above 0.7 r_link).
  *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
  *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs
@@ -223,6 +230,14 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  * ------------------------------------------------------------------------- */
 gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share, int zc_blocks,
                            int pull_blocks);
+
+/* The miss-path split policy (gd_buffer_config, adaptive share), for reports: out[0..n) of
+ * {zero-copy share, r_host, r_zc, r_link (GB/s), misses-per-batch estimate (the copy-engine
+ * staging size), host-rate samples, slow-host cap active (0/1), newest batch rated}.  The
+ * estimates come from the newest completed batch at each gd_extract (events queried, never
+ * waited on) and the miss count from the newest batch whose loop 2 ran (an epoch-tagged count
+ * the device writes to mapped host memory).  Host-only, no sync; n <= 8. */
+gd_status gd_buffer_policy_read(gd_buffer* b, double* out, int32_t n);
 
 /* ----------------------------------------------------------------------------
  * Phase 2 of the staged share ("CUDA async copy" of the staging buffer).
@@ -347,7 +362,10 @@ gd_status gd_debug_umma_gemm(int32_t mode, const void* A, int64_t lda, const voi
 gd_status gd_buffer_release(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev,
                             int64_t n_max, void* stream);
 
-/* Synchronises the handle's device and returns GD_ERR_DEVICE (and the sticky
+/* Error reporting of the device-side preconditions (no paper passage: the paper's
+ * extractor threads check on the host; here the checks run inside the kernels and
+ * cannot return a status without a sync, so they set a sticky word, CUDA sticky-error style).
+ * Synchronises the handle's device and returns GD_ERR_DEVICE (and the sticky
  * GD_DEV_* bits in *bits, if non-NULL) if a device-side check tripped since the
  * handle was created.  `handle` is a gd_graph* or a gd_buffer*. */
 gd_status gd_check_device_status(void* handle, uint32_t* bits);

@@ -24,7 +24,8 @@ EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy",
            "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config", "gd_buffer_stage_mode",
            "gd_buffer_peer_attach", "gd_buffer_peer_export_ipc", "gd_buffer_peer_attach_ipc", "gd_buffer_peer_stats",
            "gd_sage_create", "gd_sage_destroy", "gd_sage_step", "gd_sage_grads", "gd_sage_apply_sgd", "gd_sage_get",
-           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod", "gd_debug_umma_gemm"]
+           "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod", "gd_debug_umma_gemm",
+           "gd_buffer_policy_read"]
 
 
 class GdError(RuntimeError):
@@ -80,6 +81,7 @@ def _load():
     L.gd_buffer_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     L.gd_buffer_config.argtypes = [_vp, ctypes.c_int, ctypes.c_double, ctypes.c_int, ctypes.c_int]
     L.gd_buffer_stage_mode.argtypes = [_vp, ctypes.c_int]
+    L.gd_buffer_policy_read.argtypes = [_vp, _dp, _i32]
     L.gd_buffer_peer_attach.argtypes = [_vp, ctypes.c_int, ctypes.POINTER(_vp)]
     L.gd_buffer_peer_export_ipc.argtypes = [_vp, ctypes.c_void_p, ctypes.c_int64]
     L.gd_buffer_peer_attach_ipc.argtypes = [_vp, ctypes.c_int, ctypes.c_void_p]

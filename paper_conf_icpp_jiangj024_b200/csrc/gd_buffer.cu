@@ -193,6 +193,20 @@ __device__ __forceinline__ void ticket_finish(unsigned long long* ticket) {
     }
 }
 
+// The staged share's counts, published to mapped host memory: {M, K0, M - K0} for the host
+// gather of this batch, and the word h_meta[4] = (epoch << 32 | M) (one 8-byte store): the
+// host takes the newest epoch over the D slots as the latest miss count and sizes the next
+// copy-engine staging share from it without querying an event or synchronising, however far
+// ahead of the device it runs.
+__device__ __forceinline__ void publish_meta(int64_t* h_meta, long long M, long long K0, unsigned long long epoch) {
+    volatile int64_t* hm = h_meta;
+    hm[0] = M;
+    hm[1] = K0;
+    hm[2] = M - K0;
+    volatile unsigned long long* latest = (volatile unsigned long long*)(h_meta + 4);
+    *latest = (epoch << 32) | (unsigned long long)(M & 0xffffffffll);
+}
+
 __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
     GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
@@ -210,11 +224,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
             *a.ctl_out = c;
             *a.trip_count = 0;
             *a.trip_split = 0;
-            if (a.h_meta) {
-                a.h_meta[0] = 0;
-                a.h_meta[1] = 0;
-                a.h_meta[2] = 0;
-            }
+            if (a.h_meta) publish_meta(a.h_meta, 0, 0, a.epoch);
             if (a.stats) {
                 a.stats[2] = 0;
                 a.stats[3] = 0;
@@ -266,11 +276,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                     const long long Mx = base + agg, K0x = K0 < Mx ? K0 : Mx;
                     *a.trip_count = Mx;
                     *a.trip_split = K0x;
-                    if (a.h_meta) {
-                        a.h_meta[0] = Mx;
-                        a.h_meta[1] = K0x;
-                        a.h_meta[2] = Mx - K0x;
-                    }
+                    if (a.h_meta) publish_meta(a.h_meta, Mx, K0x, a.epoch);
                     if (a.stats) {
                         a.stats[2] = K0x;
                         a.stats[3] = Mx - K0x;
@@ -309,11 +315,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                     *a.ctl_out = o;
                     *a.trip_count = M;
                     *a.trip_split = K0;
-                    if (a.h_meta) {
-                        a.h_meta[0] = M;
-                        a.h_meta[1] = K0;
-                        a.h_meta[2] = M - K0;
-                    }
+                    if (a.h_meta) publish_meta(a.h_meta, M, K0, a.epoch);
                     if (a.stats) {
                         a.stats[2] = K0;
                         a.stats[3] = M - K0;
@@ -481,7 +483,8 @@ __global__ void __launch_bounds__(256) k_peer_probe(const int4* __restrict__ tri
 // node list and counts to the host gather.
 __global__ void k_peer_split(const int4* __restrict__ trip2, const int64_t* __restrict__ t2count,
                              int64_t* __restrict__ t2split, uint32_t alpha_q16, long long staged_cap,
-                             int32_t* __restrict__ h_nodes, int64_t* __restrict__ h_meta, int64_t* __restrict__ stats) {
+                             int32_t* __restrict__ h_nodes, int64_t* __restrict__ h_meta, int64_t* __restrict__ stats,
+                             unsigned long long epoch) {
     const long long M = *t2count;
     const long long K0 = staged_cap >= 0 ? (M > staged_cap ? M - staged_cap : 0)
                                          : (long long)(((unsigned long long)M * alpha_q16) >> 16);
@@ -491,11 +494,7 @@ __global__ void k_peer_split(const int4* __restrict__ trip2, const int64_t* __re
             h_nodes[k - K0] = trip2[k].x;
     if (blockIdx.x == 0 && threadIdx.x == 0) {
         *t2split = K0;
-        if (h_meta) {
-            h_meta[0] = M;
-            h_meta[1] = K0;
-            h_meta[2] = M - K0;
-        }
+        if (h_meta) publish_meta(h_meta, M, K0, epoch);
         if (stats) {
             stats[2] = K0;
             stats[3] = M - K0;
@@ -980,15 +979,15 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         const int64_t nm = b->n_max;
         GD_CUDA(cudaHostAlloc((void**)&b->stage_mem, (size_t)D * nm * b->R, cudaHostAllocMapped | cudaHostAllocPortable));
         GD_CUDA(cudaHostAlloc((void**)&b->hnodes_mem, (size_t)D * nm * sizeof(int32_t), cudaHostAllocMapped | cudaHostAllocPortable));
-        GD_CUDA(cudaHostAlloc((void**)&b->hmeta_mem, (size_t)D * 4 * sizeof(int64_t), cudaHostAllocMapped | cudaHostAllocPortable));
-        std::memset(b->hmeta_mem, 0, (size_t)D * 4 * sizeof(int64_t));
+        GD_CUDA(cudaHostAlloc((void**)&b->hmeta_mem, (size_t)D * 8 * sizeof(int64_t), cudaHostAllocMapped | cudaHostAllocPortable));
+        std::memset(b->hmeta_mem, 0, (size_t)D * 8 * sizeof(int64_t));
         b->stg.assign(D, StagedSlot());
         for (int d = 0; d < D; ++d) {
             b->stg[d].owner = b;
             b->stg[d].d = d;
             b->stg[d].staging = b->stage_mem + (size_t)d * nm * b->R;
             b->stg[d].h_nodes = b->hnodes_mem + (size_t)d * nm;
-            b->stg[d].h_meta = b->hmeta_mem + 4 * d;
+            b->stg[d].h_meta = b->hmeta_mem + 8 * d;
         }
     }
     if (b->pool && (host_threads == 0 || b->pool->threads() != host_threads)) {
@@ -1032,6 +1031,9 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     b->alpha = host_threads == 0 ? 1.0 : (zero_copy_share >= 0 ? zero_copy_share : 0.2);
     b->r_host = 0;
     b->r_zc = 0;
+    b->rate_samples = 0;
+    b->slow_host = false;
+    b->rated_batch = b->batch_counter - 1;
     if (host_threads > 0 && !b->alpha_fixed) {
         gd_status st = calibrate_link(b);
         if (st != GD_OK) return st;
@@ -1229,31 +1231,48 @@ static void CUDART_CB chunk_gather_cb(void* arg) {
 //   otherwise the link binds and the smallest zero-copy share that keeps the staged path
 //   within it is best (zero-copy loads also slow the SMs they run on):
 //   alpha = 1 - r_host / r_link.
-static void adapt_alpha(gd_buffer* b, int d) {
-    StagedSlot& ss = b->stg[d];
-    if (ss.batch < 0) return;
-    if (cudaEventQuery(b->ev_E[d]) != cudaSuccess || cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
-        cudaGetLastError();                     // that batch is still in flight
-        return;
+static void adapt_alpha(gd_buffer* b) {
+    const int64_t bc = b->batch_counter;   // the batch being enqueued; slots of bc-1 .. bc-D+1 are intact
+    // (1) misses per batch, for the copy-engine staging size: the newest batch whose loop 2
+    // has run, from the word every slot's publication also writes (no event, no sync)
+    int64_t newest_epoch = 0;
+    for (int d = 0; d < b->D; ++d) {
+        const unsigned long long w = *(volatile const unsigned long long*)(b->stg[d].h_meta + 4);
+        if ((int64_t)(w >> 32) > newest_epoch) {
+            newest_epoch = (int64_t)(w >> 32);
+            b->m_est = (double)(w & 0xffffffffull);
+        }
     }
-    // misses per batch, for the copy-engine staging size (its pop finished long ago)
-    b->m_est = (double)((volatile int64_t*)ss.h_meta)[0];
-    if (b->alpha_fixed) return;
-    // (Balancing the two paths' concurrently measured durations instead was tried and
-    // measured worse: the zero-copy share is translation-bound and its SM loads slow the
-    // copy engine's transfers, so the smallest share that keeps the link busy wins.)
-    if (b->r_link <= 0) return;
-    const double staged_rows = (double)ss.h_meta[2], zc_rows = (double)ss.h_meta[1];
-    if (staged_rows >= 2048 && ss.cpu_ms > 0) {
-        const double r = staged_rows * (double)b->R / ss.cpu_ms;
-        b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
+    if (b->alpha_fixed || b->r_link <= 0) return;
+    // (2) path rates from the newest batch whose miss paths have finished and that has not
+    // been used yet (a caller Q + 1 batches ahead still finds batch bc - Q - 1 complete)
+    for (int k = 1; k < b->D && bc - k > b->rated_batch; ++k) {
+        const int d = (int)((bc - k) % b->D);
+        StagedSlot& ss = b->stg[d];
+        if (ss.batch != bc - k) break;
+        if (cudaEventQuery(b->ev_E[d]) != cudaSuccess || cudaEventQuery(b->ev_z1[d]) != cudaSuccess) {
+            cudaGetLastError();                     // still in flight: try an older one
+            continue;
+        }
+        // (Balancing the two paths' concurrently measured durations instead was tried and
+        // measured worse: the zero-copy share is translation-bound and its SM loads slow the
+        // copy engine's transfers, so the smallest share that keeps the link busy wins.)
+        const volatile int64_t* hm = ss.h_meta;
+        const double staged_rows = (double)hm[2], zc_rows = (double)hm[1];
+        if (staged_rows >= 2048 && ss.cpu_ms > 0) {
+            const double r = staged_rows * (double)b->R / ss.cpu_ms;
+            b->r_host = b->r_host > 0 ? 0.7 * b->r_host + 0.3 * r : r;
+            b->rate_samples++;
+        }
+        float tz = 0;
+        if (zc_rows >= 2048 && cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]) == cudaSuccess && tz > 0) {
+            const double r = zc_rows * (double)b->R / tz;
+            b->r_zc = b->r_zc > 0 ? 0.7 * b->r_zc + 0.3 * r : r;
+        }
+        cudaGetLastError();
+        b->rated_batch = bc - k;
+        break;
     }
-    float tz = 0;
-    if (zc_rows >= 2048 && cudaEventElapsedTime(&tz, b->ev_z0[d], b->ev_z1[d]) == cudaSuccess && tz > 0) {
-        const double r = zc_rows * (double)b->R / tz;
-        b->r_zc = b->r_zc > 0 ? 0.7 * b->r_zc + 0.3 * r : r;
-    }
-    cudaGetLastError();
     if (b->r_host <= 0) return;
     double a;
     if (b->r_zc > 0 && b->r_zc + b->r_host <= b->r_link)
@@ -1262,11 +1281,24 @@ static void adapt_alpha(gd_buffer* b, int d) {
         a = 1.0 - b->r_host / b->r_link;
     // With copy-engine staging the zero-copy share also costs the DMA engine: its random
     // 4 KB-page reads contend for the host's DMA translation, and a share above ~0.2 was
-    // measured to collapse the copy rate (to ~17 GB/s at 0.4); cap it there.  When the host
-    // gather cannot fill the link anyway (a slow or busy host: r_host < 0.65 r_link) the copy
-    // engine has slack, and 0.3 measured 3-6% better than 0.2 (0.4 still collapses).
-    const double hi = (b->ce_mode && b->dstage) ? (b->r_host < 0.65 * b->r_link ? 0.3 : 0.2) : 0.9;
+    // measured to collapse the copy rate (to ~17 GB/s at 0.4); cap it there.  Only a host
+    // whose gather persistently cannot fill the link (>= 8 rate samples below 0.6 r_link; back
+    // above 0.7 r_link to leave) gets 0.3: the copy engine has slack there (measured 3-6%
+    // better with 6 gather threads).  The hysteresis keeps one slow warm-up batch from
+    // switching the cap.
+    if (b->rate_samples >= 8 && b->r_host < 0.6 * b->r_link) b->slow_host = true;
+    if (b->r_host > 0.7 * b->r_link) b->slow_host = false;
+    const double hi = (b->ce_mode && b->dstage) ? (b->slow_host ? 0.3 : 0.2) : 0.9;
     b->alpha = std::min(hi, std::max(0.05, a));
+}
+
+gd_status gd_buffer_policy_read(gd_buffer* b, double* out, int32_t n) {
+    if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: bad handle");
+    if (!out || n < 0) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: null output");
+    const double v[8] = {b->alpha, b->r_host * 1e-6, b->r_zc * 1e-6, b->r_link * 1e-6, b->m_est,
+                         (double)b->rate_samples, b->slow_host ? 1.0 : 0.0, (double)b->rated_batch};
+    for (int k = 0; k < n && k < 8; ++k) out[k] = v[k];
+    return GD_OK;
 }
 
 // Contiguous host-link pull rate (bytes/ms), measured once on the staging memory.
@@ -1335,7 +1367,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // every stream is done with trip / host-list slot d (batch - D)
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));
     if (staged) {
-        adapt_alpha(b, (int)((b->batch_counter + b->D - 2) % b->D));
+        adapt_alpha(b);
         ss->batch = b->batch_counter;
     }
     const uint32_t alpha_q16 = staged ? (uint32_t)std::lround(b->alpha * 65536.0) : 65536u;
@@ -1398,7 +1430,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         pa.h_nodes = h_nodes_dev;
         pa.h_meta = h_meta_dev;
     }
-    pa.stats = stats;
+    pa.stats = peer ? nullptr : stats;   // with peers, k_peer_split writes stats[2..3] (final at `done`)
     pa.ticket = b->tickets;
     pa.done_word = b->done_word;
     pa.epoch = ++b->epoch;
@@ -1439,7 +1471,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         k_peer_probe<<<148 * 2, 256, 0, b->side>>>(trip, tcount, b->peers, b->npeers, b->slots, (uint8_t*)out, b->R,
                                                   mtrip, mcount_d, b->peer_ctr);
         GD_DEBUG_AFTER("k_peer_probe", b->side);
-        k_peer_split<<<148, 256, 0, b->side>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats);
+        k_peer_split<<<148, 256, 0, b->side>>>(mtrip, mcount_d, msplit, alpha_q16, cap, h_nodes_dev, h_meta_dev, stats,
+                                              pa.epoch);
         GD_DEBUG_AFTER("k_peer_split", b->side);
         GD_CUDA(cudaEventRecord(b->ev_S, b->side));
     }

@@ -68,7 +68,8 @@ struct StagedSlot {
     gd_buffer* owner = nullptr;
     int d = 0;
     int32_t* h_nodes = nullptr;   // pinned, mapped [n_max]: node ids of the staged share
-    int64_t* h_meta = nullptr;    // pinned, mapped [4]: M, K0, staged rows, 0
+    int64_t* h_meta = nullptr;    // pinned, mapped [8]: M, K0, staged rows, -, (epoch << 32 | M) of the
+                                  // newest batch that used this slot (read for the staging size)
     uint8_t* staging = nullptr;   // pinned, mapped [n_max x R]
     double cpu_ms = 0;            // duration of the last host gather into this slot
     int64_t batch = -1;           // batch that last used this slot
@@ -128,6 +129,9 @@ struct gd_buffer {
     double r_zc = 0;                     // EMA of the zero-copy copy rate (bytes/ms)
     double r_link = 0;                   // contiguous pull rate of the host link (bytes/ms), calibrated
     bool alpha_fixed = false;
+    int64_t rate_samples = 0;            // host-gather rate samples since the last config
+    bool slow_host = false;              // r_host persistently < 0.6 r_link (zero-copy cap 0.3)
+    int64_t rated_batch = -1;            // newest batch whose path rates entered the estimates
     gd::HostGatherPool* pool = nullptr;
     // phase 2 of the staged share: copy engine (cudaMemcpyAsync pinned slot -> dstage[d]
     // on stream H, then a scatter kernel on P) or an SM pull kernel reading the pinned slot

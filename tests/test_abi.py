@@ -67,3 +67,33 @@ def test_null_handles_rejected(gd):
     assert L.gd_check_device_status(None, None) == 1
     assert b"null" in L.gd_last_error()
     assert L.gd_graph_destroy(None) == 0 and L.gd_buffer_destroy(None) == 0
+
+
+def test_plain_c_client_compiles_links_and_runs(gd, tmp_path):
+    """gd.h is a C header (gcc -std=c99, no nvcc, no CUDA headers): a plain C client takes the
+    address of every declared entry point, links against libgd.so and runs its host-only calls."""
+    names = declared_functions()
+    src = tmp_path / "client.c"
+    src.write_text(
+        '#include <stdio.h>\n#include "gd.h"\n'
+        "int main(void) {\n"
+        f"    void* syms[] = {{ {', '.join('(void*)' + n for n in names)} }};\n"
+        f"    for (unsigned i = 0; i < {len(names)}u; ++i) if (!syms[i]) return 10;\n"
+        "    int32_t fan[3] = {15, 10, 5};\n"
+        "    int64_t nm[4], em[3];\n"
+        "    if (gd_sample_bounds(1000, fan, 3, 111000000, 1600000000, nm, em) != GD_OK) return 11;\n"
+        "    if (nm[3] != 1056000 || em[2] != 880000) return 12;\n"
+        "    int32_t bad[1] = {GD_MAX_FANOUT + 1};\n"
+        "    if (gd_sample_bounds(10, bad, 1, 100, 1000, nm, em) != GD_ERR_INVALID) return 13;\n"
+        "    if (gd_last_error()[0] == 0) return 14;\n"
+        "    if (gd_extract(NULL, NULL, NULL, 0, NULL, NULL, NULL, NULL, NULL) != GD_ERR_INVALID) return 15;\n"
+        '    printf("%d\\n", gd_version());\n'
+        "    return 0;\n}\n")
+    exe = tmp_path / "client"
+    libdir = os.path.dirname(gd.LIB_PATH)
+    r = subprocess.run(["gcc", "-std=c99", "-Wall", "-Werror", "-I", os.path.join(ROOT, "include"), str(src), "-o",
+                        str(exe), "-L", libdir, "-l:libgd.so", f"-Wl,-rpath,{libdir}"], capture_output=True, text=True)
+    assert r.returncode == 0, r.stderr
+    r = subprocess.run([str(exe)], capture_output=True, text=True)
+    assert r.returncode == 0, (r.returncode, r.stderr)
+    assert int(r.stdout) == gd.lib.gd_version()

@@ -252,6 +252,55 @@ def test_release_on_its_own_stream_matches_oracle(tiny, gd, own_stream, row_byte
     assert buf.check() == 0
 
 
+def test_adaptive_split_stages_without_host_sync(gd):
+    """a caller that never synchronises (the host may run many batches ahead of the
+    device) still gets a miss-count estimate for the copy-engine staging size (each batch's
+    count is published with its epoch into mapped host memory), so the staged share starts
+    after warm-up instead of every miss going zero-copy; all 40 batches stay bit-exact."""
+    N, E, B, fan, Q, nbat = 200_000, 2_000_000, 1000, [10, 5], 4, 40
+    indptr, indices = make_graph(N, E, seed=21)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, 512)
+    order = synth.epoch_order(synth.train_nodes(N, 0.5))
+    nb, _ = O.sample_bounds(B, fan, N, E)
+    n_max = nb[-1]
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), Q * n_max, Q, n_max)
+    buf.config(4, -1.0)
+    seeds = [order[b * B:(b + 1) * B].cuda() for b in range(nbat)]
+    stats = torch.zeros((nbat, 4), dtype=torch.int64, device="cuda")
+    res, outs, aliases, pending = [], [], [], []
+    for b in range(nbat):
+        r = g.sample(seeds[b], fan, 3, b)
+        a = torch.empty(n_max, dtype=torch.int32, device="cuda")
+        out, _, _ = buf.extract(r.n_id, r.num_nodes_dev, r.max_nodes, alias=a, stats=stats[b])
+        res.append(r), outs.append(out), aliases.append(a)
+        pending.append(r)
+        if len(pending) == Q:
+            r0 = pending.pop(0)
+            buf.release(r0.n_id, r0.num_nodes_dev, r0.max_nodes)
+    torch.cuda.synchronize()
+    st = stats.cpu()
+    assert int(st[:, 1].sum()) > 0
+    assert int(st[10:, 3].sum()) > 0, st[:, 2:].tolist()        # the staged share ran
+    pol = buf.policy_read()
+    assert pol["misses_est"] > 0 and 0.05 <= pol["zero_copy_share"] <= 0.3, pol
+    ob = O.Buffer(feat, Q * n_max)
+    opend = []
+    for b in range(nbat):
+        n_id = res[b].to_host()["n_id"]
+        o_out, o_alias, o_stats = ob.extract(n_id)
+        n = len(n_id)
+        assert tuple(st[b].tolist()[:2]) == o_stats, b
+        assert int(st[b][2] + st[b][3]) == o_stats[1], b               # the split covers every miss
+        assert np.array_equal(aliases[b][:n].cpu().numpy(), o_alias), b
+        assert np.array_equal(outs[b][:n].cpu().numpy(), o_out), b
+        opend.append(n_id)
+        if len(opend) == Q:
+            ob.release(opend.pop(0))
+    compare_state(buf, ob)
+    assert buf.check() == 0
+
+
 # phase 2 of the staged share: SM pull of the pinned slot, or copy engine with the
 # default 8 MB chunk ring, with 64 KB chunks (many chunks per batch, ring reuse), or
 # with one chunk per batch (GD_STAGE_CHUNK_KB=0)

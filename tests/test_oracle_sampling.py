@@ -203,3 +203,57 @@ def test_generator_cpu_is_deterministic():
     a = synth.chung_lu_csr(5000, 40000)
     b = synth.chung_lu_csr(5000, 40000)
     assert torch.equal(a[0], b[0]) and torch.equal(a[1], b[1])
+
+
+def _py_positions(v, d, f, hop0, b, seed):
+    """R2-R3 written out in Python: Floyd over draws floor(u (j+1) / 2^64), u the Philox draw
+    word keyed (t, v, hop index, batch id) (the word itself is pinned to curand in
+    test_oracle_rng), positions ascending; f < 0 or d <= f: the whole row."""
+    if f < 0 or d <= f:
+        return list(range(d))
+    S = []
+    for t in range(f):
+        j = d - f + t
+        r = (O.draw_word(t, v, hop0, b, seed) * (j + 1)) >> 64
+        S.append(j if r in S else r)
+    return sorted(S)
+
+
+def test_sample_rows_are_keyed_by_node_hop_and_batch(tiny):
+    """Pins the wiring inside oracle_sample: every row of every hop of a
+    multi-hop sample is exactly indptr[v] + positions(v, deg v, f_h, h - 1, batch_id).  A
+    swapped or 1-based hop index, a wrong batch id or a frontier-index key fails here, which
+    the invariant and BFS pins cannot see."""
+    cfg, indptr, indices, order = tiny
+    seed = 7
+    for b, fan in ((0, [5, 5]), (3, [15, 10, 5]), (123456, [2, 3, 4, 1])):
+        seeds = synth.batch_seeds(order, 48, b % 10).numpy()
+        res = O.sample(indptr, indices, seeds, fan, seed, b)
+        checked = 0
+        for h in range(1, len(fan) + 1):
+            rp, eid = res.rowptr[h - 1], res.eid[h - 1]
+            for i in range(int(res.sizes[h - 1])):
+                v = int(res.n_id[i])
+                d = int(indptr[v + 1] - indptr[v])
+                want = [int(indptr[v]) + p for p in _py_positions(v, d, fan[h - 1], h - 1, b, seed)]
+                assert eid[rp[i]:rp[i + 1]].tolist() == want, (b, h, i, v)
+                checked += d > fan[h - 1] >= 0
+        assert checked > 50      # plenty of rows where the draws decide
+
+
+def test_star_hub_uniform_through_oracle_sample():
+    """SURVEY P3 through the whole sampler: a star hub with 6 leaves sampled with fanout 2 in
+    6000 mini-batches (batch id = the only thing that varies) picks each of the 15 leaf pairs
+    uniformly (chi-square), and the relabel puts them in ascending position order."""
+    from scipy.stats import chisquare
+    indptr, indices = csr_from_lists([[1, 2, 3, 4, 5, 6]] + [[0]] * 6)
+    seeds = np.array([0], dtype=np.int32)
+    counts = Counter()
+    for b in range(6000):
+        res = O.sample(indptr, indices, seeds, [2], 3, b)
+        pair = tuple(res.n_id[1:].tolist())
+        assert len(pair) == 2 and pair[0] < pair[1] and res.col[0].tolist() == [1, 2]
+        counts[pair] += 1
+    obs = [counts[c] for c in itertools.combinations(range(1, 7), 2)]
+    assert sum(obs) == 6000
+    assert chisquare(obs).pvalue > 1e-4
