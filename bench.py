@@ -31,6 +31,7 @@ import numpy as np  # noqa: E402
 import torch  # noqa: E402
 
 import synth  # noqa: E402
+from synth.host import HostTable, SharedArray, batch_schedule, bind_to_gpu_socket, set_interleave  # noqa: E402
 
 Q = 4   # release lag = training-queue capacity
 
@@ -53,7 +54,12 @@ def parse():
     p.add_argument("--lr", type=float, default=0.01, help="f4 SGD learning rate")
     p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
                    "peer (CUDA IPC); misses are served from peers' HBM before the host link")
-    p.add_argument("--parity-batches", type=int, default=2, help="sampled full-size parity checks vs the oracle")
+    p.add_argument("--parity-batches", type=int, default=None,
+                   help="first batches of each rank checked in full (sample outputs, alias, hits/misses, rows) vs the "
+                        "oracle; default 8 (papers100m/friendster/mag240m; 4 per rank at >= 8 ranks), 16 (products), "
+                        "all of the rank's segment (tiny)")
+    p.add_argument("--no-replay", action="store_true",
+                   help="skip the steady-state parity: the oracle's Alg. 1 replayed over the rank's whole schedule")
     p.add_argument("--prewarm-max", type=int, default=400,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
@@ -67,6 +73,71 @@ def parse():
 
 
 # ----------------------------------------------------------------------------- helpers
+# (torch.distributed directly: the reference arm must not load the product package / libgd.so)
+
+def _dist_on():
+    import torch.distributed as dist
+    return dist.is_available() and dist.is_initialized()
+
+
+def barrier():
+    if _dist_on():
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def _reduce(x: float, op, device=None) -> float:
+    if not _dist_on():
+        return float(x)
+    import torch.distributed as dist
+    t = torch.tensor([float(x)], dtype=torch.float64, device=None if dist.get_backend() == "gloo" else device)
+    dist.all_reduce(t, op=op)
+    return float(t.item())
+
+
+def max_over_ranks(x: float, device=None) -> float:
+    import torch.distributed as dist
+    return _reduce(x, dist.ReduceOp.MAX, device)
+
+
+def sum_over_ranks(x: float, device=None) -> float:
+    import torch.distributed as dist
+    return _reduce(x, dist.ReduceOp.SUM, device)
+
+
+def gather_objects(obj, world):
+    """Every rank's `obj` (a list indexed by rank) on every rank."""
+    if world == 1 or not _dist_on():
+        return [obj]
+    import torch.distributed as dist
+    out = [None] * world
+    dist.all_gather_object(out, obj)
+    return out
+
+
+def default_parity_batches(cfg, world, seg_len):
+    """SURVEY 8(d) parity plan: all batches (tiny), the first 16 (products), the first 8 per GPU
+    (papers100m / friendster / mag240m; 4 per GPU at 8 GPUs)."""
+    if cfg.name == "tiny":
+        return seg_len
+    if cfg.name == "products":
+        return 16
+    return 4 if world >= 8 else 8
+
+
+def loaded_native_libs():
+    """Shared objects of this repo mapped into this process (reference-arm hygiene)."""
+    libs = set()
+    try:
+        with open("/proc/self/maps") as f:
+            for line in f:
+                path = line.split()[-1] if line.strip() else ""
+                if path.startswith(ROOT) and ".so" in path:
+                    libs.add(os.path.relpath(path, ROOT))
+    except OSError:
+        pass
+    return sorted(libs)
+
 
 def log(*a):
     if int(os.environ.get("RANK", "0")) == 0:
@@ -121,8 +192,9 @@ class ClockSampler:
                 "reasons": reasons, "samples": len(self.rows), "source": "NVML, 200 ms"}
 
 
-def h2d_peak_gbps(device) -> float:
-    """Host-link roofline measured in-run: pinned 1 GiB cudaMemcpyAsync H2D, best of 10."""
+def h2d_peak_gbps(device, sync=None, reps: int = 10) -> float:
+    """Host-link roofline measured in-run: pinned 1 GiB cudaMemcpyAsync H2D, best of `reps`.
+    sync: called before every repetition (a barrier, so that all ranks copy at once)."""
     n = 1 << 30
     h = torch.empty(n, dtype=torch.uint8, pin_memory=True)
     h.fill_(1)
@@ -130,7 +202,9 @@ def h2d_peak_gbps(device) -> float:
     s = torch.cuda.Stream(device)
     best = 0.0
     with torch.cuda.stream(s):
-        for _ in range(10):
+        for _ in range(reps):
+            if sync is not None:
+                sync()
             a = torch.cuda.Event(enable_timing=True)
             b = torch.cuda.Event(enable_timing=True)
             a.record(s)
@@ -140,6 +214,24 @@ def h2d_peak_gbps(device) -> float:
             best = max(best, n / (a.elapsed_time(b) * 1e6))
     del h, d
     return best
+
+
+def h2d_peaks(device, rank, world):
+    """the host-link denominators at G GPUs.  `alone`: this rank's link with the
+    other ranks idle (ranks take turns between barriers); `concurrent`: every rank copies at
+    the same time (a barrier before each of the 10 repetitions), the per-GPU share of the
+    links the G GPUs contend for (PCIe switch uplinks, host DRAM)."""
+    if world == 1:
+        v = h2d_peak_gbps(device)
+        return {"alone": v, "concurrent": v}
+    alone = 0.0
+    for r in range(world):
+        barrier()
+        if r == rank:
+            alone = h2d_peak_gbps(device)
+        barrier()
+    conc = h2d_peak_gbps(device, sync=barrier)
+    return {"alone": alone, "concurrent": conc}
 
 
 def measured_peaks():
@@ -170,7 +262,6 @@ class Workload:
     """Graph, host table, seeds of one config on this rank (setup, not timed)."""
 
     def __init__(self, cfg, rank, world, device, need_host_csr):
-        from paper_conf_icpp_jiangj024_b200.multigpu import HostTable, barrier
         self.cfg = cfg
         t0 = time.time()
         indptr, indices = synth.chung_lu_csr(cfg.num_nodes, cfg.num_edges, device=device)
@@ -181,8 +272,24 @@ class Workload:
         self.deg_stats = {"max": int(deg.max()), "mean": float(cfg.num_edges / cfg.num_nodes),
                           "p99": int(torch.quantile(deg[:: max(1, cfg.num_nodes // 1_000_000)].double(), 0.99))}
         del deg
-        self.host_indptr = indptr.cpu().numpy() if need_host_csr else None
-        self.host_indices = indices.cpu().numpy() if need_host_csr else None
+        # host CSR for the oracle (parity, replay, cpu baseline): private at world 1, one shared
+        # copy at world > 1 (rank 0 writes it; "topological data ... shared")
+        self._csr_shm = []
+        if need_host_csr and world == 1:
+            self.host_indptr, self.host_indices = indptr.cpu().numpy(), indices.cpu().numpy()
+        elif need_host_csr:
+            a = SharedArray((cfg.num_nodes + 1,), np.int64, f"{cfg.name}_indptr", rank, world)
+            b = SharedArray((cfg.num_edges,), np.int32, f"{cfg.name}_indices", rank, world)
+            if rank == 0:
+                a.array[:] = indptr.cpu().numpy()
+                step = 1 << 28
+                for s0 in range(0, cfg.num_edges, step):
+                    b.array[s0:s0 + step] = indices[s0:s0 + step].cpu().numpy()
+            barrier()
+            self._csr_shm = [a, b]
+            self.host_indptr, self.host_indices = a.array, b.array
+        else:
+            self.host_indptr = self.host_indices = None
         self.indptr, self.indices = indptr, indices
         t0 = time.time()
         self.table = HostTable(cfg.host_rows, cfg.row_bytes, cfg.name, rank, world)
@@ -194,7 +301,6 @@ class Workload:
         self._barrier = barrier if world > 1 else (lambda: None)   # world 1: also under torchrun (reference arm)
         self.registered = False
         if rank == 0 and device.type == "cuda":
-            from paper_conf_icpp_jiangj024_b200.multigpu import set_interleave
             self.interleaved = world > 1 and set_interleave(True)   # the pages fault in here
             try:
                 self._register()
@@ -239,6 +345,9 @@ class Workload:
         if self.registered:
             torch.cuda.cudart().cudaHostUnregister(self.table.tensor.data_ptr())
         self.table.close()
+        self.host_indptr = self.host_indices = None
+        for a in self._csr_shm:
+            a.close()
 
     def seeds(self, b, epoch):
         if epoch not in self._orders:
@@ -266,13 +375,20 @@ def config_from_args(args):
 
 def run_ours(args, rank, world, local_rank):
     import paper_conf_icpp_jiangj024_b200 as gd
-    from paper_conf_icpp_jiangj024_b200.multigpu import barrier, batch_schedule, max_over_ranks, sum_over_ranks
 
     cfg = config_from_args(args)
     dev = torch.device("cuda", local_rank)
     torch.cuda.set_device(dev)
+    # NUMA: each rank (and the host-gather pool / CUDA callback threads it creates later) on the
+    # CPUs of its GPU's socket, so its pinned staging is first-touched there; at N = 1
+    # only with GD_NUMA_BIND=1 (one rank may use every core)
+    if os.environ.get("GD_NUMA_BIND", "1" if world > 1 else "0") == "1":
+        numa = bind_to_gpu_socket(local_rank)
+    else:
+        numa = {"bound": False, "cpus": len(os.sched_getaffinity(0))}
     want_cpu = (not args.no_cpu_baseline) and rank == 0 and world == 1 and not args.train
-    need_host_csr = want_cpu or (rank == 0 and args.parity_batches > 0)
+    want_replay = not args.no_replay
+    need_host_csr = want_cpu or want_replay or args.parity_batches != 0
     W, K = args.warmup, args.steps
     t_setup = time.time()
     wl = Workload(cfg, rank, world, dev, need_host_csr)
@@ -408,9 +524,11 @@ def run_ours(args, rank, world, local_rank):
 
     # ---- full-size sampled parity vs the oracle (untimed; first batches of this rank)
     parity = None
-    if rank == 0 and args.parity_batches > 0:
-        log("parity check ...")
-        parity = check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev)
+    n_par = args.parity_batches if args.parity_batches is not None else default_parity_batches(
+        cfg, world, len(synth.segment(wl.num_batches, rank, world)))
+    if n_par > 0:
+        log(f"parity check ({n_par} batches per rank) ...")
+        parity = check_parity(n_par, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev, world)
         buf.close()
         buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank,
                                num_nodes=cfg.num_nodes)
@@ -481,6 +599,7 @@ def run_ours(args, rank, world, local_rank):
         windows = [round(args.window / (a_.elapsed_time(b_) / 1e3), 1) for a_, b_ in zip(marks, marks[1:])]
     tg = g.timing_read()
     tb = buf.timing_read()
+    policy = buf.policy_read() if not cfg.preload else None
     st = stats[off + W:off + W + K].sum(0).cpu().tolist()
     sz = sizes_log[off + W:off + W + K].double().mean(0).cpu().tolist()
     hits, misses, miss_zc, miss_staged = (int(x) for x in st)
@@ -548,6 +667,21 @@ def run_ours(args, rank, world, local_rank):
                "read_back": f"each step's sizes + hit/miss stats copied D2H into pinned memory on the stream and "
                             f"read by the host {Q} steps later (queue depth Q, P:177; the last {Q} inside the timed "
                             f"region)"}
+    # ---- capture for the steady-state replay: this rank's buffer has run steps
+    # [0, j_win) (pre-warm, warm-up, timed, e2e); keep their per-batch sizes and hit/miss
+    # counts, the last RING batches' n_id + alias and the whole buffer state for the oracle
+    j_win = off + W + K + (0 if args.no_e2e else K)
+    replay_cap = None
+    if want_replay:
+        torch.cuda.synchronize(dev)
+        stats_h = stats[:j_win].cpu().numpy()
+        sizes_h = sizes_log[:j_win].cpu().numpy()
+        tail = {}
+        for j in range(max(0, j_win - RING), j_win):
+            s_ = j % RING
+            n_j = int(sizes_h[j][len(fan)])
+            tail[j] = (outs[s_].n_id[:n_j].cpu().numpy(), aliases[s_][:n_j].cpu().numpy())
+        replay_cap = (j_win, stats_h, sizes_h, tail, buf.snapshot())
     # ---- optional in-process sweep of the miss-stream configuration (tuning only)
     sweep = []
     j0 = off + W + K + (0 if args.no_e2e else K)
@@ -654,7 +788,8 @@ def run_ours(args, rank, world, local_rank):
     hbm_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)"
     if not hbm_peak:   # B200_PROFILING.md: fallback only when the driver-written file is absent
         hbm_peak, hbm_src = 6650.0, "of fallback: B200_PROFILING.md 6.65 TB/s (MEASURED_PEAKS.json absent)"
-    link_peak = h2d_peak_gbps(dev)
+    link_peaks = h2d_peaks(dev, rank, world)
+    link_peak = link_peaks["concurrent"]          # the denominator at G GPUs
     R = cfg.row_bytes
     region_s = ms / 1e3
     nb = max(1, tb["batches"])
@@ -693,7 +828,17 @@ def run_ours(args, rank, world, local_rank):
                  "per_path_GBps": {"zero_copy_kernel": rnd(zc_gbs), "staged_pull_or_scatter_kernel": rnd(pull_gbs),
                                    "staged_copy_engine_h2d": rnd(ce_gbs), "host_gather_phase1": rnd(host_gbs)},
                  "misses_zero_copy": miss_zc, "misses_staged": miss_staged,
-                 "peak_source": "in-run pinned 1 GiB H2D cudaMemcpyAsync, best of 10"}
+                 "peak_source": "in-run pinned 1 GiB H2D cudaMemcpyAsync, best of 10" + (
+                     ", all ranks copying at once (barrier per repetition)" if world > 1 else "")}
+    if world > 1:   # the whole job: every rank's misses over the slowest rank's region, vs the summed concurrent peaks
+        tot_bytes = sum_over_ranks(R * misses, dev)
+        tot_peak = sum_over_ranks(link_peak, dev)
+        roof_miss["rank0"] = {"achieved": roof_miss["achieved"], "peak": roof_miss["peak"], "frac": roof_miss["frac"]}
+        roof_miss["achieved"] = rnd(tot_bytes / (ms_max / 1e3) / 1e9)
+        roof_miss["peak"] = round(tot_peak, 2)
+        roof_miss["frac"] = rnd(roof_miss["achieved"] / tot_peak, 4) if tot_bytes else None
+        roof_miss["achieved_def"] = ("row bytes of all ranks' misses / the slowest rank's timed region, against the "
+                                     "sum of the per-rank concurrent H2D peaks")
     miss_busy = max(kern["miss_zero_copy_ms_per_batch"], kern["miss_staged_pull_ms_per_batch"],
                     kern["staged_copy_engine_ms_per_batch"])
     dominant = roof_miss if misses > 0 and miss_busy >= kern["gather_ms_per_batch"] else roof_gather
@@ -729,10 +874,27 @@ def run_ours(args, rank, world, local_rank):
         served_all, probed_all = sum_over_ranks(served, dev), sum_over_ranks(probed, dev)
         peer_info = {"served_rows": int(served_all), "probed_misses": int(probed_all),
                      "served_share": round(served_all / max(1, probed_all), 4), "peers_per_rank": min(world - 1, 7)}
+    # ---- steady-state parity: the oracle replays this rank's whole schedule (CPU only)
+    replay, single = None, None
+    if replay_cap is not None:
+        log(f"oracle replay of {replay_cap[0]} batches ...")
+        thr = max(2, (os.cpu_count() or 2) // world)
+        keep = want_cpu and S * R <= 48e9
+        replay, single = oracle_replay(cfg, wl, seeds_host, batch_ids, fan, S, *replay_cap, threads=thr,
+                                       keep_rows=keep, t_single=0.5 * args.cpu_seconds if want_cpu else 0.0)
+        log(f"replay: {replay}")
+    first_all = gather_objects(parity, world)
+    replay_all = gather_objects(replay, world)
+    parity_out = {"first": first_all[0] if world == 1 else first_all,
+                  "steady_state": replay_all[0] if world == 1 else replay_all,
+                  "bit_exact": all(x is None or x["bit_exact"] for x in first_all + replay_all)}
     cpu = None
     log("cpu baseline ...")
     if want_cpu:
-        cpu = cpu_baseline(cfg, wl, sched, batch_ids, fan, S, args.cpu_seconds)
+        cpu = cpu_variant_baseline(cfg, wl.table.array, wl.host_indptr, wl.host_indices, seeds_host, batch_ids, fan,
+                                   args.cpu_seconds, len(os.sched_getaffinity(0)))
+        cpu["single_thread_full_oracle"] = single
+        cpu["host_cpu"] = host_cpu_info()
     total_batches = sum_over_ranks(K, dev)
     value = total_batches / (ms_max / 1e3)
     line = {
@@ -740,14 +902,7 @@ def run_ours(args, rank, world, local_rank):
         "value": round(value, 2), "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": round(ms_max / K, 4), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-        "config": {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
-                   "feat_dim": cfg.feat_dim, "feat_bytes": R, "batch_size": cfg.batch_size, "fanouts": fan,
-                   "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
-                   "buffer_prewarm_batches": prewarm_batches,
-                   "parallelism": f"dp{world} (batch segments, no collective)",
-                   "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
-                       (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.host_rows * R * 1e-9),
-                   "host_table_rows": cfg.host_rows},
+        "config": config_dict(cfg, S, world, prewarm_batches),
         "e2e": e2e,
         # per step: seed intake + K x (sample, relabel) + col resolve + hash clear | lookup, pop/assign, hit gather
         # [+ zero-copy miss copy + peer-tag publish unless preload] [+ staged scatter when the host
@@ -764,8 +919,11 @@ def run_ours(args, rank, world, local_rank):
         "per_batch": {"n_nodes": round(sz[len(fan)], 1), "edges": [round(x, 1) for x in sz[len(fan) + 1:]],
                       "hits": hits / K, "misses": misses / K,
                       "hit_rate": round(hits / max(1, hits + misses), 4), **{k: round(v, 4) for k, v in kern.items()}},
-        "parity": parity,
+        "miss_policy": {k: (round(v, 3) if isinstance(v, float) else v) for k, v in policy.items()} if policy else None,
+        "parity": parity_out,
         "rows_check": rows_check,
+        "host_link_peaks_GBps": {k: round(v, 2) for k, v in link_peaks.items()},
+        "numa": numa,
         "windows": windows,
         "sweep": sweep or None,
         "pipeline": pipe_res or None,
@@ -796,16 +954,20 @@ def load_traffic(config_name):
         return None
 
 
-def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
-    """Full-size sampled parity: the first batches in the bench's launch configuration,
-    checked bit-exactly against the oracle (sampling outputs, alias, hit/miss, out rows)."""
+def check_parity(n_par, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev, world):
+    """Full-size cold parity: this rank's first `n_par` batches in the bench's launch
+    configuration, bit-exact against the oracle: sampling outputs (sizes, n_id, rowptr, col,
+    eid), alias, hits/misses, and the out rows (the oracle's slot rows at world 1; the closed
+    form table[n_id mod P] (P5) at world > 1, where each rank's replay buffer keeps no rows)."""
     from oracle import oracle as O
     t0 = time.time()
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
+    keep = world == 1
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes, keep_rows=keep)
     log(f"  oracle buffer ready {time.time() - t0:.1f}s")
     res_ok = True
     checked = 0
-    for j in range(min(args.parity_batches, len(sched))):
+    pend = []
+    for j in range(min(n_par, len(sched))):
         b, ep = sched[j]
         seeds = wl.seeds(b, ep)
         o = g.sample(seeds.to(dev), fan, synth.RNG_SEED, batch_ids[j], with_eid=True)
@@ -819,46 +981,179 @@ def check_parity(args, cfg, g, buf, wl, sched, batch_ids, fan, n_max, S, dev):
         for k in range(len(fan)):
             ok &= np.array_equal(h["rowptr"][k], ref.rowptr[k]) and np.array_equal(h["col"][k], ref.col[k])
             ok &= np.array_equal(h["eid"][k], ref.eid[k])
-        log(f"  batch {j}: gpu+oracle sample done {time.time() - t0:.1f}s, ok={ok}")
         o_out, o_alias, o_st = ob.extract(ref.n_id)
         n = len(ref.n_id)
         ok &= tuple(st.cpu().tolist()[:2]) == o_st
         ok &= np.array_equal(alias[:n].cpu().numpy(), o_alias)
-        ok &= np.array_equal(out[:n].cpu().numpy(), o_out)
+        got = out[:n].cpu().numpy()
+        ok &= np.array_equal(got, o_out if keep else wl.table.array[ref.n_id.astype(np.int64) % cfg.host_rows])
+        pend.append((o, ref.n_id))           # release with lag Q, as the timed loop does
+        if len(pend) == Q:
+            o0, n0 = pend.pop(0)
+            buf.release(o0.n_id, o0.num_nodes_dev, o0.max_nodes)
+            ob.release(n0)
         res_ok &= bool(ok)
         checked += 1
-    return {"batches": checked, "bit_exact": res_ok, "seconds": round(time.time() - t0, 1)}
+        log(f"  batch {j}: ok={ok} ({time.time() - t0:.1f}s)")
+    torch.cuda.synchronize(dev)
+    return {"batches": checked, "bit_exact": res_ok, "seconds": round(time.time() - t0, 1),
+            "rows_vs": "oracle slot rows" if keep else "closed form table[n_id mod P]"}
 
 
-def cpu_baseline(cfg, wl, sched, batch_ids, fan, S, budget_s):
-    """The oracle as it stands, single-threaded on this host, on a bounded sample of the same
-    workload: full steps (sample + Alg. 1 extract + release with lag Q) until budget_s."""
+def oracle_replay(cfg, wl, seeds_host, batch_ids, fan, S, j_end, stats_h, sizes_h, tail, gpu_state, threads,
+                  keep_rows, t_single=0.0):
+    """Steady-state parity: the oracle's Alg. 1 replayed over this
+    rank's WHOLE schedule [0, j_end) -- pre-warm, warm-up, timed and e2e batches, with the same
+    release lag Q -- from its own sampling (never the GPU's n_id).  Compared per batch: the 2K+1
+    block sizes and (hits, misses); for the last batches still in the bench's ring: n_id and
+    alias; at the end: the whole buffer state (map slot / refcount / valid bit, reverse map,
+    standby list in LRU order) against the GPU's snapshot.  Sampling runs `threads`-wide
+    ahead (independent per batch); Alg. 1 itself is sequential, as the paper's.
+    t_single > 0 (world 1): afterwards, the full oracle (sample + extract with rows + release)
+    on one thread from this warm state for about t_single seconds: the single-thread figure."""
+    from concurrent.futures import ThreadPoolExecutor
     from oracle import oracle as O
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
+    t0 = time.time()
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes, keep_rows=keep_rows)
+    t_buf = time.time() - t0
+    K = len(fan)
+
+    def samp(j):
+        return O.sample(wl.host_indptr, wl.host_indices, seeds_host[j].numpy(), fan, synth.RNG_SEED, batch_ids[j])
+
+    bad_sizes, bad_stats, bad_tail = [], [], []
     pend = []
-    n = 0
+    hits = misses = 0
+    with ThreadPoolExecutor(max(1, threads)) as ex:
+        futs, nxt = {}, 0
+        for j in range(j_end):
+            while nxt < min(j_end, j + 2 * max(1, threads)):
+                futs[nxt] = ex.submit(samp, nxt)
+                nxt += 1
+            ref = futs.pop(j).result()
+            if not np.array_equal(ref.sizes, sizes_h[j]):
+                bad_sizes.append(j)
+            _, alias, st = ob.extract(ref.n_id, want_out=False)
+            hits += st[0]
+            misses += st[1]
+            if st != (int(stats_h[j][0]), int(stats_h[j][1])):
+                bad_stats.append(j)
+            if j in tail:
+                g_nid, g_alias = tail[j]
+                if not (np.array_equal(g_nid, ref.n_id) and np.array_equal(g_alias, alias)):
+                    bad_tail.append(j)
+            pend.append(ref.n_id)
+            if len(pend) == Q:
+                ob.release(pend.pop(0))
+    t_replay = time.time() - t0
+    st_ok = None
+    if gpu_state is not None:
+        o = ob.state()
+        st_ok = all(np.array_equal(gpu_state[k], o[k]) for k in ("slot", "rc", "valid", "reverse", "standby"))
+    res = {"batches": j_end, "hits": int(hits), "misses": int(misses), "sizes_equal": not bad_sizes,
+           "hits_misses_equal": not bad_stats, "tail_batches_n_id_alias": len(tail), "tail_equal": not bad_tail,
+           "final_state_equal": st_ok,
+           "bit_exact": not bad_sizes and not bad_stats and not bad_tail and st_ok is not False,
+           "first_mismatch": min(bad_sizes + bad_stats + bad_tail) if (bad_sizes or bad_stats or bad_tail) else None,
+           "seconds": round(t_replay, 1), "oracle_buffer_s": round(t_buf, 1), "sampler_threads": threads}
+    single = None
+    if t_single > 0 and keep_rows:
+        n, t1 = 0, time.perf_counter()
+        while True:
+            j = j_end + n
+            ref = samp(j % len(batch_ids))
+            ob.extract(ref.n_id, want_out=True)
+            pend.append(ref.n_id)
+            if len(pend) == Q:
+                ob.release(pend.pop(0))
+            n += 1
+            el = time.perf_counter() - t1
+            if el >= t_single or n >= 10_000:
+                break
+        single = {"value": round(n / el, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
+                  "sample": f"{n} full mini-batches (sample + Alg. 1 extract with rows + release, Q={Q}) continuing "
+                            f"from the replayed steady-state buffer, {el:.1f} s on 1 host thread"}
+    return res, single
+
+
+def cpu_variant_baseline(cfg, table, indptr, indices, seeds_host, batch_ids, fan, budget_s, threads, n_target=None):
+    """SURVEY 8(d) CPU baseline: the oracle's sample + relabel on `threads` host threads, one
+    independent batch stream per thread (the paper's per-subprocess model), rows gathered
+    straight from the host table (every row host-resident: the CPU variant's data path, P:152,
+    without an SSD).  Runs until budget_s (or n_target batches in total); value = batches
+    finished / wall time of the slowest thread."""
+    from concurrent.futures import ThreadPoolExecutor
+    from oracle import oracle as O
+    R = table.shape[1]
+    CH = max(1, (16 << 20) // R)                     # gather in 16 MB chunks per thread
+    nb = len(batch_ids)
     t0 = time.perf_counter()
-    while True:
-        b, ep = sched[n % len(sched)]
-        ref = O.sample(wl.host_indptr, wl.host_indices, wl.seeds(b, ep).cpu().numpy(), fan, synth.RNG_SEED,
-                       batch_ids[n % len(sched)])
-        ob.extract(ref.n_id)
-        pend.append(ref.n_id)
-        if len(pend) == Q:
-            ob.release(pend.pop(0))
-        n += 1
-        el = time.perf_counter() - t0
-        if el >= budget_s or n >= 10_000:
-            break
-    return {"value": round(n / el, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
-            "sample": f"{n} consecutive full mini-batches of {cfg.name} (sample+extract+release, Q={Q}), "
-                      f"{el:.1f} s on 1 host thread"}
+    stop = t0 + budget_s
+
+    def work(t):
+        out = np.empty((CH, R), dtype=np.uint8)
+        done, j, rows = 0, t, 0
+        while True:
+            if n_target is not None and j >= n_target:
+                break
+            if n_target is None and time.perf_counter() >= stop:
+                break
+            ref = O.sample(indptr, indices, seeds_host[j % nb].numpy(), fan, synth.RNG_SEED, batch_ids[j % nb])
+            for s0 in range(0, len(ref.n_id), CH):
+                ids = ref.n_id[s0:s0 + CH]
+                O.gather_rows(table, ids, out[:len(ids)])
+            rows += len(ref.n_id)
+            done += 1
+            j += threads
+        return done, rows, time.perf_counter()
+
+    with ThreadPoolExecutor(threads) as ex:
+        res = list(ex.map(work, range(threads)))
+    n = sum(r[0] for r in res)
+    el = max(r[2] for r in res) - t0
+    return {"value": round(n / el, 3), "unit": "batches/s", "cores": threads, "kind": "oracle",
+            "sample": f"{n} mini-batches of {cfg.name} (oracle sample + relabel, rows gathered from the host table: "
+                      f"{sum(r[1] for r in res) * R / 2**30:.1f} GiB), one batch stream per thread on {threads} "
+                      f"threads (every core of the affinity mask), {el:.1f} s",
+            "seconds": round(el, 2)}
+
+
+def host_cpu_info():
+    import subprocess
+    info = {"affinity_cores": len(os.sched_getaffinity(0))}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            if k.strip() in ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core", "NUMA node(s)", "CPU(s)"):
+                info[k.strip()] = v.strip()
+    except Exception:  # noqa: BLE001
+        pass
+    return info
+
+
+def config_dict(cfg, S, world, prewarm):
+    """The `config` object of the JSON line; identical for both arms."""
+    R = cfg.row_bytes
+    return {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
+            "feat_dim": cfg.feat_dim, "feat_bytes": R, "batch_size": cfg.batch_size, "fanouts": list(cfg.fanouts),
+            "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
+            "buffer_prewarm_batches": prewarm,
+            "parallelism": f"dp{world} (batch segments, no collective)",
+            "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
+                (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.host_rows * R * 1e-9),
+            "host_table_rows": cfg.host_rows}
 
 
 # ----------------------------------------------------------------------- reference arm
 
 def run_reference(args, rank, world, local_rank):
-    """The oracle (oracle/) as the reference arm: W + K full steps on the host CPU."""
+    """The oracle (oracle/) as the reference arm, on the host cores; rank 0 only (the other
+    ranks exit without work).  Never loads the product package (libgd.so).
+      value: W warm-up then K timed mini-batches of the CPU variant (sample + relabel + rows
+             from the host table) spread over every core of the affinity mask (cpu_variant_baseline);
+      single_thread_full_oracle: the full oracle (Alg. 1 buffer with rows) on one thread, after
+             the GPU arm's pre-warm rule (cumulative misses >= S, checked every 8 batches)."""
     if rank != 0:
         return
     from oracle import oracle as O
@@ -870,30 +1165,59 @@ def run_reference(args, rank, world, local_rank):
     fan = list(cfg.fanouts)
     nm = O.sample_bounds(cfg.batch_size, fan, cfg.num_nodes, cfg.num_edges)[0]
     S = capacity_for(cfg, nm[-1])
-    from paper_conf_icpp_jiangj024_b200.multigpu import batch_schedule
-    sched = batch_schedule(wl.num_batches, 0, 1, args.warmup + args.steps)
+    W, K = args.warmup, args.steps
+    PRE = 0 if cfg.preload else args.prewarm_max
+    threads = len(os.sched_getaffinity(0))
+    n_all = max(W + K, threads) + PRE + 64
+    sched = batch_schedule(wl.num_batches, 0, 1, n_all)
     bids = [ep * wl.num_batches + b for b, ep in sched]
-    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes)
-    pend = []
-    t0 = None
-    for j, (b, ep) in enumerate(sched):
-        if j == args.warmup:
-            t0 = time.perf_counter()
-        ref = O.sample(wl.host_indptr, wl.host_indices, wl.seeds(b, ep).cpu().numpy(), fan, synth.RNG_SEED, bids[j])
-        ob.extract(ref.n_id)
+    seeds_host = torch.stack([wl.seeds(b, ep) for b, ep in sched]).cpu()
+    # (1) multi-core CPU variant: W warm-up batches, then K timed batches over `threads` threads
+    cpu_variant_baseline(cfg, wl.table.array, wl.host_indptr, wl.host_indices, seeds_host, bids, fan, 0, threads,
+                         n_target=W)
+    cv = cpu_variant_baseline(cfg, wl.table.array, wl.host_indptr, wl.host_indices, seeds_host[W:], bids[W:], fan, 0,
+                              threads, n_target=K)
+    v = cv["value"]
+    # (2) the full single-thread oracle from a pre-warmed buffer (the GPU arm's rule)
+    keep = S * cfg.row_bytes <= 48e9
+    ob = O.Buffer(wl.table.array, S, preload=cfg.preload, num_nodes=cfg.num_nodes, keep_rows=keep)
+    pend, jp, cum_miss = [], 0, 0
+
+    def full_step(j, want_out):
+        nonlocal cum_miss
+        ref = O.sample(wl.host_indptr, wl.host_indices, seeds_host[j].numpy(), fan, synth.RNG_SEED, bids[j])
+        _, _, st = ob.extract(ref.n_id, want_out=want_out)
+        cum_miss += st[1]
         pend.append(ref.n_id)
         if len(pend) == Q:
             ob.release(pend.pop(0))
-    el = time.perf_counter() - t0
-    v = args.steps / el
-    line = {"impl": "reference", "metric": "sampled+extracted mini-batches/s", "value": round(v, 3),
-            "unit": "batches/s", "n_gpus": world, "steps": args.steps, "warmup": args.warmup,
-            "ms_per_step": round(el * 1e3 / args.steps, 2), "higher_is_better": True, "scaling": "weak",
+
+    while jp < PRE:
+        for _ in range(8):
+            if jp < PRE:
+                full_step(jp, False)
+                jp += 1
+        if cum_miss >= S:
+            break
+    t1 = time.perf_counter()
+    n1 = 0
+    while n1 < 8 or time.perf_counter() - t1 < 6.0:
+        full_step(jp + n1, keep)
+        n1 += 1
+        if jp + n1 >= len(bids) - 1:
+            break
+    el1 = time.perf_counter() - t1
+    single = {"value": round(n1 / el1, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
+              "sample": f"{n1} full mini-batches (sample + Alg. 1 extract{' with rows' if keep else ''} + release, "
+                        f"Q={Q}) after a {jp}-batch pre-warm, {el1:.1f} s on 1 host thread"}
+    line = {"impl": "reference", "metric": "sampled+extracted mini-batches/s", "value": v,
+            "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
+            "ms_per_step": round(1e3 / v, 3) if v else None, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-            "config": {"workload": cfg.name, "batch_size": cfg.batch_size, "fanouts": fan, "buffer_slots": S},
-            "cpu_baseline": {"value": round(v, 3), "unit": "batches/s", "cores": 1, "kind": "oracle",
-                             "sample": f"{args.steps} timed full mini-batches after {args.warmup} warm-up, 1 thread"},
-            "e2e": {"value": round(v, 3), "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "config": config_dict(cfg, S, world, jp),
+            "cpu_baseline": cv, "single_thread_full_oracle": single, "host_cpu": host_cpu_info(),
+            "e2e": {"value": v, "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+            "native_libs_loaded": loaded_native_libs()}
     print(json.dumps(line), flush=True)
     wl.close()
 

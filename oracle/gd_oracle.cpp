@@ -205,6 +205,7 @@ struct OracleBuffer {
     std::vector<std::list<int32_t>::iterator> where;   /* slot -> list node (the "hash table") */
     std::vector<uint8_t> in_standby;
     std::vector<uint8_t> slots;            /* the feature buffer, S x R bytes */
+    int keep_rows;                         /* 0: bookkeeping only, no slot contents (see below) */
     int64_t hits, misses;                  /* cumulative */
 };
 
@@ -226,8 +227,13 @@ static void standby_remove(OracleBuffer* B, int32_t s) {   /* Alg. 1 line 11 */
  * (P = N is the paper's layout; P < N is the bounded table of the mag240m config). */
 static const uint8_t* feat_row(const OracleBuffer* B, int64_t v) { return B->feat + (size_t)(v % B->P) * B->R; }
 
-void* oracle_buffer_create(const uint8_t* host_feat, int64_t num_nodes, int64_t row_bytes,
-                           int64_t capacity_slots, int preload, int64_t table_rows) {
+/* keep_rows = 0 builds the same buffer without the S x R slot contents: Alg. 1's
+ * bookkeeping (map, reverse, standby list, alias, hits / misses) is unchanged, lines 30-36's
+ * row copy is skipped and extract refuses `out` (-2).  Storage only, no arithmetic: it lets
+ * full-size replays (37.5 GB of slots at mag240m, one replay per GPU) fit in host memory; the
+ * rows themselves are checked by the closed form out[i] = feat[ids[i] mod P] (P5). */
+void* oracle_buffer_create2(const uint8_t* host_feat, int64_t num_nodes, int64_t row_bytes,
+                            int64_t capacity_slots, int preload, int64_t table_rows, int keep_rows) {
     if (preload && capacity_slots < num_nodes) return nullptr;
     if (table_rows < 1 || table_rows > num_nodes) return nullptr;
     OracleBuffer* B = new OracleBuffer();
@@ -236,17 +242,23 @@ void* oracle_buffer_create(const uint8_t* host_feat, int64_t num_nodes, int64_t 
     B->reverse.assign(capacity_slots, -1);
     B->where.resize(capacity_slots);
     B->in_standby.assign(capacity_slots, 0);
-    B->slots.assign((size_t)capacity_slots * (size_t)row_bytes, 0);
+    B->keep_rows = keep_rows != 0;
+    if (B->keep_rows) B->slots.assign((size_t)capacity_slots * (size_t)row_bytes, 0);
     B->hits = B->misses = 0;
     for (int64_t s = 0; s < capacity_slots; ++s) standby_push_back(B, (int32_t)s);
     if (preload) {
         for (int64_t v = 0; v < num_nodes; ++v) {
             B->map[v] = MapEntry{(int32_t)v, 0, 1};
             B->reverse[v] = (int32_t)v;
-            std::memcpy(&B->slots[(size_t)v * row_bytes], feat_row(B, v), row_bytes);
+            if (B->keep_rows) std::memcpy(&B->slots[(size_t)v * row_bytes], feat_row(B, v), row_bytes);
         }
     }
     return B;
+}
+
+void* oracle_buffer_create(const uint8_t* host_feat, int64_t num_nodes, int64_t row_bytes,
+                           int64_t capacity_slots, int preload, int64_t table_rows) {
+    return oracle_buffer_create2(host_feat, num_nodes, row_bytes, capacity_slots, preload, table_rows, 1);
 }
 
 void oracle_buffer_destroy(void* h) { delete (OracleBuffer*)h; }
@@ -259,6 +271,7 @@ void oracle_buffer_destroy(void* h) { delete (OracleBuffer*)h; }
 int oracle_extract(void* h, const int32_t* ids, int64_t n, uint8_t* out, int32_t* alias,
                    int64_t* stats) {
     OracleBuffer* B = (OracleBuffer*)h;
+    if (out && !B->keep_rows) return -2;
     std::vector<int32_t> ids_r(n, -1);                       /* lines 3-4 */
     int64_t hits = 0, misses = 0;
     for (int64_t i = 0; i < n; ++i) {                         /* lines 6-20 */
@@ -289,7 +302,7 @@ int oracle_extract(void* h, const int32_t* ids, int64_t n, uint8_t* out, int32_t
         B->reverse[index] = id;                               /* line 28 */
         ids_r[i] = index;                                     /* line 29 */
         /* lines 30-36: load from the table (the SSD stand-in) into the slot */
-        std::memcpy(&B->slots[(size_t)index * B->R], feat_row(B, id), B->R);
+        if (B->keep_rows) std::memcpy(&B->slots[(size_t)index * B->R], feat_row(B, id), B->R);
         B->map[id].valid = 1;                                 /* line 37 */
         ++misses;
     }
@@ -315,6 +328,13 @@ int oracle_release(void* h, const int32_t* ids, int64_t n) {
         if (m.rc == 0) standby_push_back(B, m.slot);
     }
     return 0;
+}
+
+/* The CPU variant's data path (every feature row host-resident, no device buffer):
+ * out[i] = feat[ids[i] mod P], row by row in list order (the closed form of C6's out). */
+void oracle_gather_rows(const uint8_t* feat, int64_t P, int64_t R, const int32_t* ids, int64_t n, uint8_t* out) {
+    for (int64_t i = 0; i < n; ++i)
+        std::memcpy(out + (size_t)i * R, feat + (size_t)((int64_t)ids[i] % P) * R, R);
 }
 
 /* Debug snapshot of the whole state (C8).  Any pointer may be null. */
@@ -343,7 +363,7 @@ int oracle_buffer_set_state(void* h, const int32_t* map_slot, const int32_t* map
     B->standby.clear();
     std::fill(B->in_standby.begin(), B->in_standby.end(), 0);
     for (int64_t k = 0; k < standby_len; ++k) standby_push_back(B, standby[k]);
-    for (int64_t v = 0; v < B->N; ++v)
+    for (int64_t v = 0; B->keep_rows && v < B->N; ++v)
         if (B->map[v].valid && B->map[v].slot >= 0)
             std::memcpy(&B->slots[(size_t)B->map[v].slot * B->R], feat_row(B, v), B->R);
     return 0;

@@ -59,6 +59,11 @@ def lib():
         L.oracle_buffer_create.argtypes = [_u8p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
                                            ctypes.c_int64]
         L.oracle_buffer_create.restype = ctypes.c_void_p
+        L.oracle_buffer_create2.argtypes = [_u8p, ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.c_int,
+                                            ctypes.c_int64, ctypes.c_int]
+        L.oracle_buffer_create2.restype = ctypes.c_void_p
+        L.oracle_gather_rows.argtypes = [_u8p, ctypes.c_int64, ctypes.c_int64, _i32p, ctypes.c_int64, _u8p]
+        L.oracle_gather_rows.restype = None
         L.oracle_buffer_destroy.argtypes = [ctypes.c_void_p]
         L.oracle_buffer_destroy.restype = None
         L.oracle_extract.argtypes = [ctypes.c_void_p, _i32p, ctypes.c_int64, _u8p, _i32p, _i64p]
@@ -124,6 +129,17 @@ def sample_bounds(num_seeds: int, fanouts, num_nodes: int, num_edges: int):
     return n, e
 
 
+def gather_rows(feat_u8: np.ndarray, ids: np.ndarray, out: np.ndarray | None = None) -> np.ndarray:
+    """CPU-variant data path: out[i] = feat_u8[ids[i] mod P] (releases the GIL)."""
+    ids = np.ascontiguousarray(ids, dtype=np.int32)
+    P, R = feat_u8.shape
+    if out is None:
+        out = np.empty((len(ids), R), dtype=np.uint8)
+    assert out.flags.c_contiguous and out.shape[0] >= len(ids) and out.shape[1] == R
+    lib().oracle_gather_rows(_p(feat_u8, _u8p), P, R, _p(ids, _i32p), len(ids), _p(out, _u8p))
+    return out
+
+
 class SampleResult:
     def __init__(self, n_id, rowptr, col, eid, sizes):
         self.n_id, self.rowptr, self.col, self.eid, self.sizes = n_id, rowptr, col, eid, sizes
@@ -162,14 +178,18 @@ def sample(indptr: np.ndarray, indices: np.ndarray, seeds: np.ndarray, fanouts, 
 class Buffer:
     """Algorithm 1 feature buffer over a host table feat[N, R] (uint8 view)."""
 
-    def __init__(self, feat_u8: np.ndarray, capacity_slots: int, preload: bool = False, num_nodes: int | None = None):
-        """feat_u8 [P, R]: node v's row is feat_u8[v mod P]; num_nodes defaults to P."""
+    def __init__(self, feat_u8: np.ndarray, capacity_slots: int, preload: bool = False, num_nodes: int | None = None,
+                 keep_rows: bool = True):
+        """feat_u8 [P, R]: node v's row is feat_u8[v mod P]; num_nodes defaults to P.
+        keep_rows=False: bookkeeping only (no S x R slot contents; extract(want_out=True) fails)."""
         assert feat_u8.dtype == np.uint8 and feat_u8.ndim == 2 and feat_u8.flags.c_contiguous
         self.feat = feat_u8
         self.P, self.R = feat_u8.shape
         self.N = int(num_nodes) if num_nodes is not None else self.P
         self.S = int(capacity_slots)
-        self.h = lib().oracle_buffer_create(_p(feat_u8, _u8p), self.N, self.R, self.S, int(preload), self.P)
+        self.keep_rows = bool(keep_rows)
+        self.h = lib().oracle_buffer_create2(_p(feat_u8, _u8p), self.N, self.R, self.S, int(preload), self.P,
+                                             int(self.keep_rows))
         if not self.h:
             raise ValueError("oracle_buffer_create: preload requires capacity >= N, and 1 <= P <= N")
 
@@ -178,13 +198,17 @@ class Buffer:
             lib().oracle_buffer_destroy(self.h)
             self.h = None
 
-    def extract(self, ids: np.ndarray, want_out: bool = True):
+    def extract(self, ids: np.ndarray, want_out: bool | None = None):
+        if want_out is None:
+            want_out = self.keep_rows
         ids = np.ascontiguousarray(ids, dtype=np.int32)
         n = len(ids)
         out = np.zeros((n, self.R), dtype=np.uint8) if want_out else None
         alias = np.zeros(max(n, 1), dtype=np.int32)
         stats = np.zeros(2, dtype=np.int64)
         rc = lib().oracle_extract(self.h, _p(ids, _i32p), n, _p(out, _u8p), _p(alias, _i32p), _p(stats, _i64p))
+        if rc == -2:
+            raise RuntimeError("oracle_extract: a bookkeeping-only buffer (keep_rows=False) has no rows for `out`")
         if rc != 0:
             raise RuntimeError("oracle_extract: standby list ran dry (capacity rule violated)")
         return out, alias[:n], (int(stats[0]), int(stats[1]))

@@ -134,16 +134,38 @@ def test_single_process_fallbacks():
 
 
 def test_numa_helpers():
-    """NUMA interleave of the shared host table (bench.py, world > 1): node-list parsing and a
-    policy call that never raises (False on single-node hosts)."""
-    from paper_conf_icpp_jiangj024_b200 import multigpu as mg
-    assert mg._parse_list("0-1,3\n") == [0, 1, 3]
-    assert mg._parse_list("0") == [0]
-    nodes = mg.numa_nodes()
+    """NUMA placement (bench.py, world > 1): node-list parsing, an interleave policy call that
+    never raises (False on single-node hosts), and the per-rank socket binding, which is a
+    no-op (reported, not raised) where the GPU's PCIe locality is unknown or the host has one
+    node."""
+    from synth import host as H
+    assert H.parse_cpulist("0-1,3\n") == [0, 1, 3]
+    assert H.parse_cpulist("0") == [0]
+    nodes = H.numa_nodes()
     assert all(isinstance(n, int) for n in nodes)
-    ok = mg.set_interleave(True)
+    ok = H.set_interleave(True)
     assert ok == (len(nodes) >= 2) or not ok
-    mg.set_interleave(False)
+    H.set_interleave(False)
+    before = os.sched_getaffinity(0)
+    rep = H.bind_to_gpu_socket(0)
+    assert rep["cpus"] >= 1 and (rep["bound"] or os.sched_getaffinity(0) == before)
+    os.sched_setaffinity(0, before)
+
+
+def test_shared_array_refuses_a_short_shm(monkeypatch, tmp_path):
+    """Rank 0 checks the shared-memory filesystem's free space before creating the table and
+    fails with a clear message (instead of a SIGBUS mid-fill)."""
+    from synth import host as H
+    monkeypatch.setattr(H, "shm_free_bytes", lambda path: 1000)
+    with pytest.raises(RuntimeError, match="GiB free"):
+        H.HostTable(100, 64, "short", rank=0, world=2, shm_dir=str(tmp_path))
+    assert not os.listdir(tmp_path)
+    monkeypatch.setattr(H, "shm_free_bytes", lambda path: 1 << 40)
+    t = H.HostTable(100, 64, "ok", rank=0, world=2, shm_dir=str(tmp_path))
+    t.array[:] = 7
+    assert int(t.array.sum()) == 7 * 6400
+    t.close()
+    assert not os.listdir(tmp_path)
 
 
 def test_reference_arm_under_torchrun_world2():
@@ -165,3 +187,7 @@ def test_reference_arm_under_torchrun_world2():
     rec = lines[0]
     assert rec["impl"] == "reference" and rec["n_gpus"] == 2 and rec["value"] > 0
     assert rec["e2e"]["h2d_bytes_per_step"] == 0 and rec["cpu_baseline"]["kind"] == "oracle"
+    # reference-arm hygiene: the oracle only, never the product library
+    assert rec["native_libs_loaded"] == ["oracle/libgd_oracle.so"], rec["native_libs_loaded"]
+    assert rec["cpu_baseline"]["cores"] == len(os.sched_getaffinity(0))
+    assert rec["config"]["workload"] == "tiny" and rec["config"]["release_lag"] == 4

@@ -186,3 +186,33 @@ def test_bounded_table_rows_mod_p():
             B.release(pend.pop(0))
     with pytest.raises(ValueError):
         O.Buffer(feat, 600, preload=True, num_nodes=N + 1000)   # preload needs capacity >= N
+
+
+@pytest.mark.parametrize("Q,P", [(1, 200), (3, 200), (4, 61)])
+def test_bookkeeping_only_buffer_equals_full_buffer(Q, P):
+    """keep_rows=False (the full-size replays' oracle: no S x R slot contents) takes exactly the
+    same Alg. 1 decisions: alias, hits/misses and the whole state match the full buffer every
+    step; its extract refuses `out`.  gather_rows is the closed form feat[ids mod P]."""
+    rng = np.random.default_rng(Q * 7 + P)
+    N, M = 200, 25
+    feat = table(P, R=20, seed=Q)
+    A = O.Buffer(feat, Q * M, num_nodes=N)
+    B = O.Buffer(feat, Q * M, num_nodes=N, keep_rows=False)
+    pending = []
+    for step in range(80):
+        w = rng.zipf(1.5, size=300) % N
+        ids = np.array(list(dict.fromkeys(w.tolist()))[: rng.integers(1, M + 1)], dtype=np.int32)
+        out, a1, s1 = A.extract(ids)
+        none, a2, s2 = B.extract(ids)
+        assert none is None and s1 == s2 and np.array_equal(a1, a2)
+        assert np.array_equal(O.gather_rows(feat, ids), out)
+        pending.append(ids)
+        if len(pending) == Q:
+            r = pending.pop(0)
+            A.release(r)
+            B.release(r)
+        sa, sb = A.state(), B.state()
+        for k in sa:
+            assert np.array_equal(sa[k], sb[k]), k
+    with pytest.raises(RuntimeError):
+        B.extract(np.array([0], dtype=np.int32), want_out=True)
