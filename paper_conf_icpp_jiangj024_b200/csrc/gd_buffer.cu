@@ -22,6 +22,9 @@
 #include <cstdlib>
 #include <thread>
 
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
 #include "gd_common.cuh"
 #include "gd_handles.cuh"
 
@@ -554,33 +557,171 @@ __global__ void __launch_bounds__(256) k_gather_hits(const int2* __restrict__ hi
 // Warp per row, U rows in flight per warp, CPL 16-byte chunks per lane (R <= 512 * CPL):
 // all loads of U rows are issued before any store (measured 5.0 TB/s = 78% of the HBM
 // copy peak on 512-byte rows vs 4.1 TB/s for the flat chunk loop, tools/gather_bench.cu).
+// ctr != nullptr: dynamic assignment, each warp takes the next G = 8U rows from a per-launch
+// counter (the last block out re-zeroes it).  Live, the gather shares the GPU with the next
+// batch's sampling and with the miss copies, whose microsecond host loads clog the memory
+// pipeline of the SMs they run on; with a static row partition the blocks landing on those
+// SMs (or scheduled late, behind other kernels) set the kernel's duration, with dynamic
+// assignment they just take fewer rows.  ctr == nullptr: static grid-stride partition.
+template <int U, int CPL>
+__device__ __forceinline__ void gather_rows_span(const int2* __restrict__ hitlist, int64_t r0, int64_t rend,
+                                                 const uint8_t* __restrict__ slots, uint8_t* __restrict__ out,
+                                                 int64_t R, int cpr, int lane) {
+    int2 h[U];
+    uint4 v[U][CPL];
+#pragma unroll
+    for (int u = 0; u < U; ++u) h[u] = (r0 + u < rend) ? __ldg(hitlist + r0 + u) : make_int2(-1, -1);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int q = 0; q < CPL; ++q)
+            if (h[u].y >= 0 && lane + 32 * q < cpr)
+                asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+                             : "=r"(v[u][q].x), "=r"(v[u][q].y), "=r"(v[u][q].z), "=r"(v[u][q].w)
+                             : "l"((const uint4*)(slots + (int64_t)h[u].y * R) + lane + 32 * q));
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int q = 0; q < CPL; ++q)
+            if (h[u].y >= 0 && lane + 32 * q < cpr) ((uint4*)(out + (int64_t)h[u].x * R))[lane + 32 * q] = v[u][q];
+}
+
 template <int U, int CPL>
 __global__ void __launch_bounds__(256) k_gather_rows(const int2* __restrict__ hitlist, const int64_t* __restrict__ hcount,
-                                                     const uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R) {
+                                                     const uint8_t* __restrict__ slots, uint8_t* __restrict__ out, int64_t R,
+                                                     unsigned long long* __restrict__ ctr) {
     const int64_t H = *hcount;
     const int lane = threadIdx.x & 31;
-    const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
     const int cpr = (int)(R >> 4);
-    for (int64_t r0 = w * U; r0 < H; r0 += nw * U) {
-        int2 h[U];
-        uint4 v[U][CPL];
-#pragma unroll
-        for (int u = 0; u < U; ++u) h[u] = (r0 + u < H) ? __ldg(hitlist + r0 + u) : make_int2(-1, -1);
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-#pragma unroll
-            for (int q = 0; q < CPL; ++q)
-                if (h[u].y >= 0 && lane + 32 * q < cpr)
-                    asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
-                                 : "=r"(v[u][q].x), "=r"(v[u][q].y), "=r"(v[u][q].z), "=r"(v[u][q].w)
-                                 : "l"((const uint4*)(slots + (int64_t)h[u].y * R) + lane + 32 * q));
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-#pragma unroll
-            for (int q = 0; q < CPL; ++q)
-                if (h[u].y >= 0 && lane + 32 * q < cpr) ((uint4*)(out + (int64_t)h[u].x * R))[lane + 32 * q] = v[u][q];
+    if (ctr == nullptr) {
+        const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+        const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+        for (int64_t r0 = w * U; r0 < H; r0 += nw * U) gather_rows_span<U, CPL>(hitlist, r0, H, slots, out, R, cpr, lane);
+        return;
     }
+    constexpr int G = 8 * U;
+    while (true) {
+        unsigned long long g0 = 0;
+        if (lane == 0) g0 = atomicAdd(ctr, (unsigned long long)G);
+        g0 = __shfl_sync(0xffffffffu, g0, 0);
+        if ((int64_t)g0 >= H) break;
+        const int64_t gend = (int64_t)g0 + G < H ? (int64_t)g0 + G : H;
+        for (int64_t r0 = (int64_t)g0; r0 < gend; r0 += U) gather_rows_span<U, CPL>(hitlist, r0, gend, slots, out, R, cpr, lane);
+    }
+    ticket_finish(ctr);
+}
+
+// a8 variant: TMA gather.  One warp per CTA, one elected thread: a 2-D tensor map
+// over the slots ([S rows x R bytes], box = one row), `cp.async.bulk.tensor.2d.tile::gather4`
+// brings 4 hit rows (4 slot indices) into a shared-memory stage, and 4 bulk stores
+// (`cp.async.bulk.global.shared::cta`) write them to their `out` rows.  L gathers in flight per
+// CTA over P = 2L stages; a stage is reloaded once the store group that last read it is done
+// (`cp.async.bulk.wait_group.read P - L`).  Rows are taken dynamically from a per-launch counter
+// (G = 32 per grab; the last CTA out re-zeroes it).  Address generation and the data movement
+// are the TMA unit's, so the SM issues ~2 instructions per row instead of one load + one store
+// per 16 bytes per lane.  R % 16 == 0, R <= 2048 (box of R / 4 uint32 or R / 8 uint64 <= 256).
+__device__ __forceinline__ uint32_t gsm_u32(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void gsm_mbar_wait(uint32_t addr, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "GWAIT_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n\t"
+        "@!p bra GWAIT_%=;\n}\n" ::"r"(addr),
+        "r"(parity)
+        : "memory");
+}
+
+template <int L>
+__global__ void __launch_bounds__(32) k_gather_tma(const __grid_constant__ CUtensorMap tm, const int2* __restrict__ hitlist,
+                                                   const int64_t* __restrict__ hcount, uint8_t* __restrict__ out, int64_t R,
+                                                   int64_t stage_stride, unsigned long long* __restrict__ ctr) {
+    constexpr int P = 2 * L;
+    constexpr int G = 32;
+    extern __shared__ __align__(128) uint8_t gsm[];
+    __shared__ __align__(8) unsigned long long full[P];
+    __shared__ int32_t spos[P][4];
+    __shared__ int32_t s_n[P];
+    if (threadIdx.x == 0) {
+        const int64_t H = *hcount;
+        for (int st = 0; st < P; ++st) asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;\n" ::"r"(gsm_u32(&full[st])));
+        asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+        const uint32_t stage_bytes = (uint32_t)(4 * R);
+        int64_t g0 = 0, gend = 0, issued = 0, done = 0;
+        bool exhausted = false;
+        while (true) {
+            while (!exhausted && issued - done < L) {
+                if (g0 >= gend) {
+                    const unsigned long long t = atomicAdd(ctr, (unsigned long long)G);
+                    if ((int64_t)t >= H) {
+                        exhausted = true;
+                        break;
+                    }
+                    g0 = (int64_t)t;
+                    gend = g0 + G < H ? g0 + G : H;
+                }
+                const int nq = gend - g0 < 4 ? (int)(gend - g0) : 4;
+                const int st = (int)(issued % P);
+                int32_t rows[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const int2 h = __ldg(hitlist + g0 + (q < nq ? q : nq - 1));
+                    rows[q] = h.y;
+                    if (q < nq) spos[st][q] = h.x;
+                }
+                s_n[st] = nq;
+                g0 += nq;
+                // the store group that last read stage st (iteration issued - P) has finished reading
+                asm volatile("cp.async.bulk.wait_group.read %0;\n" ::"n"(P - L) : "memory");
+                const uint32_t bar = gsm_u32(&full[st]);
+                asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n" ::"r"(bar), "r"(stage_bytes) : "memory");
+                asm volatile(
+                    "cp.async.bulk.tensor.2d.shared::cta.global.tile::gather4.mbarrier::complete_tx::bytes"
+                    " [%0], [%1, {%2, %3, %4, %5, %6}], [%7];\n" ::"r"(gsm_u32(gsm + st * stage_stride)),
+                    "l"((uint64_t)&tm), "r"(0), "r"(rows[0]), "r"(rows[1]), "r"(rows[2]), "r"(rows[3]), "r"(bar)
+                    : "memory");
+                ++issued;
+            }
+            if (done == issued) break;
+            const int st = (int)(done % P);
+            gsm_mbar_wait(gsm_u32(&full[st]), (uint32_t)((done / P) & 1));
+            asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory");
+            for (int q = 0; q < s_n[st]; ++q)
+                asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;\n" ::"l"(out + (int64_t)spos[st][q] * R),
+                             "r"(gsm_u32(gsm + st * stage_stride + q * R)), "r"((uint32_t)R)
+                             : "memory");
+            asm volatile("cp.async.bulk.commit_group;\n" ::: "memory");
+            ++done;
+        }
+        asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory");
+    }
+    ticket_finish(ctr);
+}
+
+// Tensor map over the slots for k_gather_tma: dims {R / e, S}, row stride R, box {R / e, 1}
+// (e = 4 or 8 bytes), no swizzle.  Returns false when R does not fit one box.
+static bool make_slot_map(CUtensorMap* m, const void* slots, int64_t S, int64_t R) {
+    static PFN_cuTensorMapEncodeTiled_v12000 encode = nullptr;
+    if (!encode) {
+        cudaDriverEntryPointQueryResult q;
+        cudaError_t e = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", (void**)&encode, cudaEnableDefault, &q);
+        if (e != cudaSuccess || q != cudaDriverEntryPointSuccess || !encode) {
+            cudaGetLastError();
+            encode = nullptr;
+            return false;
+        }
+    }
+    if (R % 16 != 0 || S < 1 || S > (1ll << 31) - 1) return false;
+    const int64_t e = R / 4 <= 256 ? 4 : (R / 8 <= 256 ? 8 : 0);
+    if (!e) return false;
+    const cuuint64_t dims[2] = {(cuuint64_t)(R / e), (cuuint64_t)S};
+    const cuuint64_t strides[1] = {(cuuint64_t)R};
+    const cuuint32_t box[2] = {(cuuint32_t)(R / e), 1};
+    const cuuint32_t es[2] = {1, 1};
+    const CUresult r = encode(m, e == 4 ? CU_TENSOR_MAP_DATA_TYPE_UINT32 : CU_TENSOR_MAP_DATA_TYPE_INT64, 2,
+                              const_cast<void*>(slots), dims, strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                              CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    return r == CUDA_SUCCESS;
 }
 
 __global__ void k_gather_hits_w4(const int2* __restrict__ hitlist, const int64_t* __restrict__ hcount,
@@ -887,7 +1028,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     GD_ALLOC(b->trip, (int64_t)b->D * nm * sizeof(int4));
     GD_ALLOC(b->trip_count, b->D * sizeof(int64_t));
     GD_ALLOC(b->trip_split, b->D * sizeof(int64_t));
-    GD_ALLOC(b->tickets, 4 * sizeof(unsigned long long));
+    GD_ALLOC(b->tickets, 6 * sizeof(unsigned long long));
     GD_ALLOC(b->done_word, sizeof(unsigned long long));
     GD_ALLOC(b->ready, capacity_slots * sizeof(unsigned long long));
     GD_ALLOC(b->trip2, (int64_t)b->D * nm * sizeof(int4));
@@ -904,7 +1045,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     c0[1] = c0[0];
     if (cudaMemcpy(b->ctl, c0, sizeof(c0), cudaMemcpyHostToDevice) != cudaSuccess ||
         cudaMemset(b->hdr.dev_status, 0, sizeof(unsigned int)) != cudaSuccess ||
-        cudaMemset(b->tickets, 0, 4 * sizeof(unsigned long long)) != cudaSuccess ||
+        cudaMemset(b->tickets, 0, 6 * sizeof(unsigned long long)) != cudaSuccess ||
         cudaMemset(b->done_word, 0, sizeof(unsigned long long)) != cudaSuccess ||
         cudaMemset(b->trip_count, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
         cudaMemset(b->trip_split, 0, b->D * sizeof(int64_t)) != cudaSuccess ||
@@ -927,9 +1068,28 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
         cudaError_t e = cudaDeviceSynchronize();
         if (e != cudaSuccess) return fail(cuda_error(e, "gd_buffer_init: init kernels"));
     }
-    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_g, &b->side_c})
+    for (cudaStream_t* sp : {&b->side, &b->side_h, &b->side_p, &b->side_j, &b->side_c})
         if (cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
+    {   // the hit gather (stream G) at the highest stream priority: when SMs free up, the block
+        // scheduler starts its blocks before those of the sampling / miss-copy kernels beside it
+        // (env GD_GATHER_PRIORITY=0: default priority); GD_GATHER_DYNAMIC=0: static row partition
+        int lo = 0, hi = 0;
+        cudaDeviceGetStreamPriorityRange(&lo, &hi);
+        const char* e = std::getenv("GD_GATHER_PRIORITY");
+        if (cudaStreamCreateWithPriority(&b->side_g, cudaStreamNonBlocking, (e && e[0] == '0') ? lo : hi) != cudaSuccess)
+            return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
+        const char* d = std::getenv("GD_GATHER_DYNAMIC");
+        b->gather_dynamic = !(d && d[0] == '0');
+        // GD_GATHER_TMA=1: the TMA gather4 variant of a8 (rows <= 2048 B, multiples of 16)
+        const char* t = std::getenv("GD_GATHER_TMA");
+        if (t && t[0] == '1' && make_slot_map(&b->slot_map, b->slots, capacity_slots, row_bytes)) {
+            const int64_t stride = (4 * row_bytes + 127) / 128 * 128;
+            if (cudaFuncSetAttribute(k_gather_tma<4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(8 * stride)) == cudaSuccess)
+                b->gather_tma = true;
+            cudaGetLastError();
+        }
+    }
     for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G, &b->ev_S})
         if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
@@ -1484,12 +1644,18 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
 
     // a8: hits, slots -> out (stream G)
     const int t_gat = timed ? b->timer.begin(b->side_g) : -1;
-    if (b->R % 16 == 0 && b->R <= 512)
-        k_gather_rows<4, 1><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
+    unsigned long long* gctr = b->gather_dynamic ? b->tickets + 4 : nullptr;
+    if (b->gather_tma) {
+        const int64_t stride = (4 * b->R + 127) / 128 * 128, smem = 8 * stride;   // P = 8 stages
+        const int per_sm = (int)std::max<int64_t>(1, std::min<int64_t>(16, (200 << 10) / (smem + 256)));
+        k_gather_tma<4><<<148 * per_sm, 32, smem, b->side_g>>>(b->slot_map, hlist, hcnt, (uint8_t*)out, b->R, stride,
+                                                                 b->tickets + 4);
+    } else if (b->R % 16 == 0 && b->R <= 512)
+        k_gather_rows<4, 1><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0 && b->R <= 1024)
-        k_gather_rows<4, 2><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
+        k_gather_rows<4, 2><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0 && b->R <= 2048)
-        k_gather_rows<2, 4><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
+        k_gather_rows<2, 4><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0)
         k_gather_hits<4><<<148 * 8, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
     else

@@ -1,6 +1,7 @@
 // gd_handles.cuh — layouts of the two opaque handles of libgd.so.
 #pragma once
 
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -104,7 +105,10 @@ struct gd_buffer {
     int D = 0;
     int4* trip = nullptr;                // [D][n_max] {node, slot, batch position, 0}
     int64_t* trip_count = nullptr;       // [D]
-    unsigned long long* tickets = nullptr;   // [4] {ticket, finished} x 2 kernels
+    unsigned long long* tickets = nullptr;   // [6] {ticket, finished} x 3 kernels (pop, compact, gather)
+    bool gather_dynamic = true;          // hit gather: dynamic row assignment (GD_GATHER_DYNAMIC)
+    bool gather_tma = false;             // hit gather by TMA gather4 (GD_GATHER_TMA=1)
+    CUtensorMap slot_map;                // tensor map over the slots for the TMA gather
     unsigned long long* done_word = nullptr; // [1] epoch-tagged early-exit word of the pop scan
     gd::ScanState scan;
     cudaStream_t side = nullptr;         // Z: zero-copy share of the misses

@@ -359,6 +359,27 @@ def test_extract_parity_row_sizes(gd, R, mode, monkeypatch):
                  config=(4, 0.3), stage_mode=copy_engine)
 
 
+@pytest.mark.parametrize("variant", ["tma", "static", "low-priority"])
+@pytest.mark.parametrize("R", [400, 512, 1536, 2048, 12])
+def test_hit_gather_variants(gd, R, variant, monkeypatch):
+    """a8 variants (selected at buffer init): the TMA gather4 kernel (GD_GATHER_TMA=1), the
+    warp-per-row kernel with a static row partition (GD_GATHER_DYNAMIC=0) and the gather
+    stream at default priority: the same bytes, alias and state as the oracle (R = 12: the
+    4-byte kernel, whichever variant is asked for)."""
+    env = {"tma": ("GD_GATHER_TMA", "1"), "static": ("GD_GATHER_DYNAMIC", "0"),
+           "low-priority": ("GD_GATHER_PRIORITY", "0")}[variant]
+    monkeypatch.setenv(*env)
+    N, E = 20_000, 150_000
+    indptr, indices = make_graph(N, E, seed=17)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, R if R % 8 == 0 else 16)[:, :R].copy()
+    order = synth.epoch_order(synth.train_nodes(N, 0.2))
+    seeds = [order[b * 300:(b + 1) * 300].numpy() for b in range(8)]
+    nb, _ = O.sample_bounds(300, [10, 5], N, E)
+    run_schedule(gd, g, indptr.numpy(), indices.numpy(), feat, 2 * nb[-1] + 5, 2, seeds, [10, 5], check_state_every=4,
+                 config=(4, 0.3))
+
+
 def test_extract_ring_compaction(gd):
     """Many batches with a small capacity and lag: the standby ring compacts repeatedly."""
     N, E = 3000, 30000
