@@ -46,6 +46,9 @@ def parse():
     p.add_argument("--batch-size", type=int, default=None, help="f3 sweep override (Fig. 10)")
     p.add_argument("--feat-dim", type=int, default=None, help="f3 sweep override (Fig. 8)")
     p.add_argument("--buffer-frac", type=float, default=None, help="f3 sweep override (Fig. 12)")
+    p.add_argument("--table-rows", type=int, default=None,
+                   help="bounded physical host table (node v -> row v mod P, reading R15), e.g. for the dim-512 sweep point "
+                        "whose full table exceeds host RAM")
     p.add_argument("--cpu-seconds", type=float, default=12.0, help="budget of the oracle cpu_baseline sample")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-e2e", action="store_true")
@@ -370,6 +373,8 @@ def config_from_args(args):
     if args.buffer_frac is not None:
         over["buffer_frac"] = args.buffer_frac
         over["preload"] = False
+    if args.table_rows:
+        over["table_rows"] = min(args.table_rows, cfg.num_nodes)
     return dataclasses.replace(cfg, **over) if over else cfg
 
 

@@ -308,7 +308,7 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
                 a.reverse[s] = v;                               // line 28
                 a.alias[i] = s;                                 // line 29
                 a.pos_of_slot[s] = -1;
-                a.ready[s] = kReadyNone;                        // peers stop reading it (f2)
+                if (a.ready) a.ready[s] = kReadyNone;           // peers stop reading it (f2)
                 a.trip[rank] = make_int4(v, s, i, 0);
                 if (rank >= K0 && a.h_nodes) a.h_nodes[rank - K0] = v;
                 if (rank == M - 1) {
@@ -1228,6 +1228,22 @@ static gd_status set_peers(gd_buffer* b, int n, const int2* const* maps, const u
     return GD_OK;
 }
 
+// A buffer maintains its f2 publication tags (cleared by k_pop_assign on reassignment, set by
+// k_publish) only from the moment another buffer can read them: in-process attach as someone's
+// peer, or an IPC export.  Until then it skips both (a random 8-byte write per miss, twice).
+// Switching on re-initialises every tag (preload: slot s holds node s; otherwise none), so a
+// tag left from before can never vouch for a slot's current row.
+static gd_status ensure_publishing(gd_buffer* q) {
+    if (q->publish) return GD_OK;
+    DeviceGuard guard(q->hdr.device);
+    gd_status s = drain_streams(q);
+    if (s != GD_OK) return s;
+    k_init_ready<<<148 * 8, 256, 0, q->side_j>>>(q->ready, q->S, q->N, q->preload);
+    GD_CUDA(cudaStreamSynchronize(q->side_j));
+    q->publish = true;
+    return GD_OK;
+}
+
 gd_status gd_buffer_peer_attach(gd_buffer* b, int npeers, gd_buffer* const* peers) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_attach: bad handle");
     if (npeers < 0 || npeers > kMaxPeers || (npeers > 0 && !peers))
@@ -1254,6 +1270,10 @@ gd_status gd_buffer_peer_attach(gd_buffer* b, int npeers, gd_buffer* const* peer
         readys[p] = q->ready;
         slots[p] = q->slots;
     }
+    for (int p = 0; p < npeers; ++p) {
+        gd_status st = ensure_publishing(peers[p]);
+        if (st != GD_OK) return st;
+    }
     gd_status s = drain_streams(b);
     if (s != GD_OK) return s;
     return set_peers(b, npeers, maps, readys, slots);
@@ -1266,6 +1286,10 @@ gd_status gd_buffer_peer_export_ipc(gd_buffer* b, void* blob, int64_t blob_bytes
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_peer_export_ipc: bad handle");
     if (!blob || blob_bytes < GD_PEER_BLOB_BYTES) return set_error(GD_ERR_INVALID, "gd_buffer_peer_export_ipc: blob too small");
     DeviceGuard guard(b->hdr.device);
+    {
+        gd_status st = ensure_publishing(b);
+        if (st != GD_OK) return st;
+    }
     std::memset(blob, 0, GD_PEER_BLOB_BYTES);
     int64_t* h = (int64_t*)blob;
     h[0] = kBlobMagic;
@@ -1576,7 +1600,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.trip_split = tsplit;
     pa.alpha_q16 = alpha_q16;
     pa.staged_cap = cap;
-    pa.ready = b->ready;
+    pa.ready = b->publish ? b->ready : nullptr;   // f2 tags only once a peer can read them
     pa.h_nodes = nullptr;
     pa.h_meta = nullptr;
     int32_t* h_nodes_dev = nullptr;
@@ -1759,7 +1783,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaStreamWaitEvent(b->side_j, b->ev_G, 0));
     // f2: the batch's new slots are complete: publish them to peers (before `done`, so a
     // release, and with it any reuse of these slots, is ordered after the publication)
-    if (!b->preload) k_publish<<<148, 256, 0, b->side_j>>>(trip, tcount, b->ready, pa.epoch);
+    if (!b->preload && b->publish) k_publish<<<148, 256, 0, b->side_j>>>(trip, tcount, b->ready, pa.epoch);
     GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side_j));
     if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side_j));
     GD_CUDA(cudaGetLastError());

@@ -161,6 +161,7 @@ struct gd_buffer {
     // the batch's copies joined), kReadyNone from the moment the slot is reassigned.
     unsigned long long* ready = nullptr; // HBM [S]
     int npeers = 0;
+    bool publish = false;                // tags maintained (someone can read them as a peer)
     gd::PeerView peers;                  // device pointers of the peers' map / ready / slots
     std::vector<void*> ipc_opened;       // pointers opened with cudaIpcOpenMemHandle (closed at destroy)
     int4* trip2 = nullptr;               // [D][n_max] misses no peer served (compacted)
