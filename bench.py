@@ -57,6 +57,13 @@ def parse():
     p.add_argument("--lr", type=float, default=0.01, help="f4 SGD learning rate")
     p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
                    "peer (CUDA IPC); misses are served from peers' HBM before the host link")
+    p.add_argument("--samplers", type=int, default=2,
+                   help="sampler streams (P:94 'a pool of threads as samplers'), each with its own gd_workspace: "
+                        "batch j is sampled on stream j mod S, so the next batch's sampling overlaps this batch's "
+                        "(extraction stays in batch order on the caller's stream)")
+    p.add_argument("--no-peer-leg", action="store_true",
+                   help="N > 1: skip the extra f2 leg (every rank's buffer attached as NVLink peers, W + K more "
+                        "timed steps) that runs after the main measurement")
     p.add_argument("--parity-batches", type=int, default=None,
                    help="first batches of each rank checked in full (sample outputs, alias, hits/misses, rows) vs the "
                         "oracle; default 8 (papers100m/friendster/mag240m; 4 per rank at >= 8 ranks), 16 (products), "
@@ -420,7 +427,8 @@ def run_ours(args, rank, world, local_rank):
     sweep_cfgs = [tuple(float(x) for x in c.split(":")) for c in args.miss_sweep.split(",") if c]
     PRE = 0 if cfg.preload else args.prewarm_max
     n_pipe = len([x for x in args.pipeline_sweep.split(",") if x])
-    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe) * (W + K)
+    leg = world > 1 and not args.peer and not args.no_peer_leg and not cfg.preload
+    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe + int(leg)) * (W + K)
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -436,6 +444,15 @@ def run_ours(args, rank, world, local_rank):
     stats = torch.zeros((total, 4), dtype=torch.int64, device=dev)
     sizes_log = torch.zeros((total, 2 * len(fan) + 1), dtype=torch.int64, device=dev)
     main = torch.cuda.current_stream(dev)
+    NS = max(1, args.samplers)
+    samp_streams = [main] if NS == 1 else [torch.cuda.Stream(dev) for _ in range(NS)]
+    samp_ws = [None] if NS == 1 else [g.workspace() for _ in range(NS)]
+    ev_samp = [torch.cuda.Event() for _ in range(RING)]
+
+    def samplers_after(ev):       # timed regions: no sampling work before their start event
+        if NS > 1:
+            for ss in samp_streams:
+                ss.wait_event(ev)
     pending = []
     # releases on their own stream (GD_RELEASE_STREAM=0: on main); release(j - Q) is ordered after extract(j)'s bookkeeping
     # and before extract(j + 1)'s (the sequential order of Alg. 1, so the buffer state is the
@@ -477,11 +494,15 @@ def run_ours(args, rank, world, local_rank):
         last_o[0] = o
         if HOST_BOUND:
             dones[s].synchronize()         # the host, too, stays at most RING batches ahead (bounded queue)
-        main.wait_event(dones[s])          # batch j - RING is complete: its buffers are free
+        ss = samp_streams[j % NS]
+        ss.wait_event(dones[s])            # batch j - RING is complete: its buffers are free
         if model is not None:
-            main.wait_event(tdones[s])     # ... and trained (the trainer reads outs[s], feats[s])
+            ss.wait_event(tdones[s])       # ... and trained (the trainer reads outs[s], feats[s])
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
-        g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=main)
+        g.sample(sd, fan, synth.RNG_SEED, batch_ids[j], out=o, stream=ss, workspace=samp_ws[j % NS])
+        if ss is not main:
+            ev_samp[s].record(ss)
+            main.wait_event(ev_samp[s])
         dsync("sample", j)
         if rel_live[0]:
             main.wait_event(ev_rel)        # the previous step's release precedes this lookup
@@ -578,6 +599,7 @@ def run_ours(args, rank, world, local_rank):
     ev1 = torch.cuda.Event(enable_timing=True)
     with ClockSampler(local_rank) as clk:
         ev0.record(main)
+        samplers_after(ev0)
         win_ev = []
         for j in range(off + W, off + W + K):
             step(j)
@@ -651,6 +673,7 @@ def run_ours(args, rank, world, local_rank):
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(main)
+        samplers_after(e0)
         j_end = off + W + 2 * K
         for j in range(off + W + K, j_end):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats, h_ev, seen))
@@ -687,9 +710,52 @@ def run_ours(args, rank, world, local_rank):
             n_j = int(sizes_h[j][len(fan)])
             tail[j] = (outs[s_].n_id[:n_j].cpu().numpy(), aliases[s_][:n_j].cpu().numpy())
         replay_cap = (j_win, stats_h, sizes_h, tail, buf.snapshot())
+    # ---- f2 leg at N > 1 (after the main measurement and its replay window): every rank attaches
+    # the other ranks' buffers as NVLink peers (CUDA IPC, "reuse feature data loaded by other
+    # subprocesses") and runs W + K more steps; reports its rate and the share of misses peers served
+    peer_leg = None
+    if leg:
+        import torch.distributed as dist
+        torch.cuda.synchronize(dev)
+        s0, p0 = buf.peer_stats()
+        blobs = [None] * world
+        dist.all_gather_object(blobs, buf.peer_export_ipc())
+        buf.peer_attach_ipc([bl for r, bl in enumerate(blobs) if r != rank][:7])
+        barrier()
+        jl = j_win
+        for j in range(jl, jl + W):
+            step(j)
+        torch.cuda.synchronize(dev)
+        barrier()
+        pa_, pz_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        pa_.record(main)
+        samplers_after(pa_)
+        for j in range(jl + W, jl + W + K):
+            step(j)
+        main.wait_event(dones[(jl + W + K - 1) % RING])
+        if rel_live[0]:
+            main.wait_event(ev_rel)
+        pz_.record(main)
+        pz_.synchronize()
+        pl_ms = max_over_ranks(pa_.elapsed_time(pz_), dev)
+        s1, p1 = buf.peer_stats()
+        served, probed = sum_over_ranks(s1 - s0, dev), sum_over_ranks(p1 - p0, dev)
+        barrier()
+        buf.peer_attach_ipc([])
+        barrier()
+        peer_leg = {"value": round(world * K / (pl_ms / 1e3), 2), "unit": "batches/s", "steps": K,
+                    "served_rows": int(served), "probed_misses": int(probed),
+                    "served_share": round(served / max(1, probed), 4), "peers_per_rank": min(world - 1, 7),
+                    "same_device": os.environ.get("GD_BENCH_SAME_DEVICE") == "1",
+                    "def": "f2: W + K further steps with every other rank's buffer attached as a peer (misses probe the "
+                           "peers' maps and copy served rows over NVLink before the host paths); max-over-ranks time"}
+        log(f"f2 peer leg: {peer_leg}")
+        j_win_after = jl + W + K
+    else:
+        j_win_after = j_win
     # ---- optional in-process sweep of the miss-stream configuration (tuning only)
     sweep = []
-    j0 = off + W + K + (0 if args.no_e2e else K)
+    j0 = j_win_after
     for (thr, share, zcb, plb) in sweep_cfgs:
         torch.cuda.synchronize(dev)
         buf.config(int(thr), share, int(zcb), int(plb))
@@ -907,7 +973,7 @@ def run_ours(args, rank, world, local_rank):
         "value": round(value, 2), "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": round(ms_max / K, 4), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-        "config": config_dict(cfg, S, world, prewarm_batches),
+        "config": config_dict(cfg, S, world, prewarm_batches, NS),
         "e2e": e2e,
         # per step: seed intake + K x (sample, relabel) + col resolve + hash clear | lookup, pop/assign, hit gather
         # [+ zero-copy miss copy + peer-tag publish unless preload] [+ staged scatter when the host
@@ -934,6 +1000,7 @@ def run_ours(args, rank, world, local_rank):
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
         "peer": peer_info,
+        "peer_leg": peer_leg,
         "train": train_info,
         "setup_s": round(time.time() - t_setup, 1),
     }
@@ -1137,14 +1204,14 @@ def host_cpu_info():
     return info
 
 
-def config_dict(cfg, S, world, prewarm):
+def config_dict(cfg, S, world, prewarm, samplers):
     """The `config` object of the JSON line; identical for both arms."""
     R = cfg.row_bytes
     return {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
             "feat_dim": cfg.feat_dim, "feat_bytes": R, "batch_size": cfg.batch_size, "fanouts": list(cfg.fanouts),
             "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
             "buffer_prewarm_batches": prewarm,
-            "parallelism": f"dp{world} (batch segments, no collective)",
+            "parallelism": f"dp{world} (batch segments, no collective)", "sampler_streams": samplers,
             "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
                 (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.host_rows * R * 1e-9),
             "host_table_rows": cfg.host_rows}
@@ -1219,7 +1286,7 @@ def run_reference(args, rank, world, local_rank):
             "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": round(1e3 / v, 3) if v else None, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-            "config": config_dict(cfg, S, world, jp),
+            "config": config_dict(cfg, S, world, jp, max(1, args.samplers)),
             "cpu_baseline": cv, "single_thread_full_oracle": single, "host_cpu": host_cpu_info(),
             "e2e": {"value": v, "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
             "native_libs_loaded": loaded_native_libs()}

@@ -269,9 +269,9 @@ gd_status gd_buffer_stage_mode(gd_buffer* b, int copy_engine);
  * reassigned (before it is refilled); a reader checks the tag, copies, re-reads the
  * tag and falls back to the host when it changed.  Tags never repeat, so a stale copy
  * is always detected.  A buffer maintains its tags only from the moment another buffer can
- * read them (it is attached as someone's peer, or exported); that switch re-initialises every
- * tag (rows loaded before it are simply not offered), and until then its extractions skip
- * the tag writes.
+ * read them (it is attached as someone's peer, or exported): that switch rebuilds every tag
+ * from its mapping table (its streams idle, so every valid node's row is in its slot), and
+ * until then its extractions skip the tag writes.
  *   gd_buffer_peer_attach     in-process peers (same or other device; P2P access is
  *                             enabled here).  npeers = 0 detaches.  <= 7 peers; they
  *                             must have the same num_nodes, row_bytes and table rows.

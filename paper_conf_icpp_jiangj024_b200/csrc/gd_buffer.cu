@@ -1231,14 +1231,25 @@ static gd_status set_peers(gd_buffer* b, int n, const int2* const* maps, const u
 // A buffer maintains its f2 publication tags (cleared by k_pop_assign on reassignment, set by
 // k_publish) only from the moment another buffer can read them: in-process attach as someone's
 // peer, or an IPC export.  Until then it skips both (a random 8-byte write per miss, twice).
-// Switching on re-initialises every tag (preload: slot s holds node s; otherwise none), so a
-// tag left from before can never vouch for a slot's current row.
+// Switching on rebuilds every tag from the mapping table once the buffer's streams are idle
+// (so every valid node's row is in its slot): slot s of valid node v gets (epoch << 32 | v)
+// with the current epoch, every other slot none; a tag left from before can never vouch for
+// a slot's current row.
+__global__ void k_republish(const int2* __restrict__ map, int64_t N, unsigned long long* __restrict__ ready,
+                            unsigned long long epoch) {
+    for (int64_t v = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; v < N; v += (int64_t)gridDim.x * blockDim.x) {
+        const int2 m = map[v];
+        if ((m.y & 1) && m.x >= 0) ready[m.x] = (epoch << 32) | (uint32_t)v;
+    }
+}
+
 static gd_status ensure_publishing(gd_buffer* q) {
     if (q->publish) return GD_OK;
     DeviceGuard guard(q->hdr.device);
     gd_status s = drain_streams(q);
     if (s != GD_OK) return s;
-    k_init_ready<<<148 * 8, 256, 0, q->side_j>>>(q->ready, q->S, q->N, q->preload);
+    k_init_ready<<<148 * 8, 256, 0, q->side_j>>>(q->ready, q->S, q->N, 0);
+    k_republish<<<148 * 8, 256, 0, q->side_j>>>(q->map, q->N, q->ready, (unsigned long long)q->epoch);
     GD_CUDA(cudaStreamSynchronize(q->side_j));
     q->publish = true;
     return GD_OK;

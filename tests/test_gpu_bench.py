@@ -76,3 +76,5 @@ def test_bench_two_ranks_same_gpu_per_rank_parity():
     peaks = rec["host_link_peaks_GBps"]
     assert peaks["alone"] > 0 and peaks["concurrent"] > 0
     assert "rank0" in rec["roofline_miss"]
+    leg = rec["peer_leg"]                        # f2 leg: both ranks' buffers attached as peers
+    assert leg is not None and leg["value"] > 0 and leg["probed_misses"] > 0 and leg["served_rows"] >= 0
