@@ -70,7 +70,7 @@ def parse():
                         "all of the rank's segment (tiny)")
     p.add_argument("--no-replay", action="store_true",
                    help="skip the steady-state parity: the oracle's Alg. 1 replayed over the rank's whole schedule")
-    p.add_argument("--prewarm-max", type=int, default=400,
+    p.add_argument("--prewarm-max", type=int, default=1000,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
     p.add_argument("--window", type=int, default=0, help="also report batches/s per window of this many timed steps "
@@ -448,6 +448,11 @@ def run_ours(args, rank, world, local_rank):
     samp_streams = [main] if NS == 1 else [torch.cuda.Stream(dev) for _ in range(NS)]
     samp_ws = [None] if NS == 1 else [g.workspace() for _ in range(NS)]
     ev_samp = [torch.cuda.Event() for _ in range(RING)]
+    # slot s's previous batch has been released (its release reads outs[s].n_id): a sampler on
+    # its own stream must not overwrite that n_id before (on the caller's stream the release's
+    # event wait orders it)
+    ev_relslot = [torch.cuda.Event() for _ in range(RING)]
+    relslot_live = [False] * RING
 
     def samplers_after(ev):       # timed regions: no sampling work before their start event
         if NS > 1:
@@ -496,6 +501,8 @@ def run_ours(args, rank, world, local_rank):
             dones[s].synchronize()         # the host, too, stays at most RING batches ahead (bounded queue)
         ss = samp_streams[j % NS]
         ss.wait_event(dones[s])            # batch j - RING is complete: its buffers are free
+        if relslot_live[s] and ss is not main:
+            ss.wait_event(ev_relslot[s])   # ... and released
         if model is not None:
             ss.wait_event(tdones[s])       # ... and trained (the trainer reads outs[s], feats[s])
         sd = seeds_host[j] if host_inputs else seeds_dev[j]
@@ -523,13 +530,15 @@ def run_ours(args, rank, world, local_rank):
                     z.record(tstream)
                     t_events.append((a, z))
             tdones[s].record(tstream)
-        pending.append(o)
+        pending.append((o, s))
         if len(pending) == Q:
-            r = pending.pop(0)
+            r, rs = pending.pop(0)
             if rel_stream is not main:
                 ev_bk.record(main)
                 rel_stream.wait_event(ev_bk)
             buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=rel_stream)
+            ev_relslot[rs].record(rel_stream)
+            relslot_live[rs] = True
             if rel_stream is not main:
                 ev_rel.record(rel_stream)
                 rel_live[0] = True
@@ -791,7 +800,7 @@ def run_ours(args, rank, world, local_rank):
         from paper_conf_icpp_jiangj024_b200.pipeline import SETPipeline
         torch.cuda.synchronize(dev)
         while pending:                              # hand the buffer over with nothing in flight
-            r = pending.pop(0)
+            r, _ = pending.pop(0)
             buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
         torch.cuda.synchronize(dev)
         for spec in args.pipeline_sweep.split(","):
@@ -822,7 +831,7 @@ def run_ours(args, rank, world, local_rank):
     if last_o[0] is not None:
         torch.cuda.synchronize(dev)
         while pending:
-            r = pending.pop(0)
+            r, _ = pending.pop(0)
             buf.release(r.n_id, r.num_nodes_dev, r.max_nodes, stream=main)
         torch.cuda.synchronize(dev)
         lo = last_o[0]
