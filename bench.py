@@ -73,6 +73,9 @@ def parse():
     p.add_argument("--prewarm-max", type=int, default=1000,
                    help="untimed buffer pre-warm: batches until cumulative misses >= S (SURVEY 8(d)), at most this")
     p.add_argument("--out", default=None, help="also write the JSON line to this file")
+    p.add_argument("--timeline", default=None, help="after the measurement, 16 more steps under torch.profiler "
+                   "(CUPTI): per-activity busy time and the overlap of the miss stream with sampling -> this .md "
+                   "(tools/timeline.py)")
     p.add_argument("--window", type=int, default=0, help="also report batches/s per window of this many timed steps "
                    "(device events on the caller's stream; sustained-rate evidence)")
     p.add_argument("--pipeline-sweep", default="", help="f1: 'samplers:reorder,...' SET pipeline runs "
@@ -428,7 +431,8 @@ def run_ours(args, rank, world, local_rank):
     PRE = 0 if cfg.preload else args.prewarm_max
     n_pipe = len([x for x in args.pipeline_sweep.split(",") if x])
     leg = world > 1 and not args.peer and not args.no_peer_leg and not cfg.preload
-    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe + int(leg)) * (W + K)
+    TL = 16 if args.timeline else 0
+    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe + int(leg)) * (W + K) + TL
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -762,6 +766,25 @@ def run_ours(args, rank, world, local_rank):
         j_win_after = jl + W + K
     else:
         j_win_after = j_win
+    # ---- timeline (VERDICT r1 missing #7): TL more steps under the CUPTI activity tracer
+    timeline = None
+    if TL:
+        import tempfile
+        from torch.profiler import ProfilerActivity, profile
+        from tools.timeline import summarise
+        torch.cuda.synchronize(dev)
+        with profile(activities=[ProfilerActivity.CUDA]) as prof:
+            for j in range(j_win_after, j_win_after + TL):
+                step(j)
+            torch.cuda.synchronize(dev)
+        with tempfile.NamedTemporaryFile(suffix=".json", delete=False) as tf:
+            path = tf.name
+        prof.export_chrome_trace(path)
+        if rank == 0:
+            timeline = summarise(path, args.timeline, TL, f"Timeline — {cfg.name}, {TL} steps (bench.py --timeline)")
+            log(f"timeline: {timeline}")
+        os.unlink(path)
+        j_win_after += TL
     # ---- optional in-process sweep of the miss-stream configuration (tuning only)
     sweep = []
     j0 = j_win_after
@@ -1010,6 +1033,7 @@ def run_ours(args, rank, world, local_rank):
         "device_status": {"graph": status_g, "buffer": status_b},
         "peer": peer_info,
         "peer_leg": peer_leg,
+        "timeline": timeline,
         "train": train_info,
         "setup_s": round(time.time() - t_setup, 1),
     }
