@@ -216,9 +216,9 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  *                    and host gather rate r_host and the contiguous pull rate r_link of
  *                    the host link (calibrated when this call enables adaptation):
  *                    r_zc / (r_zc + r_host) if r_zc + r_host <= r_link, else
- *                    1 - r_host / r_link; clamped to [0.05, 0.9] (to [0.05, 0.2] with
- *                    copy-engine staging, [0.05, 0.3] once >= 8 host-rate samples show the
- *                    host gather below 0.6 r_link; back to 0.2 above 0.7 r_link).
+ *                    1 - r_host / r_link; clamped to [0.05, 0.9] ([0.05, 0.15] with
+ *                    copy-engine staging: a larger zero-copy share collapses the copy
+ *                    engine's rate on some hosts).
  *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
  *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs
@@ -233,7 +233,7 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
 
 /* The miss-path split policy (gd_buffer_config, adaptive share), for reports: out[0..n) of
  * {zero-copy share, r_host, r_zc, r_link (GB/s), misses-per-batch estimate (the copy-engine
- * staging size), host-rate samples, slow-host cap active (0/1), newest batch rated}.  The
+ * staging size), host-rate samples, the share's upper clamp, newest batch rated}.  The
  * estimates come from the newest completed batch at each gd_extract (events queried, never
  * waited on) and the miss count from the newest batch whose loop 2 ran (an epoch-tagged count
  * the device writes to mapped host memory).  Host-only, no sync; n <= 8. */

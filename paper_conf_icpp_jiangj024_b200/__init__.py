@@ -322,7 +322,7 @@ class FeatureBuffer:
         v = (ctypes.c_double * 8)()
         check(lib.gd_buffer_policy_read(self._h, v, 8))
         return {"zero_copy_share": v[0], "r_host_GBps": v[1], "r_zc_GBps": v[2], "r_link_GBps": v[3],
-                "misses_est": v[4], "rate_samples": int(v[5]), "slow_host": bool(v[6]), "rated_batch": int(v[7])}
+                "misses_est": v[4], "rate_samples": int(v[5]), "share_cap": v[6], "rated_batch": int(v[7])}
 
     def config(self, host_threads: int, zero_copy_share: float = -1.0, zc_blocks: int = 0, pull_blocks: int = 0):
         """gd_buffer_config: staged miss path width, zero-copy share (< 0: adaptive), copy grids."""

@@ -36,7 +36,8 @@ constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
 constexpr int kStageRing = 4;    // pinned chunk buffers of the copy-engine staging ring
 constexpr int kJobRing = 1024;   // host-function argument slots of the staged chunks
-constexpr int kTimedPairs = 5;   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
+constexpr int kTimedPairs = 5;
+constexpr double kZeroCopyCapCE = 0.15;   // adaptive zero-copy share cap with copy-engine staging   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
 
 static int64_t cdiv(int64_t a, int64_t b) { return (a + b - 1) / b; }
 
@@ -1192,7 +1193,6 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     b->r_host = 0;
     b->r_zc = 0;
     b->rate_samples = 0;
-    b->slow_host = false;
     b->rated_batch = b->batch_counter - 1;
     if (host_threads > 0 && !b->alpha_fixed) {
         gd_status st = calibrate_link(b);
@@ -1475,15 +1475,12 @@ static void adapt_alpha(gd_buffer* b) {
     else
         a = 1.0 - b->r_host / b->r_link;
     // With copy-engine staging the zero-copy share also costs the DMA engine: its random
-    // 4 KB-page reads contend for the host's DMA translation, and a share above ~0.2 was
-    // measured to collapse the copy rate (to ~17 GB/s at 0.4); cap it there.  Only a host
-    // whose gather persistently cannot fill the link (>= 8 rate samples below 0.6 r_link; back
-    // above 0.7 r_link to leave) gets 0.3: the copy engine has slack there (measured 3-6%
-    // better with 6 gather threads).  The hysteresis keeps one slow warm-up batch from
-    // switching the cap.
-    if (b->rate_samples >= 8 && b->r_host < 0.6 * b->r_link) b->slow_host = true;
-    if (b->r_host > 0.7 * b->r_link) b->slow_host = false;
-    const double hi = (b->ce_mode && b->dstage) ? (b->slow_host ? 0.3 : 0.2) : 0.9;
+    // 4 KB-page reads contend with the copy engine for the host's DMA translation, and past a
+    // box-dependent threshold the copy rate collapses (r01: ~17 GB/s at 0.4; r02, a slow-host
+    // box, papers100m: share 0.1 / 0.15 / 0.2 / 0.3 -> 450 / 500 / 197 / 319 batches/s, the copy
+    // engine 2.0 ms per batch at 0.15 and 5.1 ms at 0.2).  Cap it at 0.15, below every collapse
+    // measured; a fast host (r_host > r_link) gets 0.05 anyway.
+    const double hi = (b->ce_mode && b->dstage) ? kZeroCopyCapCE : 0.9;
     b->alpha = std::min(hi, std::max(0.05, a));
 }
 
@@ -1491,7 +1488,8 @@ gd_status gd_buffer_policy_read(gd_buffer* b, double* out, int32_t n) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: bad handle");
     if (!out || n < 0) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: null output");
     const double v[8] = {b->alpha, b->r_host * 1e-6, b->r_zc * 1e-6, b->r_link * 1e-6, b->m_est,
-                         (double)b->rate_samples, b->slow_host ? 1.0 : 0.0, (double)b->rated_batch};
+                         (double)b->rate_samples, (b->ce_mode && b->dstage) ? kZeroCopyCapCE : 0.9,
+                         (double)b->rated_batch};
     for (int k = 0; k < n && k < 8; ++k) out[k] = v[k];
     return GD_OK;
 }

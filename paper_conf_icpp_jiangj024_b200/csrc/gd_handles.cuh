@@ -134,7 +134,6 @@ struct gd_buffer {
     double r_link = 0;                   // contiguous pull rate of the host link (bytes/ms), calibrated
     bool alpha_fixed = false;
     int64_t rate_samples = 0;            // host-gather rate samples since the last config
-    bool slow_host = false;              // r_host persistently < 0.6 r_link (zero-copy cap 0.3)
     int64_t rated_batch = -1;            // newest batch whose path rates entered the estimates
     gd::HostGatherPool* pool = nullptr;
     // phase 2 of the staged share: copy engine (cudaMemcpyAsync pinned slot -> dstage[d]

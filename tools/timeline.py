@@ -18,9 +18,11 @@ CATS = [
     ("sampling (a1-a4)", lambda n, k: k == "kernel" and n.startswith(SAMPLING)),
     ("bookkeeping (a5, a6, a9)", lambda n, k: k == "kernel" and n.startswith(BOOKKEEPING)),
     ("hit gather (a8)", lambda n, k: k == "kernel" and n.startswith(("k_gather_rows", "k_gather_tma", "k_gather_hits"))),
-    ("miss zero-copy kernel (a7)", lambda n, k: k == "kernel" and n.startswith("k_miss_copy<4, 0>")),
+    ("miss zero-copy kernel (a7)", lambda n, k: k == "kernel" and n.startswith(("k_miss_copy<4, 0>", "k_miss_copy<4, false>",
+                                                                             "k_miss_copy_w4<false>", "k_miss_copy_w4<0>"))),
     ("miss copy-engine H2D (a7)", lambda n, k: k == "gpu_memcpy" and "HtoD" in n),
-    ("miss staged scatter (a7)", lambda n, k: k == "kernel" and n.startswith("k_miss_copy<4, 1>")),
+    ("miss staged scatter (a7)", lambda n, k: k == "kernel" and n.startswith(("k_miss_copy<4, 1>", "k_miss_copy<4, true>",
+                                                                           "k_miss_copy_w4<true>", "k_miss_copy_w4<1>"))),
 ]
 
 
