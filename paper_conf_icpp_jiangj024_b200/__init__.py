@@ -319,10 +319,12 @@ class FeatureBuffer:
 
     def policy_read(self):
         """gd_buffer_policy_read: the miss-path split policy's current inputs and decision."""
-        v = (ctypes.c_double * 8)()
-        check(lib.gd_buffer_policy_read(self._h, v, 8))
+        v = (ctypes.c_double * 12)()
+        check(lib.gd_buffer_policy_read(self._h, v, 12))
         return {"zero_copy_share": v[0], "r_host_GBps": v[1], "r_zc_GBps": v[2], "r_link_GBps": v[3],
-                "misses_est": v[4], "rate_samples": int(v[5]), "share_cap": v[6], "rated_batch": int(v[7])}
+                "misses_est": v[4], "rate_samples": int(v[5]), "model_share_cap": v[6], "rated_batch": int(v[7]),
+                "tuner_on": bool(v[8]), "tuner_windows": int(v[9]), "tuner_frozen": bool(v[10]),
+                "tuner_best_ns_per_miss": v[11]}
 
     def config(self, host_threads: int, zero_copy_share: float = -1.0, zc_blocks: int = 0, pull_blocks: int = 0):
         """gd_buffer_config: staged miss path width, zero-copy share (< 0: adaptive), copy grids."""

@@ -934,10 +934,10 @@ static void buffer_free(gd_buffer* b) {
     b->scan.release();
     b->timer.destroy();
     for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_ring,
-                    &b->ev_s0, &b->ev_job})
+                    &b->ev_s0, &b->ev_job, &b->ev_fin})
         for (cudaEvent_t e : *v)
             if (e) cudaEventDestroy(e);
-    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk, b->ev_S})
+    for (cudaEvent_t e : {b->ev_L, b->ev_X, b->ev_Xs, b->ev_G, b->ev_chunk, b->ev_S, b->ev_ref})
         if (e) cudaEventDestroy(e);
     for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c})
         if (s) cudaStreamDestroy(s);
@@ -1094,9 +1094,10 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     for (cudaEvent_t* ep : {&b->ev_L, &b->ev_X, &b->ev_Xs, &b->ev_G, &b->ev_S})
         if (cudaEventCreateWithFlags(ep, cudaEventDisableTiming) != cudaSuccess)
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: event"));
-    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_s0}) {
+    for (auto* v : {&b->ev_trip, &b->ev_E, &b->ev_P, &b->ev_z0, &b->ev_z1, &b->ev_p0, &b->ev_p1, &b->ev_H, &b->ev_s0,
+                    &b->ev_fin}) {
         const bool timing = (v == &b->ev_z0 || v == &b->ev_z1 || v == &b->ev_p0 || v == &b->ev_p1 || v == &b->ev_E ||
-                             v == &b->ev_s0);
+                             v == &b->ev_s0 || v == &b->ev_fin);
         v->assign(b->D, nullptr);
         for (int d = 0; d < b->D; ++d)
             if (cudaEventCreateWithFlags(&(*v)[d], timing ? cudaEventDefault : cudaEventDisableTiming) != cudaSuccess)
@@ -1194,6 +1195,15 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     b->r_zc = 0;
     b->rate_samples = 0;
     b->rated_batch = b->batch_counter - 1;
+    b->tune = ShareTuner();
+    {
+        const char* e = std::getenv("GD_SHARE_TUNER");
+        b->tune.on = host_threads > 0 && !b->alpha_fixed && b->ce_mode && !(e && e[0] == '0');
+        for (int k = 0; k < 64; ++k) b->tune.mb[k] = -1;
+        b->tune.change_batch = b->batch_counter;
+        if (!b->ev_ref) GD_CUDA(cudaEventCreate(&b->ev_ref));
+        GD_CUDA(cudaEventRecord(b->ev_ref, b->side_j));
+    }
     if (host_threads > 0 && !b->alpha_fixed) {
         gd_status st = calibrate_link(b);
         if (st != GD_OK) return st;
@@ -1478,19 +1488,116 @@ static void adapt_alpha(gd_buffer* b) {
     // 4 KB-page reads contend with the copy engine for the host's DMA translation, and past a
     // box-dependent threshold the copy rate collapses (r01: ~17 GB/s at 0.4; r02, a slow-host
     // box, papers100m: share 0.1 / 0.15 / 0.2 / 0.3 -> 450 / 500 / 197 / 319 batches/s, the copy
-    // engine 2.0 ms per batch at 0.15 and 5.1 ms at 0.2).  Cap it at 0.15, below every collapse
-    // measured; a fast host (r_host > r_link) gets 0.05 anyway.
+    // engine 2.0 ms per batch at 0.15 and 5.1 ms at 0.2).  The model's share is clamped to
+    // [0.05, 0.15], below every collapse measured; with the tuner on, it is only the start.
     const double hi = (b->ce_mode && b->dstage) ? kZeroCopyCapCE : 0.9;
-    b->alpha = std::min(hi, std::max(0.05, a));
+    const double model = std::min(hi, std::max(0.05, a));
+    if (!b->tune.on) {
+        b->alpha = model;
+        return;
+    }
+    ShareTuner& T = b->tune;
+    if (!T.have_best && T.windows == 0 && T.phase == 0 && T.w_b0 < 0) {
+        T.alpha = T.best_alpha = model;                     // start from the model
+        b->alpha = model;
+    }
+}
+
+// (3) The share tuner (ShareTuner in gd_handles.cuh).  Called at every gd_extract after the
+// estimates; reads only events that have completed and mapped host words.
+static void tune_share(gd_buffer* b) {
+    ShareTuner& T = b->tune;
+    if (!T.on || T.frozen || b->r_host <= 0) return;
+    const int64_t bc = b->batch_counter;
+    // per-batch miss counts: a slot's word belongs to its current batch once the epochs match
+    for (int d = 0; d < b->D; ++d) {
+        const StagedSlot& ss = b->stg[d];
+        if (ss.batch < 0) continue;
+        const unsigned long long w = *(volatile const unsigned long long*)(ss.h_meta + 4);
+        if ((w >> 32) == (ss.epoch & 0xffffffffull) && T.mb[ss.batch & 63] != ss.batch) {
+            T.mb[ss.batch & 63] = ss.batch;
+            T.mc[ss.batch & 63] = (int64_t)(w & 0xffffffffull);
+        }
+    }
+    // newest completed batch and its completion time
+    int64_t nb = -1;
+    float tnb = 0;
+    for (int k = 1; k < b->D && bc - k >= 0; ++k) {
+        const int d = (int)((bc - k) % b->D);
+        if (b->stg[d].batch != bc - k) break;
+        if (cudaEventQuery(b->ev_fin[d]) == cudaSuccess && cudaEventElapsedTime(&tnb, b->ev_ref, b->ev_fin[d]) == cudaSuccess) {
+            nb = bc - k;
+            break;
+        }
+        cudaGetLastError();
+    }
+    cudaGetLastError();
+    if (nb < 0) return;
+    if (T.phase == 0) {                    // settling: the window starts at the first new-share batch
+        if (nb >= T.change_batch) {
+            T.w_b0 = nb;
+            T.w_t0 = tnb;
+            T.phase = 1;
+        }
+        return;
+    }
+    constexpr int kWindow = 6;
+    if (nb - T.w_b0 < kWindow) return;
+    int64_t misses = 0;
+    bool known = true;
+    for (int64_t x = T.w_b0 + 1; x <= nb; ++x) {
+        if (T.mb[x & 63] != x) { known = false; break; }
+        misses += T.mc[x & 63];
+    }
+    if (!known || misses <= 0) {           // a count was missed (the host ran far ahead): re-measure
+        T.w_b0 = nb;
+        T.w_t0 = tnb;
+        return;
+    }
+    const double cost = (double)(tnb - T.w_t0) / (double)misses;
+    T.windows++;
+    double next;
+    if (!T.have_best || cost < T.best_cost * 0.985) {            // better: keep going this way
+        T.have_best = true;
+        T.best_alpha = T.alpha;
+        T.best_cost = cost;
+        T.fails = 0;
+        next = T.alpha + T.dir * T.step;
+    } else if (T.alpha == T.best_alpha) {                        // re-measured the best
+        T.best_cost = cost;
+        next = T.alpha + T.dir * T.step;
+    } else {                                                     // worse: try the other side
+        T.dir = -T.dir;
+        if (++T.fails >= 2) {
+            T.fails = 0;
+            T.step *= 0.5;
+        }
+        next = T.best_alpha + T.dir * T.step;
+    }
+    constexpr double kLo = 0.0, kHi = 0.4;
+    if (next < kLo || next > kHi) {                              // at a bound: the other side
+        T.dir = -T.dir;
+        next = T.best_alpha + T.dir * T.step;
+    }
+    if (T.step < 0.0124 || next < kLo || next > kHi) {
+        T.frozen = true;
+        next = T.best_alpha;
+    }
+    T.alpha = next;
+    b->alpha = next;
+    T.change_batch = bc;
+    T.phase = 0;
 }
 
 gd_status gd_buffer_policy_read(gd_buffer* b, double* out, int32_t n) {
     if (!b || b->hdr.magic != kMagicBuffer) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: bad handle");
     if (!out || n < 0) return set_error(GD_ERR_INVALID, "gd_buffer_policy_read: null output");
-    const double v[8] = {b->alpha, b->r_host * 1e-6, b->r_zc * 1e-6, b->r_link * 1e-6, b->m_est,
-                         (double)b->rate_samples, (b->ce_mode && b->dstage) ? kZeroCopyCapCE : 0.9,
-                         (double)b->rated_batch};
-    for (int k = 0; k < n && k < 8; ++k) out[k] = v[k];
+    const ShareTuner& T = b->tune;
+    const double v[12] = {b->alpha, b->r_host * 1e-6, b->r_zc * 1e-6, b->r_link * 1e-6, b->m_est,
+                          (double)b->rate_samples, (b->ce_mode && b->dstage) ? kZeroCopyCapCE : 0.9,
+                          (double)b->rated_batch, T.on ? 1.0 : 0.0, (double)T.windows, T.frozen ? 1.0 : 0.0,
+                          T.best_cost * 1e6};
+    for (int k = 0; k < n && k < 12; ++k) out[k] = v[k];
     return GD_OK;
 }
 
@@ -1561,6 +1668,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_CUDA(cudaStreamWaitEvent(st, b->ev_trip[d], 0));
     if (staged) {
         adapt_alpha(b);
+        tune_share(b);
         ss->batch = b->batch_counter;
     }
     const uint32_t alpha_q16 = staged ? (uint32_t)std::lround(b->alpha * 65536.0) : 65536u;
@@ -1627,6 +1735,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     pa.ticket = b->tickets;
     pa.done_word = b->done_word;
     pa.epoch = ++b->epoch;
+    if (staged) ss->epoch = pa.epoch;
     pa.st = b->scan.use();
     pa.st_clear = b->scan.other();
     pa.st_clear_n = b->scan.cap;
@@ -1794,6 +1903,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     // release, and with it any reuse of these slots, is ordered after the publication)
     if (!b->preload && b->publish) k_publish<<<148, 256, 0, b->side_j>>>(trip, tcount, b->ready, pa.epoch);
     GD_CUDA(cudaEventRecord(b->ev_trip[d], b->side_j));
+    GD_CUDA(cudaEventRecord(b->ev_fin[d], b->side_j));
     if (done_v) GD_CUDA(cudaEventRecord((cudaEvent_t)done_v, b->side_j));
     GD_CUDA(cudaGetLastError());
     b->inflight++;

@@ -74,6 +74,27 @@ struct StagedSlot {
     uint8_t* staging = nullptr;   // pinned, mapped [n_max x R]
     double cpu_ms = 0;            // duration of the last host gather into this slot
     int64_t batch = -1;           // batch that last used this slot
+    uint64_t epoch = 0;           // that batch's epoch (its published miss-count word carries it)
+};
+
+// Hill-climbing tuner of the zero-copy share: the cost of a share is the
+// extraction period per miss over a window of completed batches (done-to-done event time /
+// their misses); the tuner moves the share by `step` while that improves, turns back when it
+// gets worse, halves the step after failing on both sides, and freezes at the best share.
+struct ShareTuner {
+    bool on = false;
+    bool frozen = false;
+    int phase = 0;                 // 0: settling after a change, 1: measuring
+    int64_t change_batch = 0;      // first batch enqueued with the current share
+    int64_t w_b0 = -1;             // window start: batch, its completion time (ms since ev_ref)
+    double w_t0 = 0;
+    double alpha = 0.1;            // share under test
+    double best_alpha = 0.1, best_cost = 0;
+    bool have_best = false;
+    int dir = +1, fails = 0, windows = 0;
+    double step = 0.05;
+    int64_t mb[64];                // per-batch miss counts seen so far: batch id and count, ring
+    int64_t mc[64];
 };
 
 // Feature buffer + extraction workspace.
@@ -135,6 +156,9 @@ struct gd_buffer {
     bool alpha_fixed = false;
     int64_t rate_samples = 0;            // host-gather rate samples since the last config
     int64_t rated_batch = -1;            // newest batch whose path rates entered the estimates
+    ShareTuner tune;                     // GD_SHARE_TUNER=0: model-based share only
+    std::vector<cudaEvent_t> ev_fin;     // [D] timing: batch d's extraction complete (stream J join)
+    cudaEvent_t ev_ref = nullptr;        // timing reference of ev_fin
     gd::HostGatherPool* pool = nullptr;
     // phase 2 of the staged share: copy engine (cudaMemcpyAsync pinned slot -> dstage[d]
     // on stream H, then a scatter kernel on P) or an SM pull kernel reading the pinned slot

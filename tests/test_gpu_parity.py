@@ -283,7 +283,7 @@ def test_adaptive_split_stages_without_host_sync(gd):
     assert int(st[:, 1].sum()) > 0
     assert int(st[10:, 3].sum()) > 0, st[:, 2:].tolist()        # the staged share ran
     pol = buf.policy_read()
-    assert pol["misses_est"] > 0 and 0.05 <= pol["zero_copy_share"] <= 0.3, pol
+    assert pol["misses_est"] > 0 and 0.0 <= pol["zero_copy_share"] <= 0.4 and pol["tuner_on"], pol
     ob = O.Buffer(feat, Q * n_max)
     opend = []
     for b in range(nbat):
