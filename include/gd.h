@@ -218,8 +218,8 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  *                    r_zc / (r_zc + r_host) if r_zc + r_host <= r_link, else
  *                    1 - r_host / r_link; clamped to [0.05, 0.9] ([0.05, 0.15] with
  *                    copy-engine staging: a larger zero-copy share collapses the copy
- *                    engine's rate on some hosts), then (copy-engine
- *                    staging) refined by the share tuner (gd_buffer_policy_read).
+ *                    engine's rate on some hosts); GD_SHARE_TUNER=1 refines
+ *                    it by measurement (gd_buffer_policy_read).
  *   zc_blocks, pull_blocks  grid (1024-thread blocks, about one SM each) of the two
  *                    copy kernels; <= 0 keeps the current value (defaults 16 and 8).
  *                    Few whole-SM blocks keep long-latency host loads off the SMs
@@ -238,11 +238,11 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
  * tuner on (0/1), tuner windows measured, tuner frozen (0/1), tuner's best cost (ns per miss)}.
  * The estimates come from the newest completed batch at each gd_extract (events queried, never
  * waited on) and the miss count from the newest batch whose loop 2 ran (an epoch-tagged count
- * the device writes to mapped host memory).  With copy-engine staging and an adaptive share a
- * hill-climbing tuner then owns the share: it starts at the model's value, measures the
- * extraction period per miss over windows of 6 completed batches, moves the share in steps
- * (0.05, halved after failing on both sides) while that improves, and freezes at the best
- * share in [0, 0.4] (env GD_SHARE_TUNER=0: the model only).  Host-only, no sync; n <= 12. */
+ * the device writes to mapped host memory).  Optionally (env GD_SHARE_TUNER=1, copy-engine
+ * staging, adaptive share) a hill-climbing tuner owns the share: it starts at the model's value,
+ * measures the extraction period per miss over windows of 6 completed batches, moves the share
+ * in steps (0.05, halved after failing on both sides) while that improves, and freezes at the
+ * best share in [0, 0.4].  Host-only, no sync; n <= 12. */
 gd_status gd_buffer_policy_read(gd_buffer* b, double* out, int32_t n);
 
 /* ----------------------------------------------------------------------------

@@ -1198,7 +1198,10 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     b->tune = ShareTuner();
     {
         const char* e = std::getenv("GD_SHARE_TUNER");
-        b->tune.on = host_threads > 0 && !b->alpha_fixed && b->ce_mode && !(e && e[0] == '0');
+        // off by default: measured no better than the model share on a fast-host box (papers100m
+        // 511 vs 519, mag240m 923 vs 1014 batches/s) and its probes of large shares can hit the
+        // copy-engine collapse inside a short timed region; GD_SHARE_TUNER=1 enables
+        b->tune.on = host_threads > 0 && !b->alpha_fixed && b->ce_mode && (e && e[0] == '1');
         for (int k = 0; k < 64; ++k) b->tune.mb[k] = -1;
         b->tune.change_batch = b->batch_counter;
         if (!b->ev_ref) GD_CUDA(cudaEventCreate(&b->ev_ref));

@@ -252,6 +252,40 @@ def test_release_on_its_own_stream_matches_oracle(tiny, gd, own_stream, row_byte
     assert buf.check() == 0
 
 
+def test_share_tuner_runs_and_stays_exact(gd, monkeypatch):
+    """GD_SHARE_TUNER=1: the hill-climbing share tuner measures windows and moves the zero-copy
+    share (in [0, 0.4]) while the outputs and the buffer state stay the oracle's."""
+    monkeypatch.setenv("GD_SHARE_TUNER", "1")
+    N, E, B, fan, Q, nbat = 200_000, 2_000_000, 1000, [10, 5], 4, 60
+    indptr, indices = make_graph(N, E, seed=23)
+    g = gd.Graph(indptr, indices)
+    feat = table_np(N, 512)
+    order = synth.epoch_order(synth.train_nodes(N, 0.5))
+    nb, _ = O.sample_bounds(B, fan, N, E)
+    n_max = nb[-1]
+    buf = gd.FeatureBuffer(torch.from_numpy(feat), Q * n_max, Q, n_max)
+    buf.config(4, -1.0)
+    ob = O.Buffer(feat, Q * n_max)
+    pend, opend = [], []
+    for b in range(nbat):
+        r = g.sample(order[(b % 100) * B:((b % 100) + 1) * B].cuda(), fan, 3, b)
+        st = torch.zeros(4, dtype=torch.int64, device="cuda")
+        out, _, done = buf.extract(r.n_id, r.num_nodes_dev, r.max_nodes, stats=st)
+        done.synchronize()                      # completed batches let the tuner measure windows
+        n_id = r.to_host()["n_id"]
+        o_out, _, o_st = ob.extract(n_id)
+        assert tuple(st.cpu().tolist()[:2]) == o_st and np.array_equal(out[:len(n_id)].cpu().numpy(), o_out), b
+        pend.append(r), opend.append(n_id)
+        if len(pend) == Q:
+            r0 = pend.pop(0)
+            buf.release(r0.n_id, r0.num_nodes_dev, r0.max_nodes)
+            ob.release(opend.pop(0))
+    pol = buf.policy_read()
+    assert pol["tuner_on"] and pol["tuner_windows"] >= 2 and 0.0 <= pol["zero_copy_share"] <= 0.4, pol
+    compare_state(buf, ob)
+    assert buf.check() == 0
+
+
 def test_adaptive_split_stages_without_host_sync(gd):
     """a caller that never synchronises (the host may run many batches ahead of the
     device) still gets a miss-count estimate for the copy-engine staging size (each batch's
@@ -283,7 +317,7 @@ def test_adaptive_split_stages_without_host_sync(gd):
     assert int(st[:, 1].sum()) > 0
     assert int(st[10:, 3].sum()) > 0, st[:, 2:].tolist()        # the staged share ran
     pol = buf.policy_read()
-    assert pol["misses_est"] > 0 and 0.0 <= pol["zero_copy_share"] <= 0.4 and pol["tuner_on"], pol
+    assert pol["misses_est"] > 0 and 0.05 <= pol["zero_copy_share"] <= 0.15 and not pol["tuner_on"], pol
     ob = O.Buffer(feat, Q * n_max)
     opend = []
     for b in range(nbat):
