@@ -159,35 +159,49 @@ def log(*a):
 
 class ClockSampler:
     """SM clocks and throttle reasons sampled every 200 ms during the timed region, in-process
-    through NVML (spawning nvidia-smi would steal a host core from the miss-path gather)."""
+    through NVML (spawning nvidia-smi would steal a host core from the miss-path gather).
+    NVML is initialised (and queried once) when the sampler is constructed, before the timed
+    region: nvmlInit inside the region stalled the copy-engine miss path for ~100 ms in some
+    runs (20-step papers100m: 149 batches/s vs 444-485), visible only in short regions."""
+
+    BITS = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40, "sw_power_cap": 0x4}
 
     def __init__(self, gpu_index: int):
         self.gpu = gpu_index
         self.rows = []
         self._stop = threading.Event()
         self._t = None
-
-    def _run(self):
+        self._N = self._h = None
         try:
             import pynvml as N
             N.nvmlInit()
-            h = N.nvmlDeviceGetHandleByIndex(self.gpu)
+            self._N, self._h = N, N.nvmlDeviceGetHandleByIndex(gpu_index)
+            self._query()
+            self.rows.clear()
         except Exception:  # noqa: BLE001
+            self._N = None
+
+    def _query(self):
+        N, h = self._N, self._h
+        sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
+        mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
+        r = N.nvmlDeviceGetCurrentClocksEventReasons(h) if hasattr(N, "nvmlDeviceGetCurrentClocksEventReasons") \
+            else N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
+        self.rows.append((sm, mx, [k for k, b in self.BITS.items() if r & b]))
+
+    def _run(self):
+        if self._N is None:
             return
-        bits = {"hw_slowdown": 0x8, "sw_thermal_slowdown": 0x20, "hw_thermal_slowdown": 0x40,
-                "sw_power_cap": 0x4}
         while not self._stop.is_set():
             try:
-                sm = N.nvmlDeviceGetClockInfo(h, N.NVML_CLOCK_SM)
-                mx = N.nvmlDeviceGetMaxClockInfo(h, N.NVML_CLOCK_SM)
-                r = N.nvmlDeviceGetCurrentClocksEventReasons(h) if hasattr(N, "nvmlDeviceGetCurrentClocksEventReasons") \
-                    else N.nvmlDeviceGetCurrentClocksThrottleReasons(h)
-                self.rows.append((sm, mx, [k for k, b in bits.items() if r & b]))
+                self._query()
             except Exception:  # noqa: BLE001
                 pass
             self._stop.wait(0.2)
 
     def __enter__(self):
+        self._stop.clear()
+        self.rows = []
         self._t = threading.Thread(target=self._run, daemon=True)
         self._t.start()
         return self
@@ -604,13 +618,18 @@ def run_ours(args, rank, world, local_rank):
     torch.cuda.synchronize(dev)
 
     # ---- timed region (device events on the launching stream)
+    clock_sampler = ClockSampler(local_rank)     # NVML initialised here, outside the region
+    import gc
+    gc.collect()
+    gc.disable()                                  # no collector pause in the host loop of the region
+    torch.cuda.synchronize(dev)
     log("timed region ...")
     g.timing(True)
     buf.timing(True)
     train_timing[0] = True
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
-    with ClockSampler(local_rank) as clk:
+    with clock_sampler as clk:
         ev0.record(main)
         samplers_after(ev0)
         win_ev = []
@@ -631,6 +650,7 @@ def run_ours(args, rank, world, local_rank):
     g.timing(False)
     buf.timing(False)
     train_timing[0] = False
+    gc.enable()
     ms = ev0.elapsed_time(ev1)
     ms_max = max_over_ranks(ms, dev)
     windows = None
@@ -683,6 +703,8 @@ def run_ours(args, rank, world, local_rank):
         seen = [-1, 0, 0]                  # last step copied, running sum of what the host read, first step
         torch.cuda.synchronize(dev)
         barrier()
+        gc.collect()
+        gc.disable()
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(main)
@@ -701,6 +723,7 @@ def run_ours(args, rank, world, local_rank):
             main.wait_event(tdones[(off + W + 2 * K - 1) % RING])
         e1.record(main)
         e1.synchronize()
+        gc.enable()
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)
         e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s",
                "h2d_bytes_per_step": cfg.batch_size * 4,
