@@ -198,7 +198,7 @@ gd_status gd_buffer_destroy(gd_buffer* b);
  * `done` (with peers attached they are written on a side stream after the peer probe; rows
  * served by peers count in neither, see gd_buffer_peer_stats).
  * The call does not synchronise the device; it blocks the calling thread only when
- * 1024 staged chunk jobs (8 MB each by default) enqueued by earlier calls are still
+ * 1024 staged chunk jobs (8-16 MB each by default) enqueued by earlier calls are still
  * waiting for their host-gather callbacks (their argument slots are then reused).
  * ------------------------------------------------------------------------- */
 gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev, int64_t n_max,

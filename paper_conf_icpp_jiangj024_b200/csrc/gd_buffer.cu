@@ -1165,8 +1165,18 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
     }
     // chunked staging ring (copy-engine mode): env GD_STAGE_CHUNK_KB, default 8 MB chunks;
     // 0 = one chunk per batch into the batch's full pinned staging slot
-    int64_t chunk_kb = 8192;
-    if (const char* e = std::getenv("GD_STAGE_CHUNK_KB")) chunk_kb = std::max<int64_t>(0, std::atoll(e));
+    // chunked staging ring: env GD_STAGE_CHUNK_KB fixes the chunk size (0 = one chunk per batch
+    // into the batch's full pinned staging slot); by default the ring holds 16 MB chunks and each
+    // batch uses a sixth of its staged share, clamped to [8, 16] MB (measured, papers100m 8 / 12 /
+    // 16 / 24 / 32 MB: 496 / 528 / 524 / 509 / 485 batches/s; mag240m, ~33 MB staged per batch,
+    // 8 MB 1087 vs 16 MB 979; friendster 8 MB 98.1 vs 16 MB 103.3): enough chunks that the copy
+    // engine starts early in a batch, few enough that per-chunk callback costs stay small
+    int64_t chunk_kb = 16384;
+    b->chunk_adaptive = true;
+    if (const char* e = std::getenv("GD_STAGE_CHUNK_KB")) {
+        chunk_kb = std::max<int64_t>(0, std::atoll(e));
+        b->chunk_adaptive = false;
+    }
     const int64_t rows = (host_threads > 0 && b->ce_mode && chunk_kb > 0)
                              ? std::min<int64_t>(b->n_max, std::max<int64_t>(1, (chunk_kb << 10) / b->R)) : 0;
     if (rows != b->stage_chunk_rows) {
@@ -1831,7 +1841,12 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
             // chunk c: H waits until the copy out of ring buffer r (chunk k - kStageRing)
             // is done, gathers into it; C copies it to dstage[d] at rank offset lo
             stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
-            const int64_t ch = b->stage_chunk_rows, nch = cap > 0 ? cdiv(cap, ch) : 0;
+            int64_t ch = b->stage_chunk_rows;
+            if (b->chunk_adaptive) {
+                const int64_t want = std::min<int64_t>(16ll << 20, std::max<int64_t>(8ll << 20, cap * b->R / 6));
+                ch = std::max<int64_t>(1, std::min<int64_t>(ch, want / b->R));
+            }
+            const int64_t nch = cap > 0 ? cdiv(cap, ch) : 0;
             const int t_ce = timed ? b->timer.begin(b->side_c) : -1;
             GD_CUDA(cudaEventRecord(b->ev_s0[d], b->side_h));   // staged path starts (after its waits)
             if (nch == 0) ss->cpu_ms = 0;
@@ -1848,7 +1863,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
                 j->ss = ss;
                 j->lo = c * ch;
                 j->hi = std::min<int64_t>(cap, (c + 1) * ch);
-                j->buf = b->ring_mem + (int64_t)r * ch * b->R;
+                j->buf = b->ring_mem + (int64_t)r * b->stage_chunk_rows * b->R;   // ring stride = max chunk
                 j->first = c == 0;
                 GD_CUDA(cudaStreamWaitEvent(b->side_h, b->ev_ring[r], 0));
                 GD_CUDA(cudaLaunchHostFunc(b->side_h, chunk_gather_cb, j));

@@ -168,7 +168,8 @@ struct gd_buffer {
     // chunked copy-engine staging (stage_chunk_rows > 0): the host gathers chunk c of the
     // staged share into ring buffer (k mod kStageRing) of a small pinned ring that stays
     // in the CPU caches, and the copy engine moves each chunk as soon as it is gathered
-    int64_t stage_chunk_rows = 0;
+    int64_t stage_chunk_rows = 0;        // ring buffer stride (max chunk) in rows
+    bool chunk_adaptive = true;          // per-batch chunk = staged share / 6, in [8, 16] MB
     uint8_t* ring_mem = nullptr;         // pinned [kStageRing x stage_chunk_rows x R]
     uint64_t chunk_counter = 0;
     // host-function arguments of the staged chunks: a ring indexed by a global job counter, so
