@@ -66,7 +66,12 @@ struct HostGatherPool::Impl {
         }
     }
 
-    int64_t pf = 8;   // prefetch distance in rows (env GD_GATHER_PF; 0 = off)
+    int64_t pf_env = -1;   // prefetch distance in rows from env GD_GATHER_PF (0 = off), else byte-based
+
+    // Prefetch distance: ~4 KB of rows ahead (8 rows of 512 B, 4 of 1 KB, 2 of 1.5 KB), so the
+    // lines in flight per thread stay within the core's fill buffers whatever the row width
+    // (a fixed 8 rows asked for 192 lines ahead with mag240m's 1536-byte rows).
+    int64_t pf_rows() const { return pf_env >= 0 ? pf_env : std::max<int64_t>(2, 4096 / std::max<int64_t>(1, R)); }
 
     const uint8_t* row_ptr(int64_t v) const { return src + (v < P ? v : v % P) * R; }
     void prefetch_row(const uint8_t* p) const {
@@ -81,6 +86,7 @@ struct HostGatherPool::Impl {
             // software prefetch `pf` rows ahead: random rows over a table far larger than
             // the caches and the TLB reach are latency-bound per thread; prefetching every
             // line of row j + pf keeps ~pf rows of misses (and their page walks) in flight
+            const int64_t pf = pf_rows();
             for (int64_t j = lo; j < hi && j < lo + pf; ++j) prefetch_row(row_ptr(rows[j]));
             for (int64_t j = lo; j < hi; ++j) {
                 if (j + pf < hi) prefetch_row(row_ptr(rows[j + pf]));
@@ -110,7 +116,7 @@ struct HostGatherPool::Impl {
 
 HostGatherPool::HostGatherPool(int threads) : impl_(new Impl) {
     // the calling (CUDA callback) thread works too, so spawn threads-1 helpers
-    if (const char* e = std::getenv("GD_GATHER_PF")) impl_->pf = std::max(0, std::atoi(e));
+    if (const char* e = std::getenv("GD_GATHER_PF")) impl_->pf_env = std::max(0, std::atoi(e));
     for (int t = 1; t < threads; ++t) impl_->workers.emplace_back([this] { impl_->loop(); });
 }
 
