@@ -261,6 +261,17 @@ def h2d_peaks(device, rank, world):
     return {"alone": alone, "concurrent": conc}
 
 
+def anon_huge_gb():
+    """AnonHugePages of /proc/meminfo in GB (transparent huge pages in use), or None."""
+    try:
+        for line in open("/proc/meminfo"):
+            if line.startswith("AnonHugePages:"):
+                return round(int(line.split()[1]) / 1e6, 2)
+    except OSError:
+        pass
+    return None
+
+
 def measured_peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -319,6 +330,15 @@ class Workload:
             self.host_indptr = self.host_indices = None
         self.indptr, self.indices = indptr, indices
         t0 = time.time()
+        if world == 1 and os.environ.get("GD_COMPACT_MEMORY", "1") == "1":
+            # the table asks for transparent huge pages: compact host memory first so the fill's
+            # page faults find free 2 MB pages (a reused box's memory may be fragmented)
+            try:
+                with open("/proc/sys/vm/compact_memory", "w") as f:
+                    f.write("1")
+            except OSError:
+                pass
+        self.thp_before = anon_huge_gb()
         self.table = HostTable(cfg.host_rows, cfg.row_bytes, cfg.name, rank, world)
         # page-lock + map once here, so FeatureBuffer re-inits (parity / preload) skip it.
         # Multi-rank: rank 0 registers (faulting the shared pages in) and fills first; the
@@ -361,6 +381,8 @@ class Workload:
                 self.table.tensor[s:e].copy_(rows)
         if self.device.type == "cuda":
             torch.cuda.synchronize(self.device)
+        self.thp_table_gb = (round(anon_huge_gb() - self.thp_before, 2)
+                             if self.thp_before is not None and anon_huge_gb() is not None else None)
         self._barrier()
         for r in range(1, self.world):
             if self.rank == r:
@@ -1049,6 +1071,8 @@ def run_ours(args, rank, world, local_rank):
         "parity": parity_out,
         "rows_check": rows_check,
         "host_link_peaks_GBps": {k: round(v, 2) for k, v in link_peaks.items()},
+        "host_table": {"GB": round(cfg.host_rows * R / 1e9, 2), "thp_requested": bool(getattr(wl.table, "thp", False)),
+                       "huge_pages_GB_after_fill": wl.thp_table_gb},
         "numa": numa,
         "windows": windows,
         "sweep": sweep or None,
