@@ -29,9 +29,14 @@ struct HostGatherPool::Impl {
     std::vector<std::thread> workers;
     std::mutex mu;
     std::condition_variable cv_work, cv_done;
-    uint64_t generation = 0;
-    int active = 0;
-    bool stop = false;
+    // generation / active / stop are atomics so that idle workers and the waiting caller can
+    // spin on them for a short while before sleeping on the condition variables: the chunks of
+    // a batch arrive back to back, and a futex wake-up of 12 helpers plus the join cost tens of
+    // microseconds per chunk (env GD_POOL_SPIN = spin iterations, 0 = sleep at once)
+    std::atomic<uint64_t> generation{0};
+    std::atomic<int> active{0};
+    std::atomic<bool> stop{false};
+    int spin = 4000;
     // current job
     const uint8_t* src = nullptr;
     const int32_t* rows = nullptr;
@@ -99,16 +104,22 @@ struct HostGatherPool::Impl {
     void loop() {
         uint64_t seen = 0;
         while (true) {
-            {
-                std::unique_lock<std::mutex> lk(mu);
-                cv_work.wait(lk, [&] { return stop || generation != seen; });
-                if (stop) return;
-                seen = generation;
+            bool got = false;
+            for (int i = 0; i < spin && !got; ++i) {
+                if (stop.load(std::memory_order_acquire)) return;
+                got = generation.load(std::memory_order_acquire) != seen;
+                if (!got) _mm_pause();
             }
+            if (!got) {
+                std::unique_lock<std::mutex> lk(mu);
+                cv_work.wait(lk, [&] { return stop.load() || generation.load() != seen; });
+                if (stop.load()) return;
+            }
+            seen = generation.load(std::memory_order_acquire);
             work();
-            {
+            if (active.fetch_sub(1, std::memory_order_acq_rel) == 1) {
                 std::lock_guard<std::mutex> lk(mu);
-                if (--active == 0) cv_done.notify_one();
+                cv_done.notify_one();
             }
         }
     }
@@ -117,13 +128,14 @@ struct HostGatherPool::Impl {
 HostGatherPool::HostGatherPool(int threads) : impl_(new Impl) {
     // the calling (CUDA callback) thread works too, so spawn threads-1 helpers
     if (const char* e = std::getenv("GD_GATHER_PF")) impl_->pf_env = std::max(0, std::atoi(e));
+    if (const char* e = std::getenv("GD_POOL_SPIN")) impl_->spin = std::max(0, std::atoi(e));
     for (int t = 1; t < threads; ++t) impl_->workers.emplace_back([this] { impl_->loop(); });
 }
 
 HostGatherPool::~HostGatherPool() {
     {
         std::lock_guard<std::mutex> lk(impl_->mu);
-        impl_->stop = true;
+        impl_->stop.store(true);
     }
     impl_->cv_work.notify_all();
     for (auto& w : impl_->workers) w.join();
@@ -147,13 +159,16 @@ double HostGatherPool::gather(const uint8_t* src, const int32_t* rows, int64_t n
             I.P = P;
             I.nt = nt;
             I.next.store(0, std::memory_order_relaxed);
-            I.active = (int)I.workers.size();
-            ++I.generation;
+            I.active.store((int)I.workers.size(), std::memory_order_relaxed);
+            I.generation.fetch_add(1, std::memory_order_release);   // publishes the job fields
         }
         I.cv_work.notify_all();
         I.work();
-        std::unique_lock<std::mutex> lk(I.mu);
-        I.cv_done.wait(lk, [&] { return I.active == 0; });
+        for (int i = 0; i < I.spin && I.active.load(std::memory_order_acquire) != 0; ++i) _mm_pause();
+        if (I.active.load(std::memory_order_acquire) != 0) {
+            std::unique_lock<std::mutex> lk(I.mu);
+            I.cv_done.wait(lk, [&] { return I.active.load() == 0; });
+        }
     }
     return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
 }
