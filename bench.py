@@ -1320,15 +1320,18 @@ def run_reference(args, rank, world, local_rank):
     W, K = args.warmup, args.steps
     PRE = 0 if cfg.preload else args.prewarm_max
     threads = len(os.sched_getaffinity(0))
-    n_all = max(W + K, threads) + PRE + 64
+    n_all = W + -(-K // threads) * threads + PRE + 64
     sched = batch_schedule(wl.num_batches, 0, 1, n_all)
     bids = [ep * wl.num_batches + b for b, ep in sched]
     seeds_host = torch.stack([wl.seeds(b, ep) for b, ep in sched]).cpu()
     # (1) multi-core CPU variant: W warm-up batches, then K timed batches over `threads` threads
     cpu_variant_baseline(cfg, wl.table.array, wl.host_indptr, wl.host_indices, seeds_host, bids, fan, 0, threads,
                          n_target=W)
+    # K timed batches, rounded up to whole rounds of the thread pool so that every thread is busy
+    # for the whole timed span (a rate over a partly idle pool would understate the host)
+    n_timed = -(-K // threads) * threads
     cv = cpu_variant_baseline(cfg, wl.table.array, wl.host_indptr, wl.host_indices, seeds_host[W:], bids[W:], fan, 0,
-                              threads, n_target=K)
+                              threads, n_target=n_timed)
     v = cv["value"]
     # (2) the full single-thread oracle from a pre-warmed buffer (the GPU arm's rule)
     keep = S * cfg.row_bytes <= 48e9
