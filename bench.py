@@ -457,7 +457,11 @@ def run_ours(args, rank, world, local_rank):
     buf = gd.FeatureBuffer(wl.table.tensor, S, Q, n_max, preload=cfg.preload, device=local_rank,
                            num_nodes=cfg.num_nodes)
     t_register = time.time() - t0
-    host_threads = max(1, min(13, len(os.sched_getaffinity(0)) // world - 3))
+    # host-gather threads: the cores this rank may use, shared with the other ranks on them (after
+    # a NUMA bind the mask is the socket's, shared by world / sockets ranks), minus ~3 for the
+    # driver, CUDA callback and clock threads
+    sharing = max(1, world // max(1, numa.get("numa_nodes", 1))) if numa.get("bound") else world
+    host_threads = max(1, min(13, len(os.sched_getaffinity(0)) // sharing - 3))
     if "GD_HOST_THREADS" not in os.environ and not cfg.preload:
         buf.config(host_threads)
     log(f"setup: graph {wl.t_graph:.1f}s table alloc {wl.t_table_alloc:.1f}s register {t_register:.1f}s "

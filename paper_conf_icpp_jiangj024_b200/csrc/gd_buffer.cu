@@ -34,7 +34,7 @@ constexpr int kBThreads = 256;
 constexpr int kBItems = 8;
 constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
-constexpr int kStageRing = 4;    // pinned chunk buffers of the copy-engine staging ring
+constexpr int kStageRingMax = 16; // pinned chunk buffers of the copy-engine staging ring (max)
 constexpr int kJobRing = 1024;   // host-function argument slots of the staged chunks
 constexpr int kTimedPairs = 5;
 constexpr double kZeroCopyCapCE = 0.15;   // adaptive zero-copy share cap with copy-engine staging   // per gd_extract: bookkeeping, gather, zero-copy, pull/scatter, CE copy
@@ -1184,9 +1184,11 @@ gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_shar
         b->ring_mem = nullptr;
         b->stage_chunk_rows = rows;
         if (rows > 0) {
-            GD_CUDA(cudaHostAlloc((void**)&b->ring_mem, (size_t)kStageRing * rows * b->R, cudaHostAllocPortable));
+            b->stage_ring = 4;
+            if (const char* e = std::getenv("GD_STAGE_RING")) b->stage_ring = std::max(2, std::min(kStageRingMax, std::atoi(e)));
+            GD_CUDA(cudaHostAlloc((void**)&b->ring_mem, (size_t)b->stage_ring * rows * b->R, cudaHostAllocPortable));
             if (b->ev_ring.empty()) {
-                b->ev_ring.assign(kStageRing, nullptr);
+                b->ev_ring.assign(kStageRingMax, nullptr);
                 for (auto& e : b->ev_ring) GD_CUDA(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
                 GD_CUDA(cudaEventCreateWithFlags(&b->ev_chunk, cudaEventDisableTiming));
             }
@@ -1838,7 +1840,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     if (staged) {
         const uint8_t* stage_dev = nullptr;
         if (ce && b->stage_chunk_rows > 0) {
-            // chunk c: H waits until the copy out of ring buffer r (chunk k - kStageRing)
+            // chunk c: H waits until the copy out of ring buffer r (chunk k - stage_ring)
             // is done, gathers into it; C copies it to dstage[d] at rank offset lo
             stage_dev = b->dstage + (int64_t)d * b->n_max * b->R;
             int64_t ch = b->stage_chunk_rows;
@@ -1851,7 +1853,7 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
             GD_CUDA(cudaEventRecord(b->ev_s0[d], b->side_h));   // staged path starts (after its waits)
             if (nch == 0) ss->cpu_ms = 0;
             for (int64_t c = 0; c < nch; ++c) {
-                const int r = (int)(b->chunk_counter++ % kStageRing);
+                const int r = (int)(b->chunk_counter++ % b->stage_ring);
                 // The callback reads its arguments when stream H reaches it, possibly many
                 // batches after this enqueue: each chunk gets its own argument slot, reused
                 // only after its previous callback ran (a host wait that needs the caller to

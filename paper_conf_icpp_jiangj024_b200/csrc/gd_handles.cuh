@@ -166,18 +166,19 @@ struct gd_buffer {
     uint8_t* dstage = nullptr;           // HBM [D][n_max x R] (copy-engine mode)
     double m_est = 0;                    // misses of a recently completed batch
     // chunked copy-engine staging (stage_chunk_rows > 0): the host gathers chunk c of the
-    // staged share into ring buffer (k mod kStageRing) of a small pinned ring that stays
+    // staged share into ring buffer (k mod stage_ring) of a small pinned ring that stays
     // in the CPU caches, and the copy engine moves each chunk as soon as it is gathered
     int64_t stage_chunk_rows = 0;        // ring buffer stride (max chunk) in rows
     bool chunk_adaptive = true;          // per-batch chunk = staged share / 6, in [8, 16] MB
-    uint8_t* ring_mem = nullptr;         // pinned [kStageRing x stage_chunk_rows x R]
+    uint8_t* ring_mem = nullptr;         // pinned [stage_ring x stage_chunk_rows x R]
+    int stage_ring = 4;                  // ring buffers (env GD_STAGE_RING)
     uint64_t chunk_counter = 0;
     // host-function arguments of the staged chunks: a ring indexed by a global job counter, so
     // a pending callback's arguments are never rewritten by a later batch's enqueue (slot k is
     // reused only after ev_job[k], recorded after its callback, has fired)
     std::vector<cudaEvent_t> ev_job;
     uint64_t job_counter = 0;
-    std::vector<cudaEvent_t> ev_ring;    // [kStageRing] copy out of ring buffer r done
+    std::vector<cudaEvent_t> ev_ring;    // [kStageRingMax] copy out of ring buffer r done
     cudaEvent_t ev_chunk = nullptr;      // chunk gathered (re-recorded per chunk)
     std::vector<struct ChunkJob> jobs;   // [kJobRing] host-function arguments (see ev_job)
     // f2: NVLink peer feature buffers (subprocesses reuse rows another has loaded).
