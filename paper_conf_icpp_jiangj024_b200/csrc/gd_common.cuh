@@ -198,13 +198,6 @@ __device__ __forceinline__ T warp_sum(T v) {
 // are processed by blocks that start in tile order (blockIdx order or a ticket), so
 // every predecessor is running or done.  `base` is added to tile 0's prefix.
 // Returns the exclusive prefix of `tile` (same value in every lane).
-// The warp inspects a window of 256 predecessors per step (8 per lane, loaded together):
-// when every tile of a grid runs at once, inclusive prefixes spread from tile 0 one window
-// per round trip, so a 32-tile window made tile 440 of a hop's relabel walk 14 round trips
-// (the kernel then ran at ~2% SM throughput); 256 takes it to 2.  A published inclusive
-// prefix at distance i implies every tile beyond it has published (it walked through them),
-// so waiting for the whole window never waits on a tile the result does not need.
-constexpr int kLookbackPerLane = 8;
 __device__ __forceinline__ long long lookback_exclusive(unsigned long long* st, long long tile,
                                                         long long agg, long long base) {
     const int lane = threadIdx.x & 31;
@@ -214,36 +207,21 @@ __device__ __forceinline__ long long lookback_exclusive(unsigned long long* st, 
     }
     if (lane == 0) st_relaxed_u64(st + tile, kFlagA | (unsigned long long)agg);
     long long excl = 0;
-    long long t0 = tile - 1;                         // window entry i = lane * 8 + k is tile t0 - i
+    long long t = tile - 1 - lane;
     while (true) {
-        unsigned long long w[kLookbackPerLane];
+        unsigned long long w;
         int spins = 0;
         while (true) {
-            bool ready = true;
-#pragma unroll
-            for (int k = 0; k < kLookbackPerLane; ++k) {
-                const long long t = t0 - (long long)(lane * kLookbackPerLane + k);
-                w[k] = (t >= 0) ? ld_relaxed_u64(st + t) : kFlagP;
-                ready &= (w[k] >> 62) != 0;
-            }
-            if (__all_sync(0xffffffffu, ready)) break;
+            w = (t >= 0) ? ld_relaxed_u64(st + t) : kFlagP;
+            if (__all_sync(0xffffffffu, (w >> 62) != 0)) break;
             if (++spins > 8) __nanosleep(64);
         }
-        int kp = kLookbackPerLane;                   // first inclusive prefix among my entries
-#pragma unroll
-        for (int k = kLookbackPerLane - 1; k >= 0; --k)
-            if ((w[k] >> 62) == 2) kp = k;
-        const unsigned pmask = __ballot_sync(0xffffffffu, kp < kLookbackPerLane);
-        const int first_lane = pmask ? (__ffs(pmask) - 1) : 32;
-        const int first_k = __shfl_sync(0xffffffffu, kp, pmask ? first_lane : 0);
-        const int g = pmask ? first_lane * kLookbackPerLane + first_k : 32 * kLookbackPerLane;   // inclusive bound
-        long long v = 0;
-#pragma unroll
-        for (int k = 0; k < kLookbackPerLane; ++k)
-            if (lane * kLookbackPerLane + k <= g) v += (long long)(w[k] & kValMask);
+        const unsigned pmask = __ballot_sync(0xffffffffu, (w >> 62) == 2);
+        const int first_p = pmask ? (__ffs(pmask) - 1) : 32;
+        long long v = (lane <= first_p) ? (long long)(w & kValMask) : 0;
         excl += warp_sum(v);
         if (pmask) break;
-        t0 -= 32 * kLookbackPerLane;
+        t -= 32;
     }
     if (lane == 0) st_relaxed_u64(st + tile, kFlagP | (unsigned long long)(excl + agg));
     return excl;
