@@ -736,8 +736,13 @@ def run_ours(args, rank, world, local_rank):
         e0.record(main)
         samplers_after(e0)
         j_end = off + W + 2 * K
+        e2e_win = []
         for j in range(off + W + K, j_end):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats, h_ev, seen))
+            if args.window and (j - off - W - K + 1) % args.window == 0:
+                e_ = torch.cuda.Event(enable_timing=True)
+                e_.record(main)
+                e2e_win.append(e_)
         for j in range(max(off + W + K, j_end - LAG), j_end):   # the last LAG results, inside the timed region
             k = j % LAG
             h_ev[k].synchronize()
@@ -751,7 +756,11 @@ def run_ours(args, rank, world, local_rank):
         e1.synchronize()
         gc.enable()
         e2e_ms = max_over_ranks(e0.elapsed_time(e1), dev)
-        e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s",
+        e2e_windows = None
+        if e2e_win:
+            marks = [e0] + e2e_win
+            e2e_windows = [round(args.window / (a_.elapsed_time(b_) / 1e3), 1) for a_, b_ in zip(marks, marks[1:])]
+        e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s", "windows": e2e_windows,
                "h2d_bytes_per_step": cfg.batch_size * 4,
                "d2h_bytes_per_step": (2 * len(fan) + 1) * 8 + 32,
                "read_back": f"each step's sizes + hit/miss stats copied D2H into pinned memory on the stream and "
