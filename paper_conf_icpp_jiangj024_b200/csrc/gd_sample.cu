@@ -410,14 +410,40 @@ struct ColResolveArgs {
     const uint32_t* hvals;
 };
 
+// One flat pass over the concatenated edges of all hops (hop boundaries from the device sizes),
+// 4 edges per thread in flight: each edge is a dependent pair of loads (col, then the hash
+// value it names), so the loads of 4 edges are issued before any result is stored.  (A 2-D
+// grid with one row of blocks per hop left most blocks of the small hops idle: 18.5 us warm.)
+constexpr int kResolveItems = 4;
 __global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
     GD_PDL_ENTRY();
-    const int hop = blockIdx.y;
-    const int64_t e_h = a.sizes[a.K + 1 + hop];
-    int32_t* col = a.col[hop];
-    for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < e_h;
-         e += (int64_t)gridDim.x * blockDim.x)
-        col[e] = (int32_t)__ldg(a.hvals + col[e]);
+    int64_t cum[GD_MAX_HOPS + 1];
+    cum[0] = 0;
+    for (int h = 0; h < a.K; ++h) cum[h + 1] = cum[h] + a.sizes[a.K + 1 + h];
+    const int64_t total = cum[a.K];
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; base < total; base += stride * kResolveItems) {
+        int32_t* ptr[kResolveItems];
+        uint32_t slot[kResolveItems];
+#pragma unroll
+        for (int u = 0; u < kResolveItems; ++u) {
+            const int64_t e = base + (int64_t)u * stride;
+            ptr[u] = nullptr;
+            if (e < total) {
+                int h = 0;
+                while (e >= cum[h + 1]) ++h;
+                ptr[u] = a.col[h] + (e - cum[h]);
+                slot[u] = (uint32_t)*ptr[u];
+            }
+        }
+        uint32_t v[kResolveItems];
+#pragma unroll
+        for (int u = 0; u < kResolveItems; ++u)
+            if (ptr[u]) v[u] = __ldg(a.hvals + slot[u]);
+#pragma unroll
+        for (int u = 0; u < kResolveItems; ++u)
+            if (ptr[u]) *ptr[u] = (int32_t)v[u];
+    }
 }
 
 // Empties exactly the hash slots this call used: every claimed key is a node of n_id (a seed
@@ -694,16 +720,13 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         w.scan.flip();
     }
     ColResolveArgs c;
-    int64_t emax_all = 1;
-    for (int h = 0; h < num_hops; ++h) {
-        c.col[h] = out->col[h];
-        emax_all = std::max(emax_all, emax[h]);
-    }
+    for (int h = 0; h < num_hops; ++h) c.col[h] = out->col[h];
     c.sizes = out->sizes;
     c.K = num_hops;
     c.hvals = hv;
-    dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(emax_all, kThreads))),
-              (unsigned)num_hops);
+    int64_t esum = 0;
+    for (int h = 0; h < num_hops; ++h) esum += emax[h];
+    dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(esum, kThreads * kResolveItems))));
     GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
     GD_CUDA(launch_chain(k_hash_clear, dim3((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(nmax[num_hops], kThreads)))),
                          dim3(kThreads), 0, st, (const int32_t*)w.slot_of, (const int64_t*)(out->sizes + num_hops), hk, hv));
