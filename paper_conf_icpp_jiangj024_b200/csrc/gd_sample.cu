@@ -27,8 +27,9 @@ namespace gd {
 
 constexpr int kThreads = 256;
 constexpr int kWarps = kThreads / 32;
-constexpr int kRelabelItems = 8;
-constexpr int kEdgesPerTile = kThreads * kRelabelItems;   // 2048 edges per relabel block
+constexpr int kRelabelItems = 16;
+constexpr int kEdgesPerTile = kThreads * kRelabelItems;   // 4096 edges per relabel block
+static_assert((kRelabelItems * kWarps) % 32 == 0, "relabel scan layout");
 constexpr int kMaxFanSmem = GD_MAX_FANOUT;
 
 struct SampleHopArgs {
@@ -373,14 +374,25 @@ __global__ void __launch_bounds__(kThreads) k_relabel_hop(RelabelArgs a) {
     }
     __syncthreads();
     if (warp == 0) {
-        // exclusive scan over the 64 (round, warp) counts in edge order
-        const int c0 = s_cnt[2 * lane], c1 = s_cnt[2 * lane + 1];
-        const int inc = warp_inclusive_sum(c0 + c1);
-        const int ex = inc - c0 - c1;
+        // exclusive scan over the kRelabelItems x kWarps (round, warp) counts in edge order,
+        // kPer consecutive counts per lane
+        constexpr int kPer = kRelabelItems * kWarps / 32;
+        int c[kPer];
+        int sum = 0;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            c[q] = s_cnt[kPer * lane + q];
+            sum += c[q];
+        }
+        const int inc = warp_inclusive_sum(sum);
         const int agg = __shfl_sync(0xffffffffu, inc, 31);
         __syncwarp();
-        s_cnt[2 * lane] = ex;
-        s_cnt[2 * lane + 1] = ex + c0;
+        int run = inc - sum;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            s_cnt[kPer * lane + q] = run;
+            run += c[q];
+        }
         const long long base = lookback_exclusive(a.st, tile, agg, 0);
         if (lane == 0) {
             s_base = base;
