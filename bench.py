@@ -1069,7 +1069,7 @@ def run_ours(args, rank, world, local_rank):
         # [+ zero-copy miss copy unless preload] [+ staged scatter when the host path is on] [+ peer-tag
         # publish with peers attached: not in the timed region] | compact, release [| train: L x (agg, FWD GEMM,
         # DW GEMM, 2 colsum) + xent + loss + (L-1) x (DA GEMM, scatter init, scatter, relu') + SGD + L bf16 casts]
-        "gpu_launches": K * ((2 * len(fan) + 3) + 3 + (0 if cfg.preload else 1) + (2 if args.peer and world > 1 else 0)
+        "gpu_launches": K * ((2 * len(fan) + 3) + 3 + (0 if cfg.preload else 1) + (3 if args.peer and world > 1 else 0)
                              + (1 if (miss_staged > 0 or tb["miss_staged_ms"] > 1e-3) and not cfg.preload else 0) + 2
                              + (0 if model is None else 5 * model.L + 2 + 4 * (model.L - 1) + 1 + model.L)),
         "roofline": dominant,
