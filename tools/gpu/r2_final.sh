@@ -18,3 +18,7 @@ for T in memcheck racecheck synccheck; do
   GD_HOST_THREADS=2 timeout 1200 compute-sanitizer --tool $T --kernel-name regex=k_ python -m pytest tests/test_gpu_parity.py -m gpu -q \
       -k "gather_variants and 512 or tiny_evict or figure6" > gpurun_out/final/san_$T.log 2>&1; echo "san $T rc=$?"; tail -3 gpurun_out/final/san_$T.log
 done
+A="--steps 100 --warmup 8 --no-cpu-baseline --parity-batches 0 --no-replay --no-e2e"
+for C in papers100m products mag240m; do
+  timeout 900 python bench.py --config $C $A --timeline gpurun_out/final/r02_${C}_timeline.md > /dev/null 2>&1; echo "timeline $C rc=$?"
+done
