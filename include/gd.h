@@ -226,8 +226,12 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
  *                    that run sampling / bookkeeping / the hit gather.
  * Default at init: host_threads = min(13, cores - 3) (0 with preload),
  * adaptive share; env GD_HOST_THREADS / GD_ZERO_COPY_SHARE / GD_ZC_BLOCKS /
- * GD_PULL_BLOCKS override.  Synchronises the buffer's
- * internal streams; call between batches.
+ * GD_PULL_BLOCKS override.  Further knobs, read here: GD_STAGE_CHUNK_KB (fixed staging chunk;
+ * default a sixth of the batch's staged share in [8, 16] MB), GD_STAGE_RING (pinned chunk
+ * buffers, default 4), GD_POOL_SPIN (host-gather pool spin before sleeping), GD_GATHER_PF
+ * (host prefetch distance in rows), GD_SHARE_TUNER=1 (see gd_buffer_policy_read); at init:
+ * GD_GATHER_DYNAMIC / GD_GATHER_PRIORITY / GD_GATHER_TMA (hit-gather variants).  Synchronises
+ * the buffer's internal streams; call between batches.
  * ------------------------------------------------------------------------- */
 gd_status gd_buffer_config(gd_buffer* b, int host_threads, double zero_copy_share, int zc_blocks,
                            int pull_blocks);
