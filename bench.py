@@ -192,12 +192,15 @@ class ClockSampler:
     def _run(self):
         if self._N is None:
             return
+        period = float(os.environ.get("GD_CLOCK_PERIOD_S", "0.2"))
         while not self._stop.is_set():
             try:
                 self._query()
             except Exception:  # noqa: BLE001
                 pass
-            self._stop.wait(0.2)
+            if period <= 0:
+                break
+            self._stop.wait(period)
 
     def __enter__(self):
         self._stop.clear()
