@@ -1391,6 +1391,7 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable) {
     if (enable) {
         for (cudaStream_t s : {b->side, b->side_h, b->side_p, b->side_j, b->side_g, b->side_c}) GD_CUDA(cudaStreamSynchronize(s));
         b->timer.reset();
+        b->timer.reserve(kTimedPairs * 4096);   // events for 4096 batches, created before the timed region
         b->timer_host_ms = 0;
     }
     b->timer.on = enable != 0;

@@ -104,6 +104,17 @@ struct EventTimer {
         return pool[used++];
     }
     void reset() { used = 0; pairs.clear(); }
+    // Create the events of `n` more pairs now, outside the timed region: creating them on demand
+    // inside it put ~12 cudaEventCreate calls per batch on the caller's thread, which contend for
+    // the driver with the staged path's host-function callbacks (200-step papers100m: the device-
+    // timed region ran 15-25% below the untimed e2e region on the same box).
+    void reserve(int n_pairs) {
+        while ((int)pool.size() < used + 2 * n_pairs) {
+            cudaEvent_t e;
+            if (cudaEventCreate(&e) != cudaSuccess) break;
+            pool.push_back(e);
+        }
+    }
     // record the start of a group on `s`; returns the pair slot
     int begin(cudaStream_t s) {
         const int a = used;

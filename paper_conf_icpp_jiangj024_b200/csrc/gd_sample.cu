@@ -751,7 +751,10 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
 gd_status gd_graph_timing(gd_graph* g, int enable) {
     if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_graph_timing: bad handle");
     DeviceGuard guard(g->hdr.device);
-    if (enable) g->timer.reset();
+    if (enable) {
+        g->timer.reset();
+        g->timer.reserve(4096);      // events for 4096 calls, created before the timed region
+    }
     g->timer.on = enable != 0;
     return GD_OK;
 }
