@@ -653,8 +653,9 @@ def run_ours(args, rank, world, local_rank):
     gc.disable()                                  # no collector pause in the host loop of the region
     torch.cuda.synchronize(dev)
     log("timed region ...")
-    g.timing(True)
-    buf.timing(True)
+    KT = os.environ.get("GD_KERNEL_TIMING", "1") == "1"   # per-kernel event pairs in the timed region
+    g.timing(KT)
+    buf.timing(KT)
     train_timing[0] = True
     ev0 = torch.cuda.Event(enable_timing=True)
     ev1 = torch.cuda.Event(enable_timing=True)
