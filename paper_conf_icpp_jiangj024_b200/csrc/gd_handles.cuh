@@ -75,6 +75,7 @@ struct StagedSlot {
     double cpu_ms = 0;            // duration of the last host gather into this slot
     int64_t batch = -1;           // batch that last used this slot
     uint64_t epoch = 0;           // that batch's epoch (its published miss-count word carries it)
+    bool zc_timed = false;        // its zero-copy kernel was bracketed by ev_z0 / ev_z1
 };
 
 // Hill-climbing tuner of the zero-copy share: the cost of a share is the
@@ -142,9 +143,8 @@ struct gd_buffer {
     std::vector<cudaEvent_t> ev_trip;    // [D] every stream finished with trip ring slot d
     std::vector<cudaEvent_t> ev_E, ev_P; // [D] staging slot d ready in HBM or pinned / staged pull done
     std::vector<cudaEvent_t> ev_H;       // [D] host gather of slot d done (copy-engine mode)
-    std::vector<cudaEvent_t> ev_s0;      // [D] staged path of slot d started (chunked mode, timing)
     cudaStream_t side_c = nullptr;       // C: copy-engine H2D of the staged share
-    std::vector<cudaEvent_t> ev_z0, ev_z1, ev_p0, ev_p1;   // [D] timing of the two miss paths
+    std::vector<cudaEvent_t> ev_z0, ev_z1;   // [D] timing of the zero-copy path (every 8th batch)
     int64_t* trip_split = nullptr;       // [D] K0: misses [0, K0) zero-copy, [K0, M) staged
     int host_threads = 0;                // 0: staged path off (all misses zero-copy)
     int zc_blocks = 16;                  // 1024-thread blocks (~whole SMs) of the zero-copy copy
