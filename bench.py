@@ -57,6 +57,8 @@ def parse():
     p.add_argument("--lr", type=float, default=0.01, help="f4 SGD learning rate")
     p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
                    "peer (CUDA IPC); misses are served from peers' HBM before the host link")
+    p.add_argument("--sample-ahead", type=int, default=3,
+                   help="batches sampled ahead of extraction (per-batch buffer ring = Q + 1 + this)")
     p.add_argument("--samplers", type=int, default=2,
                    help="sampler streams (P:94 'a pool of threads as samplers'), each with its own gd_workspace: "
                         "batch j is sampled on stream j mod S, so the next batch's sampling overlaps this batch's "
@@ -482,7 +484,11 @@ def run_ours(args, rank, world, local_rank):
     seeds_host = seeds_dev.cpu().pin_memory()
     batch_ids = [ep * wl.num_batches + b for b, ep in sched]
 
-    RING = Q + 1   # per-batch buffers in flight: Q unreleased batches + the one being sampled
+    # per-batch buffers in flight: Q unreleased batches + the one being extracted + `--sample-ahead`
+    # batches sampled ahead of extraction (the sampler -> extractor queue: sampling of batch j
+    # waits for the release of batch j - RING, issued after extract(j - RING + Q); with RING = Q + 1
+    # that chained every sampling to the previous batch's bookkeeping)
+    RING = Q + 1 + max(0, args.sample_ahead)
     outs = [g.alloc_out(cfg.batch_size, fan) for _ in range(RING)]
     feats = [buf.alloc_out(n_max) for _ in range(RING)]
     aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(RING)]
@@ -1098,7 +1104,7 @@ def run_ours(args, rank, world, local_rank):
         "value": round(value, 2), "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
         "ms_per_step": round(ms_max / K, 4), "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-        "config": config_dict(cfg, S, world, prewarm_batches, NS),
+        "config": config_dict(cfg, S, world, prewarm_batches, NS, RING),
         "e2e": e2e,
         # per step: seed intake + K x (sample, relabel) + col resolve + hash clear | lookup, pop/assign, hit gather
         # [+ zero-copy miss copy unless preload] [+ staged scatter when the host path is on] [+ peer-tag
@@ -1333,7 +1339,7 @@ def host_cpu_info():
     return info
 
 
-def config_dict(cfg, S, world, prewarm, samplers):
+def config_dict(cfg, S, world, prewarm, samplers, ring):
     """The `config` object of the JSON line; identical for both arms."""
     R = cfg.row_bytes
     return {"workload": cfg.name, "num_nodes": cfg.num_nodes, "num_edges": cfg.num_edges,
@@ -1341,6 +1347,7 @@ def config_dict(cfg, S, world, prewarm, samplers):
             "buffer_slots": S, "buffer_frac": round(S / cfg.num_nodes, 4), "release_lag": Q,
             "buffer_prewarm_batches": prewarm,
             "parallelism": f"dp{world} (batch segments, no collective)", "sampler_streams": samplers,
+            "batches_in_flight": ring,
             "l2": "inputs larger than L2 (topology %.1f GB, slots %.1f GB, host table %.1f GB)" % (
                 (cfg.num_nodes + 1) * 8e-9 + cfg.num_edges * 4e-9, S * R * 1e-9, cfg.host_rows * R * 1e-9),
             "host_table_rows": cfg.host_rows}
@@ -1418,7 +1425,7 @@ def run_reference(args, rank, world, local_rank):
             "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": round(1e3 / v, 3) if v else None, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-            "config": config_dict(cfg, S, world, jp, max(1, args.samplers)),
+            "config": config_dict(cfg, S, world, jp, max(1, args.samplers), Q + 1 + max(0, args.sample_ahead)),
             "cpu_baseline": cv, "single_thread_full_oracle": single, "host_cpu": host_cpu_info(),
             "e2e": {"value": v, "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
             "native_libs_loaded": loaded_native_libs()}

@@ -410,6 +410,15 @@ gd_status gd_buffer_timing(gd_buffer* b, int enable);
  *          (phase 1, summed), current zero-copy share, copy-engine H2D of the staged
  *          share (copy-engine mode; 0 otherwise)}. */
 gd_status gd_buffer_timing_read(gd_buffer* b, double* ms, int64_t* batches);
+/* Sampler variant of the hops with 1 <= f <= 32 (test / A-B surface, readings R4-R5
+ * in DESIGN.md): padded = 1 (default; GD_SAMPLE_PAD=0 in the environment at gd_graph_create turns
+ * it off) draws each frontier node's neighbours into a padded [n_{h-1} x f] layout with no scan
+ * (k_sample_pad), then one pass with one decoupled look-back over (edges, new nodes) writes rowptr,
+ * the compacted col / eid and the new nodes (k_relabel_pad); padded = 0 scans the counts inside
+ * the sampling kernel (k_sample_hop + k_relabel_hop).  Outputs are identical (bit for bit) either
+ * way; hops with f = -1 or f > 32 always take the second form.  Host-only, not stream-ordered:
+ * call it between gd_sample calls.  GD_ERR_INVALID on a bad handle. */
+gd_status gd_graph_sampler(gd_graph* g, int padded);
 gd_status gd_graph_timing(gd_graph* g, int enable);
 gd_status gd_graph_timing_read(gd_graph* g, double* sample_ms, int64_t* calls);
 

@@ -159,6 +159,10 @@ class Graph:
     def check(self):
         return check_device_status(self._h)
 
+    def sampler(self, padded: bool):
+        """gd_graph_sampler: padded hops (default) or count-scan hops; identical outputs."""
+        check(lib.gd_graph_sampler(self._h, int(padded)))
+
     def timing(self, enable: bool):
         check(lib.gd_graph_timing(self._h, int(enable)))
 

@@ -21,7 +21,7 @@ DEV_BITS = {0x1: "GD_DEV_BAD_ID", 0x2: "GD_DEV_DUP_SEED", 0x4: "GD_DEV_UNDERFLOW
 EXPORTS = ["gd_last_error", "gd_version", "gd_graph_create", "gd_graph_destroy", "gd_sample_bounds", "gd_sample",
            "gd_buffer_init", "gd_buffer_destroy", "gd_extract", "gd_buffer_release", "gd_check_device_status",
            "gd_buffer_snapshot", "gd_buffer_set_state", "gd_buffer_side_stream", "gd_buffer_timing",
-           "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_buffer_config", "gd_buffer_stage_mode",
+           "gd_buffer_timing_read", "gd_graph_timing", "gd_graph_timing_read", "gd_graph_sampler", "gd_buffer_config", "gd_buffer_stage_mode",
            "gd_buffer_peer_attach", "gd_buffer_peer_export_ipc", "gd_buffer_peer_attach_ipc", "gd_buffer_peer_stats",
            "gd_sage_create", "gd_sage_destroy", "gd_sage_step", "gd_sage_grads", "gd_sage_apply_sgd", "gd_sage_get",
            "gd_workspace_create", "gd_workspace_destroy", "gd_sample_ws", "gd_buffer_init_mod", "gd_debug_umma_gemm",
@@ -95,6 +95,7 @@ def _load():
     L.gd_debug_umma_gemm.argtypes = [_i32, _vp, _i64, _vp, _i64, _vp, _i64, _i32, _i32, _vp, _vp, _i64, _i64, _i32,
                                      _i32, _i32, _i32, _vp]
     L.gd_graph_timing.argtypes = [_vp, ctypes.c_int]
+    L.gd_graph_sampler.argtypes = [_vp, ctypes.c_int]
     L.gd_graph_timing_read.argtypes = [_vp, _dp, ctypes.POINTER(_i64)]
     for name in EXPORTS:
         if name not in ("gd_last_error", "gd_version", "gd_buffer_side_stream"):

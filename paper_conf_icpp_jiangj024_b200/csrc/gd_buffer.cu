@@ -94,17 +94,31 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
     const int t = threadIdx.x, lane = t & 31;
     unsigned ball[kBItems];
     int32_t alv[kBItems];
+    // all loads of the thread's items first (ids, then their map entries), stores after: the
+    // stores to map / pos_of_slot / alias could alias `ids` for the compiler, which otherwise
+    // serialises the items' dependent round trips (node ids are distinct within a batch, so no
+    // item reads an entry another item writes)
+    int32_t vv[kBItems];
+    int2 mm[kBItems];
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k) {
+        const int64_t i = i0 + (int64_t)k * kBThreads + t;
+        vv[k] = (i < n) ? __ldg(a.ids + i) : -1;
+    }
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k)
+        mm[k] = (vv[k] >= 0 && (int64_t)vv[k] < a.N) ? a.map[vv[k]] : make_int2(-1, 0);
 #pragma unroll
     for (int k = 0; k < kBItems; ++k) {
         const int64_t i = i0 + (int64_t)k * kBThreads + t;
         bool miss = false;
         int32_t al = -1;
         if (i < n) {
-            const int32_t v = a.ids[i];
+            const int32_t v = vv[k];
             if (v < 0 || (int64_t)v >= a.N) {
                 atomicOr(a.status, GD_DEV_BAD_ID);
             } else {
-                const int2 m = a.map[v];
+                const int2 m = mm[k];
                 const int valid = m.y & 1;
                 const int rc = m.y >> 1;
                 if (valid) {                                   // Alg. 1 lines 8-13
@@ -768,17 +782,27 @@ __global__ void __launch_bounds__(kBThreads) k_release(ReleaseArgs a) {
     const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
     unsigned ball[kBItems];
     int32_t slot[kBItems];
+    int32_t vv[kBItems];
+    int2 mm[kBItems];
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k) {   // loads first (as in k_lookup)
+        const int64_t i = i0 + (int64_t)k * kBThreads + t;
+        vv[k] = (i < n) ? __ldg(a.ids + i) : -1;
+    }
+#pragma unroll
+    for (int k = 0; k < kBItems; ++k)
+        mm[k] = (vv[k] >= 0 && (int64_t)vv[k] < a.N) ? a.map[vv[k]] : make_int2(-1, 0);
 #pragma unroll
     for (int k = 0; k < kBItems; ++k) {
         const int64_t i = i0 + (int64_t)k * kBThreads + t;
         bool zero = false;
         slot[k] = -1;
         if (i < n) {
-            const int32_t v = a.ids[i];
+            const int32_t v = vv[k];
             if (v < 0 || (int64_t)v >= a.N) {
                 atomicOr(a.status, GD_DEV_BAD_ID);
             } else {
-                const int2 m = a.map[v];
+                const int2 m = mm[k];
                 const int rc = m.y >> 1;
                 if (rc <= 0) {
                     atomicOr(a.status, GD_DEV_UNDERFLOW);
@@ -1081,6 +1105,8 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
             return fail(cuda_error(cudaGetLastError(), "gd_buffer_init: stream"));
         const char* d = std::getenv("GD_GATHER_DYNAMIC");
         b->gather_dynamic = !(d && d[0] == '0');
+        if (const char* e2 = std::getenv("GD_GATHER_BPS")) b->gather_bps = std::max(1, std::min(8, std::atoi(e2)));
+        if (const char* e2 = std::getenv("GD_GATHER_U")) b->gather_u = std::atoi(e2) == 8 ? 8 : 4;
         // GD_GATHER_TMA=1: the TMA gather4 variant of a8 (rows <= 2048 B, multiples of 16)
         const char* t = std::getenv("GD_GATHER_TMA");
         if (t && t[0] == '1' && make_slot_map(&b->slot_map, b->slots, capacity_slots, row_bytes)) {
@@ -1808,12 +1834,14 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
         const int per_sm = (int)std::max<int64_t>(1, std::min<int64_t>(16, (200 << 10) / (smem + 256)));
         k_gather_tma<4><<<148 * per_sm, 32, smem, b->side_g>>>(b->slot_map, hlist, hcnt, (uint8_t*)out, b->R, stride,
                                                                  b->tickets + 4);
-    } else if (b->R % 16 == 0 && b->R <= 512)
-        k_gather_rows<4, 1><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
+    } else if (b->R % 16 == 0 && b->R <= 512 && b->gather_u == 8)
+        k_gather_rows<8, 1><<<148 * b->gather_bps, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
+    else if (b->R % 16 == 0 && b->R <= 512)
+        k_gather_rows<4, 1><<<148 * b->gather_bps, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0 && b->R <= 1024)
-        k_gather_rows<4, 2><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
+        k_gather_rows<4, 2><<<148 * b->gather_bps, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0 && b->R <= 2048)
-        k_gather_rows<2, 4><<<148 * 4, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
+        k_gather_rows<2, 4><<<148 * b->gather_bps, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R, gctr);
     else if (b->R % 16 == 0)
         k_gather_hits<4><<<148 * 8, 256, 0, b->side_g>>>(hlist, hcnt, b->slots, (uint8_t*)out, b->R);
     else

@@ -21,7 +21,12 @@ struct gd_workspace {
     int64_t slot_cap = 0;
     int32_t* seeds_ws = nullptr;    // staging for host seed arrays
     int64_t seeds_cap = 0;
+    int32_t* pslot = nullptr;       // padded hop: [pcap] hash slot of draw q = i f + r
+    int64_t* ppos = nullptr;        // padded hop: [ppos_cap] CSR position of draw q (eid requested)
+    int32_t* pcnt = nullptr;        // padded hop: [pcnt_cap] min(f, deg) of frontier node i
+    int64_t pcap = 0, ppos_cap = 0, pcnt_cap = 0;
     gd::ScanState scan;
+    void release_padded();
 };
 
 // Topology replica + its default workspace.
@@ -31,6 +36,7 @@ struct gd_graph {
     int64_t* indptr = nullptr;      // HBM int64[N+1]
     int32_t* indices = nullptr;     // HBM int32[E]
     gd_workspace ws;                // used by gd_sample
+    int sample_padded = 1;          // padded hops for 1 <= f <= 32 (GD_SAMPLE_PAD=0 / gd_graph_sampler)
     gd::EventTimer timer;           // one pair per gd_sample call
 };
 
@@ -130,6 +136,8 @@ struct gd_buffer {
     unsigned long long* tickets = nullptr;   // [6] {ticket, finished} x 3 kernels (pop, compact, gather)
     bool gather_dynamic = true;          // hit gather: dynamic row assignment (GD_GATHER_DYNAMIC)
     bool gather_tma = false;             // hit gather by TMA gather4 (GD_GATHER_TMA=1)
+    int gather_bps = 4;                  // hit gather: 256-thread blocks per SM (GD_GATHER_BPS)
+    int gather_u = 4;                    // hit gather, rows <= 512 B: rows in flight per warp (GD_GATHER_U: 4 | 8)
     CUtensorMap slot_map;                // tensor map over the slots for the TMA gather
     unsigned long long* done_word = nullptr; // [1] epoch-tagged early-exit word of the pop scan
     gd::ScanState scan;

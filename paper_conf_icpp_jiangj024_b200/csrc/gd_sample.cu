@@ -331,6 +331,223 @@ static void launch_sample_hop(const SampleHopArgs& a, int64_t n_frontier_max, cu
     }
 }
 
+// ---------------------------------------------------------------- padded hop (default, 1 <= f <= 32)
+// The hop is split where its only grid-wide dependency lies.  k_sample_pad draws every frontier
+// node's neighbours into a padded layout (node i's draw of rank r at q = i f + r) with no scan:
+// first occurrence over (frontier index, ascending position) is first occurrence over q, so the
+// hash tag kPending | q decides it exactly as the flat position did (reading R5).  k_relabel_pad
+// then makes one pass over the padded positions and one decoupled look-back over the pair
+// (edges, new nodes): it writes rowptr, the compacted col / eid, and the new nodes' local ids.
+// Compared with k_sample_hop + k_relabel_hop, the look-back chain of the sampling kernel (one
+// tile per 64-256 frontier nodes: the longest dependency chain of the hop) is gone, and the
+// relabel tiles cover ~2048 padded positions each.
+struct PadHopArgs {
+    const int64_t* indptr;
+    const int32_t* indices;
+    int64_t N;
+    const int32_t* n_id;
+    const int64_t* sizes;
+    int hop;          // 1-based
+    int fanout;       // 1..32
+    uint32_t batch;
+    uint64_t seed;
+    int32_t* pslot;   // [n_{h-1} f] hash slot of the draw at q
+    int64_t* ppos;    // [n_{h-1} f] CSR position (eid) of the draw at q, or null
+    int32_t* pcnt;    // [n_{h-1}] min(f, deg)
+    uint32_t* hkeys;
+    uint32_t* hvals;
+    uint32_t mask;
+};
+
+template <int G>
+__global__ void __launch_bounds__(kThreads) k_sample_pad(PadHopArgs a) {
+    GD_PDL_ENTRY();
+    const int64_t n_prev = a.sizes[a.hop - 1];
+    const int lane = threadIdx.x & 31;
+    const int64_t gt = (int64_t)blockIdx.x * kThreads + threadIdx.x;
+    if ((gt - lane) / G >= n_prev) return;      // the whole warp is past the frontier (warp-uniform)
+    const int64_t i = gt / G;
+    const int gl = lane & (G - 1);
+    const int gbase = lane & ~(G - 1);
+    const unsigned gmask = ((G == 32) ? 0xffffffffu : ((1u << G) - 1u)) << gbase;
+    const int f = a.fanout;
+    const bool active = i < n_prev;
+    int64_t d = 0, start = 0;
+    uint32_t v = 0;
+    if (active) {
+        v = (uint32_t)a.n_id[i];
+        if ((int32_t)v >= 0 && (int64_t)v < a.N) {
+            start = a.indptr[v];
+            d = a.indptr[v + 1] - start;
+        }
+        if (gl == 0) a.pcnt[i] = (int32_t)(d < f ? d : f);
+    }
+    const bool fl = active && d > f;           // Floyd; otherwise the row verbatim
+    int64_t sel = INT64_MAX;
+    if (fl) {
+        if (gl < f) sel = (int64_t)draw_uniform((uint32_t)gl, v, (uint32_t)(a.hop - 1), a.batch, a.seed, (uint64_t)(d - f + gl));
+    } else if (active && gl < d) {
+        sel = gl;
+    }
+    for (int s = 1; s < f; ++s) {
+        const int64_t rs = __shfl_sync(0xffffffffu, sel, gbase + s);
+        const unsigned bl = __ballot_sync(0xffffffffu, fl && gl < s && sel == rs);
+        if (fl && gl == s && (bl & gmask)) sel = d - f + s;
+    }
+    int rank = gl;
+    if (f > 1) {
+        int r = 0;
+        for (int s = 0; s < f; ++s) {
+            const int64_t o = __shfl_sync(0xffffffffu, sel, gbase + s);
+            r += (o < sel);
+        }
+        if (fl) rank = r;
+    }
+    if (sel != INT64_MAX) {
+        const uint32_t q = (uint32_t)(i * f + rank);
+        const uint32_t u = (uint32_t)__ldg(a.indices + start + sel);
+        a.pslot[q] = (int32_t)hash_insert(a.hkeys, a.hvals, a.mask, u, q);
+        if (a.ppos) a.ppos[q] = start + sel;
+    }
+}
+
+struct PadRelabelArgs {
+    const int32_t* pslot;
+    const int64_t* ppos;
+    const int32_t* pcnt;
+    int64_t* rowptr;
+    int32_t* col;
+    int64_t* eid;
+    int32_t* n_id;
+    int64_t* sizes;
+    int hop;
+    int K;
+    int fanout;
+    int nt;           // frontier nodes per tile (nt f <= kEdgesPerTile)
+    uint32_t* hkeys;
+    uint32_t* hvals;
+    int32_t* slot_of;
+    unsigned long long* st;
+    unsigned long long* st_clear;
+    int64_t st_clear_n;
+};
+
+constexpr unsigned long long kPairShift = 31;   // look-back value = edges << 31 | new nodes
+
+__global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
+    GD_PDL_ENTRY();
+    clear_tile_state(a.st_clear, a.st_clear_n);
+    const int64_t n_prev = a.sizes[a.hop - 1];
+    const int64_t tile = blockIdx.x;
+    const int64_t i0 = tile * a.nt;
+    if (i0 >= n_prev && tile != 0) return;
+    const uint32_t f = (uint32_t)a.fanout;
+    const uint32_t q0 = (uint32_t)(i0 * f);
+    const uint32_t qend = (uint32_t)((i0 + a.nt < n_prev ? i0 + a.nt : n_prev) * f);
+
+    __shared__ uint32_t s_cnt[kRelabelItems * kWarps];   // (valid << 16 | new) per (round, warp)
+    __shared__ unsigned long long s_base;
+    const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
+
+    uint32_t slot[kRelabelItems];
+    bool valid[kRelabelItems];
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
+        valid[k] = false;
+        slot[k] = 0;
+        if (q < qend) {
+            const uint32_t i = q / f;
+            if (q - i * f < (uint32_t)__ldg(a.pcnt + i)) {
+                valid[k] = true;
+                slot[k] = (uint32_t)__ldg(a.pslot + q);
+            }
+        }
+    }
+    uint32_t hv0[kRelabelItems];
+    unsigned bv[kRelabelItems], bn[kRelabelItems];
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
+        hv0[k] = valid[k] ? ld_relaxed_u32(a.hvals + slot[k]) : 0u;
+        const bool isnew = valid[k] && hv0[k] == (kPending | q);
+        bv[k] = __ballot_sync(0xffffffffu, valid[k]);
+        bn[k] = __ballot_sync(0xffffffffu, isnew);
+        if (lane == 0) s_cnt[k * kWarps + warp] = ((uint32_t)__popc(bv[k]) << 16) | (uint32_t)__popc(bn[k]);
+    }
+    __syncthreads();
+    if (warp == 0) {
+        constexpr int kPer = kRelabelItems * kWarps / 32;
+        uint32_t c[kPer];
+        uint32_t sum = 0;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            c[q] = s_cnt[kPer * lane + q];
+            sum += c[q];
+        }
+        const uint32_t inc = warp_inclusive_sum(sum);
+        const uint32_t agg = __shfl_sync(0xffffffffu, inc, 31);
+        __syncwarp();
+        uint32_t run = inc - sum;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            s_cnt[kPer * lane + q] = run;
+            run += c[q];
+        }
+        const unsigned long long agg64 = ((unsigned long long)(agg >> 16) << kPairShift) | (agg & 0xFFFFu);
+        const unsigned long long base = (unsigned long long)lookback_exclusive(a.st, tile, (long long)agg64, 0);
+        if (lane == 0) {
+            s_base = base;
+            const bool last = (n_prev == 0) ? (tile == 0) : (tile == (n_prev - 1) / a.nt);
+            if (last) {
+                const unsigned long long tot = base + agg64;
+                const int64_t edges = (int64_t)(tot >> kPairShift);
+                a.rowptr[n_prev] = edges;
+                a.sizes[a.K + a.hop] = edges;
+                a.sizes[a.hop] = n_prev + (int64_t)(tot & ((1ull << kPairShift) - 1));
+            }
+        }
+    }
+    __syncthreads();
+    const int64_t ebase = (int64_t)(s_base >> kPairShift);
+    const int64_t nbase = (int64_t)(s_base & ((1ull << kPairShift) - 1));
+    const unsigned lt = (1u << lane) - 1u;
+    // first occurrences take their local ids (n_prev + rank) and finalise the hash value
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        if (bn[k] & (1u << lane)) {
+            const uint32_t ex = s_cnt[k * kWarps + warp];
+            const int64_t local = n_prev + nbase + (ex & 0xFFFFu) + __popc(bn[k] & lt);
+            a.n_id[local] = (int32_t)a.hkeys[slot[k]];
+            st_relaxed_u32(a.hvals + slot[k], (uint32_t)local);
+            a.slot_of[local] = (int32_t)slot[k];
+            hv0[k] = (uint32_t)local;
+        }
+    }
+    // every edge's final col (no k_col_resolve for this hop): a node first seen at an earlier
+    // position q' < q of this hop is finalised by the tile owning q' (this one or an earlier one,
+    // resident or done, as the look-back already requires): wait for that store
+#pragma unroll
+    for (int k = 0; k < kRelabelItems; ++k) {
+        const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
+        if (q >= qend) continue;
+        const uint32_t ex = s_cnt[k * kWarps + warp];
+        const int64_t e = ebase + (ex >> 16) + __popc(bv[k] & lt);
+        const uint32_t i = q / f;
+        if (q == i * f) a.rowptr[i] = e;
+        if (valid[k]) {
+            uint32_t v = hv0[k];
+            int spins = 0;
+            while (v >= kPending) {
+                if (++spins > 4) __nanosleep(32);
+                v = ld_relaxed_u32(a.hvals + slot[k]);
+            }
+            a.col[e] = (int32_t)v;
+            if (a.eid) a.eid[e] = __ldg(a.ppos + q);
+        }
+    }
+}
+
 struct RelabelArgs {
     int32_t* col;
     int32_t* n_id;
@@ -431,7 +648,7 @@ __global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
     GD_PDL_ENTRY();
     int64_t cum[GD_MAX_HOPS + 1];
     cum[0] = 0;
-    for (int h = 0; h < a.K; ++h) cum[h + 1] = cum[h] + a.sizes[a.K + 1 + h];
+    for (int h = 0; h < a.K; ++h) cum[h + 1] = cum[h] + (a.col[h] ? a.sizes[a.K + 1 + h] : 0);   // null: resolved
     const int64_t total = cum[a.K];
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; base < total; base += stride * kResolveItems) {
@@ -492,7 +709,46 @@ static gd_status copy_in(void* dst, const void* src, size_t bytes) {
     return GD_OK;
 }
 
+template <int G>
+static void launch_pad_g(const PadHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
+    const unsigned nb = (unsigned)std::max<int64_t>(1, ceil_div(n_frontier_max * G, kThreads));
+    launch_chain(k_sample_pad<G>, dim3(nb), dim3(kThreads), 0, st, a);
+}
+
+static void launch_sample_pad(const PadHopArgs& a, int64_t n_frontier_max, cudaStream_t st) {
+    switch (sampler_group(a.fanout)) {
+        case 1: launch_pad_g<1>(a, n_frontier_max, st); break;
+        case 2: launch_pad_g<2>(a, n_frontier_max, st); break;
+        case 4: launch_pad_g<4>(a, n_frontier_max, st); break;
+        case 8: launch_pad_g<8>(a, n_frontier_max, st); break;
+        case 16: launch_pad_g<16>(a, n_frontier_max, st); break;
+        default: launch_pad_g<32>(a, n_frontier_max, st); break;
+    }
+}
+
+// grow-only device array (the workspace's steady state never reallocates)
+template <typename T>
+static gd_status grow(T*& p, int64_t& cap, int64_t want) {
+    if (want <= cap) return GD_OK;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    GD_CUDA(cudaMalloc(&p, std::max<int64_t>(1, want) * sizeof(T)));
+    cap = want;
+    return GD_OK;
+}
+
 }  // namespace gd
+
+void gd_workspace::release_padded() {
+    if (pslot) cudaFree(pslot);
+    if (ppos) cudaFree(ppos);
+    if (pcnt) cudaFree(pcnt);
+    pslot = nullptr;
+    ppos = nullptr;
+    pcnt = nullptr;
+    pcap = ppos_cap = pcnt_cap = 0;
+}
 
 using namespace gd;
 
@@ -537,6 +793,7 @@ gd_status gd_graph_create(const int64_t* indptr, const int32_t* indices, int64_t
     g->hdr.device = device;
     g->N = num_nodes;
     g->E = num_edges;
+    if (const char* e = std::getenv("GD_SAMPLE_PAD")) g->sample_padded = e[0] != '0';
     auto fail = [&](gd_status s) {
         gd_graph_destroy(g);
         return s;
@@ -579,6 +836,7 @@ gd_status gd_graph_destroy(gd_graph* g) {
     if (g->ws.hash) cudaFree(g->ws.hash);
     if (g->ws.slot_of) cudaFree(g->ws.slot_of);
     if (g->ws.seeds_ws) cudaFree(g->ws.seeds_ws);
+    g->ws.release_padded();
     if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
     g->ws.scan.release();
     g->timer.destroy();
@@ -602,6 +860,7 @@ gd_status gd_workspace_destroy(gd_workspace* w) {
     if (w->hash) cudaFree(w->hash);
     if (w->slot_of) cudaFree(w->slot_of);
     if (w->seeds_ws) cudaFree(w->seeds_ws);
+    w->release_padded();
     w->scan.release();
     w->magic = 0;
     delete w;
@@ -688,7 +947,59 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     GD_CUDA(launch_chain(k_seed_intake, dim3((unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads))), dim3(kThreads),
                          0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, w.slot_of, g->hdr.dev_status));
 
+    bool resolved[GD_MAX_HOPS] = {};
     for (int h = 1; h <= num_hops; ++h) {
+        const int f = fanouts[h - 1];
+        if (g->sample_padded && f >= 1 && f <= 32 && nmax[h - 1] * f < (int64_t)kPending) {
+            const int64_t np = nmax[h - 1] * f;
+            if ((s = grow(w.pslot, w.pcap, np)) != GD_OK) return s;
+            if ((s = grow(w.pcnt, w.pcnt_cap, nmax[h - 1])) != GD_OK) return s;
+            if (out->eid[h - 1] && (s = grow(w.ppos, w.ppos_cap, np)) != GD_OK) return s;
+            PadHopArgs a;
+            a.indptr = g->indptr;
+            a.indices = g->indices;
+            a.N = g->N;
+            a.n_id = out->n_id;
+            a.sizes = out->sizes;
+            a.hop = h;
+            a.fanout = f;
+            a.batch = batch_id;
+            a.seed = rng_seed;
+            a.pslot = w.pslot;
+            a.ppos = out->eid[h - 1] ? w.ppos : nullptr;
+            a.pcnt = w.pcnt;
+            a.hkeys = hk;
+            a.hvals = hv;
+            a.mask = mask;
+            launch_sample_pad(a, nmax[h - 1], st);
+            GD_DEBUG_AFTER("k_sample_pad", st);
+
+            PadRelabelArgs r;
+            r.pslot = w.pslot;
+            r.ppos = a.ppos;
+            r.pcnt = w.pcnt;
+            r.rowptr = out->rowptr[h - 1];
+            r.col = out->col[h - 1];
+            r.eid = out->eid[h - 1];
+            r.n_id = out->n_id;
+            r.sizes = out->sizes;
+            r.hop = h;
+            r.K = num_hops;
+            r.fanout = f;
+            r.nt = kEdgesPerTile / f;
+            r.hkeys = hk;
+            r.hvals = hv;
+            r.slot_of = w.slot_of;
+            r.st = w.scan.use();
+            r.st_clear = w.scan.other();
+            r.st_clear_n = w.scan.cap;
+            const int64_t et = std::max<int64_t>(1, ceil_div(nmax[h - 1], r.nt));
+            GD_CUDA(launch_chain(k_relabel_pad, dim3((unsigned)et), dim3(kThreads), 0, st, r));
+            GD_DEBUG_AFTER("k_relabel_pad", st);
+            w.scan.flip();
+            resolved[h - 1] = true;
+            continue;
+        }
         SampleHopArgs a;
         a.indptr = g->indptr;
         a.indices = g->indices;
@@ -732,19 +1043,29 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         w.scan.flip();
     }
     ColResolveArgs c;
-    for (int h = 0; h < num_hops; ++h) c.col[h] = out->col[h];
+    int64_t esum = 0;
+    for (int h = 0; h < num_hops; ++h) {
+        c.col[h] = resolved[h] ? nullptr : out->col[h];
+        if (!resolved[h]) esum += emax[h];
+    }
     c.sizes = out->sizes;
     c.K = num_hops;
     c.hvals = hv;
-    int64_t esum = 0;
-    for (int h = 0; h < num_hops; ++h) esum += emax[h];
-    dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(esum, kThreads * kResolveItems))));
-    GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
+    if (esum > 0) {   // hops of the count-scan form only (padded hops wrote their final col)
+        dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(esum, kThreads * kResolveItems))));
+        GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
+    }
     GD_CUDA(launch_chain(k_hash_clear, dim3((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(nmax[num_hops], kThreads)))),
                          dim3(kThreads), 0, st, (const int32_t*)w.slot_of, (const int64_t*)(out->sizes + num_hops), hk, hv));
         GD_DEBUG_AFTER("k_col_resolve", st);
     if (tslot >= 0) g->timer.end(tslot, st);
     GD_CUDA(cudaGetLastError());
+    return GD_OK;
+}
+
+gd_status gd_graph_sampler(gd_graph* g, int padded) {
+    if (!g || g->hdr.magic != kMagicGraph) return set_error(GD_ERR_INVALID, "gd_graph_sampler: bad handle");
+    g->sample_padded = padded != 0;
     return GD_OK;
 }
 

@@ -53,15 +53,18 @@ def tiny(gd):
 
 
 @pytest.mark.parametrize("fanouts", [(5, 5), (15, 10, 5), (25, 15), (10, 10, 10), (-1, 3), (0, 4), (40, 2),
-                                     (100,), (33, 1), (1, 1, 1, 1, 1, 1, 1, 1)])
-def test_sample_parity_tiny(tiny, gd, fanouts):
+                                     (100,), (33, 1), (1, 1, 1, 1, 1, 1, 1, 1), (32, 17, 16, 2)])
+@pytest.mark.parametrize("padded", [True, False])
+def test_sample_parity_tiny(tiny, gd, fanouts, padded):
     cfg, g, indptr, indices, order = tiny
+    g.sampler(padded)
     for b in range(6):
         seeds = synth.batch_seeds(order, cfg.batch_size, b)
         res = g.sample(seeds.cuda(), fanouts, synth.RNG_SEED, b, with_eid=True)
         torch.cuda.synchronize()
         ref = O.sample(indptr, indices, seeds.numpy(), list(fanouts), synth.RNG_SEED, b)
         compare_sample(res, ref, len(fanouts))
+    g.sampler(True)
     assert g.check() == 0
 
 
@@ -79,11 +82,13 @@ def test_sample_parity_host_seeds_and_no_eid(tiny, gd):
     compare_sample(res2, ref, 2)
 
 
-def test_sample_parity_multi_tile(gd):
+@pytest.mark.parametrize("padded", [True, False])
+def test_sample_parity_multi_tile(gd, padded):
     """~200k nodes, (15,10,5) from 1024 seeds: hundreds of tiles per hop, ragged tails."""
     N, E = 200_000, 3_000_000
     indptr, indices = make_graph(N, E, seed=9)
     g = gd.Graph(indptr, indices)
+    g.sampler(padded)
     order = synth.epoch_order(synth.train_nodes(N, 0.05))
     ip, ix = indptr.numpy(), indices.numpy()
     for b, B in [(0, 1024), (1, 1000), (2, 1), (3, 777)]:
@@ -93,12 +98,14 @@ def test_sample_parity_multi_tile(gd):
         compare_sample(res, O.sample(ip, ix, seeds.numpy(), [15, 10, 5], 3, b), 3)
 
 
-def test_sample_edge_cases(gd):
+@pytest.mark.parametrize("padded", [True, False])
+def test_sample_edge_cases(gd, padded):
     # isolated nodes, self loops, multi-edges; empty seed list
     rows = [[1, 2], [1, 0, 4], [0, 0, 4], [], [5], [2], [], [3, 3, 3, 3]]
     indptr = torch.tensor(np.cumsum([0] + [len(r) for r in rows]), dtype=torch.int64)
     indices = torch.tensor([u for r in rows for u in r], dtype=torch.int32)
     g = gd.Graph(indptr, indices)
+    g.sampler(padded)
     for seeds, fan in [([3], [2, 2]), ([6, 3], [5]), ([0, 7, 5], [1, 2, 3]), ([7], [-1, -1, -1]), ([], [2, 2])]:
         s = torch.tensor(seeds, dtype=torch.int32)
         res = g.sample(s.cuda() if len(seeds) else s.cuda(), fan, 1, 0, with_eid=True)

@@ -12,7 +12,8 @@ from __future__ import annotations
 import collections
 import json
 
-SAMPLING = ("k_seed_intake", "k_sample_hop", "k_relabel_hop", "k_col_resolve", "k_hash_clear")
+SAMPLING = ("k_seed_intake", "k_sample_hop", "k_relabel_hop", "k_sample_pad", "k_relabel_pad", "k_col_resolve",
+            "k_hash_clear")
 BOOKKEEPING = ("k_lookup", "k_pop_assign", "k_release", "k_compact")
 CATS = [
     ("sampling (a1-a4)", lambda n, k: k == "kernel" and n.startswith(SAMPLING)),
