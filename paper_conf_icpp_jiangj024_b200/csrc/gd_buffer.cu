@@ -73,7 +73,7 @@ struct LookupArgs {
     int32_t* alias;
     int2* hitlist;                   // [n - M]: {batch position, slot} of the non-misses, list order
     int64_t* hcount;                 // n - M
-    int32_t* misslist;
+    int2* misslist;                  // [M]: {batch position, node} of the misses, list order
     int64_t* mcount;
     int64_t* stats;
     unsigned long long* st;
@@ -162,7 +162,7 @@ __global__ void __launch_bounds__(kBThreads) k_lookup(LookupArgs a) {
         const int64_t i = i0 + (int64_t)k * kBThreads + t;
         const long long mrank = base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);   // misses before i
         if (ball[k] & (1u << lane))
-            a.misslist[mrank] = (int32_t)i;
+            a.misslist[mrank] = make_int2((int32_t)i, vv[k]);
         else if (i < n)
             a.hitlist[i - mrank] = make_int2((int32_t)i, alv[k]);
     }
@@ -177,7 +177,7 @@ struct PopArgs {
     int2* map;
     int32_t* reverse;
     const int32_t* ids;
-    const int32_t* misslist;
+    const int2* misslist;
     const int64_t* mcount;
     int32_t* alias;
     int4* trip;
@@ -308,18 +308,34 @@ __global__ void __launch_bounds__(kBThreads) k_pop_assign(PopArgs a) {
         const long long base = s_base;
         if (base < M) {
             const unsigned lt = (1u << lane) - 1u;
+            // loads of every item first ({position, node} of the miss, the slot's old node), then
+            // the stores: an evicted node sits in the standby list (valid, refcount 0), so k_lookup
+            // made it a hit of this batch if it is in it -- no store below aliases a load above
+            long long rk[kBItems];
+            int2 mi[kBItems];
+            int32_t oldv[kBItems];
 #pragma unroll
             for (int k = 0; k < kBItems; ++k) {
+                rk[k] = -1;
                 if (!(ball[k] & (1u << lane))) continue;
                 const long long rank = base + s_cnt[k * kBWarps + warp] + __popc(ball[k] & lt);
                 if (rank >= M) continue;
+                rk[k] = rank;
+                mi[k] = __ldg(a.misslist + rank);
+                oldv[k] = a.reverse[slot[k]];
+            }
+#pragma unroll
+            for (int k = 0; k < kBItems; ++k) {
+                const long long rank = rk[k];
+                if (rank < 0) continue;
                 const int32_t s = slot[k];
-                const int32_t i = a.misslist[rank];
-                const int32_t v = a.ids[i];
-                const int32_t old = a.reverse[s];
+                const int32_t i = mi[k].x;
+                const int32_t v = mi[k].y;
+                const int32_t old = oldv[k];
                 if (old >= 0) a.map[old] = make_int2(-1, 0);   // invalidate (R9)
-                const int2 m = a.map[v];
-                a.map[v] = make_int2(s, m.y | 1);               // lines 27, 37
+                // lines 27, 37: slot s, valid; a miss had refcount 0 before k_lookup's
+                // increment (line 19), so its refcount is 1
+                a.map[v] = make_int2(s, (1 << 1) | 1);
                 a.reverse[s] = v;                               // line 28
                 a.alias[i] = s;                                 // line 29
                 a.pos_of_slot[s] = -1;
@@ -1044,7 +1060,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
     GD_ALLOC(b->pos_of_slot, capacity_slots * sizeof(int32_t));
     GD_ALLOC(b->ring, 2 * C * sizeof(int32_t));
     GD_ALLOC(b->ctl, 2 * sizeof(GdCtl));
-    GD_ALLOC(b->misslist, nm * sizeof(int32_t));
+    GD_ALLOC(b->misslist, nm * sizeof(int2));
     GD_ALLOC(b->hitlist, (int64_t)b->D * nm * sizeof(int2));
     GD_ALLOC(b->hcount, (int64_t)b->D * sizeof(int64_t));
     GD_ALLOC(b->alias_ws, (int64_t)b->D * nm * sizeof(int32_t));

@@ -124,7 +124,7 @@ struct gd_buffer {
     GdCtl* ctl = nullptr;                // HBM [2]
     int ctl_parity = 0;
     // per-batch workspace used on the caller's stream
-    int32_t* misslist = nullptr;         // [n_max] batch positions of misses, list order
+    int2* misslist = nullptr;            // [n_max] {batch position, node} of the misses, list order
     int2* hitlist = nullptr;             // [D][n_max] {position, slot} of the hits (read on stream G)
     int64_t* hcount = nullptr;           // [D] number of hits
     int32_t* alias_ws = nullptr;         // [D][n_max] used when the caller passes alias = NULL

@@ -61,16 +61,20 @@ struct SampleHopArgs {
 __device__ __forceinline__ uint32_t hash_insert(uint32_t* __restrict__ hk, uint32_t* __restrict__ hv,
                                                 uint32_t mask, uint32_t u, uint32_t e) {
     uint32_t h = fmix32(u) & mask;
+    const uint32_t tag = kPending | e;
     while (true) {
         const uint32_t k = ld_relaxed_u32(hk + h);
         if (k == u) break;
         if (k == kEmpty) {
             const uint32_t old = atomicCAS(hk + h, kEmpty, u);
-            if (old == kEmpty || old == u) break;
+            if (old == kEmpty) {           // claimed: the value is empty (> any tag), no load first
+                atomicMin(hv + h, tag);
+                return h;
+            }
+            if (old == u) break;
         }
         h = (h + 1) & mask;
     }
-    const uint32_t tag = kPending | e;
     if (ld_relaxed_u32(hv + h) > tag) atomicMin(hv + h, tag);
     return h;
 }
@@ -456,12 +460,11 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
         const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
         valid[k] = false;
         slot[k] = 0;
-        if (q < qend) {
+        if (q < qend) {   // both loads at once (pslot past a node's count is stale but in bounds)
             const uint32_t i = q / f;
-            if (q - i * f < (uint32_t)__ldg(a.pcnt + i)) {
-                valid[k] = true;
-                slot[k] = (uint32_t)__ldg(a.pslot + q);
-            }
+            const int32_t c = __ldg(a.pcnt + i);
+            slot[k] = (uint32_t)__ldg(a.pslot + q);
+            valid[k] = q - i * f < (uint32_t)c;
         }
     }
     uint32_t hv0[kRelabelItems];
