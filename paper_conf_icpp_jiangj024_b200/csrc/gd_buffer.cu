@@ -1123,6 +1123,7 @@ gd_status gd_buffer_init_mod(const void* host_feat, int64_t table_rows, int64_t 
         b->gather_dynamic = !(d && d[0] == '0');
         if (const char* e2 = std::getenv("GD_GATHER_BPS")) b->gather_bps = std::max(1, std::min(8, std::atoi(e2)));
         if (const char* e2 = std::getenv("GD_GATHER_U")) b->gather_u = std::atoi(e2) == 8 ? 8 : 4;
+        if (const char* e2 = std::getenv("GD_ZC_AFTER_GATHER")) b->zc_after_gather = e2[0] != '0';
         // GD_GATHER_TMA=1: the TMA gather4 variant of a8 (rows <= 2048 B, multiples of 16)
         const char* t = std::getenv("GD_GATHER_TMA");
         if (t && t[0] == '1' && make_slot_map(&b->slot_map, b->slots, capacity_slots, row_bytes)) {
@@ -1865,6 +1866,10 @@ gd_status gd_extract(gd_buffer* b, const int32_t* node_ids, const int64_t* n_dev
     GD_DEBUG_AFTER("k_gather_hits", b->side_g);
     if (timed) b->timer.end(t_gat, b->side_g);
     GD_CUDA(cudaEventRecord(b->ev_G, b->side_g));
+    // zc_after_gather: the zero-copy kernel of this batch also waits for this batch's hit gather,
+    // so the two never overlap (microsecond host loads clog the memory pipeline of the SMs the
+    // gather shares with them); the gather already waits for the previous batch's copies
+    if (b->zc_after_gather && !peer) GD_CUDA(cudaStreamWaitEvent(b->side, b->ev_G, 0));
 
     // a7, zero-copy share: misses [0, K0) straight from the pinned host table (stream Z).
     // With preload every node is valid from the start and never evicted: no misses, no copy.

@@ -137,6 +137,7 @@ struct gd_buffer {
     bool gather_dynamic = true;          // hit gather: dynamic row assignment (GD_GATHER_DYNAMIC)
     bool gather_tma = false;             // hit gather by TMA gather4 (GD_GATHER_TMA=1)
     int gather_bps = 4;                  // hit gather: 256-thread blocks per SM (GD_GATHER_BPS)
+    bool zc_after_gather = false;        // zero-copy kernel of batch b after the hit gather of b (GD_ZC_AFTER_GATHER)
     int gather_u = 4;                    // hit gather, rows <= 512 B: rows in flight per warp (GD_GATHER_U: 4 | 8)
     CUtensorMap slot_map;                // tensor map over the slots for the TMA gather
     unsigned long long* done_word = nullptr; // [1] epoch-tagged early-exit word of the pop scan
