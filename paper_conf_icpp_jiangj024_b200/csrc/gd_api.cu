@@ -75,6 +75,7 @@ gd_status ScanState::ensure(int64_t tiles) {
     buf[1] = b + ncap;
     cap = ncap;
     parity = 0;
+    dirty[0] = dirty[1] = 0;
     return GD_OK;
 }
 

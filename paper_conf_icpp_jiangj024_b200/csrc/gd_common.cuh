@@ -157,6 +157,17 @@ struct ScanState {
     unsigned long long* use() const { return buf[parity]; }
     unsigned long long* other() const { return buf[parity ^ 1]; }
     void flip() { parity ^= 1; }
+    // Tiles each array's last launch may have written, tracked on the host: a launch whose tile
+    // count is known clears only what the previous launch on the other array dirtied (clearing
+    // the whole array from a small grid -- the 8-block first-hop relabel of products -- cost
+    // ~16 us of stores).  Launches that do not know their tile count record the whole array.
+    int64_t dirty[2] = {0, 0};
+    int64_t clear_n() const { return dirty[parity ^ 1]; }
+    void launched(int64_t tiles) {
+        dirty[parity] = tiles < cap ? tiles : cap;
+        dirty[parity ^ 1] = 0;
+        flip();
+    }
 };
 
 // ----------------------------------------------------------------- device side

@@ -995,11 +995,11 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
             r.slot_of = w.slot_of;
             r.st = w.scan.use();
             r.st_clear = w.scan.other();
-            r.st_clear_n = w.scan.cap;
+            r.st_clear_n = w.scan.clear_n();
             const int64_t et = std::max<int64_t>(1, ceil_div(nmax[h - 1], r.nt));
             GD_CUDA(launch_chain(k_relabel_pad, dim3((unsigned)et), dim3(kThreads), 0, st, r));
             GD_DEBUG_AFTER("k_relabel_pad", st);
-            w.scan.flip();
+            w.scan.launched(et);
             resolved[h - 1] = true;
             continue;
         }
@@ -1022,11 +1022,11 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         a.mask = mask;
         a.st = w.scan.use();
         a.st_clear = w.scan.other();
-        a.st_clear_n = w.scan.cap;
+        a.st_clear_n = w.scan.clear_n();
         a.status = g->hdr.dev_status;
         launch_sample_hop(a, nmax[h - 1], st);
         GD_DEBUG_AFTER("k_sample_hop", st);
-        w.scan.flip();
+        w.scan.launched(w.scan.cap);
 
         RelabelArgs r;
         r.col = out->col[h - 1];
@@ -1039,11 +1039,11 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         r.slot_of = w.slot_of;
         r.st = w.scan.use();
         r.st_clear = w.scan.other();
-        r.st_clear_n = w.scan.cap;
+        r.st_clear_n = w.scan.clear_n();
         const int64_t et = std::max<int64_t>(1, ceil_div(emax[h - 1], kEdgesPerTile));
         GD_CUDA(launch_chain(k_relabel_hop, dim3((unsigned)et), dim3(kThreads), 0, st, r));
         GD_DEBUG_AFTER("k_relabel_hop", st);
-        w.scan.flip();
+        w.scan.launched(et);
     }
     ColResolveArgs c;
     int64_t esum = 0;
