@@ -400,16 +400,21 @@ def test_extract_parity_row_sizes(gd, R, mode, monkeypatch):
                  config=(4, 0.3), stage_mode=copy_engine)
 
 
-@pytest.mark.parametrize("variant", ["tma", "static", "low-priority"])
+@pytest.mark.parametrize("variant", ["tma", "static", "low-priority", "u8-2bps", "zc-after-gather"])
 @pytest.mark.parametrize("R", [400, 512, 1536, 2048, 12])
 def test_hit_gather_variants(gd, R, variant, monkeypatch):
     """a8 variants (selected at buffer init): the TMA gather4 kernel (GD_GATHER_TMA=1), the
-    warp-per-row kernel with a static row partition (GD_GATHER_DYNAMIC=0) and the gather
-    stream at default priority: the same bytes, alias and state as the oracle (R = 12: the
+    warp-per-row kernel with a static row partition (GD_GATHER_DYNAMIC=0), the gather
+    stream at default priority, 8 rows in flight per warp on 2 blocks per SM (GD_GATHER_U=8,
+    GD_GATHER_BPS=2), and the zero-copy kernel ordered after the hit gather
+    (GD_ZC_AFTER_GATHER=1): the same bytes, alias and state as the oracle (R = 12: the
     4-byte kernel, whichever variant is asked for)."""
-    env = {"tma": ("GD_GATHER_TMA", "1"), "static": ("GD_GATHER_DYNAMIC", "0"),
-           "low-priority": ("GD_GATHER_PRIORITY", "0")}[variant]
-    monkeypatch.setenv(*env)
+    envs = {"tma": [("GD_GATHER_TMA", "1")], "static": [("GD_GATHER_DYNAMIC", "0")],
+            "low-priority": [("GD_GATHER_PRIORITY", "0")],
+            "u8-2bps": [("GD_GATHER_U", "8"), ("GD_GATHER_BPS", "2")],
+            "zc-after-gather": [("GD_ZC_AFTER_GATHER", "1")]}[variant]
+    for k, v in envs:
+        monkeypatch.setenv(k, v)
     N, E = 20_000, 150_000
     indptr, indices = make_graph(N, E, seed=17)
     g = gd.Graph(indptr, indices)

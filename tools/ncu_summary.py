@@ -18,7 +18,7 @@ import subprocess
 import sys
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-GO = os.path.join(ROOT, "gpurun_out")
+GO = os.environ.get("NCU_DIR", os.path.join(ROOT, "gpurun_out"))
 PROF = os.path.join(ROOT, "profiles")
 
 
