@@ -14,11 +14,15 @@
 struct gd_workspace {
     uint32_t magic = 0x47445753u;   // "GDWS"
     int device = 0;
-    uint32_t* hash = nullptr;       // keys [hcap] then values [hcap] (L2-resident); all empty
-                                    // between calls (each call clears the slots it used)
+    uint32_t* hash = nullptr;       // two tables, table t at hash + 2 t hcap: keys [hcap] then
+                                    // values [hcap] (L2-resident).  Calls alternate tables; a call
+                                    // empties the slots the previous call used in the other table
+                                    // (inside its last relabel pass), so a table is empty when used
     int64_t hcap = 0;               // power of two >= 1.25 x max_nodes[K]
-    int32_t* slot_of = nullptr;     // [slot_cap] hash slot of n_id[i] (for that clearing)
+    int32_t* slot_of = nullptr;     // [2 slot_cap] hash slot of n_id[i], table t at slot_of + t slot_cap
     int64_t slot_cap = 0;
+    int64_t* used = nullptr;        // device [2]: entries of slot_of of the last call on table t
+    int tsel = 0;                   // table of the next call
     int32_t* seeds_ws = nullptr;    // staging for host seed arrays
     int64_t seeds_cap = 0;
     int32_t* pslot = nullptr;       // padded hop: [pcap] hash slot of draw q = i f + r
@@ -36,6 +40,7 @@ struct gd_graph {
     int64_t* indptr = nullptr;      // HBM int64[N+1]
     int32_t* indices = nullptr;     // HBM int32[E]
     gd_workspace ws;                // used by gd_sample
+    int fold_clear = 1;             // padded last hop empties the previous table (GD_HASH_CLEAR_KERNEL=1: k_hash_clear)
     int sample_padded = 1;          // padded hops for 1 <= f <= 32 (GD_SAMPLE_PAD=0 / gd_graph_sampler)
     gd::EventTimer timer;           // one pair per gd_sample call
 };

@@ -434,9 +434,29 @@ struct PadRelabelArgs {
     unsigned long long* st;
     unsigned long long* st_clear;
     int64_t st_clear_n;
+    // last hop only (else null): empty the slots the previous call used in the other table
+    // (clr_slot_of[0, *clr_count)), and record this call's node count (*rec_used = n_K)
+    const int32_t* clr_slot_of;
+    const int64_t* clr_count;
+    uint32_t* clr_hk;
+    uint32_t* clr_hv;
+    int64_t* rec_used;
 };
 
-constexpr unsigned long long kPairShift = 31;   // look-back value = edges << 31 | new nodes
+constexpr unsigned long long kPairShift = 31;
+
+// Stores only (no result is read back in this call): the other table is not touched by any
+// kernel of this call, and the next call on it is stream-ordered after this one.
+__device__ __forceinline__ void clear_previous_table(const PadRelabelArgs& a) {
+    if (a.clr_slot_of == nullptr) return;
+    const int64_t n = *a.clr_count;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+        const int32_t sl = __ldg(a.clr_slot_of + i);
+        a.clr_hk[sl] = kEmpty;
+        a.clr_hv[sl] = kEmpty;
+    }
+}   // look-back value = edges << 31 | new nodes
 
 __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     GD_PDL_ENTRY();
@@ -444,7 +464,10 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     const int64_t n_prev = a.sizes[a.hop - 1];
     const int64_t tile = blockIdx.x;
     const int64_t i0 = tile * a.nt;
-    if (i0 >= n_prev && tile != 0) return;
+    if (i0 >= n_prev && tile != 0) {
+        clear_previous_table(a);
+        return;
+    }
     const uint32_t f = (uint32_t)a.fanout;
     const uint32_t q0 = (uint32_t)(i0 * f);
     const uint32_t qend = (uint32_t)((i0 + a.nt < n_prev ? i0 + a.nt : n_prev) * f);
@@ -508,6 +531,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
                 a.rowptr[n_prev] = edges;
                 a.sizes[a.K + a.hop] = edges;
                 a.sizes[a.hop] = n_prev + (int64_t)(tot & ((1ull << kPairShift) - 1));
+                if (a.rec_used) *a.rec_used = a.sizes[a.hop];
             }
         }
     }
@@ -549,6 +573,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
             if (a.eid) a.eid[e] = __ldg(a.ppos + q);
         }
     }
+    clear_previous_table(a);
 }
 
 struct RelabelArgs {
@@ -682,9 +707,10 @@ __global__ void __launch_bounds__(kThreads) k_col_resolve(ColResolveArgs a) {
 // or a neighbour, appended at its first occurrence), whose slot k_seed_intake /
 // k_relabel_hop recorded.  Replaces a memset of the whole table per call.
 __global__ void __launch_bounds__(kThreads) k_hash_clear(const int32_t* __restrict__ slot_of, const int64_t* __restrict__ n_p,
-                                                         uint32_t* hk, uint32_t* hv) {
+                                                         uint32_t* hk, uint32_t* hv, const int64_t* rec_src, int64_t* rec_dst) {
     GD_PDL_ENTRY();
     const int64_t n = *n_p;
+    if (rec_dst && blockIdx.x == 0 && threadIdx.x == 0) *rec_dst = *rec_src;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         const int32_t s = slot_of[i];
         hk[s] = kEmpty;
@@ -797,6 +823,7 @@ gd_status gd_graph_create(const int64_t* indptr, const int32_t* indices, int64_t
     g->N = num_nodes;
     g->E = num_edges;
     if (const char* e = std::getenv("GD_SAMPLE_PAD")) g->sample_padded = e[0] != '0';
+    if (const char* e = std::getenv("GD_HASH_CLEAR_KERNEL")) g->fold_clear = e[0] != '1';
     auto fail = [&](gd_status s) {
         gd_graph_destroy(g);
         return s;
@@ -838,6 +865,7 @@ gd_status gd_graph_destroy(gd_graph* g) {
     if (g->indices) cudaFree(g->indices);
     if (g->ws.hash) cudaFree(g->ws.hash);
     if (g->ws.slot_of) cudaFree(g->ws.slot_of);
+    if (g->ws.used) cudaFree(g->ws.used);
     if (g->ws.seeds_ws) cudaFree(g->ws.seeds_ws);
     g->ws.release_padded();
     if (g->hdr.dev_status) cudaFree(g->hdr.dev_status);
@@ -862,6 +890,7 @@ gd_status gd_workspace_destroy(gd_workspace* w) {
     DeviceGuard guard(w->device);
     if (w->hash) cudaFree(w->hash);
     if (w->slot_of) cudaFree(w->slot_of);
+    if (w->used) cudaFree(w->used);
     if (w->seeds_ws) cudaFree(w->seeds_ws);
     w->release_padded();
     w->scan.release();
@@ -902,21 +931,26 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
     // real batches reach 30-70% of the bound), so the per-batch clear stays small
     int64_t want = 1024;
     while (want < std::max<int64_t>(nmax[num_hops], 1) * 5 / 4 + 1) want *= 2;
-    if (want > w.hcap) {
-        if (w.hash) cudaFree(w.hash);
-        w.hash = nullptr;
-        w.hcap = 0;
-        GD_CUDA(cudaMalloc(&w.hash, 2 * want * sizeof(uint32_t)));
-        GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 2 * want * sizeof(uint32_t), st));   // empty; calls keep it so
-        w.hcap = want;
-    }
-    if (nmax[num_hops] > w.slot_cap) {
-        if (w.slot_of) cudaFree(w.slot_of);
-        w.slot_of = nullptr;
-        w.slot_cap = 0;
-        GD_CUDA(cudaMalloc(&w.slot_of, std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t)));
-        GD_CUDA(cudaMemsetAsync(w.slot_of, 0, std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t), st));
-        w.slot_cap = nmax[num_hops];
+    if (want > w.hcap || nmax[num_hops] > w.slot_cap || !w.used) {
+        // (re)allocate; both tables start empty and no call's slots are pending
+        if (want > w.hcap) {
+            if (w.hash) cudaFree(w.hash);
+            w.hash = nullptr;
+            w.hcap = 0;
+            GD_CUDA(cudaMalloc(&w.hash, 4 * want * sizeof(uint32_t)));
+            w.hcap = want;
+        }
+        if (nmax[num_hops] > w.slot_cap) {
+            if (w.slot_of) cudaFree(w.slot_of);
+            w.slot_of = nullptr;
+            w.slot_cap = 0;
+            GD_CUDA(cudaMalloc(&w.slot_of, 2 * std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t)));
+            GD_CUDA(cudaMemsetAsync(w.slot_of, 0, 2 * std::max<int64_t>(1, nmax[num_hops]) * sizeof(int32_t), st));
+            w.slot_cap = std::max<int64_t>(1, nmax[num_hops]);
+        }
+        if (!w.used) GD_CUDA(cudaMalloc(&w.used, 2 * sizeof(int64_t)));
+        GD_CUDA(cudaMemsetAsync(w.hash, 0xFF, 4 * w.hcap * sizeof(uint32_t), st));
+        GD_CUDA(cudaMemsetAsync(w.used, 0, 2 * sizeof(int64_t), st));
     }
     int64_t tiles = 1;
     for (int h = 0; h < num_hops; ++h) {
@@ -943,14 +977,18 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         seeds_d = w.seeds_ws;
     }
 
-    uint32_t* hk = w.hash;
-    uint32_t* hv = w.hash + w.hcap;
+    const int tb = w.tsel, tp = tb ^ 1;     // this call's table, the previous call's
+    w.tsel = tp;
+    uint32_t* hk = w.hash + 2 * tb * w.hcap;
+    uint32_t* hv = hk + w.hcap;
+    int32_t* slot_of = w.slot_of + tb * w.slot_cap;
     const uint32_t mask = (uint32_t)(w.hcap - 1);
     const int tslot = g->timer.on ? g->timer.begin(st) : -1;
     GD_CUDA(launch_chain(k_seed_intake, dim3((unsigned)std::max<int64_t>(1, ceil_div(num_seeds, kThreads))), dim3(kThreads),
-                         0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, w.slot_of, g->hdr.dev_status));
+                         0, st, seeds_d, num_seeds, g->N, hk, hv, mask, out->n_id, out->sizes, slot_of, g->hdr.dev_status));
 
     bool resolved[GD_MAX_HOPS] = {};
+    bool cleared_prev = false;   // the last hop's relabel emptied the previous call's table
     for (int h = 1; h <= num_hops; ++h) {
         const int f = fanouts[h - 1];
         if (g->sample_padded && f >= 1 && f <= 32 && nmax[h - 1] * f < (int64_t)kPending) {
@@ -992,7 +1030,14 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
             r.nt = kEdgesPerTile / f;
             r.hkeys = hk;
             r.hvals = hv;
-            r.slot_of = w.slot_of;
+            r.slot_of = slot_of;
+            const bool last_hop = h == num_hops && g->fold_clear;
+            r.clr_slot_of = last_hop ? w.slot_of + tp * w.slot_cap : nullptr;
+            r.clr_count = w.used + tp;
+            r.clr_hk = w.hash + 2 * tp * w.hcap;
+            r.clr_hv = r.clr_hk + w.hcap;
+            r.rec_used = last_hop ? w.used + tb : nullptr;
+            cleared_prev = cleared_prev || last_hop;
             r.st = w.scan.use();
             r.st_clear = w.scan.other();
             r.st_clear_n = w.scan.clear_n();
@@ -1036,7 +1081,7 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         r.K = num_hops;
         r.hkeys = hk;
         r.hvals = hv;
-        r.slot_of = w.slot_of;
+        r.slot_of = slot_of;
         r.st = w.scan.use();
         r.st_clear = w.scan.other();
         r.st_clear_n = w.scan.clear_n();
@@ -1058,8 +1103,12 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
         dim3 grid((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(esum, kThreads * kResolveItems))));
         GD_CUDA(launch_chain(k_col_resolve, grid, dim3(kThreads), 0, st, c));
     }
-    GD_CUDA(launch_chain(k_hash_clear, dim3((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(nmax[num_hops], kThreads)))),
-                         dim3(kThreads), 0, st, (const int32_t*)w.slot_of, (const int64_t*)(out->sizes + num_hops), hk, hv));
+    if (!cleared_prev) {   // last hop of the count-scan form: empty the previous call's table here
+        uint32_t* phk = w.hash + 2 * tp * w.hcap;
+        GD_CUDA(launch_chain(k_hash_clear, dim3((unsigned)std::min<int64_t>(148 * 8, std::max<int64_t>(1, ceil_div(nmax[num_hops], kThreads)))),
+                             dim3(kThreads), 0, st, (const int32_t*)(w.slot_of + tp * w.slot_cap), (const int64_t*)(w.used + tp),
+                             phk, phk + w.hcap, (const int64_t*)(out->sizes + num_hops), w.used + tb));
+    }
         GD_DEBUG_AFTER("k_col_resolve", st);
     if (tslot >= 0) g->timer.end(tslot, st);
     GD_CUDA(cudaGetLastError());
