@@ -545,6 +545,7 @@ def run_ours(args, rank, world, local_rank):
             log(f"  step {j}: {what} ok")
 
     last_o = [None]
+    host_wait = [0.0]     # seconds the host loop spent waiting for the bounded queue (not enqueueing)
     HOST_BOUND = os.environ.get("GD_HOST_BOUND", "1") == "1"   # GD_HOST_BOUND=0: unbounded host lookahead
 
     def step(j, host_inputs=False, host_out=None):
@@ -552,7 +553,9 @@ def run_ours(args, rank, world, local_rank):
         o = outs[s]
         last_o[0] = o
         if HOST_BOUND:
+            t_w = time.perf_counter()
             dones[s].synchronize()         # the host, too, stays at most RING batches ahead (bounded queue)
+            host_wait[0] += time.perf_counter() - t_w
         ss = samp_streams[j % NS]
         ss.wait_event(dones[s])            # batch j - RING is complete: its buffers are free
         if relslot_live[s] and ss is not main:
@@ -675,12 +678,15 @@ def run_ours(args, rank, world, local_rank):
         ev0.record(main)
         samplers_after(ev0)
         win_ev = []
+        host_wait[0] = 0.0
+        t_host0 = time.perf_counter()
         for j in range(off + W, off + W + K):
             step(j)
             if args.window and (j - off - W + 1) % args.window == 0:
                 e_ = torch.cuda.Event(enable_timing=True)
                 e_.record(main)
                 win_ev.append(e_)
+        t_host1 = time.perf_counter()
         main.wait_event(dones[(off + W + K - 1) % RING])  # the last batch's rows are all in `out`
         if rel_live[0]:
             main.wait_event(ev_rel)                          # ... and the last release is done
@@ -688,6 +694,10 @@ def run_ours(args, rank, world, local_rank):
             main.wait_event(tdones[(off + W + K - 1) % RING])   # ... and it is trained
         ev1.record(main)
         ev1.synchronize()
+    host_loop = {"enqueue_ms_per_step": round((t_host1 - t_host0) * 1e3 / K, 4),
+                 "busy_ms_per_step": round((t_host1 - t_host0 - host_wait[0]) * 1e3 / K, 4),
+                 "def": "host wall time of the timed loop per step, and the same minus the bounded-queue waits "
+                        "(the host thread's own enqueue work: Python, ctypes, the library's API calls)"}
     torch.cuda.synchronize(dev)
     g.timing(False)
     buf.timing(False)
@@ -1130,6 +1140,7 @@ def run_ours(args, rank, world, local_rank):
                        "huge_pages_GB_after_fill": wl.thp_table_gb},
         "numa": numa,
         "windows": windows,
+        "host_loop": host_loop,
         "sweep": sweep or None,
         "pipeline": pipe_res or None,
         "device_status": {"graph": status_g, "buffer": status_b},
