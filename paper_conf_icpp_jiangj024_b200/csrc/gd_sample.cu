@@ -1,20 +1,22 @@
 // gd_sample.cu — topology replica and the multi-hop sampler (rows a1-a4 of the hot path).
 //
-// One gd_sample call = 3 + 2K launches on the caller's stream, no host sync:
-//   memset(hash) ; k_seed_intake ; K x { k_sample_hop ; k_relabel_hop } ; k_col_resolve
+// One gd_sample call = 1 + 2K launches on the caller's stream (hops with 1 <= f <= 32), no host
+// sync:   k_seed_intake ; K x { k_sample_pad ; k_relabel_pad }
 //
-// k_sample_hop  (S1, a2+a3): tile of 64-256 frontier nodes per 256-thread block.  Counts
-//   cnt = min(f, deg) are scanned with a decoupled look-back (rowptr), then a group of
-//   G = pow2 >= f lanes per node (32/G nodes per warp at once; a whole warp for f > 16)
-//   draws Floyd positions with Philox (lane t = draw t, resolution by ballots, rank
-//   sort by shuffles) and inserts every neighbour into the global open-addressing hash
-//   with atomicMin of its flat position (first occurrence).  col temporarily holds the
-//   neighbour's hash slot.
-// k_relabel_hop (S2, a4): flag = "this edge is the first occurrence of a new node";
-//   warp ballots + popc give in-warp ranks (warp-aggregated compaction), a look-back scan
-//   gives the global rank; new nodes get local ids n_{h-1} + rank, are appended to n_id
-//   and finalised in the hash.
-// k_col_resolve: col[e] = local id of the slot (one launch for all hops).
+// k_sample_pad  (S1, a2+a3): G = pow2 >= f lanes per frontier node, no tiles, no scan: Floyd
+//   positions by Philox (lane t = draw t, resolution by ballots, rank sort by shuffles); the
+//   draw of rank r of node i goes to padded position q = i f + r, its neighbour into the global
+//   open-addressing hash with atomicMin(PENDING | q) (first occurrence), its hash slot to
+//   pslot[q], min(f, deg) to pcnt[i].
+// k_relabel_pad (S2, a2+a4): one pass over the padded positions, one decoupled look-back over
+//   (edges, new nodes): rowptr, compacted col / eid, new nodes' local ids n_{h-1} + rank
+//   (warp-aggregated compaction), appended to n_id and finalised in the hash; then every edge's
+//   final col (waiting for the store of a node first seen in an earlier tile).  The last hop's
+//   pass also empties the slots the previous call used in the workspace's other hash table.
+// Hops with f = -1 or f > 32 (or gd_graph_sampler(g, 0)) take the count-scan form:
+// k_sample_hop (counts + look-back -> rowptr, sampling writes col at rowptr + rank),
+// k_relabel_hop (first-occurrence flags, look-back ranks) and one k_col_resolve pass over those
+// hops' edges (+ k_hash_clear when the last hop has this form).
 #include <algorithm>
 #include <cstdlib>
 #include <cstring>
