@@ -57,8 +57,10 @@ def parse():
     p.add_argument("--lr", type=float, default=0.01, help="f4 SGD learning rate")
     p.add_argument("--peer", action="store_true", help="f2: attach every other rank's feature buffer as an NVLink "
                    "peer (CUDA IPC); misses are served from peers' HBM before the host link")
-    p.add_argument("--sample-ahead", type=int, default=3,
-                   help="batches sampled ahead of extraction (per-batch buffer ring = Q + 1 + this)")
+    p.add_argument("--sample-ahead", type=int, default=None,
+                   help="batches sampled ahead of extraction (per-batch buffer ring = Q + 1 + this); default: 3 "
+                        "when every feature is resident (sampling bounds the step), 0 with a miss path (the host "
+                        "link bounds it; sampling further ahead only adds contention for the hit gather)")
     p.add_argument("--samplers", type=int, default=2,
                    help="sampler streams (P:94 'a pool of threads as samplers'), each with its own gd_workspace: "
                         "batch j is sampled on stream j mod S, so the next batch's sampling overlaps this batch's "
@@ -488,7 +490,7 @@ def run_ours(args, rank, world, local_rank):
     # batches sampled ahead of extraction (the sampler -> extractor queue: sampling of batch j
     # waits for the release of batch j - RING, issued after extract(j - RING + Q); with RING = Q + 1
     # that chained every sampling to the previous batch's bookkeeping)
-    RING = Q + 1 + max(0, args.sample_ahead)
+    RING = Q + 1 + sample_ahead(args, cfg)
     outs = [g.alloc_out(cfg.batch_size, fan) for _ in range(RING)]
     feats = [buf.alloc_out(n_max) for _ in range(RING)]
     aliases = [torch.empty(n_max, dtype=torch.int32, device=dev) for _ in range(RING)]
@@ -1350,6 +1352,16 @@ def host_cpu_info():
     return info
 
 
+def sample_ahead(args, cfg):
+    """Batches sampled ahead of extraction.  Measured on one box each (profiles/r02_ab): products
+    (all resident, sampling-bound) 4697 -> 5260 batches/s with 3; papers100m (host-link bound)
+    the same rate with 0 or 3 (505-521) but the hit gather's live share of HBM 29-32% with 0 vs
+    22% with 3 (the extra sampling in flight holds the SM slots the gather waits for)."""
+    if args.sample_ahead is not None:
+        return max(0, args.sample_ahead)
+    return 3 if cfg.preload else 0
+
+
 def config_dict(cfg, S, world, prewarm, samplers, ring):
     """The `config` object of the JSON line; identical for both arms."""
     R = cfg.row_bytes
@@ -1436,7 +1448,7 @@ def run_reference(args, rank, world, local_rank):
             "unit": "batches/s", "n_gpus": world, "steps": K, "warmup": W,
             "ms_per_step": round(1e3 / v, 3) if v else None, "higher_is_better": True, "scaling": "weak",
             "vs_baseline": None, "dtype": "int32", "data": "synthetic (Chung-Lu power law, seeded; synth/)",
-            "config": config_dict(cfg, S, world, jp, max(1, args.samplers), Q + 1 + max(0, args.sample_ahead)),
+            "config": config_dict(cfg, S, world, jp, max(1, args.samplers), Q + 1 + sample_ahead(args, cfg)),
             "cpu_baseline": cv, "single_thread_full_oracle": single, "host_cpu": host_cpu_info(),
             "e2e": {"value": v, "unit": "batches/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
             "native_libs_loaded": loaded_native_libs()}
