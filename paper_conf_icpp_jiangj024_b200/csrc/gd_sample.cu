@@ -33,6 +33,17 @@ constexpr int kRelabelItems = 8;    // (16 measured slower: products 4345 vs 453
 constexpr int kEdgesPerTile = kThreads * kRelabelItems;   // 2048 edges per relabel block
 static_assert((kRelabelItems * kWarps) % 32 == 0, "relabel scan layout");
 constexpr int kMaxFanSmem = GD_MAX_FANOUT;
+// k_relabel_pad: padded positions per thread (<= kRelabelItems) and the launch-bounds block
+// minimum (the defaults were measured; the macros exist for same-box A/B builds)
+#ifndef GD_PAD_ITEMS
+#define GD_PAD_ITEMS 8
+#endif
+#ifndef GD_PAD_MINB
+#define GD_PAD_MINB 1
+#endif
+constexpr int kPadItems = GD_PAD_ITEMS;
+constexpr int kPadPerTile = kThreads * kPadItems;
+static_assert(kPadItems <= kRelabelItems && (kPadItems * kWarps) % 32 == 0, "relabel_pad scan layout");
 
 struct SampleHopArgs {
     const int64_t* indptr;
@@ -429,7 +440,7 @@ struct PadRelabelArgs {
     int hop;
     int K;
     int fanout;
-    int nt;           // frontier nodes per tile (nt f <= kEdgesPerTile)
+    int nt;           // frontier nodes per tile (nt f <= kPadPerTile)
     uint32_t* hkeys;
     uint32_t* hvals;
     int32_t* slot_of;
@@ -460,7 +471,7 @@ __device__ __forceinline__ void clear_previous_table(const PadRelabelArgs& a) {
     }
 }   // look-back value = edges << 31 | new nodes
 
-__global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
+__global__ void __launch_bounds__(kThreads, GD_PAD_MINB) k_relabel_pad(PadRelabelArgs a) {
     GD_PDL_ENTRY();
     clear_tile_state(a.st_clear, a.st_clear_n);
     const int64_t n_prev = a.sizes[a.hop - 1];
@@ -474,14 +485,14 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     const uint32_t q0 = (uint32_t)(i0 * f);
     const uint32_t qend = (uint32_t)((i0 + a.nt < n_prev ? i0 + a.nt : n_prev) * f);
 
-    __shared__ uint32_t s_cnt[kRelabelItems * kWarps];   // (valid << 16 | new) per (round, warp)
+    __shared__ uint32_t s_cnt[kPadItems * kWarps];   // (valid << 16 | new) per (round, warp)
     __shared__ unsigned long long s_base;
     const int t = threadIdx.x, lane = t & 31, warp = t >> 5;
 
-    uint32_t slot[kRelabelItems];
-    bool valid[kRelabelItems];
+    uint32_t slot[kPadItems];
+    bool valid[kPadItems];
 #pragma unroll
-    for (int k = 0; k < kRelabelItems; ++k) {
+    for (int k = 0; k < kPadItems; ++k) {
         const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
         valid[k] = false;
         slot[k] = 0;
@@ -492,10 +503,10 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
             valid[k] = q - i * f < (uint32_t)c;
         }
     }
-    uint32_t hv0[kRelabelItems];
-    unsigned bv[kRelabelItems], bn[kRelabelItems];
+    uint32_t hv0[kPadItems];
+    unsigned bv[kPadItems], bn[kPadItems];
 #pragma unroll
-    for (int k = 0; k < kRelabelItems; ++k) {
+    for (int k = 0; k < kPadItems; ++k) {
         const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
         hv0[k] = valid[k] ? ld_relaxed_u32(a.hvals + slot[k]) : 0u;
         const bool isnew = valid[k] && hv0[k] == (kPending | q);
@@ -505,7 +516,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     }
     __syncthreads();
     if (warp == 0) {
-        constexpr int kPer = kRelabelItems * kWarps / 32;
+        constexpr int kPer = kPadItems * kWarps / 32;
         uint32_t c[kPer];
         uint32_t sum = 0;
 #pragma unroll
@@ -543,7 +554,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     const unsigned lt = (1u << lane) - 1u;
     // first occurrences take their local ids (n_prev + rank) and finalise the hash value
 #pragma unroll
-    for (int k = 0; k < kRelabelItems; ++k) {
+    for (int k = 0; k < kPadItems; ++k) {
         if (bn[k] & (1u << lane)) {
             const uint32_t ex = s_cnt[k * kWarps + warp];
             const int64_t local = n_prev + nbase + (ex & 0xFFFFu) + __popc(bn[k] & lt);
@@ -557,7 +568,7 @@ __global__ void __launch_bounds__(kThreads) k_relabel_pad(PadRelabelArgs a) {
     // position q' < q of this hop is finalised by the tile owning q' (this one or an earlier one,
     // resident or done, as the look-back already requires): wait for that store
 #pragma unroll
-    for (int k = 0; k < kRelabelItems; ++k) {
+    for (int k = 0; k < kPadItems; ++k) {
         const uint32_t q = q0 + (uint32_t)(k * kThreads + t);
         if (q >= qend) continue;
         const uint32_t ex = s_cnt[k * kWarps + warp];
@@ -1029,7 +1040,7 @@ gd_status gd_sample_ws(gd_graph* g, gd_workspace* wsp, const int32_t* seeds, int
             r.hop = h;
             r.K = num_hops;
             r.fanout = f;
-            r.nt = kEdgesPerTile / f;
+            r.nt = kPadPerTile / f;
             r.hkeys = hk;
             r.hvals = hv;
             r.slot_of = slot_of;

@@ -20,6 +20,7 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC,-O2", "-cudart", "static",
          "--expt-relaxed-constexpr", "-I", os.path.join(ROOT, "include")]
+FLAGS += os.environ.get("GD_NVCC_EXTRA", "").split()   # A/B builds only (e.g. -DGD_PAD_ITEMS=4)
 
 
 def sources():
