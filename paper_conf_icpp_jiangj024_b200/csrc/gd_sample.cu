@@ -36,7 +36,7 @@ constexpr int kMaxFanSmem = GD_MAX_FANOUT;
 // k_relabel_pad: padded positions per thread (<= kRelabelItems) and the launch-bounds block
 // minimum (the defaults were measured; the macros exist for same-box A/B builds)
 #ifndef GD_PAD_ITEMS
-#define GD_PAD_ITEMS 8
+#define GD_PAD_ITEMS 4
 #endif
 #ifndef GD_PAD_MINB
 #define GD_PAD_MINB 1
