@@ -11,9 +11,10 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 P = os.path.join(ROOT, "profiles")
 BOXES = [("A", os.path.join(P, "r02_boxes", "boxA_{}_bench.json"), "code before the double-buffered hash, sample-ahead 3"),
          ("B", os.path.join(P, "r02_boxes", "boxB_{}_bench.json"), "code before the double-buffered hash, sample-ahead 3"),
-         ("C", os.path.join(P, "r02_boxes", "boxC_{}_bench.json"), "final kernels, sample-ahead 3"),
-         ("final", os.path.join(P, "r02_{}_bench.json"), "final code: the committed lines (products / tiny from box C, "
-                                                          "the miss-path configs from a fourth box, sample-ahead 0)")]
+         ("C", os.path.join(P, "r02_boxes", "boxC_{}_bench.json"), "double-buffered hash, sample-ahead 3"),
+         ("D", os.path.join(P, "r02_boxes", "boxD_{}_bench.json"), "sample-ahead 0 with a miss path"),
+         ("final", os.path.join(P, "r02_{}_bench.json"), "final code (4 positions per thread in k_relabel_pad): the "
+                                                          "committed lines, all from one box")]
 
 
 def cell(path):
