@@ -31,7 +31,10 @@
 namespace gd {
 
 constexpr int kBThreads = 256;
-constexpr int kBItems = 8;
+#ifndef GD_BOOK_ITEMS
+#define GD_BOOK_ITEMS 8   // entries per thread of the bookkeeping scans (macro for same-box A/B builds)
+#endif
+constexpr int kBItems = GD_BOOK_ITEMS;
 constexpr int kBTile = kBThreads * kBItems;    // 2048 entries per scan tile
 constexpr int kBWarps = kBThreads / 32;
 constexpr int kStageRingMax = 16; // pinned chunk buffers of the copy-engine staging ring (max)
@@ -53,12 +56,23 @@ __device__ __forceinline__ int block_flag_offsets(const unsigned (&ball)[kBItems
     __syncthreads();
     int agg = 0;
     if (warp == 0) {
-        const int c0 = s_cnt[2 * lane], c1 = s_cnt[2 * lane + 1];
-        const int inc = warp_inclusive_sum(c0 + c1);
+        constexpr int kPer = kBItems * kBWarps / 32;   // consecutive (round, warp) counts per lane
+        static_assert(kPer >= 1 && kBItems * kBWarps % 32 == 0, "bookkeeping scan layout");
+        int c[kPer], sum = 0;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            c[q] = s_cnt[kPer * lane + q];
+            sum += c[q];
+        }
+        const int inc = warp_inclusive_sum(sum);
         agg = __shfl_sync(0xffffffffu, inc, 31);
         __syncwarp();
-        s_cnt[2 * lane] = inc - c0 - c1;
-        s_cnt[2 * lane + 1] = inc - c1;
+        int run = inc - sum;
+#pragma unroll
+        for (int q = 0; q < kPer; ++q) {
+            s_cnt[kPer * lane + q] = run;
+            run += c[q];
+        }
     }
     return agg;
 }

@@ -1,0 +1,21 @@
+# same-box A/B of the bookkeeping scan width: A = 8 entries per thread (2048 per tile), B = 4 (1024)
+set -u
+mkdir -p gpurun_out/abso3
+L=paper_conf_icpp_jiangj024_b200/libgd.so
+cp tools/ab_libs/libgd_B.so $L
+timeout 900 python -m pytest tests/test_gpu_parity.py -m gpu -q -x > gpurun_out/abso3/pytest_B.log 2>&1; echo "pytest B=$?"; tail -1 gpurun_out/abso3/pytest_B.log
+A="--steps 400 --warmup 8 --no-cpu-baseline --parity-batches 0 --no-replay"
+for i in 1 2 3; do
+for V in A B; do
+    cp tools/ab_libs/libgd_$V.so $L
+    timeout 900 python bench.py --config products $A > gpurun_out/abso3/products_${V}_$i.json 2>/dev/null
+    python -c "import json;d=json.loads(open('gpurun_out/abso3/products_${V}_$i.json').readline());print('products $V',d['value'],d['e2e']['value'])"
+done
+done
+for i in 1 2; do
+for V in A B; do
+    cp tools/ab_libs/libgd_$V.so $L
+    timeout 900 python bench.py --config papers100m $A > gpurun_out/abso3/papers_${V}_$i.json 2>/dev/null
+    python -c "import json;d=json.loads(open('gpurun_out/abso3/papers_${V}_$i.json').readline());print('papers $V',d['value'],d['e2e']['value'],d['roofline']['frac'])"
+done
+done
