@@ -480,7 +480,7 @@ def run_ours(args, rank, world, local_rank):
     leg = world > 1 and not args.peer and not args.no_peer_leg and not cfg.preload
     TL = 16 if args.timeline else 0
     KI = 0 if os.environ.get("GD_KERNEL_TIMING", "0") == "1" else K      # instrumented region
-    total = PRE + W + K + (0 if args.no_e2e else K) + (len(sweep_cfgs) + n_pipe + int(leg)) * (W + K) + TL + KI
+    total = PRE + W + K + (0 if args.no_e2e else W + K) + (len(sweep_cfgs) + n_pipe + int(leg)) * (W + K) + TL + KI
     sched = batch_schedule(wl.num_batches, rank, world, total)
     seeds_dev = torch.stack([wl.seeds(b, ep) for b, ep in sched]).to(dev).contiguous()   # HBM-resident inputs
     seeds_host = seeds_dev.cpu().pin_memory()
@@ -756,6 +756,13 @@ def run_ours(args, rank, world, local_rank):
         h_ev = [torch.cuda.Event() for _ in range(LAG)]
         seen = [-1, 0, 0]                  # last step copied, running sum of what the host read, first step
         torch.cuda.synchronize(dev)
+        # W untimed warm-up steps through the same public-API path, as before the device-timed region
+        # (the host checks above leave the pipeline drained and the host threads cold; without them
+        # the e2e region of the default run came out 10-15% below the device-timed one on papers100m)
+        for j in range(off + W + K, off + 2 * W + K):
+            step(j, host_inputs=True, host_out=(h_sizes, h_stats, h_ev, seen))
+        torch.cuda.synchronize(dev)
+        seen[0], seen[1], seen[2] = -1, 0, 0
         barrier()
         gc.collect()
         gc.disable()
@@ -763,23 +770,23 @@ def run_ours(args, rank, world, local_rank):
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(main)
         samplers_after(e0)
-        j_end = off + W + 2 * K
+        j_end = off + 2 * W + 2 * K
         e2e_win = []
-        for j in range(off + W + K, j_end):
+        for j in range(off + 2 * W + K, j_end):
             step(j, host_inputs=True, host_out=(h_sizes, h_stats, h_ev, seen))
-            if args.window and (j - off - W - K + 1) % args.window == 0:
+            if args.window and (j - off - 2 * W - K + 1) % args.window == 0:
                 e_ = torch.cuda.Event(enable_timing=True)
                 e_.record(main)
                 e2e_win.append(e_)
-        for j in range(max(off + W + K, j_end - LAG), j_end):   # the last LAG results, inside the timed region
+        for j in range(max(off + 2 * W + K, j_end - LAG), j_end):   # the last LAG results, inside the timed region
             k = j % LAG
             h_ev[k].synchronize()
             seen[1] += int(h_sizes[k][len(fan)]) + int(h_stats[k][0]) + int(h_stats[k][1])
-        main.wait_event(dones[(off + W + 2 * K - 1) % RING])
+        main.wait_event(dones[(j_end - 1) % RING])
         if rel_live[0]:
             main.wait_event(ev_rel)
         if model is not None:
-            main.wait_event(tdones[(off + W + 2 * K - 1) % RING])
+            main.wait_event(tdones[(j_end - 1) % RING])
         e1.record(main)
         e1.synchronize()
         gc.enable()
@@ -789,6 +796,7 @@ def run_ours(args, rank, world, local_rank):
             marks = [e0] + e2e_win
             e2e_windows = [round(args.window / (a_.elapsed_time(b_) / 1e3), 1) for a_, b_ in zip(marks, marks[1:])]
         e2e = {"value": round(world * K / (e2e_ms / 1e3), 2), "unit": "batches/s", "windows": e2e_windows,
+               "warmup_steps": W,
                "h2d_bytes_per_step": cfg.batch_size * 4,
                "d2h_bytes_per_step": (2 * len(fan) + 1) * 8 + 32,
                "read_back": f"each step's sizes + hit/miss stats copied D2H into pinned memory on the stream and "
@@ -797,7 +805,7 @@ def run_ours(args, rank, world, local_rank):
     # ---- capture for the steady-state replay: this rank's buffer has run steps
     # [0, j_win) (pre-warm, warm-up, timed, e2e); keep their per-batch sizes and hit/miss
     # counts, the last RING batches' n_id + alias and the whole buffer state for the oracle
-    j_win = off + W + K + (0 if args.no_e2e else K)
+    j_win = off + W + K + (0 if args.no_e2e else W + K)
     replay_cap = None
     if want_replay:
         torch.cuda.synchronize(dev)
