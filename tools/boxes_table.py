@@ -13,7 +13,8 @@ BOXES = [("A", os.path.join(P, "r02_boxes", "boxA_{}_bench.json"), "code before 
          ("B", os.path.join(P, "r02_boxes", "boxB_{}_bench.json"), "code before the double-buffered hash, sample-ahead 3"),
          ("C", os.path.join(P, "r02_boxes", "boxC_{}_bench.json"), "double-buffered hash, sample-ahead 3"),
          ("D", os.path.join(P, "r02_boxes", "boxD_{}_bench.json"), "sample-ahead 0 with a miss path"),
-         ("final", os.path.join(P, "r02_{}_bench.json"), "final code (4 positions per thread in k_relabel_pad): the "
+         ("E", os.path.join(P, "r02_boxes", "boxE_{}_bench.json"), "4 positions per thread in k_relabel_pad"),
+         ("final", os.path.join(P, "r02_{}_bench.json"), "final code (e2e region with its own warm-up steps): the "
                                                           "committed lines, all from one box")]
 
 
